@@ -270,7 +270,8 @@ alt_status alt_tune(alt_op_kind op, const void *op_params, alt_dtype dtype,
  *  consumer edge_dst[e] (-1 = graph output); edge_numel[e] = its element
  *  count (shape proxy for Alg. 1 line 10).  edge_in_idx[e] = input slot of
  *  the tensor at its consumer (0 = first input).
- *  tuned[e] = 1 if e carries a tuned layout (output of a complex op).
+ *  edge_layout[e] = the tuned layout of e (output of a complex op, chosen by
+ *  alt_tune) or NULL.  An IDENTITY layout is the empty sequence (A21).
  * Outputs per edge: src_edge[e] = the tuned edge whose layout e carries
  *  (-1 = none / default layout); conversion[e] = 1 if Alg. 1 inserts a
  *  conversion op on e (complex -> complex edge).  In this library the
@@ -279,7 +280,7 @@ alt_status alt_tune(alt_op_kind op, const void *op_params, alt_dtype dtype,
 alt_status alt_plan_chain(int32_t n_ops, const int32_t *op_kind, int32_t n_edges,
                           const int32_t *edge_src, const int32_t *edge_dst,
                           const int32_t *edge_in_idx, const int64_t *edge_numel,
-                          const int32_t *tuned, int32_t *src_edge,
+                          const alt_layout *edge_layout, int32_t *src_edge,
                           int32_t *conversion);
 
 #ifdef __cplusplus

@@ -1,0 +1,252 @@
+// capi.cpp — the C-ABI of libalt.so (include/alt.h): validation and dispatch.
+#include <cuda_runtime.h>
+
+#include <atomic>
+#include <cstring>
+#include <new>
+
+#include "alt.h"
+#include "layout.h"
+#include "ops.h"
+
+namespace alt {
+const char *last_error();
+static std::atomic<uint64_t> g_launches{0};
+void count_launch(int n) { g_launches.fetch_add((uint64_t)n, std::memory_order_relaxed); }
+static thread_local alt_kernel_cfg g_last_plan{};
+void set_last_plan(const alt_kernel_cfg &c) { g_last_plan = c; }
+
+// device (or managed) pointer?  Host pointers are rejected: no CPU fallback.
+static bool is_device_ptr(const void *p) {
+  if (!p) return false;
+  cudaPointerAttributes at{};
+  if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged;
+}
+
+static bool shape_is(const Layout *L, int r, const int64_t *s) {
+  if (L->lrank != r) return false;
+  for (int d = 0; d < r; d++)
+    if (L->lshape[d] != s[d]) return false;
+  return true;
+}
+
+static alt_status fill_epi(const alt_epilogue *e, const Layout *yl, OpEpilogue *o) {
+  *o = OpEpilogue{};
+  if (!e) return ALT_OK;
+  if (e->act < 0 || e->act > 2) { set_error("epilogue: unknown activation %d", e->act); return ALT_E_INVALID; }
+  o->scale = e->scale;
+  o->bias = e->bias;
+  o->act = e->act;
+  if ((e->scale && !is_device_ptr(e->scale)) || (e->bias && !is_device_ptr(e->bias))) {
+    set_error("epilogue: scale / bias must be device pointers");
+    return ALT_E_INVALID;
+  }
+  if (e->residual) {
+    if (!e->residual_l) { set_error("epilogue: residual without layout"); return ALT_E_INVALID; }
+    if (!is_device_ptr(e->residual)) { set_error("epilogue: residual must be a device pointer"); return ALT_E_INVALID; }
+    Layout *rl = &e->residual_l->impl;
+    if (!shape_is(rl, yl->lrank, yl->lshape)) { set_error("epilogue: residual logical shape != output"); return ALT_E_SHAPE; }
+    o->residual = e->residual;
+    o->residual_l = rl;
+  }
+  return ALT_OK;
+}
+}  // namespace alt
+
+using namespace alt;
+
+extern "C" {
+
+const char *alt_status_str(alt_status s) {
+  switch (s) {
+    case ALT_OK: return "ALT_OK";
+    case ALT_E_INVALID: return "ALT_E_INVALID";
+    case ALT_E_SHAPE: return "ALT_E_SHAPE";
+    case ALT_E_NONDIVISIBLE: return "ALT_E_NONDIVISIBLE";
+    case ALT_E_LOSSY: return "ALT_E_LOSSY";
+    case ALT_E_UNSUPPORTED: return "ALT_E_UNSUPPORTED";
+    case ALT_E_CUDA: return "ALT_E_CUDA";
+    case ALT_E_NOMEM: return "ALT_E_NOMEM";
+  }
+  return "ALT_E_?";
+}
+
+const char *alt_last_error(void) { return alt::last_error(); }
+
+alt_status alt_layout_create(int32_t logical_rank, const int64_t *logical_shape,
+                             const alt_prim *prims, int32_t nprims, alt_layout *out) {
+  if (!out) { set_error("alt_layout_create: out is NULL"); return ALT_E_INVALID; }
+  *out = nullptr;
+  alt_layout_s *h = new (std::nothrow) alt_layout_s();
+  if (!h) return ALT_E_NOMEM;
+  alt_status st = compile_layout(logical_rank, logical_shape, prims, nprims, &h->impl);
+  if (st != ALT_OK) { delete h; return st; }
+  *out = h;
+  set_error("");
+  return ALT_OK;
+}
+
+alt_status alt_layout_destroy(alt_layout l) {
+  delete l;
+  return ALT_OK;
+}
+
+alt_status alt_layout_query(alt_layout l, int32_t *phys_rank, int64_t *phys_shape,
+                            int64_t *phys_numel, uint32_t *flags) {
+  if (!l) { set_error("alt_layout_query: NULL layout"); return ALT_E_INVALID; }
+  const Layout &L = l->impl;
+  if (phys_rank) *phys_rank = L.prank;
+  if (phys_shape) for (int d = 0; d < L.prank; d++) phys_shape[d] = L.pshape[d];
+  if (phys_numel) *phys_numel = L.pnumel;
+  if (flags) *flags = L.flags;
+  return ALT_OK;
+}
+
+alt_status alt_layout_logical(alt_layout l, int32_t *logical_rank, int64_t *logical_shape) {
+  if (!l) { set_error("alt_layout_logical: NULL layout"); return ALT_E_INVALID; }
+  if (logical_rank) *logical_rank = l->impl.lrank;
+  if (logical_shape) for (int d = 0; d < l->impl.lrank; d++) logical_shape[d] = l->impl.lshape[d];
+  return ALT_OK;
+}
+
+alt_status alt_layout_phys_to_logical(alt_layout l, int64_t j, int64_t *logical_coords, int32_t *valid) {
+  if (!l || !logical_coords || !valid) { set_error("phys_to_logical: NULL argument"); return ALT_E_INVALID; }
+  const Layout &L = l->impl;
+  if (j < 0 || j >= L.pnumel) { set_error("phys_to_logical: index out of range"); return ALT_E_INVALID; }
+  int64_t c[kMaxP];
+  for (int d = L.prank - 1; d >= 0; d--) { c[d] = j % L.pshape[d]; j /= L.pshape[d]; }
+  *valid = host_G(L.desc, c, logical_coords) ? 1 : 0;
+  return ALT_OK;
+}
+
+alt_status alt_layout_logical_to_phys(alt_layout l, const int64_t *logical_coords, int64_t *j) {
+  if (!l || !logical_coords || !j) { set_error("logical_to_phys: NULL argument"); return ALT_E_INVALID; }
+  const Layout &L = l->impl;
+  for (int d = 0; d < L.lrank; d++)
+    if (logical_coords[d] < 0 || logical_coords[d] >= L.lshape[d]) { set_error("logical_to_phys: out of range"); return ALT_E_INVALID; }
+  int64_t c[kMaxP];
+  if (!host_F(L.desc, logical_coords, c)) { set_error("element has no copy"); return ALT_E_LOSSY; }
+  int64_t o = 0;
+  for (int d = 0; d < L.prank; d++) o += c[d] * L.pstride[d];
+  *j = o;
+  return ALT_OK;
+}
+
+alt_status alt_relayout(alt_layout src_l, const void *src, alt_layout dst_l, void *dst,
+                        alt_dtype dtype, alt_stream_t stream) {
+  if (!src_l || !dst_l) { set_error("alt_relayout: NULL layout"); return ALT_E_INVALID; }
+  if (dtype != ALT_F32 && dtype != ALT_BF16) { set_error("alt_relayout: bad dtype"); return ALT_E_INVALID; }
+  if (!is_device_ptr(src) || !is_device_ptr(dst)) { set_error("alt_relayout: src/dst must be device pointers"); return ALT_E_INVALID; }
+  return relayout_launch(&src_l->impl, src, &dst_l->impl, dst, dtype == ALT_BF16 ? 2 : 4,
+                         reinterpret_cast<cudaStream_t>(stream));
+}
+
+alt_status alt_conv2d(const alt_conv2d_params *p, alt_layout x_l, const void *x, alt_layout w_l,
+                      const void *w, alt_layout y_l, void *y, alt_dtype dtype,
+                      const alt_epilogue *epi, const alt_kernel_cfg *cfg, alt_stream_t stream) {
+  if (!p || !x_l || !w_l || !y_l) { set_error("alt_conv2d: NULL argument"); return ALT_E_INVALID; }
+  if (dtype != ALT_F32 && dtype != ALT_BF16) { set_error("alt_conv2d: bad dtype"); return ALT_E_INVALID; }
+  if (p->N < 0 || p->C < 1 || p->H < 1 || p->W < 1 || p->K < 1 || p->R < 1 || p->S < 1 ||
+      p->stride_h < 1 || p->stride_w < 1 || p->pad_h < 0 || p->pad_w < 0) {
+    set_error("alt_conv2d: bad geometry");
+    return ALT_E_INVALID;
+  }
+  if (p->dil_h > 1 || p->dil_w > 1) { set_error("alt_conv2d: dilation > 1 not supported (NEXT)"); return ALT_E_UNSUPPORTED; }
+  const int32_t G = p->groups < 1 ? 1 : p->groups;
+  if (p->C % G || p->K % G) { set_error("alt_conv2d: groups must divide C and K"); return ALT_E_INVALID; }
+  const int64_t Ho = (p->H + 2 * p->pad_h - p->R) / p->stride_h + 1;
+  const int64_t Wo = (p->W + 2 * p->pad_w - p->S) / p->stride_w + 1;
+  if (Ho < 1 || Wo < 1) { set_error("alt_conv2d: empty output"); return ALT_E_INVALID; }
+  const int64_t xs[4] = {p->N, p->C, p->H, p->W}, ws[4] = {p->K, p->C / G, p->R, p->S},
+                ys[4] = {p->N, p->K, Ho, Wo};
+  if (p->N > 0 && (!shape_is(&x_l->impl, 4, xs) || !shape_is(&w_l->impl, 4, ws) || !shape_is(&y_l->impl, 4, ys))) {
+    set_error("alt_conv2d: layout logical shapes do not match x[N,C,H,W] / w[K,C/g,R,S] / y[N,K,Ho,Wo]");
+    return ALT_E_SHAPE;
+  }
+  if (p->N == 0) return ALT_OK;
+  if (!is_device_ptr(x) || !is_device_ptr(w) || !is_device_ptr(y)) { set_error("alt_conv2d: x/w/y must be device pointers"); return ALT_E_INVALID; }
+  ConvProblem P{};
+  P.N = p->N; P.C = p->C; P.H = p->H; P.W = p->W; P.K = p->K; P.R = p->R; P.S = p->S;
+  P.Ho = Ho; P.Wo = Wo;
+  P.Vh = p->stride_h; P.Vw = p->stride_w; P.ph = p->pad_h; P.pw = p->pad_w; P.groups = G;
+  P.xl = &x_l->impl; P.wl = &w_l->impl; P.yl = &y_l->impl;
+  P.x = x; P.w = w; P.y = y; P.dtype = dtype;
+  alt_status st = fill_epi(epi, P.yl, &P.epi);
+  if (st != ALT_OK) return st;
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  const int32_t path = cfg ? cfg->path : ALT_PATH_AUTO;
+  alt_kernel_cfg used{};
+  if (path == ALT_PATH_TC || (path == ALT_PATH_AUTO && G == 1)) {
+    st = tc_conv(P, cfg, s, &used);
+    if (st != ALT_E_UNSUPPORTED || path == ALT_PATH_TC) {
+      if (st == ALT_OK) set_last_plan(used);
+      return st;
+    }
+  }
+  if (path == ALT_PATH_DW || (path == ALT_PATH_AUTO && G == p->C && G == p->K)) {
+    st = dw_conv(P, s, &used);
+    if (st != ALT_E_UNSUPPORTED || path == ALT_PATH_DW) {
+      if (st == ALT_OK) set_last_plan(used);
+      return st;
+    }
+  }
+  st = simt_conv(P, s);
+  if (st == ALT_OK) {
+    used = alt_kernel_cfg{};
+    used.path = ALT_PATH_SIMT;
+    set_last_plan(used);
+  }
+  return st;
+}
+
+alt_status alt_matmul(int64_t M, int64_t N, int64_t K, alt_layout a_l, const void *a,
+                      alt_layout b_l, const void *b, alt_layout c_l, void *c, alt_dtype dtype,
+                      const alt_epilogue *epi, const alt_kernel_cfg *cfg, alt_stream_t stream) {
+  if (!a_l || !b_l || !c_l) { set_error("alt_matmul: NULL layout"); return ALT_E_INVALID; }
+  if (dtype != ALT_F32 && dtype != ALT_BF16) { set_error("alt_matmul: bad dtype"); return ALT_E_INVALID; }
+  if (M < 0 || N < 1 || K < 1) { set_error("alt_matmul: bad sizes"); return ALT_E_INVALID; }
+  const int64_t as[2] = {M, K}, bs[2] = {K, N}, cs[2] = {M, N};
+  if (M > 0 && (!shape_is(&a_l->impl, 2, as) || !shape_is(&b_l->impl, 2, bs) || !shape_is(&c_l->impl, 2, cs))) {
+    set_error("alt_matmul: layout logical shapes do not match A[M,K] / B[K,N] / C[M,N]");
+    return ALT_E_SHAPE;
+  }
+  if (M == 0) return ALT_OK;
+  if (!is_device_ptr(a) || !is_device_ptr(b) || !is_device_ptr(c)) { set_error("alt_matmul: A/B/C must be device pointers"); return ALT_E_INVALID; }
+  GemmProblem P{};
+  P.M = M; P.N = N; P.K = K;
+  P.al = &a_l->impl; P.bl = &b_l->impl; P.cl = &c_l->impl;
+  P.a = a; P.b = b; P.c = c; P.dtype = dtype;
+  alt_status st = fill_epi(epi, P.cl, &P.epi);
+  if (st != ALT_OK) return st;
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  const int32_t path = cfg ? cfg->path : ALT_PATH_AUTO;
+  alt_kernel_cfg used{};
+  if (path == ALT_PATH_TC || path == ALT_PATH_AUTO) {
+    st = tc_gemm(P, cfg, s, &used);
+    if (st != ALT_E_UNSUPPORTED || path == ALT_PATH_TC) {
+      if (st == ALT_OK) set_last_plan(used);
+      return st;
+    }
+  }
+  st = simt_gemm(P, s);
+  if (st == ALT_OK) {
+    used = alt_kernel_cfg{};
+    used.path = ALT_PATH_SIMT;
+    set_last_plan(used);
+  }
+  return st;
+}
+
+alt_status alt_last_plan(alt_kernel_cfg *cfg) {
+  if (!cfg) return ALT_E_INVALID;
+  *cfg = g_last_plan;
+  return ALT_OK;
+}
+
+uint64_t alt_launch_count(void) { return g_launches.load(); }
+
+}  // extern "C"

@@ -1,0 +1,49 @@
+// ops.h — internal operator descriptions passed from the C-ABI layer
+// (capi.cpp) to the kernel launchers.
+#pragma once
+#include <cuda_runtime.h>
+
+#include "layout.h"
+
+namespace alt {
+
+struct OpEpilogue {
+  const float *scale = nullptr;
+  const float *bias = nullptr;
+  const void *residual = nullptr;
+  Layout *residual_l = nullptr;
+  int32_t act = 0;
+};
+
+struct ConvProblem {
+  int64_t N, C, H, W, K, R, S, Ho, Wo;
+  int32_t Vh, Vw, ph, pw, groups;
+  Layout *xl, *wl, *yl;
+  const void *x, *w;
+  void *y;
+  alt_dtype dtype;
+  OpEpilogue epi;
+};
+
+struct GemmProblem {
+  int64_t M, N, K;
+  Layout *al, *bl, *cl;
+  const void *a, *b;
+  void *c;
+  alt_dtype dtype;
+  OpEpilogue epi;
+};
+
+alt_status relayout_launch(Layout *S, const void *src, Layout *D, void *dst, int wb,
+                           cudaStream_t stream);
+alt_status simt_conv(const ConvProblem &P, cudaStream_t stream);
+alt_status simt_gemm(const GemmProblem &P, cudaStream_t stream);
+// tensor-core path; returns ALT_E_UNSUPPORTED (without launching) when the
+// layouts / shapes cannot be served, filling *why
+alt_status tc_conv(const ConvProblem &P, const alt_kernel_cfg *cfg, cudaStream_t stream,
+                   alt_kernel_cfg *used);
+alt_status tc_gemm(const GemmProblem &P, const alt_kernel_cfg *cfg, cudaStream_t stream,
+                   alt_kernel_cfg *used);
+alt_status dw_conv(const ConvProblem &P, cudaStream_t stream, alt_kernel_cfg *used);
+
+}  // namespace alt

@@ -1,0 +1,148 @@
+"""GPU parity of alt_conv2d / alt_matmul against the fp64 oracle, every path
+(tensor-core tcgen05, SIMT generic, depthwise), many layouts, fused
+epilogue, pad-zero / unfold-copy consistency of outputs, invariants I2
+(layout independence) and I3 (pad/unfold input == direct conv)."""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import paper_conf_eurosys_xuxpwwwdxcwc23_b200 as alt
+from paper_conf_eurosys_xuxpwwwdxcwc23_b200 import layouts as LY
+from paper_conf_eurosys_xuxpwwwdxcwc23_b200 import synth
+from tests.helpers import assert_parity, make_operand, read_output, words
+
+pytestmark = pytest.mark.gpu
+
+
+def run_conv(name, N, C, H, W, K, R, S, V, pad, xp, wp, yp, dtype, groups=1, epi=False,
+             res_p=None, act=0, cfg=None, expect_path=None):
+    x = synth.activations(name + "x", (N, C, H, W))
+    w = synth.weights(name + "w", (K, C // groups, R, S))
+    Ho, Wo = (H + 2 * pad - R) // V + 1, (W + 2 * pad - S) // V + 1
+    Xo, xph, xd = make_operand(name, xp, x, dtype)
+    Wo_, wph, wd = make_operand(name, wp, w, dtype)
+    p = alt.conv_params(N, C, H, W, K, R, S, V, pad, groups)
+    Lx, Lw, Ly = alt.Layout(x.shape, xp), alt.Layout(w.shape, wp), alt.Layout((N, K, Ho, Wo), yp)
+    y = torch.full(Ly.phys_shape, 3.0, dtype=dtype, device="cuda")  # poison
+    kw = {}
+    ref_kw = {}
+    if epi:
+        sc, bi = synth.bn_scale(name + "s", K), synth.bn_bias(name + "b", K)
+        kw.update(scale=sc.cuda(), bias=bi.cuda())
+        ref_kw.update(scale=sc.double().numpy(), bias=bi.double().numpy())
+    if res_p is not None:
+        r = synth.activations(name + "r", (N, K, Ho, Wo))
+        Ro, rph, rd = make_operand(name + "r", res_p, r, dtype)
+        kw.update(residual=rd, residual_l=alt.Layout((N, K, Ho, Wo), res_p))
+        ref_kw.update(res_l=Ro, residual=rph)
+    alt.conv2d(p, Lx, xd, Lw, wd, Ly, y, act=act, cfg=cfg, **kw)
+    plan = alt.last_plan()
+    torch.cuda.synchronize()
+    if expect_path is not None:
+        assert plan["path"] == expect_path, plan
+    pd = dict(N=N, C=C, H=H, W=W, K=K, R=R, S=S, stride_h=V, stride_w=V, pad_h=pad, pad_w=pad,
+              groups=groups)
+    ref = oracle.conv2d(pd, Xo, xph, Wo_, wph, act=act, **ref_kw)
+    got = read_output(oracle.Layout((N, K, Ho, Wo), yp), y, dtype)
+    return assert_parity(got, ref, dtype), plan
+
+
+# ---------------------------------------------------------------- config 1 --
+D1 = dict(N=1, C=16, H=14, W=14, K=32, R=3, S=3, V=1, pad=1)
+D1_LAYOUTS = [
+    ("NCHW", [], [], []),
+    ("NCHW4c/KCRS4k4c", LY.nchwxc(16, 4), LY.kcrs_yk_xc(32, 16, 4, 4), LY.nchwxc(32, 4)),
+    ("NHWC/KRSC", LY.nhwc(), [("reorder", [0, 2, 3, 1])], LY.nhwc()),
+    ("NCHW8c/KCRS16k8c", LY.nchwxc(16, 8), LY.kcrs_yk_xc(32, 16, 16, 8), LY.nchwxc(32, 16)),
+    ("tiled unfold in/out", LY.conv_input_tiled(16, 8, 14, 14, 3, 3, 7, 7, 1, 1),
+     LY.kcrs_paper(32, 16, 16, 8), LY.conv_output_tiled(32, 16, 14, 14, 7, 7)),
+    ("padded NCHW16c", LY.nchwxc(16, 16, pad_hw=1), LY.kcrs_yk_xc(32, 16, 32, 16), LY.nchwxc(32, 32)),
+]
+
+
+@pytest.mark.parametrize("lay", D1_LAYOUTS, ids=[l[0] for l in D1_LAYOUTS])
+@pytest.mark.parametrize("dtype", [torch.float32, torch.bfloat16])
+@pytest.mark.parametrize("path", [alt.PATH_AUTO, alt.PATH_SIMT])
+def test_config1_conv_layouts(lay, dtype, path):
+    _, xp, wp, yp = lay
+    run_conv("d1" + lay[0], **D1, xp=xp, wp=wp, yp=yp, dtype=dtype, cfg={"path": path})
+
+
+@pytest.mark.parametrize("dtype", [torch.float32, torch.bfloat16])
+@pytest.mark.parametrize("act", [0, 1, 2])
+def test_epilogue_scale_bias_residual_act(dtype, act):
+    run_conv("epi", 2, 16, 9, 11, 24, 3, 3, 1, 1, LY.nchwxc(16, 8), LY.kcrs_yk_xc(24, 16, 8, 8),
+             LY.nchwxc(24, 8), dtype, epi=True, res_p=LY.nhwc(), act=act)
+
+
+def test_output_pad_and_unfold_copies_written():
+    """The epilogue writes the consumer's tiled + padded input layout
+    directly (propagation, Fig. 5b): zeros in pads, all unfold copies."""
+    yp = LY.conv_input_tiled(16, 8, 14, 14, 3, 3, 7, 7, 1, 1)
+    run_conv("propout", 2, 16, 14, 14, 16, 3, 3, 1, 1, LY.nchwxc(16, 16), LY.kcrs_yk_xc(16, 16, 16, 16),
+             yp, torch.bfloat16, epi=True, act=1)
+
+
+@pytest.mark.parametrize("dtype", [torch.float32, torch.bfloat16])
+def test_depthwise_and_grouped(dtype):
+    run_conv("dw", 2, 32, 14, 14, 32, 3, 3, 1, 1, LY.nchwxc(32, 8), [], LY.nchwxc(32, 8), dtype,
+             groups=32, epi=True, act=2)
+    run_conv("dw2", 2, 32, 15, 15, 32, 3, 3, 2, 1, LY.nchwxc(32, 16), [], LY.nchwxc(32, 16), dtype,
+             groups=32)
+    run_conv("grp", 2, 16, 9, 9, 32, 3, 3, 1, 1, [], [], [], dtype, groups=4)
+
+
+@pytest.mark.parametrize("dtype", [torch.float32, torch.bfloat16])
+def test_layout_independence_I2(dtype):
+    outs = []
+    for i, (_, xp, wp, yp) in enumerate(D1_LAYOUTS):
+        outs.append(run_conv("i2", **D1, xp=xp, wp=wp, yp=yp, dtype=dtype)[0])
+    assert max(outs) <= (1e-5 if dtype == torch.float32 else 2e-2)
+
+
+def test_pad_unfold_input_equals_direct_I3():
+    # same data, semantic padding vs materialised pad + unfold input layouts
+    for xp in ([], LY.nchwxc(16, 8, pad_hw=1), LY.conv_input_tiled(16, 8, 14, 14, 3, 3, 7, 7, 1, 1)):
+        run_conv("i3", **D1, xp=xp, wp=LY.kcrs_yk_xc(32, 16, 16, 8), yp=LY.nchwxc(32, 16),
+                 dtype=torch.float32)
+
+
+# -------------------------------------------------------------------- GEMM --
+def run_gemm(name, M, N, K, ap, bp, cp, dtype, epi=False, cfg=None, expect_path=None):
+    A = synth.activations(name + "A", (M, K))
+    B = synth.weights(name + "B", (K, N))
+    Ao, aph, ad = make_operand(name + "A", ap, A, dtype)
+    Bo, bph, bd = make_operand(name + "B", bp, B, dtype)
+    La, Lb, Lc = alt.Layout((M, K), ap), alt.Layout((K, N), bp), alt.Layout((M, N), cp)
+    c = torch.full(Lc.phys_shape, 5.0, dtype=dtype, device="cuda")
+    kw, ref_kw = {}, {}
+    if epi:
+        bi = synth.bn_bias(name + "b", N)
+        kw.update(bias=bi.cuda(), act=1)
+        ref_kw.update(bias=bi.double().numpy(), act=1)
+    alt.matmul(M, N, K, La, ad, Lb, bd, Lc, c, cfg=cfg, **kw)
+    plan = alt.last_plan()
+    torch.cuda.synchronize()
+    if expect_path is not None:
+        assert plan["path"] == expect_path, plan
+    ref = oracle.gemm(Ao, aph, Bo, bph, **ref_kw)
+    got = read_output(oracle.Layout((M, N), cp), c, dtype)
+    return assert_parity(got, ref, dtype), plan
+
+
+GEMM_LAYOUTS = [
+    ("MK/KN/MN", [], [], []),
+    ("MK/NK(col)/MN", [], LY.transpose2(), []),
+    ("tiled template", LY.gemm_a_tiled(256, 192, 64, 64), LY.gemm_b_tiled_kn(192, 128, 64, 64),
+     LY.gemm_c_tiled(256, 128, 64, 64)),
+    ("NKn", [("split", 0, [16, 16]), ("reorder", [0, 2, 1])], LY.gemm_nkn_b(192, 128), []),
+]
+
+
+@pytest.mark.parametrize("lay", GEMM_LAYOUTS, ids=[l[0] for l in GEMM_LAYOUTS])
+@pytest.mark.parametrize("dtype", [torch.float32, torch.bfloat16])
+@pytest.mark.parametrize("path", [alt.PATH_AUTO, alt.PATH_SIMT])
+def test_gemm_layouts(lay, dtype, path):
+    _, ap, bp, cp = lay
+    run_gemm("g" + lay[0], 256, 128, 192, ap, bp, cp, dtype, epi=True, cfg={"path": path})
