@@ -146,3 +146,72 @@ GEMM_LAYOUTS = [
 def test_gemm_layouts(lay, dtype, path):
     _, ap, bp, cp = lay
     run_gemm("g" + lay[0], 256, 128, 192, ap, bp, cp, dtype, epi=True, cfg={"path": path})
+
+
+# ------------------------------------------------------ tensor-core path --
+TC_CASES = [
+    # name, (N, C, H, W, K, R, S, V, pad), x prims, w prims, y prims
+    ("NCHW64c 3x3", (2, 64, 14, 14, 128, 3, 3, 1, 1), LY.nchwxc(64, 64), LY.kcrs_yk_xc(128, 64, 128, 64),
+     LY.nchwxc(128, 64)),
+    ("NHWC 3x3 C128", (2, 128, 10, 12, 64, 3, 3, 1, 1), LY.nhwc(), [("reorder", [0, 2, 3, 1])], LY.nhwc()),
+    ("NCHW16c/KCRS16k16c", (2, 32, 9, 9, 64, 3, 3, 1, 1), LY.nchwxc(32, 16), LY.kcrs_yk_xc(64, 32, 16, 16),
+     LY.nchwxc(64, 16)),
+    ("NCHW8c/KCRS32k8c", (2, 16, 11, 7, 64, 3, 3, 1, 1), LY.nchwxc(16, 8), LY.kcrs_yk_xc(64, 16, 32, 8),
+     LY.nchwxc(64, 8)),
+    ("NCHW32c stride2", (4, 64, 15, 15, 64, 3, 3, 2, 1), LY.nchwxc(64, 32), LY.kcrs_yk_xc(64, 64, 64, 32),
+     LY.nchwxc(64, 32)),
+    ("1x1 stride2", (4, 128, 14, 14, 256, 1, 1, 2, 0), LY.nchwxc(128, 64), LY.kcrs_yk_xc(256, 128, 64, 64),
+     LY.nchwxc(256, 64)),
+    ("conv1 C3->8 7x7 s2", (2, 3, 32, 32, 64, 7, 7, 2, 3), LY.nchwxc(3, 8, pad_c=5),
+     LY.kcrs_yk_xc(64, 3, 64, 8, pad_c=5), LY.nchwxc(64, 64)),
+    ("padded input", (2, 64, 14, 14, 64, 3, 3, 1, 1), LY.nchwxc(64, 64, pad_hw=1),
+     LY.kcrs_yk_xc(64, 64, 64, 64), LY.nchwxc(64, 64)),
+    ("unfold tiled input", (2, 64, 14, 14, 64, 3, 3, 1, 1),
+     LY.conv_input_tiled(64, 64, 14, 14, 3, 3, 8, 8, 1, 1), LY.kcrs_yk_xc(64, 64, 64, 64), LY.nchwxc(64, 64)),
+    ("unfold tiled input s2 it16", (2, 32, 30, 30, 64, 3, 3, 2, 1),
+     LY.conv_input_tiled(32, 16, 30, 30, 3, 3, 8, 8, 2, 1), LY.kcrs_yk_xc(64, 32, 64, 16), LY.nchwxc(64, 32)),
+    ("unfold out tiled", (2, 64, 14, 14, 128, 3, 3, 1, 1), LY.nchwxc(64, 64), LY.kcrs_yk_xc(128, 64, 128, 64),
+     LY.conv_output_tiled(128, 16, 14, 14, 7, 7)),
+]
+
+
+@pytest.mark.parametrize("case", TC_CASES, ids=[c[0] for c in TC_CASES])
+def test_tc_conv(case):
+    name, (N, C, H, W, K, R, S, V, pad), xp, wp, yp = case
+    run_conv("tc" + name, N, C, H, W, K, R, S, V, pad, xp, wp, yp, torch.bfloat16, epi=True, act=1,
+             cfg={"path": alt.PATH_TC}, expect_path=alt.PATH_TC)
+
+
+def test_tc_unavailable_layout_falls_back_to_simt():
+    """ht = 7 unfold tiles cannot hold a 128-row tensor-core tile: AUTO runs
+    the generic path (still exact), TC reports ALT_E_UNSUPPORTED."""
+    xp = LY.conv_input_tiled(64, 64, 14, 14, 3, 3, 7, 7, 1, 1)
+    _, plan = run_conv("fallback", 2, 64, 14, 14, 64, 3, 3, 1, 1, xp, LY.kcrs_yk_xc(64, 64, 64, 64),
+                       LY.nchwxc(64, 64), torch.bfloat16)
+    assert plan["path"] == alt.PATH_SIMT
+    with pytest.raises(alt.AltError) as e:
+        run_conv("fallback", 2, 64, 14, 14, 64, 3, 3, 1, 1, xp, LY.kcrs_yk_xc(64, 64, 64, 64),
+                 LY.nchwxc(64, 64), torch.bfloat16, cfg={"path": alt.PATH_TC})
+    assert e.value.code == alt._alt.ALT_E_UNSUPPORTED
+
+
+@pytest.mark.parametrize("bn", [64, 128, 256])
+def test_tc_conv_block_n_and_residual(bn):
+    run_conv("tcbn", 2, 64, 16, 16, 256, 3, 3, 1, 1, LY.nchwxc(64, 64), LY.kcrs_yk_xc(256, 64, 256, 64),
+             LY.nchwxc(256, 64), torch.bfloat16, epi=True, res_p=LY.nchwxc(256, 64), act=1,
+             cfg={"path": alt.PATH_TC, "block_n": bn}, expect_path=alt.PATH_TC)
+
+
+TC_GEMM = [
+    ("MK/NK", [], LY.transpose2(), []),
+    ("tiled K-major", LY.gemm_a_tiled(384, 256, 128, 64), LY.gemm_b_tiled_nk(256, 192, 64, 64),
+     LY.gemm_c_tiled(384, 192, 128, 64)),
+    ("tiled mt=64 kt=32", LY.gemm_a_tiled(384, 256, 64, 32), LY.gemm_b_tiled_nk(256, 192, 64, 32), []),
+]
+
+
+@pytest.mark.parametrize("case", TC_GEMM, ids=[c[0] for c in TC_GEMM])
+def test_tc_gemm(case):
+    name, ap, bp, cp = case
+    run_gemm("tcg" + name, 384, 192, 256, ap, bp, cp, torch.bfloat16, epi=True, cfg={"path": alt.PATH_TC},
+             expect_path=alt.PATH_TC)
