@@ -17,14 +17,21 @@ static thread_local alt_kernel_cfg g_last_plan{};
 void set_last_plan(const alt_kernel_cfg &c) { g_last_plan = c; }
 
 // device (or managed) pointer?  Host pointers are rejected: no CPU fallback.
+// Validated pointers are remembered (direct-mapped, per thread) so the hot
+// path does not pay cudaPointerGetAttributes on every call.
 static bool is_device_ptr(const void *p) {
   if (!p) return false;
+  static thread_local const void *seen[512] = {};
+  const size_t h = (reinterpret_cast<uintptr_t>(p) >> 8) & 511;
+  if (seen[h] == p) return true;
   cudaPointerAttributes at{};
   if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
     cudaGetLastError();
     return false;
   }
-  return at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged;
+  const bool ok = at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged;
+  if (ok) seen[h] = p;
+  return ok;
 }
 
 static bool shape_is(const Layout *L, int r, const int64_t *s) {

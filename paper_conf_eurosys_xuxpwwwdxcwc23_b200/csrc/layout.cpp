@@ -8,6 +8,7 @@
 
 #include <cuda_runtime.h>
 
+#include <atomic>
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
@@ -179,6 +180,8 @@ alt_status compile_layout(int32_t lrank, const int64_t *lshape, const alt_prim *
     set_error("alt_layout_create: bad rank %d / nprims %d", lrank, np);
     return ALT_E_INVALID;
   }
+  static std::atomic<uint64_t> next_serial{1};
+  L->serial = next_serial.fetch_add(1);
   LayoutDesc &D = L->desc;
   memset(&D, 0, sizeof(D));
   L->lrank = lrank;

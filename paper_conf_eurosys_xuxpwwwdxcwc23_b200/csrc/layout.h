@@ -62,6 +62,7 @@ struct Affine {
 };
 
 struct Layout {
+  uint64_t serial = 0;  // unique per created layout (plan-cache keys)
   int32_t lrank = 0;
   int64_t lshape[kMaxL] = {};
   int32_t np = 0;

@@ -13,20 +13,27 @@
 // PHYSICAL dims and an affine rule for box coordinates; the innermost
 // physical dim (a channel tile of x elements) becomes the 16/32/64/128-byte
 // K-major row of a UMMA canonical smem layout (swizzle = row bytes).  No data
-// is converted to run on the tensor cores.
+// is converted to run on the tensor cores.  The output is written
+// the same way in reverse (TMA store boxes cut from y's layout), so a layer
+// writes its consumer's layout directly (propagation, Fig. 5b).
 //
-// Kernel: one CTA per 128 x BLOCK_N output tile, 6 warps:
-//   warp 0     TMA producer (one elected thread), STAGES-deep smem ring
-//   warp 1     TMEM allocator + single-thread tcgen05.mma issuer (M=128)
+// Persistent kernel, one CTA per SM, 6 warps:
+//   warp 0     TMA producer (one thread), STAGES-deep smem ring
+//   warp 1     TMEM allocator + single-thread tcgen05.mma issuer (M = 128),
+//              accumulator double-buffered in TMEM (2 x BLOCK_N columns)
 //   warps 2-5  epilogue: tcgen05.ld -> act(scale*acc + bias + residual) ->
-//              stored through the output layout (propagation, Fig. 5b)
+//              bf16 -> swizzled smem -> TMA store (or the generic writer for
+//              layouts with pads / unfold copies); overlaps the next tile's MMA
 #include <cuda.h>
 #include <cudaTypedefs.h>
 #include <cuda_runtime.h>
 
 #include <algorithm>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
+#include <mutex>
+#include <unordered_map>
 #include <vector>
 
 #include "epilogue.cuh"
@@ -35,41 +42,55 @@
 
 namespace alt {
 
-void set_last_plan(const alt_kernel_cfg &c);
-
 enum Var { V_N0 = 0, V_PT, V_PR, V_QT, V_QR, V_GT, V_GR, V_R, V_S, V_ONE, NVAR };
 
+// box-coordinate rule for one tensor map: coord[d] = sum_k coef[d][k] * var[k]
 struct OperandMap {
   int32_t coef[5][NVAR];
   int32_t divp, divq, divg;
   int32_t slab_bytes;
   int32_t oob0;  // dim-0 coordinate that makes a box all zeros
-  int32_t _pad;
+  int32_t sw;    // slab width (channels)
 };
 
 struct TcArgs {
-  OperandMap A, B;
+  OperandMap A, B, O;
+  int32_t out_mode;      // 1: TMA-store epilogue, 0: generic writer
   int32_t is_conv;
   int32_t N, K, Ho, Wo;  // output: conv y[N,K,Ho,Wo]; GEMM: N=1, Ho=1, Wo=M, K=cols
   int32_t tile_n, tile_h, tile_w;
   int32_t mt_h, mt_w;    // # tiles along h, w (n is the slowest)
+  int32_t num_n_tiles, num_tiles;
   int32_t S, Gc;
   int32_t total_slabs, spi, num_iters;
   int32_t sw;
-  int32_t vec_out;       // output fast path (single copy, contiguous channel runs)
-  const int64_t *yrd[4];
   Writer yw;
   EpiParams epi;
+  uint64_t *dbg;         // optional per-CTA timestamps (ALT_TC_DEBUG)
 };
 
 constexpr int kThreads = 192;
+constexpr int kStageBytesA = 128 * 64 * 2;
+constexpr int kOutStage = 128 * 64 * 2;  // one 64-column bf16 chunk of the tile
 
 template <int BN, int STAGES>
 struct TcSmem {
-  static constexpr int kA = 128 * 64 * 2;  // bytes per stage, A
-  static constexpr int kB = BN * 64 * 2;   // bytes per stage, B
-  static constexpr int kBytes = STAGES * (kA + kB) + 1024 /*barriers*/ + 1024 /*align slack*/;
+  static constexpr int kB = BN * 64 * 2;
+  static constexpr int kRing = STAGES * (kStageBytesA + kB);
+  static constexpr int kOut = kRing;                       // staging for TMA stores
+  static constexpr int kScale = kOut + kOutStage;          // BN floats
+  static constexpr int kBias = kScale + BN * 4;            // BN floats
+  static constexpr int kBar = kBias + BN * 4;              // barriers
+  static constexpr int kBytes = kBar + 256 + 1024 /*align slack*/;
 };
+
+__device__ __forceinline__ uint64_t gtimer() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+#define DBG(slot) \
+  if (a.dbg) a.dbg[(size_t)blockIdx.x * 8 + (slot)] = gtimer()
 
 __device__ __forceinline__ void coords(const OperandMap &m, const int32_t (&v)[NVAR], int32_t (&c)[5]) {
 #pragma unroll
@@ -81,185 +102,259 @@ __device__ __forceinline__ void coords(const OperandMap &m, const int32_t (&v)[N
   }
 }
 
-template <typename OutT>
-__device__ __forceinline__ void store_vec(OutT *y, int64_t off, const float *v);
-template <>
-__device__ __forceinline__ void store_vec<uint16_t>(uint16_t *y, int64_t off, const float *v) {
-  uint4 u;
-  u.x = (uint32_t)f32_to_bf16_rne(v[0]) | ((uint32_t)f32_to_bf16_rne(v[1]) << 16);
-  u.y = (uint32_t)f32_to_bf16_rne(v[2]) | ((uint32_t)f32_to_bf16_rne(v[3]) << 16);
-  u.z = (uint32_t)f32_to_bf16_rne(v[4]) | ((uint32_t)f32_to_bf16_rne(v[5]) << 16);
-  u.w = (uint32_t)f32_to_bf16_rne(v[6]) | ((uint32_t)f32_to_bf16_rne(v[7]) << 16);
-  *reinterpret_cast<uint4 *>(y + off) = u;
+__device__ __forceinline__ void named_bar(int id, int n) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory");
 }
-template <>
-__device__ __forceinline__ void store_vec<float>(float *y, int64_t off, const float *v) {
-  *reinterpret_cast<float4 *>(y + off) = make_float4(v[0], v[1], v[2], v[3]);
-  *reinterpret_cast<float4 *>(y + off + 4) = make_float4(v[4], v[5], v[6], v[7]);
+__device__ __forceinline__ void fence_async_smem() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+__device__ __forceinline__ void tma_store_5d(const CUtensorMap *m, const void *src, int32_t c0, int32_t c1,
+                                             int32_t c2, int32_t c3, int32_t c4) {
+  asm volatile(
+      "cp.async.bulk.tensor.5d.global.shared::cta.tile.bulk_group [%0, {%2, %3, %4, %5, %6}], [%1];" ::"l"(
+          reinterpret_cast<uint64_t>(m)),
+      "r"(sm100::smem_u32(src)), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(c4)
+      : "memory");
 }
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 
-template <int BN, int STAGES, typename OutT>
-__global__ void __launch_bounds__(kThreads, 1)
-    k_tc_igemm(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-               const __grid_constant__ TcArgs a, OutT *__restrict__ y) {
-  using namespace sm100;
-  extern __shared__ __align__(1024) unsigned char smem_raw[];
-  // 1024-align the ring (swizzle atoms)
-  unsigned char *smem = reinterpret_cast<unsigned char *>(
-      (reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  constexpr int kA = TcSmem<BN, STAGES>::kA, kB = TcSmem<BN, STAGES>::kB;
-  unsigned char *sA = smem;
-  unsigned char *sB = smem + STAGES * kA;
-  uint64_t *full = reinterpret_cast<uint64_t *>(smem + STAGES * (kA + kB));
-  uint64_t *empty = full + STAGES;
-  uint64_t *tmem_full = empty + STAGES;
-  uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(tmem_full + 1);
-
-  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
-  // M tile -> (n0, p0, q0); N tile -> k0
-  const int mt = blockIdx.x;
+struct TileCoord { int n0, p0, q0, k0; };
+__device__ __forceinline__ TileCoord tile_coord(const TcArgs &a, int tile, int BN) {
+  const int mt = tile / a.num_n_tiles, nt = tile % a.num_n_tiles;
   const int tw_i = mt % a.mt_w;
   const int th_i = (mt / a.mt_w) % a.mt_h;
   const int tn_i = mt / (a.mt_w * a.mt_h);
-  const int n0 = tn_i * a.tile_n, p0 = th_i * a.tile_h, q0 = tw_i * a.tile_w;
-  const int k0 = blockIdx.y * BN;
+  return {tn_i * a.tile_n, th_i * a.tile_h, tw_i * a.tile_w, nt * BN};
+}
 
+template <int BN, int STAGES>
+__global__ void __launch_bounds__(kThreads, 1)
+    k_tc_conv(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+              const __grid_constant__ CUtensorMap tmY, const __grid_constant__ TcArgs a, uint16_t *__restrict__ y) {
+  using namespace sm100;
+  using L = TcSmem<BN, STAGES>;
+  extern __shared__ __align__(1024) unsigned char smem_raw[];
+  unsigned char *smem = reinterpret_cast<unsigned char *>(
+      (reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  unsigned char *sA = smem;
+  unsigned char *sB = smem + STAGES * kStageBytesA;
+  unsigned char *sOut = smem + L::kOut;
+  float *sScale = reinterpret_cast<float *>(smem + L::kScale);
+  float *sBias = reinterpret_cast<float *>(smem + L::kBias);
+  uint64_t *full = reinterpret_cast<uint64_t *>(smem + L::kBar);
+  uint64_t *empty = full + STAGES;
+  uint64_t *tfull = empty + STAGES;   // [2]
+  uint64_t *tempty = tfull + 2;       // [2]
+  uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(tempty + 2);
+
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  if (threadIdx.x == 0) { DBG(0); }
   if (warp == 0 && lane == 0) {
     tma_prefetch(&tmA);
     tma_prefetch(&tmB);
+    if (a.out_mode) tma_prefetch(&tmY);
     for (int s = 0; s < STAGES; s++) {
       mbar_init(&full[s], 1);
       mbar_init(&empty[s], 1);
     }
-    mbar_init(tmem_full, 1);
+    for (int s = 0; s < 2; s++) {
+      mbar_init(&tfull[s], 1);
+      mbar_init(&tempty[s], 128);
+    }
     fence_mbar_init();
   }
-  if (warp == 1) tmem_alloc<(BN < 32 ? 32 : BN)>(tmem_slot);
+  if (warp == 1) tmem_alloc<2 * BN>(tmem_slot);
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
+  if (threadIdx.x == 0) { DBG(1); }
 
   if (warp == 0) {
     if (lane == 0) {
-      // ------------------------------------------------ TMA producer
-      int32_t va[NVAR], vb[NVAR];
-      va[V_N0] = n0;
-      va[V_PT] = p0 / a.A.divp; va[V_PR] = p0 % a.A.divp;
-      va[V_QT] = q0 / a.A.divq; va[V_QR] = q0 % a.A.divq;
-      va[V_ONE] = 1;
-      vb[V_N0] = 0; vb[V_PT] = 0; vb[V_PR] = 0;
-      vb[V_QT] = k0 / a.B.divq; vb[V_QR] = k0 % a.B.divq;
-      vb[V_ONE] = 1;
-      const int RS_G = a.Gc;
-      for (int it = 0; it < a.num_iters; it++) {
-        const int stage = it % STAGES, round = it / STAGES;
-        if (round > 0) mbar_wait(&empty[stage], (round - 1) & 1);
-        mbar_expect_tx(&full[stage], kA + kB);
-        for (int j = 0; j < a.spi; j++) {
-          const int slab = it * a.spi + j;
-          const bool valid = slab < a.total_slabs;
-          const int sl = valid ? slab : 0;
-          const int tap = sl / RS_G, g = sl % RS_G;
-          const int r = tap / a.S, s = tap % a.S;
-          va[V_GT] = g / a.A.divg; va[V_GR] = g % a.A.divg; va[V_R] = r; va[V_S] = s;
-          vb[V_GT] = g / a.B.divg; vb[V_GR] = g % a.B.divg; vb[V_R] = r; vb[V_S] = s;
-          int32_t ca[5], cb[5];
-          coords(a.A, va, ca);
-          coords(a.B, vb, cb);
-          if (!valid) { ca[0] = a.A.oob0; cb[0] = a.B.oob0; }
-          tma_load_5d(sA + stage * kA + j * a.A.slab_bytes, &tmA, &full[stage], ca[0], ca[1], ca[2], ca[3], ca[4]);
-          tma_load_5d(sB + stage * kB + j * a.B.slab_bytes, &tmB, &full[stage], cb[0], cb[1], cb[2], cb[3], cb[4]);
+      // ------------------------------------------------------ TMA producer
+      int it = 0;
+      for (int tile = blockIdx.x; tile < a.num_tiles; tile += gridDim.x) {
+        const TileCoord tc = tile_coord(a, tile, BN);
+        int32_t va[NVAR], vb[NVAR];
+        va[V_N0] = tc.n0;
+        va[V_PT] = tc.p0 / a.A.divp; va[V_PR] = tc.p0 % a.A.divp;
+        va[V_QT] = tc.q0 / a.A.divq; va[V_QR] = tc.q0 % a.A.divq;
+        va[V_ONE] = 1;
+        vb[V_N0] = 0; vb[V_PT] = 0; vb[V_PR] = 0;
+        vb[V_QT] = tc.k0 / a.B.divq; vb[V_QR] = tc.k0 % a.B.divq;
+        vb[V_ONE] = 1;
+        for (int kit = 0; kit < a.num_iters; kit++, it++) {
+          const int stage = it % STAGES, round = it / STAGES;
+          if (round > 0) mbar_wait(&empty[stage], (round - 1) & 1);
+          mbar_expect_tx(&full[stage], kStageBytesA + L::kB);
+          for (int j = 0; j < a.spi; j++) {
+            const int slab = kit * a.spi + j;
+            const bool valid = slab < a.total_slabs;
+            const int sl = valid ? slab : 0;
+            const int tap = sl / a.Gc, g = sl % a.Gc;
+            const int r = tap / a.S, s = tap % a.S;
+            va[V_GT] = g / a.A.divg; va[V_GR] = g % a.A.divg; va[V_R] = r; va[V_S] = s;
+            vb[V_GT] = g / a.B.divg; vb[V_GR] = g % a.B.divg; vb[V_R] = r; vb[V_S] = s;
+            int32_t ca[5], cb[5];
+            coords(a.A, va, ca);
+            coords(a.B, vb, cb);
+            if (!valid) { ca[0] = a.A.oob0; cb[0] = a.B.oob0; }
+            tma_load_5d(sA + stage * kStageBytesA + j * a.A.slab_bytes, &tmA, &full[stage], ca[0], ca[1], ca[2],
+                        ca[3], ca[4]);
+            tma_load_5d(sB + stage * L::kB + j * a.B.slab_bytes, &tmB, &full[stage], cb[0], cb[1], cb[2], cb[3],
+                        cb[4]);
+          }
         }
       }
     }
   } else if (warp == 1) {
     if (lane == 0) {
-      // ------------------------------------------------ MMA issuer
+      // ------------------------------------------------------ MMA issuer
       constexpr uint32_t idesc = idesc_f32acc(1 /*bf16*/, 128, BN);
       const int sw = a.sw;
       const uint32_t layout = sw == 8 ? 0u : (sw == 16 ? 6u : (sw == 32 ? 4u : 2u));
       const uint32_t sbo = sw == 8 ? 128u : (uint32_t)(8 * sw * 2);
       const uint32_t aS = (uint32_t)a.A.slab_bytes, bS = (uint32_t)a.B.slab_bytes;
       const uint32_t lboA = sw == 8 ? aS : 16u, lboB = sw == 8 ? bS : 16u;
-      for (int it = 0; it < a.num_iters; it++) {
-        const int stage = it % STAGES, round = it / STAGES;
-        mbar_wait(&full[stage], round & 1);
+      int it = 0, i = 0;
+      for (int tile = blockIdx.x; tile < a.num_tiles; tile += gridDim.x, i++) {
+        const int acc = i & 1, use = i >> 1;
+        if (use > 0) mbar_wait(&tempty[acc], (use - 1) & 1);
         tc_fence_after();
-        const uint32_t baseA = smem_u32(sA + stage * kA), baseB = smem_u32(sB + stage * kB);
+        const uint32_t d = tmem + (uint32_t)(acc * BN);
+        for (int kit = 0; kit < a.num_iters; kit++, it++) {
+          const int stage = it % STAGES, round = it / STAGES;
+          mbar_wait(&full[stage], round & 1);
+          tc_fence_after();
+          const uint32_t baseA = smem_u32(sA + stage * kStageBytesA), baseB = smem_u32(sB + stage * L::kB);
 #pragma unroll
-        for (int kk = 0; kk < 4; kk++) {
-          const int kc = kk * 16;
-          const int slab = kc / sw;
-          const uint32_t off = (uint32_t)((kc % sw) * 2);
-          const uint64_t ad = smem_desc(baseA + slab * aS + off, lboA, sbo, layout);
-          const uint64_t bd = smem_desc(baseB + slab * bS + off, lboB, sbo, layout);
-          mma_bf16(tmem, ad, bd, idesc, (it | kk) != 0);
+          for (int kk = 0; kk < 4; kk++) {
+            const int kc = kk * 16;
+            const int slab = kc / sw;
+            const uint32_t off = (uint32_t)((kc % sw) * 2);
+            const uint64_t ad = smem_desc(baseA + slab * aS + off, lboA, sbo, layout);
+            const uint64_t bd = smem_desc(baseB + slab * bS + off, lboB, sbo, layout);
+            mma_bf16(d, ad, bd, idesc, (kit | kk) != 0);
+          }
+          mma_commit(&empty[stage]);
         }
-        mma_commit(&empty[stage]);
+        mma_commit(&tfull[acc]);
       }
-      mma_commit(tmem_full);
     }
   } else {
-    // -------------------------------------------------- epilogue warps
-    const int wq = warp & 3;
-    const int row = wq * 32 + lane;
+    // -------------------------------------------------------- epilogue
+    const int et = threadIdx.x - 64;       // 0..127
+    const int wq = warp & 3;               // TMEM lane quarter of this warp
+    const int row = wq * 32 + lane;        // accumulator row = tile row
     const int tn = a.tile_h * a.tile_w;
-    const int n = n0 + row / tn, p = p0 + (row / a.tile_w) % a.tile_h, q = q0 + row % a.tile_w;
-    const bool vrow = n < a.N && p < a.Ho && q < a.Wo;
-    mbar_wait(tmem_full, 0);
-    tc_fence_after();
-    int64_t base = 0;
-    if (vrow && a.vec_out) {
-      base = a.is_conv ? (__ldg(a.yrd[0] + n) + __ldg(a.yrd[2] + p) + __ldg(a.yrd[3] + q))
-                       : __ldg(a.yrd[0] + q);
-    }
+    const int sw_o = a.O.sw;
+    const int pitch = sw_o * 2;            // bytes per row in a staging slab
+    const int swz = pitch == 128 ? 3 : (pitch == 64 ? 2 : (pitch == 32 ? 1 : 0));
+    int i = 0;
+    for (int tile = blockIdx.x; tile < a.num_tiles; tile += gridDim.x, i++) {
+      const int acc = i & 1, use = i >> 1;
+      const TileCoord tc = tile_coord(a, tile, BN);
+      // per-tile scale / bias into smem (previous tile finished with them)
+      named_bar(1, 128);
+      for (int c = et; c < BN; c += 128) {
+        const int k = tc.k0 + c;
+        sScale[c] = (a.epi.scale && k < a.K) ? __ldg(a.epi.scale + k) : 1.f;
+        sBias[c] = (a.epi.bias && k < a.K) ? __ldg(a.epi.bias + k) : 0.f;
+      }
+      named_bar(1, 128);
+      const int n = tc.n0 + row / tn, p = tc.p0 + (row / a.tile_w) % a.tile_h, q = tc.q0 + row % a.tile_w;
+      const bool vrow = n < a.N && p < a.Ho && q < a.Wo;
+      mbar_wait(&tfull[acc], use & 1);
+      tc_fence_after();
 #pragma unroll 1
-    for (int c0 = 0; c0 < BN; c0 += 32) {
-      uint32_t raw[32];
-      tmem_ld_32x32b_x32(tmem + ((uint32_t)(wq * 32) << 16) + (uint32_t)c0, raw);
-      tmem_ld_wait();
-      if (!vrow) continue;
-      float v[32];
-#pragma unroll
-      for (int j = 0; j < 32; j++) {
-        const int k = k0 + c0 + j;
-        float t = __uint_as_float(raw[j]);
-        if (k < a.K) {
-          if (a.epi.scale) t *= __ldg(a.epi.scale + k);
-          if (a.epi.bias) t += __ldg(a.epi.bias + k);
+      for (int c0 = 0; c0 < BN; c0 += 64) {
+        uint32_t raw[64];
+        const uint32_t taddr = tmem + ((uint32_t)(wq * 32) << 16) + (uint32_t)(acc * BN + c0);
+        tmem_ld_32x32b_x32(taddr, *reinterpret_cast<uint32_t(*)[32]>(raw));
+        tmem_ld_32x32b_x32(taddr + 32, *reinterpret_cast<uint32_t(*)[32]>(raw + 32));
+        tmem_ld_wait();
+        if (c0 + 64 >= BN) {  // accumulator buffer drained: MMA may reuse it
+          tc_fence_before();
+          mbar_arrive(&tempty[acc]);
         }
-        v[j] = t;
-      }
-      if (a.epi.residual) {
-        const OutT *res = static_cast<const OutT *>(a.epi.residual);
-#pragma unroll 4
-        for (int j = 0; j < 32; j++) {
-          const int k = k0 + c0 + j;
-          if (k >= a.K) break;
-          const int64_t o = a.is_conv ? a.epi.res.off4(n, k, p, q) : a.epi.res.off2(q, k);
-          if (o >= 0) v[j] += load_as_f32<OutT>(res, o);
+        float v[64];
+#pragma unroll
+        for (int j = 0; j < 64; j++) v[j] = __uint_as_float(raw[j]) * sScale[c0 + j] + sBias[c0 + j];
+        if (a.epi.residual && vrow) {
+          const uint16_t *res = static_cast<const uint16_t *>(a.epi.residual);
+#pragma unroll
+          for (int j = 0; j < 64; j++) {
+            const int k = tc.k0 + c0 + j;
+            if (k < a.K) {
+              const int64_t o = a.is_conv ? a.epi.res.off4(n, k, p, q) : a.epi.res.off2(q, k);
+              if (o >= 0) v[j] += bf16_to_f32(__ldg(res + o));
+            }
+          }
         }
-      }
 #pragma unroll
-      for (int j = 0; j < 32; j++) v[j] = apply_act(v[j], a.epi.act);
-      if (a.vec_out && k0 + c0 + 32 <= a.K) {
-        const int64_t *rk = a.is_conv ? a.yrd[1] : a.yrd[1];
+        for (int j = 0; j < 64; j++) v[j] = apply_act(v[j], a.epi.act);
+        if (a.out_mode) {
+          // staging buffer free once the previous chunk's TMA store read it
+          if (et == 0) bulk_wait_read0();
+          named_bar(1, 128);
+          // row `row`: 64 channels -> 64/sw_o slabs of `pitch` bytes, swizzled
 #pragma unroll
-        for (int j = 0; j < 32; j += 8) store_vec<OutT>(y, base + __ldg(rk + k0 + c0 + j), v + j);
-      } else {
-        for (int j = 0; j < 32; j++) {
-          const int k = k0 + c0 + j;
-          if (k >= a.K) break;
-          if (a.is_conv) write4<OutT>(a.yw, y, n, k, p, q, from_f32<OutT>(v[j]));
-          else write2<OutT>(a.yw, y, q, k, from_f32<OutT>(v[j]));
+          for (int c = 0; c < 8; c++) {  // 8 chunks of 16 B = 8 channels
+            const int ch = c * 8;
+            const int slab = ch / sw_o;
+            const int within = (ch % sw_o) * 2;  // byte offset in the slab row
+            uint32_t off = (uint32_t)(row * pitch + within);
+            off ^= ((off >> 7) & ((1u << swz) - 1u)) << 4;
+            uint4 u;
+            u.x = (uint32_t)f32_to_bf16_rne(v[ch + 0]) | ((uint32_t)f32_to_bf16_rne(v[ch + 1]) << 16);
+            u.y = (uint32_t)f32_to_bf16_rne(v[ch + 2]) | ((uint32_t)f32_to_bf16_rne(v[ch + 3]) << 16);
+            u.z = (uint32_t)f32_to_bf16_rne(v[ch + 4]) | ((uint32_t)f32_to_bf16_rne(v[ch + 5]) << 16);
+            u.w = (uint32_t)f32_to_bf16_rne(v[ch + 6]) | ((uint32_t)f32_to_bf16_rne(v[ch + 7]) << 16);
+            *reinterpret_cast<uint4 *>(sOut + slab * 128 * pitch + off) = u;
+          }
+          fence_async_smem();
+          named_bar(1, 128);
+          if (et == 0) {
+            int32_t vo[NVAR];
+            vo[V_N0] = tc.n0;
+            vo[V_PT] = tc.p0 / a.O.divp; vo[V_PR] = tc.p0 % a.O.divp;
+            vo[V_QT] = tc.q0 / a.O.divq; vo[V_QR] = tc.q0 % a.O.divq;
+            vo[V_R] = 0; vo[V_S] = 0; vo[V_ONE] = 1;
+            const int nslab = 64 / sw_o;
+            for (int j = 0; j < nslab; j++) {
+              if (tc.k0 + c0 + j * sw_o >= a.K) break;  // channels past K: nothing to store
+              const int g = (tc.k0 + c0) / sw_o + j;
+              vo[V_GT] = g / a.O.divg; vo[V_GR] = g % a.O.divg;
+              int32_t co[5];
+              coords(a.O, vo, co);
+              tma_store_5d(&tmY, sOut + j * 128 * pitch, co[0], co[1], co[2], co[3], co[4]);
+            }
+            bulk_commit();
+          }
+        } else if (vrow) {
+          // generic layouts: every copy / pad position through the writer
+#pragma unroll 1
+          for (int j = 0; j < 64; j++) {
+            const int k = tc.k0 + c0 + j;
+            if (k >= a.K) break;
+            float t = 0.f;
+#pragma unroll
+            for (int jj = 0; jj < 64; jj++) t = (jj == j) ? v[jj] : t;
+            const uint16_t h = f32_to_bf16_rne(t);
+            if (a.is_conv) write4<uint16_t>(a.yw, y, n, k, p, q, h);
+            else write2<uint16_t>(a.yw, y, q, k, h);
+          }
         }
       }
     }
+    if (et == 0) { DBG(5); }
+    if (et == 0 && a.out_mode) bulk_wait0();
   }
   tc_fence_before();
   __syncthreads();
-  if (warp == 1) tmem_dealloc<(BN < 32 ? 32 : BN)>(tmem);
+  if (warp == 1) tmem_dealloc<2 * BN>(tmem);
+  if (threadIdx.x == 32) { DBG(6); }
 }
 
 // =========================================================== host planner ==
@@ -288,6 +383,9 @@ struct View {
   int64_t xlo = 0;  // channel run (extent of the stride-1 channel dim)
 };
 
+// Cut a TMA view out of a compiled layout: per logical dim a role (rows n/h/w,
+// channel c, filter taps r/s).  Requires the layout's affine map (split /
+// reorder / pad / unfold sequences); see DESIGN.md §5.
 static bool build_view(const Layout &L, const RoleInfo *roles, int sw, View *out, char *why) {
   auto fail = [&](const char *m) { snprintf(why, 160, "%s", m); return false; };
   if (!L.separable || !L.aff.ok) return fail("layout not separable-affine");
@@ -299,7 +397,6 @@ static bool build_view(const Layout &L, const RoleInfo *roles, int sw, View *out
     const int d = L.pdim_owner[p];
     plist[d][nphys[d]++] = p;
   }
-  // channel: stride-1 innermost dim
   for (int d = 0; d < L.lrank; d++) {
     const RoleInfo &ri = roles[d];
     const int64_t off = L.aff.off[d];
@@ -398,7 +495,7 @@ static bool build_view(const Layout &L, const RoleInfo *roles, int sw, View *out
             hi.coef[VT] = 1;
           }
         } else {
-          // unfold (overlapped tiles): tile must sit inside one
+          // unfold (overlapped tiles): the M tile must sit inside one
           // layout tile; Eq. (1) gives the in-tile offset
           if (ch % ri.V) return fail("unfold stride not a multiple of conv stride");
           const int64_t ht = ch / ri.V;  // windows per layout tile (Eq. 1's w)
@@ -431,8 +528,7 @@ static bool build_view(const Layout &L, const RoleInfo *roles, int sw, View *out
     for (int i = 1; i < v.rank && !merged; i++) {
       for (int j = 1; j < v.rank && !merged; j++) {
         if (i == j || v.d[i].box != 1 || v.d[j].box != 1) continue;
-        // i outer, j inner
-        if (v.d[i].stride != v.d[j].stride * v.d[j].extent) continue;
+        if (v.d[i].stride != v.d[j].stride * v.d[j].extent) continue;  // i outer, j inner
         VDim m = v.d[j];
         m.extent = v.d[i].extent * v.d[j].extent;
         for (int k = 0; k < NVAR; k++) m.coef[k] = (int32_t)(v.d[i].coef[k] * v.d[j].extent + v.d[j].coef[k]);
@@ -444,7 +540,6 @@ static bool build_view(const Layout &L, const RoleInfo *roles, int sw, View *out
     }
     if (!merged) return fail("more than 5 TMA dims and no mergeable pair");
   }
-  // TMA: strides (dims >= 1) must be 16-byte multiples
   *out = v;
   return true;
 }
@@ -505,28 +600,7 @@ static bool encode_view(const View &v, const void *base, int esize, int sw, CUte
   for (int i = 1; i < v.rank; i++) rows *= (int64_t)((v.d[i].box + v.d[i].estride - 1) / v.d[i].estride);
   om->slab_bytes = (int32_t)(rows * row_bytes);
   om->oob0 = (int32_t)v.d[0].extent;
-  return true;
-}
-
-// output fast path: single copy per element, no pads, channel runs of 8
-static bool out_vec_ok(const Layout &L, int chan_dim, int esize) {
-  if (!L.separable || (L.flags & (ALT_HAS_PAD | ALT_HAS_UNFOLD))) return false;
-  for (int d = 0; d < L.lrank; d++)
-    if (L.max_copies[d] != 1) return false;
-  const int V = 8;
-  const auto &rk = L.rd[chan_dim];
-  if (rk.size() % V) return false;
-  for (size_t k = 0; k < rk.size(); k += V) {
-    if (rk[k] < 0 || rk[k] % V) return false;
-    for (int j = 1; j < V; j++)
-      if (rk[k + j] != rk[k] + j) return false;
-  }
-  for (int d = 0; d < L.lrank; d++) {
-    if (d == chan_dim) continue;
-    for (int64_t o : L.rd[d])
-      if (o < 0 || o % V) return false;
-  }
-  (void)esize;
+  om->sw = sw;
   return true;
 }
 
@@ -534,42 +608,139 @@ alt_status make_reader(Layout *L, Reader *r);
 alt_status make_writer(Layout *L, Writer *w);
 alt_status make_epi(const OpEpilogue &e, EpiParams *p);
 
-static int pow2_floor(int64_t x) {
-  int p = 1;
-  while ((int64_t)p * 2 <= x) p *= 2;
-  return p;
+// ---- optional per-CTA timestamps (env ALT_TC_DEBUG=1; developer tool)
+static uint64_t *debug_buffer() {
+  static uint64_t *buf = nullptr;
+  static bool init = false;
+  if (!init) {
+    init = true;
+    const char *e = getenv("ALT_TC_DEBUG");
+    if (e && e[0] == '1' && cudaMalloc(&buf, (size_t)8 * 8 << 20) != cudaSuccess) buf = nullptr;
+  }
+  return buf;
 }
 
-template <int BN, int STAGES, typename OutT>
-static cudaError_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const TcArgs &a, OutT *y, dim3 grid,
-                             cudaStream_t s) {
-  auto kern = k_tc_igemm<BN, STAGES, OutT>;
+}  // namespace alt
+extern "C" int alt__debug_tc(uint64_t *host, int64_t n) {
+  uint64_t *b = alt::debug_buffer();
+  if (!b) return -1;
+  return cudaMemcpy(host, b, (size_t)n * 8, cudaMemcpyDeviceToHost) == cudaSuccess ? 0 : -1;
+}
+namespace alt {
+
+static int num_sms() {
+  static int n = 0;
+  if (!n) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+    if (n <= 0) n = 148;
+  }
+  return n;
+}
+
+template <int BN, int STAGES>
+static cudaError_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUtensorMap &ty, const TcArgs &a,
+                             uint16_t *y, int grid, cudaStream_t s) {
+  auto kern = k_tc_conv<BN, STAGES>;
   const int smem = TcSmem<BN, STAGES>::kBytes;
-  cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  kern<<<grid, kThreads, smem, s>>>(ta, tb, a, y);
+  static_assert(TcSmem<BN, STAGES>::kBytes <= 232448, "smem budget");
+  static bool attr_set = false;  // once per instantiation (not capture-safe to repeat)
+  if (!attr_set) {
+    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    attr_set = true;
+  }
+  kern<<<grid, kThreads, smem, s>>>(ta, tb, ty, a, y);
   return cudaGetLastError();
 }
 
-// common driver for conv and GEMM (GEMM: N=1, H=W... expressed via roles)
+// ---- launch-plan cache: everything the host derives for a call, keyed by
+// the call's arguments (layout serials, pointers, geometry, epilogue, cfg)
+struct TcKey {
+  int64_t v[40];
+  bool operator==(const TcKey &o) const { return memcmp(v, o.v, sizeof(v)) == 0; }
+};
+struct TcKeyHash {
+  size_t operator()(const TcKey &k) const {
+    uint64_t h = 1469598103934665603ull;
+    for (int i = 0; i < 40; i++) h = (h ^ (uint64_t)k.v[i]) * 1099511628211ull;
+    return (size_t)h;
+  }
+};
+struct TcPlan {
+  CUtensorMap ta, tb, ty;
+  TcArgs a;
+  int grid;
+  int BN, stages;
+  alt_kernel_cfg used;
+};
+static std::mutex g_tc_mu;
+static std::unordered_map<TcKey, TcPlan, TcKeyHash> g_tc_cache;
+
+static cudaError_t launch_plan(const TcPlan &pl, void *y, cudaStream_t stream) {
+  uint16_t *yy = static_cast<uint16_t *>(y);
+  if (pl.BN == 64) return launch_tc<64, 8>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+  if (pl.BN == 128) {
+    if (pl.stages == 4) return launch_tc<128, 4>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+    return launch_tc<128, 6>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+  }
+  if (pl.stages == 3) return launch_tc<256, 3>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+  return launch_tc<256, 4>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+}
+
+// common driver for conv and GEMM
 struct TcProblem {
   bool is_conv;
   Layout *al, *bl, *yl;
   const void *a, *b;
   void *y;
-  RoleInfo ra[kMaxL], rb[kMaxL];
+  RoleInfo ra[kMaxL], rb[kMaxL], ry[kMaxL];
   int64_t N, K, Ho, Wo;       // output geometry (GEMM: 1, cols, 1, M)
   int64_t R, S, C;            // taps and reduction channels
-  int y_chan_dim;             // channel dim of y's logical shape
   OpEpilogue epi;
 };
 
 static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t stream, alt_kernel_cfg *used,
                          int tile_n_fixed, int tile_h_fixed) {
   char why[160] = "";
-  // slab width: largest power of two <= 64 dividing both channel runs
-  // (determined after the views are built; try 64 down to 8)
+  TcKey key;
+  memset(&key, 0, sizeof(key));
+  {
+    int64_t *k = key.v;
+    int i = 0;
+    k[i++] = P.is_conv;
+    k[i++] = (int64_t)P.al->serial; k[i++] = (int64_t)P.bl->serial; k[i++] = (int64_t)P.yl->serial;
+    k[i++] = (int64_t)(uintptr_t)P.a; k[i++] = (int64_t)(uintptr_t)P.b; k[i++] = (int64_t)(uintptr_t)P.y;
+    k[i++] = P.N; k[i++] = P.K; k[i++] = P.Ho; k[i++] = P.Wo; k[i++] = P.R; k[i++] = P.S; k[i++] = P.C;
+    for (int d = 0; d < 4; d++) {
+      k[i++] = ((int64_t)P.ra[d].role << 48) | ((int64_t)P.ra[d].V << 32) | ((int64_t)P.ra[d].pad << 16) |
+               P.ra[d].win;
+    }
+    k[i++] = (int64_t)(uintptr_t)P.epi.scale; k[i++] = (int64_t)(uintptr_t)P.epi.bias;
+    k[i++] = (int64_t)(uintptr_t)P.epi.residual;
+    k[i++] = P.epi.residual_l ? (int64_t)P.epi.residual_l->serial : 0;
+    k[i++] = P.epi.act;
+    if (cfg) {
+      k[i++] = cfg->block_n; k[i++] = cfg->tile_n; k[i++] = cfg->tile_h; k[i++] = cfg->tile_w;
+      k[i++] = cfg->stages;
+    }
+    int dev = 0;
+    cudaGetDevice(&dev);
+    k[i++] = dev;
+  }
+  {
+    std::lock_guard<std::mutex> g(g_tc_mu);
+    auto it = g_tc_cache.find(key);
+    if (it != g_tc_cache.end()) {
+      cudaError_t e = launch_plan(it->second, P.y, stream);
+      count_launch();
+      if (e != cudaSuccess) { set_error("tc launch failed: %s", cudaGetErrorString(e)); return ALT_E_CUDA; }
+      if (used) *used = it->second.used;
+      return ALT_OK;
+    }
+  }
   const int esize = 2;
-  // M-tile candidates
+  // M-tile candidates (tile_n x tile_h x tile_w = 128 output pixels)
   struct Cand { int tn, th, tw; };
   std::vector<Cand> cands;
   if (cfg && cfg->tile_n * cfg->tile_h * cfg->tile_w == 128) {
@@ -585,7 +756,7 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
         if (tn > 1 && (tn > P.N)) continue;
         cands.push_back({tn, th, tw});
       }
-    // prefer the least wasted rows: coverage = ceil(Ho/th)*th*ceil(Wo/tw)*tw*ceil(N/tn)*tn
+    // least wasted rows first, then longer contiguous runs
     std::stable_sort(cands.begin(), cands.end(), [&](const Cand &x, const Cand &y) {
       auto cov = [&](const Cand &c) {
         return (double)((P.Ho + c.th - 1) / c.th * c.th) * ((P.Wo + c.tw - 1) / c.tw * c.tw) *
@@ -593,41 +764,63 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       };
       double a = cov(x), b = cov(y);
       if (a != b) return a < b;
-      return x.tw > y.tw;  // longer contiguous runs first
+      return x.tw > y.tw;
     });
   }
-  int BN = cfg && cfg->block_n ? cfg->block_n : (P.K >= 256 && P.K % 256 == 0 ? 256 : (P.K >= 128 ? 128 : 64));
+  int BN = cfg && cfg->block_n ? cfg->block_n : (P.K > 128 ? 256 : (P.K > 64 ? 128 : 64));
   if (BN != 64 && BN != 128 && BN != 256) { set_error("tc: block_n must be 64/128/256"); return ALT_E_UNSUPPORTED; }
   for (const Cand &c : cands) {
-    RoleInfo ra[kMaxL], rb[kMaxL];
+    RoleInfo ra[kMaxL], rb[kMaxL], ry[kMaxL];
     memcpy(ra, P.ra, sizeof(ra));
     memcpy(rb, P.rb, sizeof(rb));
+    memcpy(ry, P.ry, sizeof(ry));
     for (int d = 0; d < kMaxL; d++) {
-      if (ra[d].role == R_N) ra[d].tile = c.tn;
-      if (ra[d].role == R_H) ra[d].tile = c.th;
-      if (ra[d].role == R_W) ra[d].tile = c.tw;
+      for (RoleInfo *r : {&ra[d], &ry[d]}) {
+        if (r->role == R_N) r->tile = c.tn;
+        if (r->role == R_H) r->tile = c.th;
+        if (r->role == R_W) r->tile = c.tw;
+      }
       if (rb[d].role == R_W) rb[d].tile = BN;
     }
     for (int sw = 64; sw >= 8; sw /= 2) {
       View va, vb;
       if (!build_view(*P.al, ra, sw, &va, why)) continue;
       if (!build_view(*P.bl, rb, sw, &vb, why)) continue;
-      // check TMA row count = 128 for A and BN for B
       int64_t rowsA = 1, rowsB = 1;
       for (int i = 1; i < va.rank; i++) rowsA *= (va.d[i].box + va.d[i].estride - 1) / va.d[i].estride;
       for (int i = 1; i < vb.rank; i++) rowsB *= (vb.d[i].box + vb.d[i].estride - 1) / vb.d[i].estride;
       if (rowsA != 128 || rowsB != BN) { snprintf(why, 160, "rows A %lld B %lld", (long long)rowsA, (long long)rowsB); continue; }
-      CUtensorMap ta, tb;
-      TcArgs a;
+      TcPlan pl;
+      TcArgs &a = pl.a;
       memset(&a, 0, sizeof(a));
-      if (!encode_view(va, P.a, esize, sw, &ta, &a.A, why)) continue;
-      if (!encode_view(vb, P.b, esize, sw, &tb, &a.B, why)) continue;
+      if (!encode_view(va, P.a, esize, sw, &pl.ta, &a.A, why)) continue;
+      if (!encode_view(vb, P.b, esize, sw, &pl.tb, &a.B, why)) continue;
+      // output: TMA-store view when y holds one copy per element (no pads /
+      // unfold duplicates) and a >= 8-channel contiguous run, else the writer
+      a.out_mode = 0;
+      memset(&pl.ty, 0, sizeof(pl.ty));
+      if (!(P.yl->flags & (ALT_HAS_PAD | ALT_HAS_UNFOLD))) {
+        char why2[160];
+        for (int so = 64; so >= 8 && !a.out_mode; so /= 2) {
+          View vy;
+          if (!build_view(*P.yl, ry, so, &vy, why2)) continue;
+          int64_t rowsY = 1;
+          for (int i = 1; i < vy.rank; i++) rowsY *= vy.d[i].box;
+          if (rowsY != 128) continue;
+          if (encode_view(vy, P.y, esize, so, &pl.ty, &a.O, why2)) a.out_mode = 1;
+        }
+      }
       a.is_conv = P.is_conv;
       a.N = (int32_t)P.N; a.K = (int32_t)P.K; a.Ho = (int32_t)P.Ho; a.Wo = (int32_t)P.Wo;
       a.tile_n = c.tn; a.tile_h = c.th; a.tile_w = c.tw;
       a.mt_h = (int32_t)((P.Ho + c.th - 1) / c.th);
       a.mt_w = (int32_t)((P.Wo + c.tw - 1) / c.tw);
       const int64_t mt_n = (P.N + c.tn - 1) / c.tn;
+      const int64_t mtiles = mt_n * a.mt_h * a.mt_w;
+      const int64_t ntiles = (P.K + BN - 1) / BN;
+      if (mtiles * ntiles > 0x7fffffff) { set_error("tc: too many tiles"); return ALT_E_UNSUPPORTED; }
+      a.num_n_tiles = (int32_t)ntiles;
+      a.num_tiles = (int32_t)(mtiles * ntiles);
       a.S = (int32_t)P.S;
       a.Gc = (int32_t)((P.C + sw - 1) / sw);
       a.total_slabs = (int32_t)(P.R * P.S * a.Gc);
@@ -637,34 +830,28 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       alt_status st;
       if ((st = make_epi(P.epi, &a.epi)) != ALT_OK) return st;
       if ((st = make_writer(P.yl, &a.yw)) != ALT_OK) return st;
-      a.vec_out = out_vec_ok(*P.yl, P.y_chan_dim, esize) ? 1 : 0;
-      if (a.vec_out) {
-        SepDev sd{};
-        if ((st = device_tables(P.yl, &sd, nullptr)) != ALT_OK) return st;
-        if (P.is_conv) {
-          a.yrd[0] = sd.rd[0]; a.yrd[1] = sd.rd[1]; a.yrd[2] = sd.rd[2]; a.yrd[3] = sd.rd[3];
-        } else {
-          a.yrd[0] = sd.rd[0]; a.yrd[1] = sd.rd[1];
-        }
-      }
-      const int64_t mtiles = mt_n * a.mt_h * a.mt_w;
-      const int64_t ntiles = (P.K + BN - 1) / BN;
-      if (mtiles > 0x7fffffff || ntiles > 65535) { set_error("tc: grid too large"); return ALT_E_UNSUPPORTED; }
-      dim3 grid((unsigned)mtiles, (unsigned)ntiles);
-      cudaError_t e;
-      uint16_t *y = static_cast<uint16_t *>(P.y);
-      if (BN == 64) e = launch_tc<64, 6, uint16_t>(ta, tb, a, y, grid, stream);
-      else if (BN == 128) e = launch_tc<128, 4, uint16_t>(ta, tb, a, y, grid, stream);
-      else e = launch_tc<256, 4, uint16_t>(ta, tb, a, y, grid, stream);
-      count_launch();
-      if (e != cudaSuccess) { set_error("tc launch failed: %s", cudaGetErrorString(e)); return ALT_E_CUDA; }
+      a.dbg = debug_buffer();
+      pl.grid = (int)std::min<int64_t>(a.num_tiles, num_sms());
+      pl.BN = BN;
+      pl.stages = BN == 64 ? 8 : (BN == 128 ? 6 : 4);
+      if (cfg && BN == 128 && cfg->stages == 4) pl.stages = 4;
+      if (cfg && BN == 256 && cfg->stages == 3) pl.stages = 3;
       alt_kernel_cfg u{};
       u.path = ALT_PATH_TC;
       u.block_m = 128;
       u.block_n = BN;
       u.block_k = 64;
-      u.stages = BN == 64 ? 6 : 4;
+      u.stages = pl.stages;
       u.tile_n = c.tn; u.tile_h = c.th; u.tile_w = c.tw;
+      pl.used = u;
+      cudaError_t e = launch_plan(pl, P.y, stream);
+      count_launch();
+      if (e != cudaSuccess) { set_error("tc launch failed: %s", cudaGetErrorString(e)); return ALT_E_CUDA; }
+      {
+        std::lock_guard<std::mutex> g(g_tc_mu);
+        if (g_tc_cache.size() > 4096) g_tc_cache.clear();
+        g_tc_cache.emplace(key, pl);
+      }
       if (used) *used = u;
       return ALT_OK;
     }
@@ -680,18 +867,21 @@ alt_status tc_conv(const ConvProblem &P, const alt_kernel_cfg *cfg, cudaStream_t
   T.is_conv = true;
   T.al = P.xl; T.bl = P.wl; T.yl = P.yl;
   T.a = P.x; T.b = P.w; T.y = P.y;
-  // x logical (n, c, h, w); w logical (k, c, r, s)
+  // x logical (n, c, h, w); w logical (k, c, r, s); y logical (n, k, p, q)
   T.ra[0].role = R_N;
   T.ra[1].role = R_C;
   T.ra[2] = RoleInfo{R_H, 1, P.Vh, P.ph, (int)P.R, 1};
   T.ra[3] = RoleInfo{R_W, 1, P.Vw, P.pw, (int)P.S, 1};
-  T.rb[0] = RoleInfo{R_W, 1, 1, 0, 1};
+  T.rb[0] = RoleInfo{R_W, 1, 1, 0, 1, 0};
   T.rb[1].role = R_C;
   T.rb[2].role = R_TR;
   T.rb[3].role = R_TS;
+  T.ry[0].role = R_N;
+  T.ry[1].role = R_C;
+  T.ry[2] = RoleInfo{R_H, 1, 1, 0, 1, 0};
+  T.ry[3] = RoleInfo{R_W, 1, 1, 0, 1, 0};
   T.N = P.N; T.K = P.K; T.Ho = P.Ho; T.Wo = P.Wo;
   T.R = P.R; T.S = P.S; T.C = P.C;
-  T.y_chan_dim = 1;
   T.epi = P.epi;
   if (P.N * P.Ho * P.Wo >= (1ll << 31)) { set_error("tc: too many output pixels"); return ALT_E_UNSUPPORTED; }
   return tc_run(T, cfg, stream, used, 0, 0);
@@ -703,15 +893,17 @@ alt_status tc_gemm(const GemmProblem &P, const alt_kernel_cfg *cfg, cudaStream_t
   T.is_conv = false;
   T.al = P.al; T.bl = P.bl; T.yl = P.cl;
   T.a = P.a; T.b = P.b; T.y = P.c;
-  // A logical (m, k): m = rows (W role), k = reduction; B logical (k, n)
-  T.ra[0] = RoleInfo{R_W, 128, 1, 0, 1};
+  // A logical (m, k): m = rows (W role), k = reduction; B logical (k, n); C (m, n)
+  T.ra[0] = RoleInfo{R_W, 128, 1, 0, 1, 0};
   T.ra[1].role = R_C;
   T.rb[0].role = R_C;
-  T.rb[1] = RoleInfo{R_W, 1, 1, 0, 1};
+  T.rb[1] = RoleInfo{R_W, 1, 1, 0, 1, 0};
+  T.ry[0] = RoleInfo{R_W, 128, 1, 0, 1, 0};
+  T.ry[1].role = R_C;
   T.N = 1; T.K = P.N; T.Ho = 1; T.Wo = P.M;
   T.R = 1; T.S = 1; T.C = P.K;
-  T.y_chan_dim = 1;
   T.epi = P.epi;
+  if (P.M >= (1ll << 31)) { set_error("tc: M too large"); return ALT_E_UNSUPPORTED; }
   return tc_run(T, cfg, stream, used, 1, 1);
 }
 

@@ -1,0 +1,9 @@
+cd $GRAFT_REPO_ROOT
+timeout 600 python -m pytest tests -q -x -m gpu 2>&1 | tail -5
+timeout 600 python bench.py --steps 10 --warmup 3 --no-cpu-baseline > gpurun_out/bench5.json 2> gpurun_out/bench5.err
+tail -2 gpurun_out/bench5.err
+python -c "
+import json; d=json.loads(open('gpurun_out/bench5.json').read().strip().splitlines()[-1])
+for l in d.pop('per_layer'): print(l)
+print({k: d[k] for k in ('value','ms_per_step','gpu_launches','e2e','clocks')}, d['roofline']['achieved'])
+"
