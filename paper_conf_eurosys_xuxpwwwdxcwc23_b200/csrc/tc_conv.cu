@@ -69,7 +69,7 @@ struct TcArgs {
   uint64_t *dbg;         // optional per-CTA timestamps (ALT_TC_DEBUG)
 };
 
-constexpr int kThreads = 192;
+constexpr int kThreads = 320;  // producer, MMA, 8 epilogue warps
 constexpr int kStageBytesA = 128 * 64 * 2;
 constexpr int kOutStage = 128 * 64 * 2;  // one 64-column bf16 chunk of the tile
 
@@ -77,11 +77,9 @@ template <int BN, int STAGES>
 struct TcSmem {
   static constexpr int kB = BN * 64 * 2;
   static constexpr int kRing = STAGES * (kStageBytesA + kB);
-  static constexpr int kOut = kRing;                       // staging for TMA stores
-  static constexpr int kScale = kOut + kOutStage;          // BN floats
-  static constexpr int kBias = kScale + BN * 4;            // BN floats
-  static constexpr int kBar = kBias + BN * 4;              // barriers
-  static constexpr int kBytes = kBar + 256 + 1024 /*align slack*/;
+  static constexpr int kOut = kRing;                       // 2 staging buffers for TMA stores
+  static constexpr int kBar = kOut + 2 * kOutStage;        // barriers
+  static constexpr int kBytes = kBar + 128 + 1008 /*1024-B alignment slack*/;
 };
 
 __device__ __forceinline__ uint64_t gtimer() {
@@ -90,7 +88,7 @@ __device__ __forceinline__ uint64_t gtimer() {
   return t;
 }
 #define DBG(slot) \
-  if (a.dbg) a.dbg[(size_t)blockIdx.x * 8 + (slot)] = gtimer()
+  if (a.dbg) a.dbg[(size_t)blockIdx.x * 32 + (slot)] = gtimer()
 
 __device__ __forceinline__ void coords(const OperandMap &m, const int32_t (&v)[NVAR], int32_t (&c)[5]) {
 #pragma unroll
@@ -115,8 +113,35 @@ __device__ __forceinline__ void tma_store_5d(const CUtensorMap *m, const void *s
       : "memory");
 }
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
-__device__ __forceinline__ void bulk_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_read1() { asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+
+// Out-of-line slow paths of the epilogue (kept out of the hot loop body).
+// residual values of one row's 32 channels, read through the residual layout
+static __device__ __noinline__ void residual_chunk(const EpiParams &e, int is_conv, int K, int n, int p, int q,
+                                                   int kb, float *out) {
+  const uint16_t *res = static_cast<const uint16_t *>(e.residual);
+  for (int j = 0; j < 32; j++) {
+    const int k = kb + j;
+    float r = 0.f;
+    if (k < K) {
+      const int64_t o = is_conv ? e.res.off4(n, k, p, q) : e.res.off2(q, k);
+      if (o >= 0) r = bf16_to_f32(__ldg(res + o));
+    }
+    out[j] = r;
+  }
+}
+// one row's 32 channels through the generic writer (pads, unfold copies)
+static __device__ __noinline__ void write_chunk(const Writer &w, int is_conv, int K, uint16_t *y, int n, int p,
+                                                int q, int kb, const uint32_t *pk) {
+  for (int j = 0; j < 32; j++) {
+    const int k = kb + j;
+    if (k >= K) break;
+    const uint16_t h = (uint16_t)(j & 1 ? pk[j >> 1] >> 16 : pk[j >> 1] & 0xffff);
+    if (is_conv) write4<uint16_t>(w, y, n, k, p, q, h);
+    else write2<uint16_t>(w, y, q, k, h);
+  }
+}
 
 struct TileCoord { int n0, p0, q0, k0; };
 __device__ __forceinline__ TileCoord tile_coord(const TcArgs &a, int tile, int BN) {
@@ -139,8 +164,6 @@ __global__ void __launch_bounds__(kThreads, 1)
   unsigned char *sA = smem;
   unsigned char *sB = smem + STAGES * kStageBytesA;
   unsigned char *sOut = smem + L::kOut;
-  float *sScale = reinterpret_cast<float *>(smem + L::kScale);
-  float *sBias = reinterpret_cast<float *>(smem + L::kBias);
   uint64_t *full = reinterpret_cast<uint64_t *>(smem + L::kBar);
   uint64_t *empty = full + STAGES;
   uint64_t *tfull = empty + STAGES;   // [2]
@@ -159,7 +182,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
     for (int s = 0; s < 2; s++) {
       mbar_init(&tfull[s], 1);
-      mbar_init(&tempty[s], 128);
+      mbar_init(&tempty[s], 256);
     }
     fence_mbar_init();
   }
@@ -171,40 +194,41 @@ __global__ void __launch_bounds__(kThreads, 1)
   if (threadIdx.x == 0) { DBG(1); }
 
   if (warp == 0) {
-    if (lane == 0) {
-      // ------------------------------------------------------ TMA producer
-      int it = 0;
-      for (int tile = blockIdx.x; tile < a.num_tiles; tile += gridDim.x) {
-        const TileCoord tc = tile_coord(a, tile, BN);
-        int32_t va[NVAR], vb[NVAR];
-        va[V_N0] = tc.n0;
-        va[V_PT] = tc.p0 / a.A.divp; va[V_PR] = tc.p0 % a.A.divp;
-        va[V_QT] = tc.q0 / a.A.divq; va[V_QR] = tc.q0 % a.A.divq;
-        va[V_ONE] = 1;
-        vb[V_N0] = 0; vb[V_PT] = 0; vb[V_PR] = 0;
-        vb[V_QT] = tc.k0 / a.B.divq; vb[V_QR] = tc.k0 % a.B.divq;
-        vb[V_ONE] = 1;
-        for (int kit = 0; kit < a.num_iters; kit++, it++) {
-          const int stage = it % STAGES, round = it / STAGES;
-          if (round > 0) mbar_wait(&empty[stage], (round - 1) & 1);
-          mbar_expect_tx(&full[stage], kStageBytesA + L::kB);
-          for (int j = 0; j < a.spi; j++) {
-            const int slab = kit * a.spi + j;
-            const bool valid = slab < a.total_slabs;
-            const int sl = valid ? slab : 0;
-            const int tap = sl / a.Gc, g = sl % a.Gc;
-            const int r = tap / a.S, s = tap % a.S;
-            va[V_GT] = g / a.A.divg; va[V_GR] = g % a.A.divg; va[V_R] = r; va[V_S] = s;
-            vb[V_GT] = g / a.B.divg; vb[V_GR] = g % a.B.divg; vb[V_R] = r; vb[V_S] = s;
-            int32_t ca[5], cb[5];
-            coords(a.A, va, ca);
-            coords(a.B, vb, cb);
-            if (!valid) { ca[0] = a.A.oob0; cb[0] = a.B.oob0; }
-            tma_load_5d(sA + stage * kStageBytesA + j * a.A.slab_bytes, &tmA, &full[stage], ca[0], ca[1], ca[2],
-                        ca[3], ca[4]);
-            tma_load_5d(sB + stage * L::kB + j * a.B.slab_bytes, &tmB, &full[stage], cb[0], cb[1], cb[2], cb[3],
-                        cb[4]);
-          }
+    // -------------------------------------------------------- TMA producer
+    // lane j < 8 issues A slab j of a stage, lane 16 + j issues B slab j:
+    // the box coordinates of all slabs are computed in parallel.
+    const bool isA = lane < 16;
+    const int j = lane & 15;
+    const OperandMap &om = isA ? a.A : a.B;
+    const CUtensorMap *tmap = isA ? &tmA : &tmB;
+    unsigned char *sbase = isA ? sA : sB;
+    const int sbytes = isA ? kStageBytesA : L::kB;
+    const bool active = j < a.spi;
+    int it = 0;
+    for (int tile = blockIdx.x; tile < a.num_tiles; tile += gridDim.x) {
+      const TileCoord tc = tile_coord(a, tile, BN);
+      int32_t v[NVAR];
+      const int pp = isA ? tc.p0 : 0, qq = isA ? tc.q0 : tc.k0;
+      v[V_N0] = isA ? tc.n0 : 0;
+      v[V_PT] = pp / om.divp; v[V_PR] = pp % om.divp;
+      v[V_QT] = qq / om.divq; v[V_QR] = qq % om.divq;
+      v[V_ONE] = 1;
+      for (int kit = 0; kit < a.num_iters; kit++, it++) {
+        const int stage = it % STAGES, round = it / STAGES;
+        if (round > 0) mbar_wait(&empty[stage], (round - 1) & 1);
+        if (lane == 0) mbar_expect_tx(&full[stage], kStageBytesA + L::kB);
+        __syncwarp();
+        if (active) {
+          const int slab = kit * a.spi + j;
+          const bool valid = slab < a.total_slabs;
+          const int sl = valid ? slab : 0;
+          const int tap = sl / a.Gc, g = sl % a.Gc;
+          v[V_R] = tap / a.S; v[V_S] = tap % a.S;
+          v[V_GT] = g / om.divg; v[V_GR] = g % om.divg;
+          int32_t c[5];
+          coords(om, v, c);
+          if (!valid) c[0] = om.oob0;
+          tma_load_5d(sbase + stage * sbytes + j * om.slab_bytes, tmap, &full[stage], c[0], c[1], c[2], c[3], c[4]);
         }
       }
     }
@@ -240,116 +264,135 @@ __global__ void __launch_bounds__(kThreads, 1)
           mma_commit(&empty[stage]);
         }
         mma_commit(&tfull[acc]);
+        if (i == 0) { DBG(3); }
       }
     }
   } else {
     // -------------------------------------------------------- epilogue
-    const int et = threadIdx.x - 64;       // 0..127
-    const int wq = warp & 3;               // TMEM lane quarter of this warp
+    // 8 warps: warp w reads TMEM lane quarter (w % 4) (hardware rule) and
+    // column half (w - 2) / 4 of every 64-column chunk.
+    const int et = threadIdx.x - 64;       // 0..255
+    const int wq = warp & 3;
+    const int half = (warp - 2) >> 2;
     const int row = wq * 32 + lane;        // accumulator row = tile row
     const int tn = a.tile_h * a.tile_w;
     const int sw_o = a.O.sw;
     const int pitch = sw_o * 2;            // bytes per row in a staging slab
     const int swz = pitch == 128 ? 3 : (pitch == 64 ? 2 : (pitch == 32 ? 1 : 0));
+    const uint32_t sOut_u32 = smem_u32(sOut);
+    // activation as a clamp: none (-inf, inf), ReLU [0, inf), ReLU6 [0, 6]
+    const float act_lo = a.epi.act == 0 ? -INFINITY : 0.f;
+    const float act_hi = a.epi.act == 2 ? 6.f : INFINITY;
     int i = 0;
     for (int tile = blockIdx.x; tile < a.num_tiles; tile += gridDim.x, i++) {
       const int acc = i & 1, use = i >> 1;
       const TileCoord tc = tile_coord(a, tile, BN);
-      // per-tile scale / bias into smem (previous tile finished with them)
-      named_bar(1, 128);
-      for (int c = et; c < BN; c += 128) {
-        const int k = tc.k0 + c;
-        sScale[c] = (a.epi.scale && k < a.K) ? __ldg(a.epi.scale + k) : 1.f;
-        sBias[c] = (a.epi.bias && k < a.K) ? __ldg(a.epi.bias + k) : 0.f;
-      }
-      named_bar(1, 128);
       const int n = tc.n0 + row / tn, p = tc.p0 + (row / a.tile_w) % a.tile_h, q = tc.q0 + row % a.tile_w;
       const bool vrow = n < a.N && p < a.Ho && q < a.Wo;
+      // origin of this warp's 32-row sub-box of the output tile
+      const int r0 = wq * 32;
+      const int sn = tc.n0 + r0 / tn, sp = tc.p0 + (r0 / a.tile_w) % a.tile_h, sq = tc.q0 + r0 % a.tile_w;
+      int32_t vo[NVAR];
+      vo[V_N0] = sn;
+      vo[V_PT] = sp / a.O.divp; vo[V_PR] = sp % a.O.divp;
+      vo[V_QT] = sq / a.O.divq; vo[V_QR] = sq % a.O.divq;
+      vo[V_R] = 0; vo[V_S] = 0; vo[V_ONE] = 1;
       mbar_wait(&tfull[acc], use & 1);
+      if (et == 0 && i == 0) { DBG(2); }
       tc_fence_after();
 #pragma unroll 1
       for (int c0 = 0; c0 < BN; c0 += 64) {
-        uint32_t raw[64];
-        const uint32_t taddr = tmem + ((uint32_t)(wq * 32) << 16) + (uint32_t)(acc * BN + c0);
-        tmem_ld_32x32b_x32(taddr, *reinterpret_cast<uint32_t(*)[32]>(raw));
-        tmem_ld_32x32b_x32(taddr + 32, *reinterpret_cast<uint32_t(*)[32]>(raw + 32));
+        const int cb = c0 + half * 32;     // first column of this thread's 32
+        uint32_t raw[32];
+        tmem_ld_32x32b_x32(tmem + ((uint32_t)(wq * 32) << 16) + (uint32_t)(acc * BN + cb), raw);
         tmem_ld_wait();
+        if (et == 0 && i == 0) { DBG(8 + (c0 >> 6) * 4); }
         if (c0 + 64 >= BN) {  // accumulator buffer drained: MMA may reuse it
           tc_fence_before();
           mbar_arrive(&tempty[acc]);
         }
-        float v[64];
+        float v[32];
+        // per-channel scale / bias (L1-resident after the first row)
+        const int kb = tc.k0 + cb;
+        // scale / bias are never NULL here (the host substitutes ones / zeros);
+        // a ragged last chunk clamps its indices (those channels are not stored)
+        if (kb + 32 <= a.K) {
+          const float4 *s4 = reinterpret_cast<const float4 *>(a.epi.scale + kb);
+          const float4 *b4 = reinterpret_cast<const float4 *>(a.epi.bias + kb);
 #pragma unroll
-        for (int j = 0; j < 64; j++) v[j] = __uint_as_float(raw[j]) * sScale[c0 + j] + sBias[c0 + j];
-        if (a.epi.residual && vrow) {
-          const uint16_t *res = static_cast<const uint16_t *>(a.epi.residual);
+          for (int j = 0; j < 8; j++) {
+            const float4 sc = __ldg(s4 + j), bi = __ldg(b4 + j);
+            v[4 * j + 0] = fmaf(__uint_as_float(raw[4 * j + 0]), sc.x, bi.x);
+            v[4 * j + 1] = fmaf(__uint_as_float(raw[4 * j + 1]), sc.y, bi.y);
+            v[4 * j + 2] = fmaf(__uint_as_float(raw[4 * j + 2]), sc.z, bi.z);
+            v[4 * j + 3] = fmaf(__uint_as_float(raw[4 * j + 3]), sc.w, bi.w);
+          }
+        } else {
 #pragma unroll
-          for (int j = 0; j < 64; j++) {
-            const int k = tc.k0 + c0 + j;
-            if (k < a.K) {
-              const int64_t o = a.is_conv ? a.epi.res.off4(n, k, p, q) : a.epi.res.off2(q, k);
-              if (o >= 0) v[j] += bf16_to_f32(__ldg(res + o));
-            }
+          for (int j = 0; j < 32; j++) {
+            const int k = min(kb + j, a.K - 1);
+            v[j] = fmaf(__uint_as_float(raw[j]), __ldg(a.epi.scale + k), __ldg(a.epi.bias + k));
           }
         }
+        if (a.epi.residual && vrow) {
+          float rv[32];  // local memory, touched only when a residual exists
+          residual_chunk(a.epi, a.is_conv, a.K, n, p, q, kb, rv);
 #pragma unroll
-        for (int j = 0; j < 64; j++) v[j] = apply_act(v[j], a.epi.act);
+          for (int j = 0; j < 32; j++) v[j] += rv[j];
+        }
+        uint32_t pk[16];
+#pragma unroll
+        for (int j = 0; j < 16; j++) {
+          const __nv_bfloat162 h2 = __floats2bfloat162_rn(fminf(fmaxf(v[2 * j], act_lo), act_hi),
+                                                          fminf(fmaxf(v[2 * j + 1], act_lo), act_hi));
+          pk[j] = *reinterpret_cast<const uint32_t *>(&h2);
+        }
+        if (et == 0 && i == 0) { DBG(9 + (c0 >> 6) * 4); }
         if (a.out_mode) {
-          // staging buffer free once the previous chunk's TMA store read it
-          if (et == 0) bulk_wait_read0();
-          named_bar(1, 128);
-          // row `row`: 64 channels -> 64/sw_o slabs of `pitch` bytes, swizzled
+          // Each warp stores its own 32-row x 32-channel sub-tile: private
+          // double-buffered staging, swizzled rows, one TMA store per slab;
+          // no CTA-wide barrier.  Buffer `buf` is free once the store issued
+          // two chunks ago has read it (<= 1 store group in flight per warp).
+          const int buf = (c0 >> 6) & 1;
+          if (lane == 0) bulk_wait_read1();
+          __syncwarp();
+          const uint32_t wbase = sOut_u32 + (uint32_t)((warp - 2) * 4096 + buf * 2048);
 #pragma unroll
-          for (int c = 0; c < 8; c++) {  // 8 chunks of 16 B = 8 channels
+          for (int c = 0; c < 4; c++) {  // 4 x 16 B = this thread's 32 channels
             const int ch = c * 8;
             const int slab = ch / sw_o;
-            const int within = (ch % sw_o) * 2;  // byte offset in the slab row
-            uint32_t off = (uint32_t)(row * pitch + within);
+            uint32_t off = (uint32_t)(lane * pitch + (ch % sw_o) * 2);
             off ^= ((off >> 7) & ((1u << swz) - 1u)) << 4;
-            uint4 u;
-            u.x = (uint32_t)f32_to_bf16_rne(v[ch + 0]) | ((uint32_t)f32_to_bf16_rne(v[ch + 1]) << 16);
-            u.y = (uint32_t)f32_to_bf16_rne(v[ch + 2]) | ((uint32_t)f32_to_bf16_rne(v[ch + 3]) << 16);
-            u.z = (uint32_t)f32_to_bf16_rne(v[ch + 4]) | ((uint32_t)f32_to_bf16_rne(v[ch + 5]) << 16);
-            u.w = (uint32_t)f32_to_bf16_rne(v[ch + 6]) | ((uint32_t)f32_to_bf16_rne(v[ch + 7]) << 16);
-            *reinterpret_cast<uint4 *>(sOut + slab * 128 * pitch + off) = u;
+            const uint32_t addr = wbase + (uint32_t)(slab * 32 * pitch) + off;
+            asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "r"(pk[4 * c]),
+                         "r"(pk[4 * c + 1]), "r"(pk[4 * c + 2]), "r"(pk[4 * c + 3])
+                         : "memory");
           }
+          if (et == 0 && i == 0) { DBG(10 + (c0 >> 6) * 4); }
           fence_async_smem();
-          named_bar(1, 128);
-          if (et == 0) {
-            int32_t vo[NVAR];
-            vo[V_N0] = tc.n0;
-            vo[V_PT] = tc.p0 / a.O.divp; vo[V_PR] = tc.p0 % a.O.divp;
-            vo[V_QT] = tc.q0 / a.O.divq; vo[V_QR] = tc.q0 % a.O.divq;
-            vo[V_R] = 0; vo[V_S] = 0; vo[V_ONE] = 1;
-            const int nslab = 64 / sw_o;
+          __syncwarp();
+          if (lane == 0) {
+            const int nslab = 32 / sw_o;
             for (int j = 0; j < nslab; j++) {
-              if (tc.k0 + c0 + j * sw_o >= a.K) break;  // channels past K: nothing to store
-              const int g = (tc.k0 + c0) / sw_o + j;
+              if (kb + j * sw_o >= a.K) break;  // channels past K: nothing to store
+              const int g = kb / sw_o + j;
               vo[V_GT] = g / a.O.divg; vo[V_GR] = g % a.O.divg;
               int32_t co[5];
               coords(a.O, vo, co);
-              tma_store_5d(&tmY, sOut + j * 128 * pitch, co[0], co[1], co[2], co[3], co[4]);
+              tma_store_5d(&tmY, sOut + (warp - 2) * 4096 + buf * 2048 + j * 32 * pitch, co[0], co[1], co[2],
+                           co[3], co[4]);
             }
             bulk_commit();
+            if (et == 0 && i == 0) { DBG(11 + (c0 >> 6) * 4); }
           }
         } else if (vrow) {
           // generic layouts: every copy / pad position through the writer
-#pragma unroll 1
-          for (int j = 0; j < 64; j++) {
-            const int k = tc.k0 + c0 + j;
-            if (k >= a.K) break;
-            float t = 0.f;
-#pragma unroll
-            for (int jj = 0; jj < 64; jj++) t = (jj == j) ? v[jj] : t;
-            const uint16_t h = f32_to_bf16_rne(t);
-            if (a.is_conv) write4<uint16_t>(a.yw, y, n, k, p, q, h);
-            else write2<uint16_t>(a.yw, y, q, k, h);
-          }
+          write_chunk(a.yw, a.is_conv, a.K, y, n, p, q, kb, pk);
         }
       }
     }
     if (et == 0) { DBG(5); }
-    if (et == 0 && a.out_mode) bulk_wait0();
+    if (lane == 0 && a.out_mode) bulk_wait0();
   }
   tc_fence_before();
   __syncthreads();
@@ -615,7 +658,7 @@ static uint64_t *debug_buffer() {
   if (!init) {
     init = true;
     const char *e = getenv("ALT_TC_DEBUG");
-    if (e && e[0] == '1' && cudaMalloc(&buf, (size_t)8 * 8 << 20) != cudaSuccess) buf = nullptr;
+    if (e && e[0] == '1' && cudaMalloc(&buf, (size_t)32 * 8 << 20) != cudaSuccess) buf = nullptr;
   }
   return buf;
 }
@@ -627,6 +670,33 @@ extern "C" int alt__debug_tc(uint64_t *host, int64_t n) {
   return cudaMemcpy(host, b, (size_t)n * 8, cudaMemcpyDeviceToHost) == cudaSuccess ? 0 : -1;
 }
 namespace alt {
+
+// per-device ones / zeros vectors (never freed: process lifetime)
+static alt_status identity_epilogue(int64_t K, const float **ones, const float **zeros) {
+  static std::mutex mu;
+  struct Buf { int dev; int64_t cap; float *ones, *zeros; };
+  static std::vector<Buf> bufs;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  std::lock_guard<std::mutex> g(mu);
+  for (auto &b : bufs) {
+    if (b.dev == dev && b.cap >= K) { *ones = b.ones; *zeros = b.zeros; return ALT_OK; }
+  }
+  const int64_t cap = std::max<int64_t>(K, 4096);
+  std::vector<float> h1(cap, 1.f);
+  float *d1 = nullptr, *d0 = nullptr;
+  if (cudaMalloc(&d1, cap * 4) != cudaSuccess || cudaMalloc(&d0, cap * 4) != cudaSuccess) {
+    cudaGetLastError();
+    set_error("identity epilogue buffers: out of memory");
+    return ALT_E_NOMEM;
+  }
+  cudaMemcpy(d1, h1.data(), cap * 4, cudaMemcpyHostToDevice);
+  cudaMemset(d0, 0, cap * 4);
+  bufs.push_back({dev, cap, d1, d0});
+  *ones = d1;
+  *zeros = d0;
+  return ALT_OK;
+}
 
 static int num_sms() {
   static int n = 0;
@@ -775,11 +845,17 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
     memcpy(rb, P.rb, sizeof(rb));
     memcpy(ry, P.ry, sizeof(ry));
     for (int d = 0; d < kMaxL; d++) {
-      for (RoleInfo *r : {&ra[d], &ry[d]}) {
-        if (r->role == R_N) r->tile = c.tn;
-        if (r->role == R_H) r->tile = c.th;
-        if (r->role == R_W) r->tile = c.tw;
-      }
+      if (ra[d].role == R_N) ra[d].tile = c.tn;
+      if (ra[d].role == R_H) ra[d].tile = c.th;
+      if (ra[d].role == R_W) ra[d].tile = c.tw;
+      // output stores are per epilogue warp: a 32-row sub-box of the tile
+      // (rows are (n, h, w) with w fastest, all extents powers of two)
+      const int sw_w = c.tw >= 32 ? 32 : c.tw;
+      const int sw_h = c.tw >= 32 ? 1 : (c.tw * c.th >= 32 ? 32 / c.tw : c.th);
+      const int sw_n = 32 / (sw_w * sw_h);
+      if (ry[d].role == R_N) ry[d].tile = sw_n;
+      if (ry[d].role == R_H) ry[d].tile = sw_h;
+      if (ry[d].role == R_W) ry[d].tile = sw_w;
       if (rb[d].role == R_W) rb[d].tile = BN;
     }
     for (int sw = 64; sw >= 8; sw /= 2) {
@@ -801,12 +877,12 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       memset(&pl.ty, 0, sizeof(pl.ty));
       if (!(P.yl->flags & (ALT_HAS_PAD | ALT_HAS_UNFOLD))) {
         char why2[160];
-        for (int so = 64; so >= 8 && !a.out_mode; so /= 2) {
+        for (int so = 32; so >= 8 && !a.out_mode; so /= 2) {
           View vy;
           if (!build_view(*P.yl, ry, so, &vy, why2)) continue;
           int64_t rowsY = 1;
           for (int i = 1; i < vy.rank; i++) rowsY *= vy.d[i].box;
-          if (rowsY != 128) continue;
+          if (rowsY != 32) continue;
           if (encode_view(vy, P.y, esize, so, &pl.ty, &a.O, why2)) a.out_mode = 1;
         }
       }
@@ -829,6 +905,14 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       a.sw = sw;
       alt_status st;
       if ((st = make_epi(P.epi, &a.epi)) != ALT_OK) return st;
+      // the kernel always applies scale * acc + bias: absent ones become the
+      // identity (device-resident ones / zeros, grown on demand)
+      if (!a.epi.scale || !a.epi.bias) {
+        const float *ones = nullptr, *zeros = nullptr;
+        if ((st = identity_epilogue(P.K, &ones, &zeros)) != ALT_OK) return st;
+        if (!a.epi.scale) a.epi.scale = ones;
+        if (!a.epi.bias) a.epi.bias = zeros;
+      }
       if ((st = make_writer(P.yl, &a.yw)) != ALT_OK) return st;
       a.dbg = debug_buffer();
       pl.grid = (int)std::min<int64_t>(a.num_tiles, num_sms());

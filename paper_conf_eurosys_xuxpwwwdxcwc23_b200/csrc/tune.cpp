@@ -1,0 +1,308 @@
+// tune.cpp — alt_tune: ALT's joint layout + loop tuning (§5)
+// replaced by a bounded grid measured on the device.
+//
+// Conv template (GPU form): x = N C/it H W it (optionally with
+// the conv zero padding materialised: pad(H), pad(W), reading A7),
+// w = K/ot' C/it R S ot' it (c innermost: K-major B operand, reading A11),
+// y = N K/ot Ho Wo ot; kernel ("loop") parameters: BLOCK_N and the
+// (tile_n x tile_h x tile_w) output-pixel tile.  C is padded to a multiple of
+// 8 first when needed (reading A2: non-divisible tiling = pad then split).
+// GEMM template: A = M/mt K/kt mt kt, B = N/nt K/kt nt kt
+// (K innermost), C = M/mt N/nt mt nt.
+//
+// Each point: compile the layouts, allocate operands in them (values do not
+// affect timing), run `warmup` launches, then `reps` launches each preceded
+// by an L2 flush (a 2x-L2 memset, not timed), timed with CUDA events on the
+// caller's stream.  The fastest point is returned.  Parity of the tuner is
+// unpinned by the paper (reading A19): the result is only required to be a
+// valid layout pair whose kernels are oracle-exact.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cfloat>
+#include <cstring>
+#include <vector>
+
+#include "alt.h"
+#include "layout.h"
+#include "ops.h"
+
+namespace alt {
+
+namespace {
+
+alt_prim P_split(int dim, std::initializer_list<int64_t> f) {
+  alt_prim p{};
+  p.kind = ALT_SPLIT;
+  p.dim = dim;
+  p.n = (int32_t)f.size();
+  int i = 0;
+  for (int64_t x : f) p.v[i++] = x;
+  return p;
+}
+alt_prim P_reorder(std::initializer_list<int64_t> perm) {
+  alt_prim p{};
+  p.kind = ALT_REORDER;
+  p.n = (int32_t)perm.size();
+  int i = 0;
+  for (int64_t x : perm) p.v[i++] = x;
+  return p;
+}
+alt_prim P_pad(int dim, int64_t lo, int64_t hi) {
+  alt_prim p{};
+  p.kind = ALT_PAD;
+  p.dim = dim;
+  p.v[0] = lo;
+  p.v[1] = hi;
+  return p;
+}
+
+struct Seq {
+  std::vector<alt_prim> p;
+};
+
+// N C/x H W x, with C padded to Cp and optional materialised conv padding
+Seq act_layout(int64_t C, int64_t Cp, int64_t x, int64_t pad_hw) {
+  Seq s;
+  if (Cp != C) s.p.push_back(P_pad(1, 0, Cp - C));
+  if (pad_hw) {
+    s.p.push_back(P_pad(2, pad_hw, pad_hw));
+    s.p.push_back(P_pad(3, pad_hw, pad_hw));
+  }
+  s.p.push_back(P_split(1, {Cp / x, x}));
+  s.p.push_back(P_reorder({0, 1, 3, 4, 2}));
+  return s;
+}
+// K/y C/x R S y x (c innermost), C padded to Cp
+Seq wgt_layout(int64_t K, int64_t C, int64_t Cp, int64_t y, int64_t x) {
+  Seq s;
+  if (Cp != C) s.p.push_back(P_pad(1, 0, Cp - C));
+  s.p.push_back(P_split(0, {K / y, y}));
+  s.p.push_back(P_split(2, {Cp / x, x}));
+  s.p.push_back(P_reorder({0, 2, 4, 5, 1, 3}));
+  return s;
+}
+Seq tiled2(int64_t R0, int64_t R1, int64_t t0, int64_t t1, bool swap_inner) {
+  // [R0/t0][R1/t1][t0][t1]  (swap_inner: [R1/t1][R0/t0][t1][t0])
+  Seq s;
+  s.p.push_back(P_split(0, {R0 / t0, t0}));
+  s.p.push_back(P_split(2, {R1 / t1, t1}));
+  if (swap_inner) s.p.push_back(P_reorder({2, 0, 3, 1}));
+  else s.p.push_back(P_reorder({0, 2, 1, 3}));
+  return s;
+}
+
+struct Scratch {
+  std::vector<void *> bufs;
+  void *get(size_t bytes, cudaStream_t s) {
+    void *p = nullptr;
+    if (cudaMallocAsync(&p, bytes, s) != cudaSuccess) return nullptr;
+    cudaMemsetAsync(p, 0, bytes, s);
+    bufs.push_back(p);
+    return p;
+  }
+  void release(cudaStream_t s) {
+    for (void *p : bufs) cudaFreeAsync(p, s);
+    bufs.clear();
+  }
+};
+
+struct LayoutHolder {
+  alt_layout h = nullptr;
+  ~LayoutHolder() { if (h) alt_layout_destroy(h); }
+};
+
+std::vector<int64_t> vals_or(const alt_tune_space *sp, int i, std::initializer_list<int64_t> def) {
+  std::vector<int64_t> v;
+  if (sp && sp->nvals[i] > 0) {
+    for (int k = 0; k < sp->nvals[i] && k < ALT_TUNE_MAX_VALS; k++) v.push_back(sp->vals[i][k]);
+  } else {
+    v.assign(def.begin(), def.end());
+  }
+  return v;
+}
+
+// time one callable (launches on `s`) with an L2 flush before every rep
+template <typename F>
+float time_point(F &&launch, cudaStream_t s, void *flush, size_t flush_bytes, int warmup, int reps,
+                 alt_status *st) {
+  for (int i = 0; i < warmup; i++) {
+    *st = launch();
+    if (*st != ALT_OK) return FLT_MAX;
+  }
+  cudaEvent_t e0, e1;
+  cudaEventCreate(&e0);
+  cudaEventCreate(&e1);
+  float total = 0.f;
+  for (int i = 0; i < reps; i++) {
+    if (flush) cudaMemsetAsync(flush, i & 0xff, flush_bytes, s);
+    cudaEventRecord(e0, s);
+    *st = launch();
+    cudaEventRecord(e1, s);
+    if (*st != ALT_OK) break;
+    cudaEventSynchronize(e1);
+    float ms = 0.f;
+    cudaEventElapsedTime(&ms, e0, e1);
+    total += ms;
+  }
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  if (*st != ALT_OK) return FLT_MAX;
+  return total / reps * 1000.f;  // us
+}
+
+}  // namespace
+}  // namespace alt
+
+using namespace alt;
+
+extern "C" alt_status alt_tune(alt_op_kind op, const void *op_params, alt_dtype dtype, const alt_tune_space *space,
+                               alt_stream_t stream_, alt_tune_result *out, float *all_us) {
+  if (!op_params || !out) { set_error("alt_tune: NULL argument"); return ALT_E_INVALID; }
+  if (dtype != ALT_BF16 && dtype != ALT_F32) { set_error("alt_tune: bad dtype"); return ALT_E_INVALID; }
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream_);
+  const int esize = dtype == ALT_BF16 ? 2 : 4;
+  const int max_points = space && space->max_points > 0 ? std::min(space->max_points, 4096) : 64;
+  const int warmup = space && space->warmup > 0 ? space->warmup : 2;
+  const int reps = space && space->reps > 0 ? space->reps : 5;
+  memset(out, 0, sizeof(*out));
+  out->best_us = FLT_MAX;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  int l2 = 0;
+  cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, dev);
+  const size_t flush_bytes = (size_t)std::max(l2, 1 << 20) * 2;
+  Scratch scratch;
+  void *flush = scratch.get(flush_bytes, s);
+  int measured = 0;
+
+  auto record = [&](const Seq *xs, const Seq *ws, const Seq *ys, const alt_kernel_cfg &cfg, float us) {
+    if (all_us && measured < max_points) all_us[measured] = us;
+    measured++;
+    if (us < out->best_us) {
+      out->best_us = us;
+      out->cfg = cfg;
+      const Seq *seqs[3] = {xs, ws, ys};
+      for (int i = 0; i < 3; i++) {
+        out->nprims[i] = seqs[i] ? (int32_t)seqs[i]->p.size() : 0;
+        for (int k = 0; k < out->nprims[i]; k++) out->prims[i][k] = seqs[i]->p[k];
+      }
+    }
+  };
+
+  if (op == ALT_OP_CONV2D) {
+    const alt_conv2d_params &p = *static_cast<const alt_conv2d_params *>(op_params);
+    if (p.groups > 1) { set_error("alt_tune: grouped conv has no template (NEXT)"); scratch.release(s); return ALT_E_UNSUPPORTED; }
+    const int64_t Ho = (p.H + 2 * p.pad_h - p.R) / p.stride_h + 1, Wo = (p.W + 2 * p.pad_w - p.S) / p.stride_w + 1;
+    const int64_t Cp = p.C % 8 ? (p.C + 7) / 8 * 8 : p.C;
+    const int64_t xl[4] = {p.N, p.C, p.H, p.W}, wl[4] = {p.K, p.C, p.R, p.S}, yl[4] = {p.N, p.K, Ho, Wo};
+    void *x = scratch.get((size_t)p.N * Cp * (p.H + 2 * p.pad_h) * (p.W + 2 * p.pad_w) * esize, s);
+    void *w = scratch.get((size_t)p.K * Cp * p.R * p.S * esize, s);
+    void *y = scratch.get((size_t)p.N * p.K * Ho * Wo * esize, s);
+    if (!x || !w || !y || !flush) { scratch.release(s); set_error("alt_tune: scratch allocation failed"); return ALT_E_NOMEM; }
+    std::vector<int64_t> its = vals_or(space, 0, {64, 32, 16, 8, 128, 256});
+    std::vector<int64_t> ots = vals_or(space, 1, {64, 32});
+    std::vector<int64_t> bns = vals_or(space, 6, {256, 128, 64});
+    std::vector<int64_t> pads = vals_or(space, 7, {0});
+    std::vector<int64_t> ths = vals_or(space, 4, {0});  // 0 = kernel heuristic
+    std::vector<int64_t> tws = vals_or(space, 5, {0});
+    for (int64_t it : its) {
+      if (it > Cp || Cp % it || it % 8) continue;
+      if (space && space->fix_x) { if (it != its[0]) continue; }
+      for (int64_t ot : ots) {
+        if (ot > p.K || p.K % ot) continue;
+        for (int64_t bn : bns) {
+          if (bn > 64 && bn > p.K) continue;
+          const int64_t y_w = std::min<int64_t>(bn, p.K);
+          if (p.K % y_w) continue;
+          for (int64_t pad : pads) {
+            for (int64_t th : ths) {
+              for (int64_t tw : tws) {
+                if (measured >= max_points) break;
+                Seq xs = act_layout(p.C, Cp, it, pad ? p.pad_h : 0);
+                Seq ws = wgt_layout(p.K, p.C, Cp, y_w, it);
+                Seq ys = act_layout(p.K, p.K, ot, 0);
+                LayoutHolder Lx, Lw, Ly;
+                if (space && space->fix_x && space->fixed_x) {
+                  Lx.h = nullptr;
+                } else if (alt_layout_create(4, xl, xs.p.data(), (int32_t)xs.p.size(), &Lx.h) != ALT_OK) {
+                  continue;
+                }
+                if (alt_layout_create(4, wl, ws.p.data(), (int32_t)ws.p.size(), &Lw.h) != ALT_OK) continue;
+                if (alt_layout_create(4, yl, ys.p.data(), (int32_t)ys.p.size(), &Ly.h) != ALT_OK) continue;
+                alt_layout xh = Lx.h ? Lx.h : space->fixed_x;
+                alt_kernel_cfg cfg{};
+                cfg.path = ALT_PATH_AUTO;
+                cfg.block_n = (int32_t)bn;
+                if (th && tw) {
+                  cfg.tile_h = (int32_t)th;
+                  cfg.tile_w = (int32_t)tw;
+                  cfg.tile_n = (int32_t)(128 / (th * tw));
+                  if (cfg.tile_n < 1) continue;
+                }
+                alt_status st = ALT_OK;
+                const float us = time_point(
+                    [&]() { return alt_conv2d(&p, xh, x, Lw.h, w, Ly.h, y, dtype, nullptr, &cfg, stream_); }, s, flush,
+                    flush_bytes, warmup, reps, &st);
+                if (st != ALT_OK) continue;
+                alt_kernel_cfg used{};
+                alt_last_plan(&used);
+                record(Lx.h ? &xs : nullptr, &ws, &ys, used, us);
+              }
+            }
+          }
+        }
+      }
+    }
+  } else if (op == ALT_OP_MATMUL) {
+    const alt_matmul_params &g = *static_cast<const alt_matmul_params *>(op_params);
+    void *a = scratch.get((size_t)g.M * g.K * esize, s);
+    void *b = scratch.get((size_t)g.K * g.N * esize, s);
+    void *c = scratch.get((size_t)g.M * g.N * esize, s);
+    if (!a || !b || !c || !flush) { scratch.release(s); set_error("alt_tune: scratch allocation failed"); return ALT_E_NOMEM; }
+    const int64_t al[2] = {g.M, g.K}, bl[2] = {g.K, g.N}, cl[2] = {g.M, g.N};
+    std::vector<int64_t> mts = vals_or(space, 0, {128, 256, 64});
+    std::vector<int64_t> kts = vals_or(space, 1, {64, 32});
+    std::vector<int64_t> nts = vals_or(space, 2, {128, 256, 64});
+    std::vector<int64_t> bns = vals_or(space, 6, {256, 128});
+    for (int64_t mt : mts) {
+      if (g.M % mt) continue;
+      for (int64_t kt : kts) {
+        if (g.K % kt) continue;
+        for (int64_t nt : nts) {
+          if (g.N % nt) continue;
+          for (int64_t bn : bns) {
+            if (measured >= max_points) break;
+            if (bn > g.N) continue;
+            Seq as = tiled2(g.M, g.K, mt, kt, false);
+            Seq bs = tiled2(g.K, g.N, kt, nt, true);   // N/nt K/kt nt kt
+            Seq cs = tiled2(g.M, g.N, mt, nt, false);
+            LayoutHolder La, Lb, Lc;
+            if (alt_layout_create(2, al, as.p.data(), (int32_t)as.p.size(), &La.h) != ALT_OK) continue;
+            if (alt_layout_create(2, bl, bs.p.data(), (int32_t)bs.p.size(), &Lb.h) != ALT_OK) continue;
+            if (alt_layout_create(2, cl, cs.p.data(), (int32_t)cs.p.size(), &Lc.h) != ALT_OK) continue;
+            alt_kernel_cfg cfg{};
+            cfg.block_n = (int32_t)bn;
+            alt_status st = ALT_OK;
+            const float us = time_point(
+                [&]() { return alt_matmul(g.M, g.N, g.K, La.h, a, Lb.h, b, Lc.h, c, dtype, nullptr, &cfg, stream_); },
+                s, flush, flush_bytes, warmup, reps, &st);
+            if (st != ALT_OK) continue;
+            alt_kernel_cfg used{};
+            alt_last_plan(&used);
+            record(&as, &bs, &cs, used, us);
+          }
+        }
+      }
+    }
+  } else {
+    scratch.release(s);
+    set_error("alt_tune: unknown op");
+    return ALT_E_INVALID;
+  }
+  scratch.release(s);
+  cudaStreamSynchronize(s);
+  out->measured = measured;
+  if (measured == 0) { set_error("alt_tune: no valid grid point"); return ALT_E_UNSUPPORTED; }
+  return ALT_OK;
+}
