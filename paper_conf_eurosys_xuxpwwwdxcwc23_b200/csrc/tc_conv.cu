@@ -73,9 +73,9 @@ constexpr int kThreads = 320;  // producer, MMA, 8 epilogue warps
 constexpr int kStageBytesA = 128 * 64 * 2;
 constexpr int kOutStage = 128 * 64 * 2;  // one 64-column bf16 chunk of the tile
 
-template <int BN, int STAGES>
+template <int BN, int STAGES, int CG = 1>
 struct TcSmem {
-  static constexpr int kB = BN * 64 * 2;
+  static constexpr int kB = (BN / CG) * 64 * 2;  // this CTA's share of the B tile
   static constexpr int kRing = STAGES * (kStageBytesA + kB);
   static constexpr int kOut = kRing;                       // 2 staging buffers for TMA stores
   static constexpr int kBar = kOut + 2 * kOutStage;        // barriers
@@ -144,20 +144,24 @@ static __device__ __noinline__ void write_chunk(const Writer &w, int is_conv, in
 }
 
 struct TileCoord { int n0, p0, q0, k0; };
-__device__ __forceinline__ TileCoord tile_coord(const TcArgs &a, int tile, int BN) {
-  const int mt = tile / a.num_n_tiles, nt = tile % a.num_n_tiles;
+// work unit `tile` -> this CTA's 128-row M tile and the unit's N tile; with a
+// CTA pair (CG = 2) a unit is two consecutive M tiles, one per CTA rank
+__device__ __forceinline__ TileCoord tile_coord(const TcArgs &a, int tile, int BN, int CG, int rank) {
+  const int mt = (tile / a.num_n_tiles) * CG + rank, nt = tile % a.num_n_tiles;
   const int tw_i = mt % a.mt_w;
   const int th_i = (mt / a.mt_w) % a.mt_h;
   const int tn_i = mt / (a.mt_w * a.mt_h);
   return {tn_i * a.tile_n, th_i * a.tile_h, tw_i * a.tile_w, nt * BN};
 }
 
-template <int BN, int STAGES>
+template <int BN, int STAGES, int CG>
 __global__ void __launch_bounds__(kThreads, 1)
     k_tc_conv(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
               const __grid_constant__ CUtensorMap tmY, const __grid_constant__ TcArgs a, uint16_t *__restrict__ y) {
   using namespace sm100;
-  using L = TcSmem<BN, STAGES>;
+  using L = TcSmem<BN, STAGES, CG>;
+  const int rank = CG == 2 ? (int)cluster_ctarank() : 0;
+  const int unit0 = blockIdx.x / CG, unit_step = gridDim.x / CG;
   extern __shared__ __align__(1024) unsigned char smem_raw[];
   unsigned char *smem = reinterpret_cast<unsigned char *>(
       (reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -182,13 +186,14 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
     for (int s = 0; s < 2; s++) {
       mbar_init(&tfull[s], 1);
-      mbar_init(&tempty[s], 256);
+      mbar_init(&tempty[s], 256 * CG);  // every epilogue thread of the pair
     }
     fence_mbar_init();
   }
-  if (warp == 1) tmem_alloc<2 * BN>(tmem_slot);
+  if (warp == 1) tmem_alloc<2 * BN, CG>(tmem_slot);
   tc_fence_before();
   __syncthreads();
+  if constexpr (CG == 2) cluster_sync();  // peer barriers initialised before any remote arrive
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
   if (threadIdx.x == 0) { DBG(1); }
@@ -205,10 +210,11 @@ __global__ void __launch_bounds__(kThreads, 1)
     const int sbytes = isA ? kStageBytesA : L::kB;
     const bool active = j < a.spi;
     int it = 0;
-    for (int tile = blockIdx.x; tile < a.num_tiles; tile += gridDim.x) {
-      const TileCoord tc = tile_coord(a, tile, BN);
+    for (int tile = unit0; tile < a.num_tiles; tile += unit_step) {
+      const TileCoord tc = tile_coord(a, tile, BN, CG, rank);
       int32_t v[NVAR];
-      const int pp = isA ? tc.p0 : 0, qq = isA ? tc.q0 : tc.k0;
+      // B rows of this CTA: its 1/CG share of the unit's BN output channels
+      const int pp = isA ? tc.p0 : 0, qq = isA ? tc.q0 : tc.k0 + rank * (BN / CG);
       v[V_N0] = isA ? tc.n0 : 0;
       v[V_PT] = pp / om.divp; v[V_PR] = pp % om.divp;
       v[V_QT] = qq / om.divq; v[V_QR] = qq % om.divq;
@@ -216,7 +222,8 @@ __global__ void __launch_bounds__(kThreads, 1)
       for (int kit = 0; kit < a.num_iters; kit++, it++) {
         const int stage = it % STAGES, round = it / STAGES;
         if (round > 0) mbar_wait(&empty[stage], (round - 1) & 1);
-        if (lane == 0) mbar_expect_tx(&full[stage], kStageBytesA + L::kB);
+        // the leader's full barrier counts the bytes of both CTAs of a pair
+        if (lane == 0 && rank == 0) mbar_expect_tx(&full[stage], CG * (kStageBytesA + L::kB));
         __syncwarp();
         if (active) {
           const int slab = kit * a.spi + j;
@@ -228,21 +235,27 @@ __global__ void __launch_bounds__(kThreads, 1)
           int32_t c[5];
           coords(om, v, c);
           if (!valid) c[0] = om.oob0;
-          tma_load_5d(sbase + stage * sbytes + j * om.slab_bytes, tmap, &full[stage], c[0], c[1], c[2], c[3], c[4]);
+          if constexpr (CG == 2)
+            tma_load_5d_2cta(sbase + stage * sbytes + j * om.slab_bytes, tmap, &full[stage], c[0], c[1], c[2], c[3],
+                             c[4]);
+          else
+            tma_load_5d(sbase + stage * sbytes + j * om.slab_bytes, tmap, &full[stage], c[0], c[1], c[2], c[3],
+                        c[4]);
         }
       }
     }
   } else if (warp == 1) {
-    if (lane == 0) {
+    if (lane == 0 && rank == 0) {
       // ------------------------------------------------------ MMA issuer
-      constexpr uint32_t idesc = idesc_f32acc(1 /*bf16*/, 128, BN);
+      // (the leader CTA issues for the pair: M = 128 * CG)
+      constexpr uint32_t idesc = idesc_f32acc(1 /*bf16*/, 128 * CG, BN);
       const int sw = a.sw;
       const uint32_t layout = sw == 8 ? 0u : (sw == 16 ? 6u : (sw == 32 ? 4u : 2u));
       const uint32_t sbo = sw == 8 ? 128u : (uint32_t)(8 * sw * 2);
       const uint32_t aS = (uint32_t)a.A.slab_bytes, bS = (uint32_t)a.B.slab_bytes;
       const uint32_t lboA = sw == 8 ? aS : 16u, lboB = sw == 8 ? bS : 16u;
       int it = 0, i = 0;
-      for (int tile = blockIdx.x; tile < a.num_tiles; tile += gridDim.x, i++) {
+      for (int tile = unit0; tile < a.num_tiles; tile += unit_step, i++) {
         const int acc = i & 1, use = i >> 1;
         if (use > 0) mbar_wait(&tempty[acc], (use - 1) & 1);
         tc_fence_after();
@@ -259,11 +272,14 @@ __global__ void __launch_bounds__(kThreads, 1)
             const uint32_t off = (uint32_t)((kc % sw) * 2);
             const uint64_t ad = smem_desc(baseA + slab * aS + off, lboA, sbo, layout);
             const uint64_t bd = smem_desc(baseB + slab * bS + off, lboB, sbo, layout);
-            mma_bf16(d, ad, bd, idesc, (kit | kk) != 0);
+            if constexpr (CG == 2) mma_bf16_2cta(d, ad, bd, idesc, (kit | kk) != 0);
+            else mma_bf16(d, ad, bd, idesc, (kit | kk) != 0);
           }
-          mma_commit(&empty[stage]);
+          if constexpr (CG == 2) mma_commit_2cta(&empty[stage], 0x3);  // frees the stage in both CTAs
+          else mma_commit(&empty[stage]);
         }
-        mma_commit(&tfull[acc]);
+        if constexpr (CG == 2) mma_commit_2cta(&tfull[acc], 0x3);
+        else mma_commit(&tfull[acc]);
         if (i == 0) { DBG(3); }
       }
     }
@@ -284,9 +300,9 @@ __global__ void __launch_bounds__(kThreads, 1)
     const float act_lo = a.epi.act == 0 ? -INFINITY : 0.f;
     const float act_hi = a.epi.act == 2 ? 6.f : INFINITY;
     int i = 0;
-    for (int tile = blockIdx.x; tile < a.num_tiles; tile += gridDim.x, i++) {
+    for (int tile = unit0; tile < a.num_tiles; tile += unit_step, i++) {
       const int acc = i & 1, use = i >> 1;
-      const TileCoord tc = tile_coord(a, tile, BN);
+      const TileCoord tc = tile_coord(a, tile, BN, CG, rank);
       const int n = tc.n0 + row / tn, p = tc.p0 + (row / a.tile_w) % a.tile_h, q = tc.q0 + row % a.tile_w;
       const bool vrow = n < a.N && p < a.Ho && q < a.Wo;
       // origin of this warp's 32-row sub-box of the output tile
@@ -309,7 +325,8 @@ __global__ void __launch_bounds__(kThreads, 1)
         if (et == 0 && i == 0) { DBG(8 + (c0 >> 6) * 4); }
         if (c0 + 64 >= BN) {  // accumulator buffer drained: MMA may reuse it
           tc_fence_before();
-          mbar_arrive(&tempty[acc]);
+          if constexpr (CG == 2) mbar_arrive_cluster(&tempty[acc], 0);  // the leader's MMA waits
+          else mbar_arrive(&tempty[acc]);
         }
         float v[32];
         // per-channel scale / bias (L1-resident after the first row)
@@ -396,7 +413,8 @@ __global__ void __launch_bounds__(kThreads, 1)
   }
   tc_fence_before();
   __syncthreads();
-  if (warp == 1) tmem_dealloc<2 * BN>(tmem);
+  if constexpr (CG == 2) cluster_sync();  // the pair's MMAs and epilogues are done
+  if (warp == 1) tmem_dealloc<2 * BN, CG>(tmem);
   if (threadIdx.x == 32) { DBG(6); }
 }
 
@@ -709,18 +727,36 @@ static int num_sms() {
   return n;
 }
 
-template <int BN, int STAGES>
+template <int BN, int STAGES, int CG_>
 static cudaError_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUtensorMap &ty, const TcArgs &a,
                              uint16_t *y, int grid, cudaStream_t s) {
-  auto kern = k_tc_conv<BN, STAGES>;
-  const int smem = TcSmem<BN, STAGES>::kBytes;
-  static_assert(TcSmem<BN, STAGES>::kBytes <= 232448, "smem budget");
+  constexpr int CG = CG_;
+  auto kern = k_tc_conv<BN, STAGES, CG>;
+  const int smem = TcSmem<BN, STAGES, CG>::kBytes;
+  static_assert(TcSmem<BN, STAGES, CG>::kBytes <= 232448, "smem budget");
   static bool attr_set = false;  // once per instantiation (not capture-safe to repeat)
   if (!attr_set) {
     cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (CG == 2) cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 0);
     attr_set = true;
   }
-  kern<<<grid, kThreads, smem, s>>>(ta, tb, ty, a, y);
+  if constexpr (CG == 1) {
+    kern<<<grid, kThreads, smem, s>>>(ta, tb, ty, a, y);
+  } else {
+    cudaLaunchConfig_t lc{};
+    lc.gridDim = dim3((unsigned)grid);
+    lc.blockDim = dim3(kThreads);
+    lc.dynamicSmemBytes = smem;
+    lc.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = 2;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    lc.attrs = at;
+    lc.numAttrs = 1;
+    cudaLaunchKernelEx(&lc, kern, ta, tb, ty, a, y);
+  }
   return cudaGetLastError();
 }
 
@@ -741,7 +777,7 @@ struct TcPlan {
   CUtensorMap ta, tb, ty;
   TcArgs a;
   int grid;
-  int BN, stages;
+  int BN, stages, cg;
   alt_kernel_cfg used;
 };
 static std::mutex g_tc_mu;
@@ -749,13 +785,17 @@ static std::unordered_map<TcKey, TcPlan, TcKeyHash> g_tc_cache;
 
 static cudaError_t launch_plan(const TcPlan &pl, void *y, cudaStream_t stream) {
   uint16_t *yy = static_cast<uint16_t *>(y);
-  if (pl.BN == 64) return launch_tc<64, 8>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
-  if (pl.BN == 128) {
-    if (pl.stages == 4) return launch_tc<128, 4>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
-    return launch_tc<128, 6>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+  if (pl.cg == 2) {
+    if (pl.BN == 128) return launch_tc<128, 8, 2>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+    return launch_tc<256, 6, 2>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
   }
-  if (pl.stages == 3) return launch_tc<256, 3>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
-  return launch_tc<256, 4>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+  if (pl.BN == 64) return launch_tc<64, 8, 1>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+  if (pl.BN == 128) {
+    if (pl.stages == 4) return launch_tc<128, 4, 1>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+    return launch_tc<128, 6, 1>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+  }
+  if (pl.stages == 3) return launch_tc<256, 3, 1>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+  return launch_tc<256, 4, 1>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
 }
 
 // common driver for conv and GEMM
@@ -793,6 +833,7 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
     if (cfg) {
       k[i++] = cfg->block_n; k[i++] = cfg->tile_n; k[i++] = cfg->tile_h; k[i++] = cfg->tile_w;
       k[i++] = cfg->stages;
+      k[i++] = cfg->cta_pair;
     }
     int dev = 0;
     cudaGetDevice(&dev);
@@ -839,6 +880,10 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
   }
   int BN = cfg && cfg->block_n ? cfg->block_n : (P.K > 128 ? 256 : (P.K > 64 ? 128 : 64));
   if (BN != 64 && BN != 128 && BN != 256) { set_error("tc: block_n must be 64/128/256"); return ALT_E_UNSUPPORTED; }
+  // CTA pair (tcgen05 cta_group::2, M = 256): cfg->cta_pair 1 = pair,
+  // 2 = single CTA, 0 = pair when BLOCK_N >= 128
+  const int cg = (cfg && cfg->cta_pair == 2) ? 1 : ((cfg && cfg->cta_pair == 1) || BN >= 128 ? 2 : 1);
+  if (cg == 2 && BN < 128) { set_error("tc: a CTA pair needs block_n >= 128"); return ALT_E_UNSUPPORTED; }
   for (const Cand &c : cands) {
     RoleInfo ra[kMaxL], rb[kMaxL], ry[kMaxL];
     memcpy(ra, P.ra, sizeof(ra));
@@ -856,7 +901,7 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       if (ry[d].role == R_N) ry[d].tile = sw_n;
       if (ry[d].role == R_H) ry[d].tile = sw_h;
       if (ry[d].role == R_W) ry[d].tile = sw_w;
-      if (rb[d].role == R_W) rb[d].tile = BN;
+      if (rb[d].role == R_W) rb[d].tile = BN / cg;
     }
     for (int sw = 64; sw >= 8; sw /= 2) {
       View va, vb;
@@ -865,7 +910,7 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       int64_t rowsA = 1, rowsB = 1;
       for (int i = 1; i < va.rank; i++) rowsA *= (va.d[i].box + va.d[i].estride - 1) / va.d[i].estride;
       for (int i = 1; i < vb.rank; i++) rowsB *= (vb.d[i].box + vb.d[i].estride - 1) / vb.d[i].estride;
-      if (rowsA != 128 || rowsB != BN) { snprintf(why, 160, "rows A %lld B %lld", (long long)rowsA, (long long)rowsB); continue; }
+      if (rowsA != 128 || rowsB != BN / cg) { snprintf(why, 160, "rows A %lld B %lld", (long long)rowsA, (long long)rowsB); continue; }
       TcPlan pl;
       TcArgs &a = pl.a;
       memset(&a, 0, sizeof(a));
@@ -896,7 +941,7 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       const int64_t ntiles = (P.K + BN - 1) / BN;
       if (mtiles * ntiles > 0x7fffffff) { set_error("tc: too many tiles"); return ALT_E_UNSUPPORTED; }
       a.num_n_tiles = (int32_t)ntiles;
-      a.num_tiles = (int32_t)(mtiles * ntiles);
+      a.num_tiles = (int32_t)(((mtiles + cg - 1) / cg) * ntiles);  // work units
       a.S = (int32_t)P.S;
       a.Gc = (int32_t)((P.C + sw - 1) / sw);
       a.total_slabs = (int32_t)(P.R * P.S * a.Gc);
@@ -915,14 +960,16 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       }
       if ((st = make_writer(P.yl, &a.yw)) != ALT_OK) return st;
       a.dbg = debug_buffer();
-      pl.grid = (int)std::min<int64_t>(a.num_tiles, num_sms());
+      pl.grid = (int)std::min<int64_t>((int64_t)a.num_tiles * cg, num_sms() / cg * cg);
       pl.BN = BN;
-      pl.stages = BN == 64 ? 8 : (BN == 128 ? 6 : 4);
+      pl.cg = cg;
+      pl.stages = cg == 2 ? (BN == 128 ? 8 : 6) : (BN == 64 ? 8 : (BN == 128 ? 6 : 4));
       if (cfg && BN == 128 && cfg->stages == 4) pl.stages = 4;
       if (cfg && BN == 256 && cfg->stages == 3) pl.stages = 3;
       alt_kernel_cfg u{};
       u.path = ALT_PATH_TC;
-      u.block_m = 128;
+      u.block_m = 128 * cg;
+      u.cta_pair = cg == 2 ? 1 : 2;
       u.block_n = BN;
       u.block_k = 64;
       u.stages = pl.stages;
