@@ -210,6 +210,16 @@ alt_status alt_matmul(int64_t M, int64_t N, int64_t K, alt_layout a_l,
                       const alt_epilogue *epi, const alt_kernel_cfg *cfg,
                       alt_stream_t stream);
 
+/* 2-D pooling on declared layouts (support op of the ResNet chains; not one
+ * of the paper's operators).  Uses p's N, C, H, W, R, S (window),
+ * stride and pad; K and groups are ignored.  x [N,C,H,W] -> y [N,C,Ho,Wo]:
+ * kind 0 = max (padded taps skipped), 1 = average over in-bounds taps.
+ * y is written through its layout (pad zeros, every unfold copy). */
+typedef enum { ALT_POOL_MAX = 0, ALT_POOL_AVG = 1 } alt_pool_kind;
+alt_status alt_pool2d(const alt_conv2d_params *p, alt_layout x_l, const void *x,
+                      alt_layout y_l, void *y, alt_dtype dtype, int32_t kind,
+                      alt_stream_t stream);
+
 /* Describes which kernel the last alt_conv2d / alt_matmul on this thread
  * chose (alt_path) and its resolved cfg; for tests and the tuner. */
 alt_status alt_last_plan(alt_kernel_cfg *cfg);

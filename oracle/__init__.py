@@ -87,6 +87,7 @@ def lib():
         L.orc_conv2d_unfold_native.argtypes = [c_p, c_ll, c_ll, c_p, c_p, c_p]
         L.orc_gemm_f64.argtypes = [c_ll, c_ll, c_ll, c_p, c_p, c_p, c_p, c_p, c_i,
                                    c_ll, c_ll, c_p]
+        L.orc_pool2d_f64.argtypes = [c_p, c_p, c_i, c_p]
         _lib = L
     return _lib
 
@@ -312,6 +313,17 @@ def gemm(a_l: Layout, a, b_l: Layout, b, scale=None, bias=None, res_l=None, resi
     B = b_l.read_f64(b)
     R = res_l.read_f64(residual) if residual is not None else None
     return gemm_f64(A, B, scale, bias, R, act, rows)
+
+
+def pool2d_f64(x: np.ndarray, R: int, S: int, stride: int, pad: int, kind: str = "max") -> np.ndarray:
+    """O9: max / average pooling over in-bounds taps (support op)."""
+    x = _f64(x)
+    N, C, H, W = x.shape
+    Ho, Wo = (H + 2 * pad - R) // stride + 1, (W + 2 * pad - S) // stride + 1
+    pr = np.array([N, C, H, W, R, S, stride, stride, pad, pad], np.int64)
+    y = np.zeros((N, C, Ho, Wo), np.float64)
+    lib().orc_pool2d_f64(_ptr(pr), _ptr(x), 0 if kind == "max" else 1, _ptr(y))
+    return y
 
 
 def bf16_bits_to_f64(u16: np.ndarray) -> np.ndarray:

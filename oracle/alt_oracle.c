@@ -573,3 +573,33 @@ void orc_gemm_f64(long long M, long long N, long long K, const double *A,
 
 /* sizeof for the Python wrapper */
 long long orc_layout_sizeof(void) { return (long long)sizeof(orc_layout); }
+
+/* ------------------------------------------------------------------ O9 --- */
+/* 2-D pooling (support op of the ResNet chains; not one of the
+ * paper's operators): y[n,c,p,q] = max (kind 0) or mean (kind 1) of
+ * x[n, c, p V_h - pad_h + r, q V_w - pad_w + s] over the in-bounds taps of the
+ * R x S window.  p[] = {N,C,H,W,R,S,Vh,Vw,ph,pw}. */
+void orc_pool2d_f64(const long long *p, const double *x, int kind, double *y) {
+  long long N = p[0], C = p[1], H = p[2], W = p[3], R = p[4], S = p[5];
+  long long Vh = p[6], Vw = p[7], ph = p[8], pw = p[9];
+  long long Ho = (H + 2 * ph - R) / Vh + 1, Wo = (W + 2 * pw - S) / Vw + 1;
+#pragma omp parallel for collapse(2) schedule(static)
+  for (long long n = 0; n < N; n++)
+    for (long long c = 0; c < C; c++)
+      for (long long oh = 0; oh < Ho; oh++)
+        for (long long ow = 0; ow < Wo; ow++) {
+          double acc = kind == 0 ? -INFINITY : 0.0;
+          long long cnt = 0;
+          for (long long r = 0; r < R; r++)
+            for (long long s = 0; s < S; s++) {
+              long long ih = oh * Vh - ph + r, iw = ow * Vw - pw + s;
+              if (ih < 0 || ih >= H || iw < 0 || iw >= W) continue;
+              double v = x[((n * C + c) * H + ih) * W + iw];
+              if (kind == 0) acc = v > acc ? v : acc;
+              else acc += v;
+              cnt++;
+            }
+          if (kind == 1) acc = cnt ? acc / (double)cnt : 0.0;
+          y[((n * C + c) * Ho + oh) * Wo + ow] = acc;
+        }
+}

@@ -100,9 +100,10 @@ _lib.alt_last_plan.argtypes = [_p]
 _lib.alt_launch_count.restype = ctypes.c_uint64
 _lib.alt_tune.argtypes = [ctypes.c_int, _p, ctypes.c_int, _p, _p, _p, _p]
 _lib.alt_plan_chain.argtypes = [_i32, _p, _i32, _p, _p, _p, _p, _p, _p, _p]
+_lib.alt_pool2d.argtypes = [_p, _p, _p, _p, _p, ctypes.c_int, ctypes.c_int32, _p]
 for _f in ("alt_layout_create", "alt_layout_destroy", "alt_layout_query", "alt_layout_logical",
            "alt_layout_phys_to_logical", "alt_layout_logical_to_phys", "alt_relayout",
-           "alt_conv2d", "alt_matmul", "alt_last_plan", "alt_tune", "alt_plan_chain"):
+           "alt_conv2d", "alt_matmul", "alt_last_plan", "alt_tune", "alt_plan_chain", "alt_pool2d"):
     getattr(_lib, _f).restype = ctypes.c_int
 
 
@@ -301,6 +302,13 @@ def matmul(M, N, K, a_l: Layout, a, b_l: Layout, b, c_l: Layout, c, scale=None, 
     return c
 
 
+def pool2d(p: ConvParams, x_l: Layout, x, y_l: Layout, y, kind: str = "max", stream=None):
+    """alt_pool2d: max / average pooling through declared layouts."""
+    _check(_lib.alt_pool2d(ctypes.byref(p), x_l.handle, _ptr(x), y_l.handle, _ptr(y), _dtype_code(x),
+                           0 if kind == "max" else 1, _stream_ptr(stream)), "alt_pool2d")
+    return y
+
+
 def last_plan() -> dict:
     c = KernelCfg()
     _check(_lib.alt_last_plan(ctypes.byref(c)), "alt_last_plan")
@@ -353,4 +361,4 @@ def plan_chain(op_kind: Sequence[int], edges: Sequence[tuple], edge_layouts: Seq
 EXPORTED = ["alt_status_str", "alt_last_error", "alt_layout_create", "alt_layout_destroy",
             "alt_layout_query", "alt_layout_logical", "alt_layout_phys_to_logical",
             "alt_layout_logical_to_phys", "alt_relayout", "alt_conv2d", "alt_matmul",
-            "alt_last_plan", "alt_launch_count", "alt_tune", "alt_plan_chain"]
+            "alt_last_plan", "alt_launch_count", "alt_tune", "alt_plan_chain", "alt_pool2d"]

@@ -1,0 +1,161 @@
+"""Layer chains on ALT layouts with layout propagation (SURVEY §8a rows a5,
+a7, a8, a10): ResNet-18 and MobileNet-V2 conv chains (folded BN + ReLU /
+ReLU6, residual adds, max-pool) executed through the C-ABI.
+
+Propagation (Alg. 1, plus the producer-side half of Fig. 5b):
+every tensor is stored in the input layout its first complex consumer wants;
+the producer (a conv's fused epilogue, the pool, or the input "pad" op)
+writes that layout directly, so no standalone conversion kernel runs inside
+the chain.  `alt_plan_chain` reports where Alg. 1 itself would insert
+conversion ops (complex -> complex edges) — here they are fused.
+"""
+from __future__ import annotations
+
+import math
+
+import torch
+
+from . import _alt as A
+from . import layouts as LY
+from . import nets, synth
+
+
+def chan_tile(C: int) -> int:
+    """largest power of two <= 64 dividing C (>= 8 for the tensor-core path)"""
+    x = 64
+    while x > 1 and C % x:
+        x //= 2
+    return x
+
+
+def act_prims(C: int):
+    if C % 8:
+        Cp = (C + 7) // 8 * 8
+        return LY.nchwxc(C, 8, pad_c=Cp - C)
+    return LY.nchwxc(C, chan_tile(C))
+
+
+def block_n(K: int) -> int:
+    return 64 if K <= 64 else (128 if K <= 128 else 256)
+
+
+def wgt_prims(L: nets.ConvShape):
+    if L.groups > 1:
+        return []
+    x = 8 if L.C % 8 else chan_tile(L.C)
+    pad_c = (L.C + 7) // 8 * 8 - L.C if L.C % 8 else 0
+    bn = block_n(L.K)
+    y = min(L.K, bn)
+    while L.K % y:
+        y //= 2
+    return LY.kcrs_yk_xc(L.K, L.C, y, x, pad_c=pad_c)
+
+
+class Chain:
+    """Device state + launch sequence of one network chain at batch N."""
+
+    def __init__(self, ops, N: int, dev, dtype=torch.bfloat16, name="chain", img_hw=224):
+        self.ops, self.N, self.dev, self.dtype = ops, N, dev, dtype
+        # logical shapes of every tensor
+        shapes = {"img": (N, 3, img_hw, img_hw)}
+        for op in ops:
+            if op[0] == "conv":
+                L = op[1]
+                Ho, Wo = L.out_hw()
+                shapes[op[5]] = (N, L.K, Ho, Wo)
+            else:
+                _, k, s, p, src, dst = op
+                n, c, h, w = shapes[src]
+                shapes[dst] = (n, c, (h + 2 * p - k) // s + 1, (w + 2 * p - k) // s + 1)
+        self.shapes = shapes
+        # layout of each tensor: the input layout of its first consumer (the
+        # same NCHW[x]c family for every consumer here, see act_prims)
+        self.layouts = {t: A.Layout(shp, act_prims(shp[1])) for t, shp in shapes.items()}
+        self.img_plain = A.Layout(shapes["img"], [])
+        self.buf = {t: torch.zeros(self.layouts[t].phys_shape, dtype=dtype, device=dev) for t in shapes}
+        self.img = synth.activations(name + "img", shapes["img"]).to(dtype).to(dev)
+        self.launch_ops = []
+        gen_w = {}
+        for i, op in enumerate(ops):
+            if op[0] != "conv":
+                continue
+            L = op[1]
+            wl0 = A.Layout((L.K, L.C // L.groups, L.R, L.S), [])
+            wl = A.Layout((L.K, L.C // L.groups, L.R, L.S), wgt_prims(L))
+            w0 = synth.weights(name + "w" + L.name, (L.K, L.C // L.groups, L.R, L.S)).to(dtype).to(dev)
+            w = torch.zeros(wl.phys_shape, dtype=dtype, device=dev)
+            A.relayout(wl0, w0, wl, w)  # weights: converted offline
+            sc = synth.bn_scale(name + "s" + L.name, L.K).to(dev)
+            bi = synth.bn_bias(name + "b" + L.name, L.K).to(dev)
+            gen_w[i] = (wl, w, sc, bi)
+        self.weights = gen_w
+        torch.cuda.synchronize(dev) if dev.type == "cuda" else None
+        self.flops = sum(op[1].flops(N) for op in ops if op[0] == "conv")
+
+    # ------------------------------------------------------------ planning
+    def plan(self):
+        """Alg. 1 over the chain's DAG via alt_plan_chain.  Returns
+        (recorded_conversions, standalone_conversion_launches)."""
+        ops = self.ops
+        kinds = [0 if op[0] == "conv" else 2 for op in ops] + [2]   # + the input pad op
+        pad_op = len(ops)
+        producer = {"img": pad_op}
+        for i, op in enumerate(ops):
+            producer[op[5]] = i
+        edges, lays = [], []
+        consumed = set()
+        for i, op in enumerate(ops):
+            srcs = [op[2]] if op[0] == "conv" else [op[4]]
+            if op[0] == "conv" and op[3] is not None:
+                srcs.append(op[3])  # residual input (slot 1)
+            for slot, t in enumerate(srcs):
+                n = 1
+                for s in self.shapes[t]:
+                    n *= s
+                p = producer[t]
+                edges.append((p, i, slot, n))
+                tuned = p < len(ops) and ops[p][0] == "conv"
+                lays.append(self.layouts[t] if tuned and not self.layouts[t].identity else None)
+                consumed.add(t)
+        src_edge, conversion = A.plan_chain(kinds, edges, lays)
+        return sum(conversion), 0
+
+    # ------------------------------------------------------------- running
+    def run(self, stream=None):
+        """One forward pass: the input pad op converts the image into conv1's
+        layout, then every op writes its consumer's layout directly."""
+        A.relayout(self.img_plain, self.img, self.layouts["img"], self.buf["img"], stream=stream)
+        for i, op in enumerate(self.ops):
+            if op[0] == "conv":
+                L, src, res, relu, dst = op[1], op[2], op[3], op[4], op[5]
+                wl, w, sc, bi = self.weights[i]
+                p = A.conv_params(self.N, L.C, L.H, L.W, L.K, L.R, L.S, L.stride, L.pad, L.groups)
+                kw = {}
+                if res is not None:
+                    kw = dict(residual=self.buf[res], residual_l=self.layouts[res])
+                act = ("relu6" if self._relu6 else "relu") if relu else None
+                A.conv2d(p, self.layouts[src], self.buf[src], wl, w, self.layouts[dst], self.buf[dst],
+                         scale=sc, bias=bi, act=act, stream=stream, **kw)
+            else:
+                _, k, s, pd, src, dst = op
+                n, c, h, w_ = self.shapes[src]
+                p = A.conv_params(n, c, h, w_, c, k, k, s, pd)
+                A.pool2d(p, self.layouts[src], self.buf[src], self.layouts[dst], self.buf[dst], "max",
+                         stream=stream)
+        return self.buf[self.ops[-1][5]]
+
+    _relu6 = False
+
+    @property
+    def out_name(self):
+        return self.ops[-1][5]
+
+
+def resnet18(N, dev, dtype=torch.bfloat16, img_hw=224):
+    return Chain(nets.resnet18_chain(img_hw), N, dev, dtype, "r18", img_hw)
+
+
+def mobilenet_v2(N, dev, dtype=torch.bfloat16, img_hw=224):
+    c = Chain(nets.mobilenet_v2_chain(img_hw), N, dev, dtype, "mv2", img_hw)
+    c._relu6 = True
+    return c

@@ -248,6 +248,34 @@ alt_status alt_matmul(int64_t M, int64_t N, int64_t K, alt_layout a_l, const voi
   return st;
 }
 
+alt_status alt_pool2d(const alt_conv2d_params *p, alt_layout x_l, const void *x, alt_layout y_l, void *y,
+                      alt_dtype dtype, int32_t kind, alt_stream_t stream) {
+  if (!p || !x_l || !y_l) { set_error("alt_pool2d: NULL argument"); return ALT_E_INVALID; }
+  if (dtype != ALT_F32 && dtype != ALT_BF16) { set_error("alt_pool2d: bad dtype"); return ALT_E_INVALID; }
+  if (kind != ALT_POOL_MAX && kind != ALT_POOL_AVG) { set_error("alt_pool2d: bad kind"); return ALT_E_INVALID; }
+  if (p->N < 0 || p->C < 1 || p->H < 1 || p->W < 1 || p->R < 1 || p->S < 1 || p->stride_h < 1 ||
+      p->stride_w < 1 || p->pad_h < 0 || p->pad_w < 0) {
+    set_error("alt_pool2d: bad geometry");
+    return ALT_E_INVALID;
+  }
+  const int64_t Ho = (p->H + 2 * p->pad_h - p->R) / p->stride_h + 1;
+  const int64_t Wo = (p->W + 2 * p->pad_w - p->S) / p->stride_w + 1;
+  const int64_t xs[4] = {p->N, p->C, p->H, p->W}, ys[4] = {p->N, p->C, Ho, Wo};
+  if (p->N > 0 && (!shape_is(&x_l->impl, 4, xs) || !shape_is(&y_l->impl, 4, ys))) {
+    set_error("alt_pool2d: layout logical shapes do not match x[N,C,H,W] / y[N,C,Ho,Wo]");
+    return ALT_E_SHAPE;
+  }
+  if (p->N == 0) return ALT_OK;
+  if (!is_device_ptr(x) || !is_device_ptr(y)) { set_error("alt_pool2d: x/y must be device pointers"); return ALT_E_INVALID; }
+  ConvProblem P{};
+  P.N = p->N; P.C = p->C; P.H = p->H; P.W = p->W; P.K = p->C; P.R = p->R; P.S = p->S;
+  P.Ho = Ho; P.Wo = Wo; P.Vh = p->stride_h; P.Vw = p->stride_w; P.ph = p->pad_h; P.pw = p->pad_w;
+  P.groups = 1;
+  P.xl = &x_l->impl; P.yl = &y_l->impl; P.wl = nullptr;
+  P.x = x; P.y = y; P.dtype = dtype;
+  return pool2d(P, kind, reinterpret_cast<cudaStream_t>(stream));
+}
+
 alt_status alt_last_plan(alt_kernel_cfg *cfg) {
   if (!cfg) return ALT_E_INVALID;
   *cfg = g_last_plan;

@@ -161,4 +161,66 @@ alt_status dw_conv(const ConvProblem &P, cudaStream_t stream, alt_kernel_cfg *us
   return ALT_OK;
 }
 
+// ------------------------------------------------------------------ pooling
+// Support op of the ResNet chains (not one of the paper's operators, SURVEY
+// K10): max / average over an R x S window; padded taps are skipped (max) or
+// excluded from the count (avg, count_include_pad = false).
+struct PoolArgs {
+  int32_t N, C, H, W, Ho, Wo, R, S, Vh, Vw, ph, pw, kind;
+  Reader xr;
+  Writer yw;
+};
+
+template <typename T>
+__global__ void __launch_bounds__(256) k_pool(PoolArgs a, const T *__restrict__ x, T *__restrict__ y) {
+  const int64_t total = (int64_t)a.N * a.C * a.Ho * a.Wo;
+  for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
+       idx += (int64_t)gridDim.x * blockDim.x) {
+    // channel fastest: neighbouring threads read neighbouring channels
+    const int c = (int)(idx % a.C);
+    int64_t t = idx / a.C;
+    const int q = (int)(t % a.Wo);
+    t /= a.Wo;
+    const int p = (int)(t % a.Ho);
+    const int n = (int)(t / a.Ho);
+    float acc = a.kind == 0 ? -INFINITY : 0.f;
+    int cnt = 0;
+    for (int r = 0; r < a.R; r++) {
+      const int ih = p * a.Vh - a.ph + r;
+      if (ih < 0 || ih >= a.H) continue;
+      for (int s = 0; s < a.S; s++) {
+        const int iw = q * a.Vw - a.pw + s;
+        if (iw < 0 || iw >= a.W) continue;
+        const int64_t o = a.xr.off4(n, c, ih, iw);
+        if (o < 0) continue;
+        const float v = load_as_f32<T>(x, o);
+        acc = a.kind == 0 ? fmaxf(acc, v) : acc + v;
+        cnt++;
+      }
+    }
+    if (a.kind == 1) acc = cnt ? acc / (float)cnt : 0.f;
+    write4<T>(a.yw, y, n, c, p, q, from_f32<T>(acc));
+  }
+}
+
+alt_status pool2d(const ConvProblem &P, int kind, cudaStream_t stream) {
+  PoolArgs a{};
+  a.N = (int32_t)P.N; a.C = (int32_t)P.C; a.H = (int32_t)P.H; a.W = (int32_t)P.W;
+  a.Ho = (int32_t)P.Ho; a.Wo = (int32_t)P.Wo; a.R = (int32_t)P.R; a.S = (int32_t)P.S;
+  a.Vh = P.Vh; a.Vw = P.Vw; a.ph = P.ph; a.pw = P.pw; a.kind = kind;
+  alt_status st;
+  if ((st = make_reader(P.xl, &a.xr)) != ALT_OK) return st;
+  if ((st = make_writer(P.yl, &a.yw)) != ALT_OK) return st;
+  const int64_t total = P.N * P.C * P.Ho * P.Wo;
+  if (total == 0) return ALT_OK;
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((total + 255) / 256, 148 * 32));
+  if (P.dtype == ALT_BF16)
+    k_pool<uint16_t><<<grid, 256, 0, stream>>>(a, static_cast<const uint16_t *>(P.x), static_cast<uint16_t *>(P.y));
+  else
+    k_pool<float><<<grid, 256, 0, stream>>>(a, static_cast<const float *>(P.x), static_cast<float *>(P.y));
+  count_launch();
+  if (cudaGetLastError() != cudaSuccess) { set_error("pool launch failed"); return ALT_E_CUDA; }
+  return ALT_OK;
+}
+
 }  // namespace alt

@@ -45,5 +45,6 @@ alt_status tc_conv(const ConvProblem &P, const alt_kernel_cfg *cfg, cudaStream_t
 alt_status tc_gemm(const GemmProblem &P, const alt_kernel_cfg *cfg, cudaStream_t stream,
                    alt_kernel_cfg *used);
 alt_status dw_conv(const ConvProblem &P, cudaStream_t stream, alt_kernel_cfg *used);
+alt_status pool2d(const ConvProblem &P, int kind, cudaStream_t stream);
 
 }  // namespace alt

@@ -67,6 +67,47 @@ __global__ void __launch_bounds__(256) k_relayout_sep(SepPair P, const T *__rest
   }
 }
 
+// --------------------------------------------------------------- K_GATHER --
+// One 16-byte dst vector per thread along the dst innermost dim (logical dim
+// a); the other dims are decoded once per vector, the V elements gather
+// through a's tables.  Neighbouring threads hold neighbouring vectors, so each
+// of the V gathers is coalesced across the warp.  Serves pad / unfold layouts.
+template <typename T>
+__global__ void __launch_bounds__(256) k_relayout_gather(SepPair P, int32_t a, const T *__restrict__ src,
+                                                         T *__restrict__ dst, uint32_t nvec) {
+  constexpr int V = 16 / sizeof(T);
+  for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < nvec; v += gridDim.x * blockDim.x) {
+    uint32_t rem = v * V;
+    int32_t combo[kMaxL];
+#pragma unroll
+    for (int d = 0; d < kMaxL; d++) combo[d] = 0;
+    for (int p = P.prank - 1; p >= 0; p--) {
+      uint32_t q, r;
+      P.pdiv[p].divmod(rem, q, r);
+      combo[P.powner[p]] += (int32_t)r * P.prad[p];
+      rem = q;
+    }
+    int64_t base = 0;
+    bool ok = true;
+    for (int d = 0; d < P.lrank; d++) {
+      if (d == a) continue;
+      const int32_t i = __ldg(P.rev[d] + combo[d]);
+      if (i < 0) { ok = false; break; }
+      base += __ldg(P.rd[d] + i);
+    }
+    T val[V];
+#pragma unroll
+    for (int j = 0; j < V; j++) {
+      val[j] = 0;
+      if (ok) {
+        const int32_t i = __ldg(P.rev[a] + combo[a] + j);
+        if (i >= 0) val[j] = src[base + __ldg(P.rd[a] + i)];
+      }
+    }
+    reinterpret_cast<uint4 *>(dst)[v] = *reinterpret_cast<const uint4 *>(val);
+  }
+}
+
 // ----------------------------------------------------------------- K_TILE --
 struct TilePlan {
   SepPair P;
@@ -219,6 +260,291 @@ static bool fill_pair(Layout *S, Layout *D, const SepDev &ss, const SepDev &ds, 
   return true;
 }
 
+// ===================================================== strided permutation ==
+// Fast path for layouts built from split / reorder only (no pad, no unfold):
+// both are permutations of a common refinement of the logical digits, so the
+// conversion is a strided permutation copy.  Dims are coalesced, then either
+//   K_PCOPY  (dst-innermost == src-innermost): 16-byte vector copy, or
+//   K_PTRANS (they differ): 2-D tiles staged through shared memory with
+//            16-byte global loads along the src-contiguous dim and 16-byte
+//            global stores along the dst-contiguous dim.
+struct PermDims {
+  int32_t nd;                  // batch dims (outer, excluding X / Y)
+  FastDiv ext[kMaxP];
+  int64_t sstr[kMaxP], dstr[kMaxP];
+  int64_t ex, ey;              // extents of X (dst stride 1) and Y (src stride 1)
+  int64_t sx, dy;              // src stride of X, dst stride of Y
+};
+
+struct RDim { int64_t ext, sstr, dstr; };
+
+static bool refine_perm(const Layout &S, const Layout &D, std::vector<RDim> &out) {
+  const uint32_t bad = ALT_HAS_PAD | ALT_HAS_UNFOLD;
+  if (!S.separable || !D.separable || !S.aff.ok || !D.aff.ok || (S.flags & bad) || (D.flags & bad)) return false;
+  if (!(S.flags & ALT_LOSSLESS) || !(D.flags & ALT_LOSSLESS)) return false;
+  out.clear();
+  for (int d = 0; d < S.lrank; d++) {
+    struct Dig { int64_t coef, ext, str; };
+    auto digits = [&](const Layout &L) {
+      std::vector<Dig> v;
+      for (int p = 0; p < L.prank; p++)
+        if (L.pdim_owner[p] == d && L.pshape[p] > 1) v.push_back({L.aff.coef[p], L.pshape[p], L.pstride[p]});
+      std::sort(v.begin(), v.end(), [](const Dig &a, const Dig &b) { return a.coef < b.coef; });
+      return v;
+    };
+    std::vector<Dig> sd = digits(S), dd = digits(D);
+    if (S.lshape[d] == 1) continue;
+    // place values of both digit systems must form one divisibility chain
+    std::vector<int64_t> pv;
+    for (auto &g : sd) { pv.push_back(g.coef); pv.push_back(g.coef * g.ext); }
+    for (auto &g : dd) { pv.push_back(g.coef); pv.push_back(g.coef * g.ext); }
+    std::sort(pv.begin(), pv.end());
+    pv.erase(std::unique(pv.begin(), pv.end()), pv.end());
+    if (pv.empty() || pv.front() != 1 || pv.back() != S.lshape[d]) return false;
+    for (size_t i = 0; i + 1 < pv.size(); i++) {
+      if (pv[i + 1] % pv[i]) return false;
+      const int64_t v = pv[i], e = pv[i + 1] / pv[i];
+      auto stride_in = [&](const std::vector<Dig> &ds, int64_t *str) {
+        for (auto &g : ds)
+          if (v >= g.coef && v < g.coef * g.ext) {
+            if (v % g.coef) return false;
+            *str = g.str * (v / g.coef);
+            return (v * e) <= g.coef * g.ext;
+          }
+        return false;
+      };
+      RDim r{e, 0, 0};
+      if (!stride_in(sd, &r.sstr) || !stride_in(dd, &r.dstr)) return false;
+      out.push_back(r);
+    }
+  }
+  // dst row-major order, then coalesce dims nested in both layouts
+  std::sort(out.begin(), out.end(), [](const RDim &a, const RDim &b) { return a.dstr > b.dstr; });
+  std::vector<RDim> c;
+  for (const RDim &r : out) {
+    if (!c.empty() && c.back().dstr == r.dstr * r.ext && c.back().sstr == r.sstr * r.ext) {
+      c.back().ext *= r.ext;
+      c.back().dstr = r.dstr;
+      c.back().sstr = r.sstr;
+    } else {
+      c.push_back(r);
+    }
+  }
+  out = c;
+  return true;
+}
+
+template <typename T>
+__device__ __forceinline__ uint4 ld16(const T *p) { return __ldg(reinterpret_cast<const uint4 *>(p)); }
+
+// vector copy: each thread moves VPT vectors of 16 bytes along X (contiguous
+// in both layouts); batch dims decoded per vector
+template <typename T>
+__global__ void __launch_bounds__(256) k_perm_copy(PermDims P, const T *__restrict__ src, T *__restrict__ dst,
+                                                   uint32_t nvec) {
+  constexpr int V = 16 / sizeof(T);
+  const uint32_t vx = (uint32_t)(P.ex / V);  // vectors per X run
+  for (uint32_t v0 = blockIdx.x * blockDim.x * 4 + threadIdx.x; v0 < nvec; v0 += gridDim.x * blockDim.x * 4) {
+    uint4 val[4];
+    int64_t doff[4];
+    bool ok[4];
+#pragma unroll
+    for (int u = 0; u < 4; u++) {
+      const uint32_t v = v0 + u * blockDim.x;
+      ok[u] = v < nvec;
+      if (!ok[u]) continue;
+      uint32_t rem = v / vx;
+      const uint32_t xi = (v - rem * vx) * V;
+      int64_t so = (int64_t)xi * P.sx;
+      for (int k = P.nd - 1; k >= 0; k--) {
+        uint32_t q, r;
+        P.ext[k].divmod(rem, q, r);
+        so += (int64_t)r * P.sstr[k];
+        rem = q;
+      }
+      doff[u] = (int64_t)v * V;
+      val[u] = ld16(src + so);
+    }
+#pragma unroll
+    for (int u = 0; u < 4; u++)
+      if (ok[u]) *reinterpret_cast<uint4 *>(dst + doff[u]) = val[u];
+  }
+}
+
+// transpose tiles: X (dst stride 1) x Y (src stride 1), TX x TY elements
+template <typename T, int TX, int TY>
+__global__ void __launch_bounds__(256) k_perm_trans(PermDims P, const T *__restrict__ src, T *__restrict__ dst,
+                                                    uint32_t ntiles) {
+  constexpr int V = 16 / sizeof(T);
+  // rows of TY elements; the 16-byte vector slots of row x are XOR-swizzled
+  // by (x / 8) so the column walks of the store phase spread over the banks
+  constexpr int NV = TY / V;
+  __shared__ __align__(16) T tile[TX * TY];
+  auto at = [](int x, int y) { return x * TY + ((((y / V) ^ ((x >> 3) % NV)) * V) + (y % V)); };
+  const uint32_t tx_n = (uint32_t)((P.ex + TX - 1) / TX), ty_n = (uint32_t)((P.ey + TY - 1) / TY);
+  for (uint32_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    uint32_t rem = t;
+    const uint32_t cx = rem % tx_n;
+    rem /= tx_n;
+    const uint32_t cy = rem % ty_n;
+    rem /= ty_n;
+    int64_t sb = 0, db = 0;
+    for (int k = P.nd - 1; k >= 0; k--) {
+      uint32_t q, r;
+      P.ext[k].divmod(rem, q, r);
+      sb += (int64_t)r * P.sstr[k];
+      db += (int64_t)r * P.dstr[k];
+      rem = q;
+    }
+    const int64_t x0 = (int64_t)cx * TX, y0 = (int64_t)cy * TY;
+    const int nx = (int)(P.ex - x0 < TX ? P.ex - x0 : TX), ny = (int)(P.ey - y0 < TY ? P.ey - y0 : TY);
+    sb += x0 * P.sx + y0;
+    db += y0 * P.dy + x0;
+    __syncthreads();
+    if constexpr (TY >= 4 * V) {
+      // wide Y: tile rows x; 16-byte loads along y, column-walk stores
+      for (int e = threadIdx.x; e < TX * (TY / V); e += blockDim.x) {
+        const int x = e / (TY / V), y = (e % (TY / V)) * V;
+        if (x >= nx || y >= ny) continue;
+        const T *s = src + sb + (int64_t)x * P.sx + y;
+        if (y + V <= ny && ((reinterpret_cast<uintptr_t>(s) & 15) == 0)) {
+          *reinterpret_cast<uint4 *>(&tile[at(x, y)]) = ld16(s);
+        } else {
+          for (int j = 0; j < V && y + j < ny; j++) tile[at(x, y + j)] = s[j];
+        }
+      }
+      __syncthreads();
+      for (int e = threadIdx.x; e < TY * (TX / V); e += blockDim.x) {
+        const int y = e / (TX / V), x = (e % (TX / V)) * V;
+        if (y >= ny || x >= nx) continue;
+        T *d = dst + db + (int64_t)y * P.dy + x;
+        if (x + V <= nx && ((reinterpret_cast<uintptr_t>(d) & 15) == 0)) {
+          T v[V];
+#pragma unroll
+          for (int j = 0; j < V; j++) v[j] = tile[at(x + j, y)];
+          *reinterpret_cast<uint4 *>(d) = *reinterpret_cast<const uint4 *>(v);
+        } else {
+          for (int j = 0; j < V && x + j < nx; j++) d[j] = tile[at(x + j, y)];
+        }
+      }
+    } else {
+      // narrow Y (a few vectors per src run): tile rows y; neighbouring
+      // threads load neighbouring x (coalesced when the runs are adjacent) and
+      // scatter into rows y, stores are 16-byte vectors along x
+      for (int e = threadIdx.x; e < TX * (TY / V); e += blockDim.x) {
+        const int x = e % TX, y = (e / TX) * V;
+        if (x >= nx || y >= ny) continue;
+        const T *s = src + sb + (int64_t)x * P.sx + y;
+        if (y + V <= ny && ((reinterpret_cast<uintptr_t>(s) & 15) == 0)) {
+          const uint4 u = ld16(s);
+          const T *uv = reinterpret_cast<const T *>(&u);
+#pragma unroll
+          for (int j = 0; j < V; j++) tile[(y + j) * TX + x] = uv[j];
+        } else {
+          for (int j = 0; j < V && y + j < ny; j++) tile[(y + j) * TX + x] = s[j];
+        }
+      }
+      __syncthreads();
+      for (int e = threadIdx.x; e < TY * (TX / V); e += blockDim.x) {
+        const int y = e / (TX / V), x = (e % (TX / V)) * V;
+        if (y >= ny || x >= nx) continue;
+        T *d = dst + db + (int64_t)y * P.dy + x;
+        if (x + V <= nx && ((reinterpret_cast<uintptr_t>(d) & 15) == 0)) {
+          *reinterpret_cast<uint4 *>(d) = *reinterpret_cast<const uint4 *>(&tile[y * TX + x]);
+        } else {
+          for (int j = 0; j < V && x + j < nx; j++) d[j] = tile[y * TX + x + j];
+        }
+      }
+    }
+  }
+}
+
+static bool perm_launch(Layout *S, const void *src, Layout *D, void *dst, int wb, cudaStream_t stream, int nsm,
+                        alt_status *st) {
+  std::vector<RDim> r;
+  if (!refine_perm(*S, *D, r)) return false;
+  int ix = -1, iy = -1;
+  for (int i = 0; i < (int)r.size(); i++) {
+    if (r[i].dstr == 1) ix = i;
+    if (r[i].sstr == 1) iy = i;
+  }
+  if (ix < 0 || iy < 0) return false;
+  const int V = 16 / wb;
+  PermDims P{};
+  int nd = 0;
+  for (int i = 0; i < (int)r.size(); i++) {
+    if (i == ix || i == iy) continue;
+    if (nd >= kMaxP || r[i].ext >= (1ll << 31)) return false;
+    P.ext[nd] = FastDiv((uint32_t)r[i].ext);
+    P.sstr[nd] = r[i].sstr;
+    P.dstr[nd] = r[i].dstr;
+    nd++;
+  }
+  P.nd = nd;
+  P.ex = r[ix].ext;
+  P.sx = r[ix].sstr;
+  if ((reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst)) & 15) return false;
+  if (ix == iy) {
+    // same innermost dim: vector copy (needs whole vectors and aligned runs)
+    if (P.ex % V) return false;
+    for (int k = 0; k < nd; k++)
+      if (P.sstr[k] % V) return false;
+    const int64_t nvec = D->pnumel / V;
+    if (nvec >= (1ll << 31)) return false;
+    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((nvec + 1023) / 1024, (int64_t)nsm * 8));
+    if (wb == 2) k_perm_copy<uint16_t><<<grid, 256, 0, stream>>>(P, (const uint16_t *)src, (uint16_t *)dst, (uint32_t)nvec);
+    else k_perm_copy<uint32_t><<<grid, 256, 0, stream>>>(P, (const uint32_t *)src, (uint32_t *)dst, (uint32_t)nvec);
+  } else {
+    P.ey = r[iy].ext;
+    P.dy = r[iy].dstr;
+    // tile shape: TX x TY elements (16 KB), the pair wasting
+    // the fewest elements on ragged edges (larger square-ish tiles on ties)
+    const int64_t area = 16384 / wb;  // 16 KB of shared memory per tile
+    int TX = 8;
+    double best = 1e30;
+    for (int tx = 8; tx <= (wb == 2 ? 1024 : 512); tx *= 2) {
+      const int64_t ty = area / tx;
+      if (ty < 8) break;
+      const double waste = (double)((P.ex + tx - 1) / tx * tx) * ((P.ey + ty - 1) / ty * ty) / ((double)P.ex * P.ey);
+      const double score = waste * 1.0 + 1e-3 * std::abs(std::log2((double)tx / ty));
+      if (score < best) { best = score; TX = tx; }
+    }
+    const int64_t TY = area / TX;
+    const int64_t tiles = ((P.ex + TX - 1) / TX) * ((P.ey + TY - 1) / TY) * (D->pnumel / (P.ex * P.ey));
+    if (tiles >= (1ll << 31)) return false;
+    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, (int64_t)nsm * 8));
+    const uint32_t nt = (uint32_t)tiles;
+#define PT(T, X, A) k_perm_trans<T, X, A / X><<<grid, 256, 0, stream>>>(P, (const T *)src, (T *)dst, nt)
+    if (wb == 2) {
+      switch (TX) {
+        case 8: PT(uint16_t, 8, 8192); break;
+        case 16: PT(uint16_t, 16, 8192); break;
+        case 32: PT(uint16_t, 32, 8192); break;
+        case 64: PT(uint16_t, 64, 8192); break;
+        case 128: PT(uint16_t, 128, 8192); break;
+        case 256: PT(uint16_t, 256, 8192); break;
+        case 512: PT(uint16_t, 512, 8192); break;
+        default: PT(uint16_t, 1024, 8192); break;
+      }
+    } else {
+      switch (TX) {
+        case 8: PT(uint32_t, 8, 4096); break;
+        case 16: PT(uint32_t, 16, 4096); break;
+        case 32: PT(uint32_t, 32, 4096); break;
+        case 64: PT(uint32_t, 64, 4096); break;
+        case 128: PT(uint32_t, 128, 4096); break;
+        case 256: PT(uint32_t, 256, 4096); break;
+        default: PT(uint32_t, 512, 4096); break;
+      }
+    }
+#undef PT
+  }
+  count_launch();
+  *st = cudaGetLastError() == cudaSuccess ? ALT_OK : ALT_E_CUDA;
+  if (*st != ALT_OK) set_error("relayout (permutation) launch failed");
+  return true;
+}
+
 alt_status relayout_launch(Layout *S, const void *src, Layout *D, void *dst, int wb,
                            cudaStream_t stream) {
   if (S->lrank != D->lrank) { set_error("alt_relayout: logical ranks differ"); return ALT_E_SHAPE; }
@@ -231,6 +557,10 @@ alt_status relayout_launch(Layout *S, const void *src, Layout *D, void *dst, int
   st = device_tables(D, &ds, &ddesc);
   if (st != ALT_OK) return st;
   const int nsm = sm_count();
+  {
+    alt_status pst = ALT_OK;
+    if (perm_launch(S, src, D, dst, wb, stream, nsm, &pst)) return pst;
+  }
 
   if (S->separable && D->separable) {
     // every element dst holds must have a copy in src
@@ -288,7 +618,7 @@ alt_status relayout_launch(Layout *S, const void *src, Layout *D, void *dst, int
       int p1 = -1;
       for (int p = 0; p < D->prank; p++)
         if (D->pdim_owner[p] == b && D->pdim_rad[p] == 1 && D->pshape[p] > 1) p1 = p;
-      if (p1 >= 0 && p1 != p0) {
+      if (p1 >= 0 && p1 != p0 && E0 % (16 / wb) != 0) {  // else K_GATHER below is faster
         TilePlan TP{};
         TP.P = P;
         TP.p0 = p0;
@@ -331,6 +661,20 @@ alt_status relayout_launch(Layout *S, const void *src, Layout *D, void *dst, int
         count_launch();
         if (cudaGetLastError() != cudaSuccess) { set_error("relayout launch failed"); return ALT_E_CUDA; }
         return ALT_OK;
+      }
+      // ---- K_GATHER: 16-byte dst vectors along the dst innermost dim
+      {
+        const int VV = 16 / wb;
+        bool ok = E0 % VV == 0 && D->pdim_rad[p0] == 1 && ((reinterpret_cast<uintptr_t>(dst) & 15) == 0);
+        if (ok) {
+          const uint32_t nv = (uint32_t)(elems / VV);
+          const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((nv + 255) / 256, (int64_t)nsm * 16));
+          if (wb == 2) k_relayout_gather<uint16_t><<<grid, 256, 0, stream>>>(P, a, (const uint16_t *)src, (uint16_t *)dst, nv);
+          else k_relayout_gather<uint32_t><<<grid, 256, 0, stream>>>(P, a, (const uint32_t *)src, (uint32_t *)dst, nv);
+          count_launch();
+          if (cudaGetLastError() != cudaSuccess) { set_error("relayout launch failed"); return ALT_E_CUDA; }
+          return ALT_OK;
+        }
       }
       // ---- K_SEP scalar
       uint32_t nvec = (uint32_t)elems;

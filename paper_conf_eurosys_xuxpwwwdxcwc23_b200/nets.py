@@ -67,16 +67,17 @@ RESNET50 = [
 ]
 
 
-def resnet18_chain():
+def resnet18_chain(img: int = 224):
     """ResNet-18 conv chain (torchvision): conv1 7x7 s2 + maxpool 3x3 s2,
     4 stages x 2 BasicBlocks (3x3 convs, 1x1 s2 downsample on stages 2-4),
     folded BN + ReLU, residual adds.  Returns a list of ops:
       ("conv", ConvShape, input_id, residual_id or None, relu, out_id)
       ("maxpool", k, s, p, input_id, out_id)
     ids name activation tensors."""
-    ops = [("conv", _c("conv1", 3, 224, 64, 7, 2, 3), "img", None, True, "c1"),
+    ops = [("conv", _c("conv1", 3, img, 64, 7, 2, 3), "img", None, True, "c1"),
            ("maxpool", 3, 2, 1, "c1", "p1")]
-    cur, C, H = "p1", 64, 56
+    h1 = (img + 6 - 7) // 2 + 1
+    cur, C, H = "p1", 64, (h1 + 2 - 3) // 2 + 1
     for stage, (K, stride) in enumerate([(64, 1), (128, 2), (256, 2), (512, 2)]):
         for blk in range(2):
             s = stride if blk == 0 else 1
@@ -93,7 +94,7 @@ def resnet18_chain():
     return ops
 
 
-def mobilenet_v2_chain():
+def mobilenet_v2_chain(img: int = 224):
     """MobileNet-V2 (torchvision, width 1.0, 224): stem 3x3 s2 -> 17
     inverted-residual blocks (expand 1x1 + ReLU6, depthwise 3x3 + ReLU6,
     project 1x1 linear, residual add when stride 1 and C_in == C_out) ->
@@ -101,8 +102,8 @@ def mobilenet_v2_chain():
     resnet18_chain (relu flag means ReLU6 here)."""
     cfg = [(1, 16, 1, 1), (6, 24, 2, 2), (6, 32, 3, 2), (6, 64, 4, 2), (6, 96, 3, 1), (6, 160, 3, 2),
            (6, 320, 1, 1)]
-    ops = [("conv", _c("stem", 3, 224, 32, 3, 2, 1), "img", None, True, "stem")]
-    cur, C, H = "stem", 32, 112
+    ops = [("conv", _c("stem", 3, img, 32, 3, 2, 1), "img", None, True, "stem")]
+    cur, C, H = "stem", 32, (img + 2 - 3) // 2 + 1
     bi = 0
     for t, c, n, s in cfg:
         for i in range(n):

@@ -1,0 +1,119 @@
+"""GPU chains with layout propagation: ResNet-18
+and MobileNet-V2 conv chains on small images, checked layer by layer against
+the fp64 oracle (teacher-forced: each layer's oracle is fed the GPU's own
+input of that layer), zero standalone conversion launches
+inside the chain, pooling parity, and alt_tune on a small conv."""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import paper_conf_eurosys_xuxpwwwdxcwc23_b200 as alt
+from paper_conf_eurosys_xuxpwwwdxcwc23_b200 import chain as CH
+from paper_conf_eurosys_xuxpwwwdxcwc23_b200 import layouts as LY
+from paper_conf_eurosys_xuxpwwwdxcwc23_b200 import synth
+from tests.helpers import BF16_TOL, make_operand, norm_rel, read_output, words
+
+pytestmark = pytest.mark.gpu
+
+
+def _check_chain(ch: CH.Chain, relu6: bool):
+    dev = torch.device("cuda")
+    n0 = alt.launch_count()
+    ch.run()
+    torch.cuda.synchronize()
+    launches = alt.launch_count() - n0
+    # one launch per op plus the input "pad" op that converts the image
+    # (Fig. 5b): no standalone conversion kernel inside the chain
+    assert launches == len(ch.ops) + 1, launches
+    recorded, launched = ch.plan()
+    assert recorded >= 1 and launched == 0
+    worst = 0.0
+    for i, op in enumerate(ch.ops):
+        if op[0] == "conv":
+            L, src, res, relu, dst = op[1], op[2], op[3], op[4], op[5]
+            wl, w, sc, bi = ch.weights[i]
+            Ox = oracle.Layout(ch.shapes[src], ch.layouts[src].prims)
+            Ow = oracle.Layout(wl.logical_shape, wl.prims)
+            pd = dict(N=ch.N, C=L.C, H=L.H, W=L.W, K=L.K, R=L.R, S=L.S, stride_h=L.stride,
+                      stride_w=L.stride, pad_h=L.pad, pad_w=L.pad, groups=L.groups)
+            kw = {}
+            if res is not None:
+                kw = dict(res_l=oracle.Layout(ch.shapes[res], ch.layouts[res].prims),
+                          residual=words(ch.buf[res]).reshape(ch.layouts[res].phys_shape))
+            act = (2 if relu6 else 1) if relu else 0
+            ref = oracle.conv2d(pd, Ox, words(ch.buf[src]).reshape(Ox.phys_shape), Ow,
+                                words(w).reshape(Ow.phys_shape), scale=sc.double().cpu().numpy(),
+                                bias=bi.double().cpu().numpy(), act=act, **kw)
+            got = read_output(oracle.Layout(ch.shapes[dst], ch.layouts[dst].prims), ch.buf[dst],
+                              torch.bfloat16)
+            err = norm_rel(got, ref)
+            worst = max(worst, err)
+            assert err <= BF16_TOL, (L.name, err)
+        else:
+            _, k, s, p, src, dst = op
+            Ox = oracle.Layout(ch.shapes[src], ch.layouts[src].prims)
+            xin = Ox.read_f64(words(ch.buf[src]))
+            ref = oracle.pool2d_f64(xin, k, k, s, p, "max")
+            got = read_output(oracle.Layout(ch.shapes[dst], ch.layouts[dst].prims), ch.buf[dst],
+                              torch.bfloat16)
+            assert np.array_equal(got, ref)   # max of bf16 values is exact
+    return worst
+
+
+def test_resnet18_chain_small():
+    ch = CH.resnet18(2, torch.device("cuda"), img_hw=64)
+    _check_chain(ch, relu6=False)
+
+
+def test_mobilenet_v2_chain_small():
+    ch = CH.mobilenet_v2(2, torch.device("cuda"), img_hw=64)
+    _check_chain(ch, relu6=True)
+
+
+@pytest.mark.parametrize("kind", ["max", "avg"])
+def test_pool_parity(kind):
+    x = synth.activations("pool" + kind, (2, 32, 17, 15))
+    xp = LY.nchwxc(32, 8)
+    Ox, xph, xd = make_operand("pool", xp, x, torch.bfloat16)
+    Lx = alt.Layout(x.shape, xp)
+    yp = LY.nchwxc(32, 16, pad_hw=1)
+    Ly = alt.Layout((2, 32, 9, 8), yp)
+    y = torch.full(Ly.phys_shape, 7.0, dtype=torch.bfloat16, device="cuda")
+    alt.pool2d(alt.conv_params(2, 32, 17, 15, 32, 3, 3, 2, 1), Lx, xd, Ly, y, kind)
+    torch.cuda.synchronize()
+    ref = oracle.pool2d_f64(Ox.read_f64(xph), 3, 3, 2, 1, kind)
+    got = read_output(oracle.Layout((2, 32, 9, 8), yp), y, torch.bfloat16)
+    if kind == "max":
+        assert np.array_equal(got, ref)
+    else:  # fp32 mean rounded once to bf16
+        assert norm_rel(got, ref) <= 4e-3
+
+
+def test_tune_conv_small():
+    """alt_tune (bounded grid, parity unpinned A19): the winner is a valid
+    layout pair whose conv is oracle-exact."""
+    p = alt.conv_params(4, 64, 14, 14, 128, 3, 3, 1, 1)
+    res = alt.tune("conv2d", p, alt.ALT_BF16, {0: [64, 32], 1: [64], 6: [128, 256]}, max_points=8,
+                   warmup=1, reps=3)
+    assert res["measured"] >= 2 and res["best_us"] > 0
+    assert all(t >= res["best_us"] for t in res["all_us"])
+    x = synth.activations("tunex", (4, 64, 14, 14))
+    w = synth.weights("tunew", (128, 64, 3, 3))
+    Ox, xph, xd = make_operand("tunex", res["x"], x, torch.bfloat16)
+    Ow, wph, wd = make_operand("tunew", res["w"], w, torch.bfloat16)
+    Ly = alt.Layout((4, 128, 14, 14), res["y"])
+    y = torch.zeros(Ly.phys_shape, dtype=torch.bfloat16, device="cuda")
+    alt.conv2d(p, alt.Layout(x.shape, res["x"]), xd, alt.Layout(w.shape, res["w"]), wd, Ly, y,
+               cfg=res["cfg"])
+    torch.cuda.synchronize()
+    ref = oracle.conv2d(dict(N=4, C=64, H=14, W=14, K=128, R=3, S=3, pad_h=1, pad_w=1), Ox, xph, Ow, wph)
+    got = read_output(oracle.Layout((4, 128, 14, 14), res["y"]), y, torch.bfloat16)
+    assert norm_rel(got, ref) <= BF16_TOL
+
+
+def test_tune_gemm_small():
+    g = alt._alt.MatmulParams(512, 256, 256)
+    res = alt.tune("matmul", g, alt.ALT_BF16, {0: [128], 1: [64], 2: [128, 256], 6: [256]}, max_points=4,
+                   warmup=1, reps=3)
+    assert res["measured"] >= 1 and res["best_us"] > 0

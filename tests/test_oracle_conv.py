@@ -217,3 +217,16 @@ def test_gemm_through_tiled_layouts():
         got = oracle.gemm(La, La.materialize(A.view(np.uint32)), lb,
                           lb.materialize(B.view(np.uint32)))
         np.testing.assert_allclose(got, want, rtol=1e-12, atol=1e-12)
+
+
+def test_pool_vs_torch_float64():
+    """O9 pooling vs torch max_pool2d / avg_pool2d (count_include_pad=False)."""
+    rng = np.random.default_rng(11)
+    x = rng.uniform(-1, 1, (2, 5, 13, 11))
+    for k, s, p in [(3, 2, 1), (2, 2, 0), (3, 1, 1)]:
+        got = oracle.pool2d_f64(x, k, k, s, p, "max")
+        ref = torch.nn.functional.max_pool2d(torch.from_numpy(x), k, s, p).numpy()
+        assert np.array_equal(got, ref)
+        got = oracle.pool2d_f64(x, k, k, s, p, "avg")
+        ref = torch.nn.functional.avg_pool2d(torch.from_numpy(x), k, s, p, count_include_pad=False).numpy()
+        np.testing.assert_allclose(got, ref, rtol=1e-12, atol=1e-14)
