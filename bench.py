@@ -121,10 +121,14 @@ def plan_layer(L, N):
     hit = tunecache.lookup("conv2d", L, N)
     if hit is not None:
         return hit
-    Cp = L.C if L.C % 8 == 0 else (L.C + 7) // 8 * 8
+    bn = 256 if L.K % 256 == 0 else (128 if L.K % 128 == 0 else 64)
+    if L.C % 8:
+        # few channels (conv1): window-folded input, K rows = (s, c) runs
+        return {"x": LY.conv_input_wfold(L.C, L.S, L.stride, L.pad), "w": LY.kcrs_wfold(L.K, L.C, L.S),
+                "y": LY.nchwxc(L.K, min(L.K, 64)), "cfg": {"path": 1, "block_n": bn}}
+    Cp = L.C
     x = min(Cp, 64)
     xp = LY.nchwxc(L.C, x, pad_c=Cp - L.C)
-    bn = 256 if L.K % 256 == 0 else (128 if L.K % 128 == 0 else 64)
     wp = LY.kcrs_yk_xc(L.K, L.C, min(L.K, bn), x, pad_c=Cp - L.C)
     yp = LY.nchwxc(L.K, min(L.K, 64))
     return {"x": xp, "w": wp, "y": yp, "cfg": {"path": 1, "block_n": bn}}

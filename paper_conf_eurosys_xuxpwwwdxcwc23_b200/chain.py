@@ -42,6 +42,8 @@ def block_n(K: int) -> int:
 def wgt_prims(L: nets.ConvShape):
     if L.groups > 1:
         return []
+    if L.C % 8:
+        return LY.kcrs_wfold(L.K, L.C, L.S)
     x = 8 if L.C % 8 else chan_tile(L.C)
     pad_c = (L.C + 7) // 8 * 8 - L.C if L.C % 8 else 0
     bn = block_n(L.K)
@@ -71,6 +73,11 @@ class Chain:
         # layout of each tensor: the input layout of its first consumer (the
         # same NCHW[x]c family for every consumer here, see act_prims)
         self.layouts = {t: A.Layout(shp, act_prims(shp[1])) for t, shp in shapes.items()}
+        # a few-channel first conv (C = 3) reads the image window-folded
+        # (reading A23): the input pad op writes that layout directly
+        L0 = ops[0][1]
+        if ops[0][0] == "conv" and ops[0][2] == "img" and L0.C % 8 and L0.groups == 1:
+            self.layouts["img"] = A.Layout(shapes["img"], LY.conv_input_wfold(L0.C, L0.S, L0.stride, L0.pad))
         self.img_plain = A.Layout(shapes["img"], [])
         self.buf = {t: torch.zeros(self.layouts[t].phys_shape, dtype=dtype, device=dev) for t in shapes}
         self.img = synth.activations(name + "img", shapes["img"]).to(dtype).to(dev)

@@ -108,6 +108,86 @@ __global__ void __launch_bounds__(256) k_relayout_gather(SepPair P, int32_t a, c
   }
 }
 
+// ----------------------------------------------------------------- K_GVEC --
+// One 16-byte dst vector per thread for layouts whose innermost dst dims are
+// too short for K_GATHER / K_TILE (e.g. a 4-channel run inside an unfolded
+// window, reading A23): the physical coordinate is decoded once per vector
+// and then stepped with carries; only the logical dims whose coordinate
+// changed are looked up again.
+template <typename T>
+__global__ void __launch_bounds__(256) k_relayout_gvec(SepPair P, const T *__restrict__ src,
+                                                       T *__restrict__ dst, uint32_t nvec) {
+  // all per-dim arrays are indexed with compile-time indices (registers)
+  constexpr int V = 16 / sizeof(T);
+  for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < nvec; v += gridDim.x * blockDim.x) {
+    uint32_t rem = v * V;
+    int32_t coord[kMaxP];
+    int32_t combo[kMaxL];
+#pragma unroll
+    for (int d = 0; d < kMaxL; d++) combo[d] = 0;
+#pragma unroll
+    for (int p = kMaxP - 1; p >= 0; p--) {
+      coord[p] = 0;
+      if (p < P.prank) {
+        uint32_t q, r;
+        P.pdiv[p].divmod(rem, q, r);
+        coord[p] = (int32_t)r;
+#pragma unroll
+        for (int d = 0; d < kMaxL; d++)
+          if (P.powner[p] == d) combo[d] += (int32_t)r * P.prad[p];
+        rem = q;
+      }
+    }
+    int64_t part[kMaxL];
+    uint32_t zero = 0;  // bit d: logical dim d sits on a structural zero
+#pragma unroll
+    for (int d = 0; d < kMaxL; d++) {
+      part[d] = 0;
+      if (d < P.lrank) {
+        const int32_t i = __ldg(P.rev[d] + combo[d]);
+        if (i < 0) zero |= 1u << d;
+        else part[d] = __ldg(P.rd[d] + i);
+      }
+    }
+    T val[V];
+#pragma unroll
+    for (int j = 0; j < V; j++) {
+      int64_t off = 0;
+#pragma unroll
+      for (int d = 0; d < kMaxL; d++) off += part[d];
+      val[j] = zero ? T(0) : src[off];
+      if (j + 1 < V) {
+        uint32_t dirty = 0;
+        bool carry = true;
+#pragma unroll
+        for (int p = kMaxP - 1; p >= 0; p--) {
+          if (carry && p < P.prank) {
+            const int o = P.powner[p];
+            dirty |= 1u << o;
+            const int32_t c = coord[p] + 1;
+            const bool wrap = c >= (int32_t)P.pdiv[p].d;
+            coord[p] = wrap ? 0 : c;
+            const int32_t delta = wrap ? -(c - 1) * P.prad[p] : P.prad[p];
+#pragma unroll
+            for (int d = 0; d < kMaxL; d++)
+              if (o == d) combo[d] += delta;
+            carry = wrap;
+          }
+        }
+#pragma unroll
+        for (int d = 0; d < kMaxL; d++) {
+          if (d < P.lrank && (dirty >> d & 1)) {
+            const int32_t i = __ldg(P.rev[d] + combo[d]);
+            part[d] = i < 0 ? 0 : __ldg(P.rd[d] + i);
+            zero = i < 0 ? (zero | 1u << d) : (zero & ~(1u << d));
+          }
+        }
+      }
+    }
+    reinterpret_cast<uint4 *>(dst)[v] = *reinterpret_cast<const uint4 *>(val);
+  }
+}
+
 // ----------------------------------------------------------------- K_TILE --
 struct TilePlan {
   SepPair P;
@@ -618,6 +698,17 @@ alt_status relayout_launch(Layout *S, const void *src, Layout *D, void *dst, int
       int p1 = -1;
       for (int p = 0; p < D->prank; p++)
         if (D->pdim_owner[p] == b && D->pdim_rad[p] == 1 && D->pshape[p] > 1) p1 = p;
+      const bool gvec_ok = elems % (16 / wb) == 0 && (reinterpret_cast<uintptr_t>(dst) & 15) == 0;
+      if (gvec_ok && E0 < 16 / wb) {
+        // ---- K_GVEC: short innermost runs (one 16-byte vector spans dims)
+        const uint32_t nv = (uint32_t)(elems / (16 / wb));
+        const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((nv + 255) / 256, (int64_t)nsm * 16));
+        if (wb == 2) k_relayout_gvec<uint16_t><<<grid, 256, 0, stream>>>(P, (const uint16_t *)src, (uint16_t *)dst, nv);
+        else k_relayout_gvec<uint32_t><<<grid, 256, 0, stream>>>(P, (const uint32_t *)src, (uint32_t *)dst, nv);
+        count_launch();
+        if (cudaGetLastError() != cudaSuccess) { set_error("relayout launch failed"); return ALT_E_CUDA; }
+        return ALT_OK;
+      }
       if (p1 >= 0 && p1 != p0 && E0 % (16 / wb) != 0) {  // else K_GATHER below is faster
         TilePlan TP{};
         TP.P = P;

@@ -444,23 +444,93 @@ struct View {
   int64_t xlo = 0;  // channel run (extent of the stride-1 channel dim)
 };
 
+// The part of a compiled layout a TMA view needs: physical extents / strides
+// and the affine map i_d = sum_p coef_p j_p + off_d (separable layouts).
+// Physical dims of extent 1 are ignored, which is how fold_window() below
+// drops a dim it merged into another.
+struct LView {
+  bool ok = false;
+  int lrank = 0, prank = 0;
+  int64_t pshape[kMaxP] = {}, pstride[kMaxP] = {}, coef[kMaxP] = {};
+  int32_t owner[kMaxP] = {};
+  int64_t off[kMaxL] = {};
+};
+
+static LView lview(const Layout &L) {
+  LView v;
+  v.ok = L.separable && L.aff.ok;
+  v.lrank = L.lrank;
+  v.prank = L.prank;
+  for (int p = 0; p < L.prank; p++) {
+    v.pshape[p] = L.pshape[p];
+    v.pstride[p] = L.pstride[p];
+    v.coef[p] = L.aff.coef[p];
+    v.owner[p] = L.pdim_owner[p];
+  }
+  for (int d = 0; d < L.lrank; d++) v.off[d] = L.aff.off[d];
+  return v;
+}
+
+// Window folding (unfold with one conv window per layout tile):
+// when x's W dim is unfold(B = E >= S, step = conv stride) of the conv-padded
+// row, stored [.. Wt][Wi][C] with the channel run innermost, the (Wi, C)
+// pair is one contiguous run of E*C elements per output column — the whole
+// filter row's reduction.  With the weights stored [.. S'][C] (S padded to E)
+// the conv is the same sum as a conv with S = 1, stride 1, no W padding and
+// E*C channels: x'(n, s*C + c, h, q) = x(n, c, h, V q + s - pad).  This turns
+// a few-channel layer (conv1, C = 3) into 64-element K rows instead of
+// 16-byte slabs per tap.
+static bool fold_window(const LView &x, const LView &w, int64_t S, int Vw, int pw, int64_t Wo, LView *xo,
+                        LView *wo, int64_t *Cfold) {
+  if (!x.ok || !w.ok || x.lrank != 4 || w.lrank != 4) return false;
+  int xw[kMaxP], nxw = 0, xc = -1, nxc = 0, ws = -1, nws = 0, wc = -1, nwc = 0;
+  for (int p = 0; p < x.prank; p++) {
+    if (x.pshape[p] == 1) continue;
+    if (x.owner[p] == 3) xw[nxw++] = p;
+    if (x.owner[p] == 1) { xc = p; nxc++; }
+  }
+  for (int p = 0; p < w.prank; p++) {
+    if (w.pshape[p] == 1) continue;
+    if (w.owner[p] == 3) { ws = p; nws++; }
+    if (w.owner[p] == 1) { wc = p; nwc++; }
+  }
+  if (nxw != 2 || nxc != 1 || nws != 1 || nwc != 1) return false;
+  // Wi = the inner of the two (stride 1 unfolds give both coefficient 1)
+  const int wi = x.pstride[xw[0]] < x.pstride[xw[1]] ? xw[0] : xw[1], wt = wi == xw[0] ? xw[1] : xw[0];
+  if (x.coef[wi] != 1 || x.coef[wt] != Vw || x.off[3] != -pw || x.pshape[wt] < Wo) return false;
+  const int64_t E = x.pshape[wi], C = x.pshape[xc];
+  if (E < S || x.pstride[xc] != 1 || x.coef[xc] != 1 || x.off[1] != 0 || x.pstride[wi] != C) return false;
+  if (w.pshape[ws] != E || w.coef[ws] != 1 || w.off[3] != 0 || w.pstride[ws] != C) return false;
+  if (w.pshape[wc] != C || w.pstride[wc] != 1 || w.coef[wc] != 1 || w.off[1] != 0) return false;
+  *xo = x;
+  *wo = w;
+  xo->pshape[xc] = E * C;
+  xo->pshape[wi] = 1;
+  xo->coef[wt] = 1;
+  xo->off[3] = 0;
+  wo->pshape[wc] = E * C;
+  wo->pshape[ws] = 1;
+  *Cfold = E * C;
+  return true;
+}
+
 // Cut a TMA view out of a compiled layout: per logical dim a role (rows n/h/w,
 // channel c, filter taps r/s).  Requires the layout's affine map (split /
 // reorder / pad / unfold sequences); see DESIGN.md §5.
-static bool build_view(const Layout &L, const RoleInfo *roles, int sw, View *out, char *why) {
+static bool build_view(const LView &L, const RoleInfo *roles, int sw, View *out, char *why) {
   auto fail = [&](const char *m) { snprintf(why, 160, "%s", m); return false; };
-  if (!L.separable || !L.aff.ok) return fail("layout not separable-affine");
+  if (!L.ok) return fail("layout not separable-affine");
   View v;
   int nphys[kMaxL] = {};
   int plist[kMaxL][kMaxP];
   for (int p = 0; p < L.prank; p++) {
     if (L.pshape[p] == 1) continue;
-    const int d = L.pdim_owner[p];
+    const int d = L.owner[p];
     plist[d][nphys[d]++] = p;
   }
   for (int d = 0; d < L.lrank; d++) {
     const RoleInfo &ri = roles[d];
-    const int64_t off = L.aff.off[d];
+    const int64_t off = L.off[d];
     auto add = [&](int p, int box, int es, int order) -> VDim & {
       VDim &x = v.d[v.rank++];
       x.extent = L.pshape[p];
@@ -478,12 +548,12 @@ static bool build_view(const Layout &L, const RoleInfo *roles, int sw, View *out
         int plo = -1, phi = -1;
         for (int i = 0; i < nphys[d]; i++) {
           const int p = plist[d][i];
-          if (L.aff.coef[p] == 1) plo = p; else phi = p;
+          if (L.coef[p] == 1) plo = p; else phi = p;
         }
         if (plo < 0 || L.pstride[plo] != 1) return fail("channel tile is not the innermost (stride-1) dim");
         const int64_t xlo = L.pshape[plo];
         if (xlo % sw) return fail("slab width does not divide channel tile");
-        if (phi >= 0 && L.aff.coef[phi] != xlo) return fail("channel digits not a plain split");
+        if (phi >= 0 && L.coef[phi] != xlo) return fail("channel digits not a plain split");
         v.xlo = xlo;
         v.divg = (int)(xlo / sw);
         VDim &lo = add(plo, sw, 1, 0);
@@ -496,7 +566,7 @@ static bool build_view(const Layout &L, const RoleInfo *roles, int sw, View *out
       }
       case R_N: {
         if (nphys[d] == 0) { if (ri.tile != 1) return fail("tile_n > 1 on a size-1 dim"); break; }
-        if (nphys[d] != 1 || L.aff.coef[plist[d][0]] != 1 || off != 0) return fail("batch dim must be plain");
+        if (nphys[d] != 1 || L.coef[plist[d][0]] != 1 || off != 0) return fail("batch dim must be plain");
         VDim &x = add(plist[d][0], ri.tile, 1, 50);
         x.coef[V_N0] = 1;
         break;
@@ -504,7 +574,7 @@ static bool build_view(const Layout &L, const RoleInfo *roles, int sw, View *out
       case R_TR:
       case R_TS: {
         if (nphys[d] == 0) break;
-        if (nphys[d] != 1 || L.aff.coef[plist[d][0]] != 1 || off != 0) return fail("filter tap dim must be plain");
+        if (nphys[d] != 1 || L.coef[plist[d][0]] != 1 || off != 0) return fail("filter tap dim must be plain");
         VDim &x = add(plist[d][0], 1, 1, 100);
         x.coef[ri.role == R_TR ? V_R : V_S] = 1;
         break;
@@ -521,7 +591,7 @@ static bool build_view(const Layout &L, const RoleInfo *roles, int sw, View *out
         }
         if (nphys[d] == 1) {
           const int p = plist[d][0];
-          if (L.aff.coef[p] != 1) return fail("spatial dim coefficient != 1");
+          if (L.coef[p] != 1) return fail("spatial dim coefficient != 1");
           const int box = ri.tile * ri.V;
           if (box > 256) return fail("box > 256");
           VDim &x = add(p, box, ri.V, base_order);
@@ -533,11 +603,12 @@ static bool build_view(const Layout &L, const RoleInfo *roles, int sw, View *out
         if (nphys[d] != 2) return fail("spatial dim with >2 physical dims");
         int plo = -1, phi = -1;
         for (int i = 0; i < 2; i++) {
-          const int p = plist[d][i];
-          if (L.aff.coef[p] == 1 && plo < 0) plo = p; else phi = p;
+          const int p = plist[d][i], o = plist[d][1 - i];
+          // the in-tile digit: coefficient 1, and the inner one when both are 1
+          if (L.coef[p] == 1 && (L.coef[o] != 1 || L.pstride[p] < L.pstride[o])) plo = p; else phi = p;
         }
         if (plo < 0 || phi < 0) return fail("spatial digits without unit coefficient");
-        const int64_t Elo = L.pshape[plo], ch = L.aff.coef[phi];
+        const int64_t Elo = L.pshape[plo], ch = L.coef[phi];
         if (ch == Elo) {
           // plain split (GEMM-like): no window, no stride, no padding
           if (ri.V != 1 || ri.win != 1 || ri.pad != 0 || off != 0) return fail("split spatial dim with window/stride");
@@ -802,6 +873,7 @@ static cudaError_t launch_plan(const TcPlan &pl, void *y, cudaStream_t stream) {
 struct TcProblem {
   bool is_conv;
   Layout *al, *bl, *yl;
+  LView va, vb, vy;           // what build_view sees (folded views for conv1-like layers)
   const void *a, *b;
   void *y;
   RoleInfo ra[kMaxL], rb[kMaxL], ry[kMaxL];
@@ -905,8 +977,8 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
     }
     for (int sw = 64; sw >= 8; sw /= 2) {
       View va, vb;
-      if (!build_view(*P.al, ra, sw, &va, why)) continue;
-      if (!build_view(*P.bl, rb, sw, &vb, why)) continue;
+      if (!build_view(P.va, ra, sw, &va, why)) continue;
+      if (!build_view(P.vb, rb, sw, &vb, why)) continue;
       int64_t rowsA = 1, rowsB = 1;
       for (int i = 1; i < va.rank; i++) rowsA *= (va.d[i].box + va.d[i].estride - 1) / va.d[i].estride;
       for (int i = 1; i < vb.rank; i++) rowsB *= (vb.d[i].box + vb.d[i].estride - 1) / vb.d[i].estride;
@@ -924,7 +996,7 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
         char why2[160];
         for (int so = 32; so >= 8 && !a.out_mode; so /= 2) {
           View vy;
-          if (!build_view(*P.yl, ry, so, &vy, why2)) continue;
+          if (!build_view(P.vy, ry, so, &vy, why2)) continue;
           int64_t rowsY = 1;
           for (int i = 1; i < vy.rank; i++) rowsY *= vy.d[i].box;
           if (rowsY != 32) continue;
@@ -1014,6 +1086,16 @@ alt_status tc_conv(const ConvProblem &P, const alt_kernel_cfg *cfg, cudaStream_t
   T.N = P.N; T.K = P.K; T.Ho = P.Ho; T.Wo = P.Wo;
   T.R = P.R; T.S = P.S; T.C = P.C;
   T.epi = P.epi;
+  T.va = lview(*P.xl); T.vb = lview(*P.wl); T.vy = lview(*P.yl);
+  {
+    LView xf, wf;
+    int64_t Cf = 0;
+    if (fold_window(T.va, T.vb, P.S, P.Vw, P.pw, P.Wo, &xf, &wf, &Cf)) {
+      T.va = xf; T.vb = wf;
+      T.ra[3] = RoleInfo{R_W, 1, 1, 0, 1, 0};
+      T.S = 1; T.C = Cf;
+    }
+  }
   if (P.N * P.Ho * P.Wo >= (1ll << 31)) { set_error("tc: too many output pixels"); return ALT_E_UNSUPPORTED; }
   return tc_run(T, cfg, stream, used, 0, 0);
 }
@@ -1034,6 +1116,7 @@ alt_status tc_gemm(const GemmProblem &P, const alt_kernel_cfg *cfg, cudaStream_t
   T.N = 1; T.K = P.N; T.Ho = 1; T.Wo = P.M;
   T.R = 1; T.S = 1; T.C = P.K;
   T.epi = P.epi;
+  T.va = lview(*P.al); T.vb = lview(*P.bl); T.vy = lview(*P.cl);
   if (P.M >= (1ll << 31)) { set_error("tc: M too large"); return ALT_E_UNSUPPORTED; }
   return tc_run(T, cfg, stream, used, 1, 1);
 }

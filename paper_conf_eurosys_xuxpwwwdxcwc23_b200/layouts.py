@@ -88,3 +88,39 @@ def gemm_nkn_b(K: int, N: int, n: int = 16):
 
 def transpose2():
     return [("reorder", [1, 0])]
+
+
+def fold_extent(C: int, S: int):
+    """(Cp, E) for the window-folded layouts: channels padded to Cp, windows
+    of E >= S columns, E * Cp a power of two >= 16 (one K row of 32..128 B)."""
+    Cp = 4 if C <= 4 else (C + 7) // 8 * 8
+    E = 1
+    while E < S or (E * Cp) < 16:
+        E *= 2
+    return Cp, E
+
+
+def conv_input_wfold(C: int, S: int, stride: int, pad: int):
+    """N H W/V E Cp: pad W by the conv padding, unfold(B = E, step = V) so
+    each layout tile holds one output column's filter window (P:727-749,
+    reading A23), channels innermost.  The tensor-core conv then reduces over
+    the contiguous (window, channel) run — few-channel layers (conv1)."""
+    Cp, E = fold_extent(C, S)
+    pr = []
+    if Cp > C:
+        pr.append(("pad", 1, 0, Cp - C))
+    # hi padding grows by E - S so the last output column's window is whole
+    pr += [("pad", 3, pad, pad + E - S), ("unfold", 3, E, stride), ("reorder", [0, 2, 3, 4, 1])]
+    return pr
+
+
+def kcrs_wfold(K: int, C: int, S: int):
+    """Weights K R E Cp for conv_input_wfold inputs (S zero-padded to E)."""
+    Cp, E = fold_extent(C, S)
+    pr = []
+    if Cp > C:
+        pr.append(("pad", 1, 0, Cp - C))
+    if E > S:
+        pr.append(("pad", 3, 0, E - S))
+    pr.append(("reorder", [0, 2, 3, 1]))
+    return pr

@@ -22,6 +22,7 @@ def cases():
         ("R5 images NCHW->pad(C)+NCHW8c", (N, 3, 224, 224), [], LY.nchwxc(3, 8, pad_c=5)),
         ("R6 row-major->[M/128][K/64][128][64]", (8192, 3072), [], LY.gemm_a_tiled(8192, 3072, 128, 64)),
         ("R7 KCRS->KCRS16k16c", (512, 512, 3, 3), [], LY.kcrs_yk_xc(512, 512, 16, 16)),
+        ("R8 images NCHW->window-folded conv1 input", (N, 3, 224, 224), [], LY.conv_input_wfold(3, 7, 2, 3)),
     ]
 
 

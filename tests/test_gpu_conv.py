@@ -172,6 +172,13 @@ TC_CASES = [
      LY.conv_input_tiled(32, 16, 30, 30, 3, 3, 8, 8, 2, 1), LY.kcrs_yk_xc(64, 32, 64, 16), LY.nchwxc(64, 32)),
     ("unfold out tiled", (2, 64, 14, 14, 128, 3, 3, 1, 1), LY.nchwxc(64, 64), LY.kcrs_yk_xc(128, 64, 128, 64),
      LY.conv_output_tiled(128, 16, 14, 14, 7, 7)),
+    # window-folded input (unfold B = E, step = V; reading A23): conv1-like
+    ("wfold conv1 C3 7x7 s2", (2, 3, 38, 38, 64, 7, 7, 2, 3), LY.conv_input_wfold(3, 7, 2, 3),
+     LY.kcrs_wfold(64, 3, 7), LY.nchwxc(64, 64)),
+    ("wfold C3 3x3 s2 K32", (3, 3, 30, 26, 32, 3, 3, 2, 1), LY.conv_input_wfold(3, 3, 2, 1),
+     LY.kcrs_wfold(32, 3, 3), LY.nchwxc(32, 32)),
+    ("wfold C16 3x3 s1", (2, 16, 12, 20, 64, 3, 3, 1, 1), LY.conv_input_wfold(16, 3, 1, 1),
+     LY.kcrs_wfold(64, 16, 3), LY.nhwc()),
 ]
 
 

@@ -63,6 +63,9 @@ D6 = [
     ("R7 KCRS->KCRS16k16c", (512, 512, 3, 3), [], LY.kcrs_yk_xc(512, 512, 16, 16)),
     ("unfold src -> NCHW", (2, 16, 28, 28), LY.conv_input_tiled(16, 8, 28, 28, 3, 3, 7, 7, 1, 1), []),
     ("stride-2 tiles", (2, 16, 28, 28), [], LY.conv_input_tiled(16, 16, 28, 28, 3, 3, 4, 7, 2, 1)),
+    ("R8 images -> window-folded 7x7 s2", (3, 3, 50, 46), [], LY.conv_input_wfold(3, 7, 2, 3)),
+    ("R8 images -> window-folded 3x3 s2", (2, 3, 33, 31), [], LY.conv_input_wfold(3, 3, 2, 1)),
+    ("window-folded C16 s1 -> NHWC", (2, 16, 9, 13), LY.conv_input_wfold(16, 3, 1, 1), LY.nhwc()),
 ]
 
 
