@@ -190,9 +190,12 @@ typedef struct {
   int32_t block_n;     /* 32..256, multiple of 16 */
   int32_t block_k;     /* 64 */
   int32_t stages;      /* smem pipeline depth */
-  int32_t cta_pair;    /* 1 = tcgen05 cta_group::2 (reserved) */
+  int32_t cta_pair;    /* 0 auto, 1 = tcgen05 cta_group::2 CTA pair, 2 = one CTA */
   int32_t tile_n, tile_h, tile_w;
-  int32_t _pad;
+  int32_t split_k;     /* tensor-core path: 0 auto, 1 none, s = the reduction
+                          is cut into s ranges whose fp32 partial tiles are
+                          summed in split order by the last CTA to finish
+                          (deterministic); for grids smaller than the GPU */
 } alt_kernel_cfg;
 
 alt_status alt_conv2d(const alt_conv2d_params *p, alt_layout x_l, const void *x,

@@ -34,6 +34,7 @@
 #include <cstring>
 #include <mutex>
 #include <unordered_map>
+#include <type_traits>
 #include <vector>
 
 #include "epilogue.cuh"
@@ -55,7 +56,7 @@ struct OperandMap {
 
 struct TcArgs {
   OperandMap A, B, O;
-  int32_t out_mode;      // 1: TMA-store epilogue, 0: generic writer
+  int32_t out_mode;      // 1: TMA-store epilogue, 2: direct 16-byte stores, 0: generic writer
   int32_t is_conv;
   int32_t N, K, Ho, Wo;  // output: conv y[N,K,Ho,Wo]; GEMM: N=1, Ho=1, Wo=M, K=cols
   int32_t tile_n, tile_h, tile_w;
@@ -65,8 +66,14 @@ struct TcArgs {
   int32_t total_slabs, spi, num_iters;
   int32_t sw;
   Writer yw;
+  Reader yr;             // out_mode 2: owner offsets of y
   EpiParams epi;
   uint64_t *dbg;         // optional per-CTA timestamps (ALT_TC_DEBUG)
+  // split-K: work unit = (output tile, reduction range); partial fp32 tiles
+  // in ws[cta_tile][split][BN/32][128][32], arrivals counted in cnt[cta_tile]
+  int32_t splits;
+  float *ws;
+  int32_t *cnt;
 };
 
 constexpr int kThreads = 320;  // producer, MMA, 8 epilogue warps
@@ -78,8 +85,9 @@ struct TcSmem {
   static constexpr int kB = (BN / CG) * 64 * 2;  // this CTA's share of the B tile
   static constexpr int kRing = STAGES * (kStageBytesA + kB);
   static constexpr int kOut = kRing;                       // 2 staging buffers for TMA stores
-  static constexpr int kBar = kOut + 2 * kOutStage;        // barriers
-  static constexpr int kBytes = kBar + 128 + 1008 /*1024-B alignment slack*/;
+  static constexpr int kSB = kOut + 2 * kOutStage;         // scale / bias of the tile (2 x BN floats)
+  static constexpr int kBar = kSB + 2 * BN * 4;             // barriers
+  static constexpr int kBytes = kBar + 256 + 1008 /*1024-B alignment slack*/;
 };
 
 __device__ __forceinline__ uint64_t gtimer() {
@@ -87,6 +95,9 @@ __device__ __forceinline__ uint64_t gtimer() {
   asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
   return t;
 }
+#ifndef ALT_DBG_TILE
+#define ALT_DBG_TILE 0  // which of a CTA's tiles the epilogue timestamps follow
+#endif
 #define DBG(slot) \
   if (a.dbg) a.dbg[(size_t)blockIdx.x * 32 + (slot)] = gtimer()
 
@@ -102,6 +113,17 @@ __device__ __forceinline__ void coords(const OperandMap &m, const int32_t (&v)[N
 
 __device__ __forceinline__ void named_bar(int id, int n) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory");
+}
+// two floats -> packed bf16x2 (lo = a), optionally with ReLU in the convert
+__device__ __forceinline__ uint32_t pack_bf16x2(float a, float b) {
+  uint32_t r;
+  asm("cvt.rn.bf16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(b), "f"(a));
+  return r;
+}
+__device__ __forceinline__ uint32_t pack_bf16x2_relu(float a, float b) {
+  uint32_t r;
+  asm("cvt.rn.relu.bf16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(b), "f"(a));
+  return r;
 }
 __device__ __forceinline__ void fence_async_smem() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 __device__ __forceinline__ void tma_store_5d(const CUtensorMap *m, const void *src, int32_t c0, int32_t c1,
@@ -143,6 +165,26 @@ static __device__ __noinline__ void write_chunk(const Writer &w, int is_conv, in
   }
 }
 
+// split-K: the tile's value = sum of the splits' partials in split order
+// (all read back from the workspace, this CTA's own included), so the result
+// does not depend on which CTA finishes last.  Out of line: the split path
+// is rare and must not cost the common path registers.
+static __device__ __noinline__ void split_total(const float *wt, int splits, int BN, int cb, int row, float *out) {
+  float t[32];
+#pragma unroll
+  for (int j = 0; j < 32; j++) t[j] = 0.f;
+  for (int s = 0; s < splits; s++) {
+    const float4 *src = reinterpret_cast<const float4 *>(wt + (size_t)s * (128 * BN) + ((size_t)(cb >> 5) * 128 + row) * 32);
+#pragma unroll
+    for (int j = 0; j < 8; j++) {
+      const float4 f = __ldcg(src + j);
+      t[4 * j] += f.x; t[4 * j + 1] += f.y; t[4 * j + 2] += f.z; t[4 * j + 3] += f.w;
+    }
+  }
+#pragma unroll
+  for (int j = 0; j < 32; j++) out[j] = t[j];
+}
+
 struct TileCoord { int n0, p0, q0, k0; };
 // work unit `tile` -> this CTA's 128-row M tile and the unit's N tile; with a
 // CTA pair (CG = 2) a unit is two consecutive M tiles, one per CTA rank
@@ -168,25 +210,28 @@ __global__ void __launch_bounds__(kThreads, 1)
   unsigned char *sA = smem;
   unsigned char *sB = smem + STAGES * kStageBytesA;
   unsigned char *sOut = smem + L::kOut;
+  float *sScale = reinterpret_cast<float *>(smem + L::kSB);
+  float *sBias = sScale + BN;
   uint64_t *full = reinterpret_cast<uint64_t *>(smem + L::kBar);
   uint64_t *empty = full + STAGES;
   uint64_t *tfull = empty + STAGES;   // [2]
   uint64_t *tempty = tfull + 2;       // [2]
   uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(tempty + 2);
+  volatile int32_t *last_flag = reinterpret_cast<volatile int32_t *>(tmem_slot + 1);
 
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
   if (threadIdx.x == 0) { DBG(0); }
   if (warp == 0 && lane == 0) {
     tma_prefetch(&tmA);
     tma_prefetch(&tmB);
-    if (a.out_mode) tma_prefetch(&tmY);
+    if (a.out_mode == 1) tma_prefetch(&tmY);
     for (int s = 0; s < STAGES; s++) {
       mbar_init(&full[s], 1);
       mbar_init(&empty[s], 1);
     }
     for (int s = 0; s < 2; s++) {
       mbar_init(&tfull[s], 1);
-      mbar_init(&tempty[s], 256 * CG);  // every epilogue thread of the pair
+      mbar_init(&tempty[s], 8 * CG);  // every epilogue warp of the pair
     }
     fence_mbar_init();
   }
@@ -211,7 +256,9 @@ __global__ void __launch_bounds__(kThreads, 1)
     const bool active = j < a.spi;
     int it = 0;
     for (int tile = unit0; tile < a.num_tiles; tile += unit_step) {
-      const TileCoord tc = tile_coord(a, tile, BN, CG, rank);
+      const int mn = tile / a.splits, sp = tile - mn * a.splits;
+      const TileCoord tc = tile_coord(a, mn, BN, CG, rank);
+      const int k_begin = sp * a.num_iters / a.splits, k_end = (sp + 1) * a.num_iters / a.splits;
       int32_t v[NVAR];
       // B rows of this CTA: its 1/CG share of the unit's BN output channels
       const int pp = isA ? tc.p0 : 0, qq = isA ? tc.q0 : tc.k0 + rank * (BN / CG);
@@ -219,7 +266,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       v[V_PT] = pp / om.divp; v[V_PR] = pp % om.divp;
       v[V_QT] = qq / om.divq; v[V_QR] = qq % om.divq;
       v[V_ONE] = 1;
-      for (int kit = 0; kit < a.num_iters; kit++, it++) {
+      for (int kit = k_begin; kit < k_end; kit++, it++) {
         const int stage = it % STAGES, round = it / STAGES;
         if (round > 0) mbar_wait(&empty[stage], (round - 1) & 1);
         // the leader's full barrier counts the bytes of both CTAs of a pair
@@ -260,7 +307,9 @@ __global__ void __launch_bounds__(kThreads, 1)
         if (use > 0) mbar_wait(&tempty[acc], (use - 1) & 1);
         tc_fence_after();
         const uint32_t d = tmem + (uint32_t)(acc * BN);
-        for (int kit = 0; kit < a.num_iters; kit++, it++) {
+        const int sp = tile % a.splits;
+        const int k_begin = sp * a.num_iters / a.splits, k_end = (sp + 1) * a.num_iters / a.splits;
+        for (int kit = k_begin; kit < k_end; kit++, it++) {
           const int stage = it % STAGES, round = it / STAGES;
           mbar_wait(&full[stage], round & 1);
           tc_fence_after();
@@ -272,8 +321,9 @@ __global__ void __launch_bounds__(kThreads, 1)
             const uint32_t off = (uint32_t)((kc % sw) * 2);
             const uint64_t ad = smem_desc(baseA + slab * aS + off, lboA, sbo, layout);
             const uint64_t bd = smem_desc(baseB + slab * bS + off, lboB, sbo, layout);
-            if constexpr (CG == 2) mma_bf16_2cta(d, ad, bd, idesc, (kit | kk) != 0);
-            else mma_bf16(d, ad, bd, idesc, (kit | kk) != 0);
+            const bool accum = kit != k_begin || kk != 0;
+            if constexpr (CG == 2) mma_bf16_2cta(d, ad, bd, idesc, accum);
+            else mma_bf16(d, ad, bd, idesc, accum);
           }
           if constexpr (CG == 2) mma_commit_2cta(&empty[stage], 0x3);  // frees the stage in both CTAs
           else mma_commit(&empty[stage]);
@@ -292,124 +342,226 @@ __global__ void __launch_bounds__(kThreads, 1)
     const int half = (warp - 2) >> 2;
     const int row = wq * 32 + lane;        // accumulator row = tile row
     const int tn = a.tile_h * a.tile_w;
-    const int sw_o = a.O.sw;
+    const int sw_o = a.out_mode == 1 ? a.O.sw : 32;
     const int pitch = sw_o * 2;            // bytes per row in a staging slab
     const int swz = pitch == 128 ? 3 : (pitch == 64 ? 2 : (pitch == 32 ? 1 : 0));
-    const uint32_t sOut_u32 = smem_u32(sOut);
-    // activation as a clamp: none (-inf, inf), ReLU [0, inf), ReLU6 [0, 6]
-    const float act_lo = a.epi.act == 0 ? -INFINITY : 0.f;
-    const float act_hi = a.epi.act == 2 ? 6.f : INFINITY;
+    // this thread's four 16-byte pieces inside a (swizzled) staging buffer
+    uint32_t soff[4];
+#pragma unroll
+    for (int c = 0; c < 4; c++) {
+      const int ch = c * 8;
+      uint32_t off = (uint32_t)(lane * pitch + (ch % sw_o) * 2);
+      off ^= ((off >> 7) & ((1u << swz) - 1u)) << 4;
+      soff[c] = (uint32_t)((ch / sw_o) * 32 * pitch) + off;
+    }
+    const uint32_t wbuf = smem_u32(sOut) + (uint32_t)((warp - 2) * 4096);
+    const int act = a.epi.act;
+    // scale / bias of a tile's BN channels, one per thread, fetched one tile
+    // ahead into registers and staged in smem (ragged channels clamp)
+    auto fetch_sb = [&](int tile, float &fs, float &fb) {
+      fs = 1.f; fb = 0.f;
+      if (tile < a.num_tiles && et < BN) {
+        const int k = min(tile_coord(a, tile / a.splits, BN, CG, rank).k0 + et, a.K - 1);
+        fs = __ldg(a.epi.scale + k);
+        fb = __ldg(a.epi.bias + k);
+      }
+    };
+    float pf_s, pf_b;
+    fetch_sb(unit0, pf_s, pf_b);
     int i = 0;
     for (int tile = unit0; tile < a.num_tiles; tile += unit_step, i++) {
       const int acc = i & 1, use = i >> 1;
-      const TileCoord tc = tile_coord(a, tile, BN, CG, rank);
+      const int mn = tile / a.splits, ksp = tile - mn * a.splits;
+      const TileCoord tc = tile_coord(a, mn, BN, CG, rank);
+      named_bar(2, 256);  // every epilogue warp is done with the previous tile's values
+      if (et < BN) { sScale[et] = pf_s; sBias[et] = pf_b; }
+      named_bar(2, 256);
+      fetch_sb(tile + unit_step, pf_s, pf_b);
       const int n = tc.n0 + row / tn, p = tc.p0 + (row / a.tile_w) % a.tile_h, q = tc.q0 + row % a.tile_w;
       const bool vrow = n < a.N && p < a.Ho && q < a.Wo;
-      // origin of this warp's 32-row sub-box of the output tile
-      const int r0 = wq * 32;
-      const int sn = tc.n0 + r0 / tn, sp = tc.p0 + (r0 / a.tile_w) % a.tile_h, sq = tc.q0 + r0 % a.tile_w;
-      int32_t vo[NVAR];
-      vo[V_N0] = sn;
-      vo[V_PT] = sp / a.O.divp; vo[V_PR] = sp % a.O.divp;
-      vo[V_QT] = sq / a.O.divq; vo[V_QR] = sq % a.O.divq;
-      vo[V_R] = 0; vo[V_S] = 0; vo[V_ONE] = 1;
+      int64_t yrow = 0;  // out_mode 2: offset of this thread's output row
+      if (a.out_mode == 2 && vrow)
+        yrow = a.is_conv ? __ldg(a.yr.rd[0] + n) + __ldg(a.yr.rd[2] + p) + __ldg(a.yr.rd[3] + q) : __ldg(a.yr.rd[0] + q);
+      // TMA-store coordinates of this warp's 32-row sub-box, less the
+      // channel-slab terms (added per store)
+      int32_t cbase[5];
+      if (a.out_mode == 1 && lane == 0) {
+        const int r0 = wq * 32;
+        const int sn = tc.n0 + r0 / tn, sp = tc.p0 + (r0 / a.tile_w) % a.tile_h, sq = tc.q0 + r0 % a.tile_w;
+        int32_t vo[NVAR];
+        vo[V_N0] = sn;
+        vo[V_PT] = sp / a.O.divp; vo[V_PR] = sp % a.O.divp;
+        vo[V_QT] = sq / a.O.divq; vo[V_QR] = sq % a.O.divq;
+        vo[V_GT] = 0; vo[V_GR] = 0; vo[V_R] = 0; vo[V_S] = 0; vo[V_ONE] = 1;
+        coords(a.O, vo, cbase);
+      }
       mbar_wait(&tfull[acc], use & 1);
-      if (et == 0 && i == 0) { DBG(2); }
+      if (et == 0 && i == ALT_DBG_TILE) { DBG(2); }
       tc_fence_after();
+      const float *wsl = nullptr;  // this CTA tile's partials (split-K)
+      if (a.splits > 1) {
+        const size_t cta_tile = (size_t)mn * CG + rank;
+        float *wt = a.ws + cta_tile * (size_t)a.splits * (128 * BN);
+        float *mine = wt + (size_t)ksp * (128 * BN);
 #pragma unroll 1
-      for (int c0 = 0; c0 < BN; c0 += 64) {
-        const int cb = c0 + half * 32;     // first column of this thread's 32
-        uint32_t raw[32];
-        tmem_ld_32x32b_x32(tmem + ((uint32_t)(wq * 32) << 16) + (uint32_t)(acc * BN + cb), raw);
-        tmem_ld_wait();
-        if (et == 0 && i == 0) { DBG(8 + (c0 >> 6) * 4); }
-        if (c0 + 64 >= BN) {  // accumulator buffer drained: MMA may reuse it
+        for (int c0 = 0; c0 < BN; c0 += 64) {
+          const int cb = c0 + half * 32;
+          uint32_t raw[32];
+          tmem_ld_32x32b_x32(tmem + ((uint32_t)(wq * 32) << 16) + (uint32_t)(acc * BN + cb), raw);
+          tmem_ld_wait();
+          uint4 *dst = reinterpret_cast<uint4 *>(mine + ((size_t)(cb >> 5) * 128 + row) * 32);
+#pragma unroll
+          for (int j = 0; j < 8; j++) dst[j] = make_uint4(raw[4 * j], raw[4 * j + 1], raw[4 * j + 2], raw[4 * j + 3]);
+        }
+        __threadfence();
+        named_bar(1, 256);
+        if (et == 0) *last_flag = atomicAdd(a.cnt + cta_tile, 1) == a.splits - 1;
+        named_bar(1, 256);
+        if (!*last_flag) {  // another CTA finishes this tile: free the accumulator
           tc_fence_before();
-          if constexpr (CG == 2) mbar_arrive_cluster(&tempty[acc], 0);  // the leader's MMA waits
-          else mbar_arrive(&tempty[acc]);
-        }
-        float v[32];
-        // per-channel scale / bias (L1-resident after the first row)
-        const int kb = tc.k0 + cb;
-        // scale / bias are never NULL here (the host substitutes ones / zeros);
-        // a ragged last chunk clamps its indices (those channels are not stored)
-        if (kb + 32 <= a.K) {
-          const float4 *s4 = reinterpret_cast<const float4 *>(a.epi.scale + kb);
-          const float4 *b4 = reinterpret_cast<const float4 *>(a.epi.bias + kb);
-#pragma unroll
-          for (int j = 0; j < 8; j++) {
-            const float4 sc = __ldg(s4 + j), bi = __ldg(b4 + j);
-            v[4 * j + 0] = fmaf(__uint_as_float(raw[4 * j + 0]), sc.x, bi.x);
-            v[4 * j + 1] = fmaf(__uint_as_float(raw[4 * j + 1]), sc.y, bi.y);
-            v[4 * j + 2] = fmaf(__uint_as_float(raw[4 * j + 2]), sc.z, bi.z);
-            v[4 * j + 3] = fmaf(__uint_as_float(raw[4 * j + 3]), sc.w, bi.w);
-          }
-        } else {
-#pragma unroll
-          for (int j = 0; j < 32; j++) {
-            const int k = min(kb + j, a.K - 1);
-            v[j] = fmaf(__uint_as_float(raw[j]), __ldg(a.epi.scale + k), __ldg(a.epi.bias + k));
-          }
-        }
-        if (a.epi.residual && vrow) {
-          float rv[32];  // local memory, touched only when a residual exists
-          residual_chunk(a.epi, a.is_conv, a.K, n, p, q, kb, rv);
-#pragma unroll
-          for (int j = 0; j < 32; j++) v[j] += rv[j];
-        }
-        uint32_t pk[16];
-#pragma unroll
-        for (int j = 0; j < 16; j++) {
-          const __nv_bfloat162 h2 = __floats2bfloat162_rn(fminf(fmaxf(v[2 * j], act_lo), act_hi),
-                                                          fminf(fmaxf(v[2 * j + 1], act_lo), act_hi));
-          pk[j] = *reinterpret_cast<const uint32_t *>(&h2);
-        }
-        if (et == 0 && i == 0) { DBG(9 + (c0 >> 6) * 4); }
-        if (a.out_mode) {
-          // Each warp stores its own 32-row x 32-channel sub-tile: private
-          // double-buffered staging, swizzled rows, one TMA store per slab;
-          // no CTA-wide barrier.  Buffer `buf` is free once the store issued
-          // two chunks ago has read it (<= 1 store group in flight per warp).
-          const int buf = (c0 >> 6) & 1;
-          if (lane == 0) bulk_wait_read1();
-          __syncwarp();
-          const uint32_t wbase = sOut_u32 + (uint32_t)((warp - 2) * 4096 + buf * 2048);
-#pragma unroll
-          for (int c = 0; c < 4; c++) {  // 4 x 16 B = this thread's 32 channels
-            const int ch = c * 8;
-            const int slab = ch / sw_o;
-            uint32_t off = (uint32_t)(lane * pitch + (ch % sw_o) * 2);
-            off ^= ((off >> 7) & ((1u << swz) - 1u)) << 4;
-            const uint32_t addr = wbase + (uint32_t)(slab * 32 * pitch) + off;
-            asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "r"(pk[4 * c]),
-                         "r"(pk[4 * c + 1]), "r"(pk[4 * c + 2]), "r"(pk[4 * c + 3])
-                         : "memory");
-          }
-          if (et == 0 && i == 0) { DBG(10 + (c0 >> 6) * 4); }
-          fence_async_smem();
           __syncwarp();
           if (lane == 0) {
-            const int nslab = 32 / sw_o;
-            for (int j = 0; j < nslab; j++) {
-              if (kb + j * sw_o >= a.K) break;  // channels past K: nothing to store
-              const int g = kb / sw_o + j;
-              vo[V_GT] = g / a.O.divg; vo[V_GR] = g % a.O.divg;
-              int32_t co[5];
-              coords(a.O, vo, co);
-              tma_store_5d(&tmY, sOut + (warp - 2) * 4096 + buf * 2048 + j * 32 * pitch, co[0], co[1], co[2],
-                           co[3], co[4]);
-            }
-            bulk_commit();
-            if (et == 0 && i == 0) { DBG(11 + (c0 >> 6) * 4); }
+            if constexpr (CG == 2) mbar_arrive_cluster(&tempty[acc], 0);
+            else mbar_arrive(&tempty[acc]);
           }
-        } else if (vrow) {
-          // generic layouts: every copy / pad position through the writer
-          write_chunk(a.yw, a.is_conv, a.K, y, n, p, q, kb, pk);
+          continue;
         }
+        __threadfence();
+        if (et == 0) a.cnt[cta_tile] = 0;  // ready for the next launch
+        wsl = wt;
       }
+      // TMEM reads are software-pipelined (TMEM read is 32 B/clk per SM):
+      // on the plain path (TMA-store output, no residual, no split) chunk
+      // c + 1's load is issued as soon as chunk c's values are consumed, so
+      // it overlaps chunk c's conversion and store.  That variant makes no
+      // function calls while a load is in flight (a call would save / restore
+      // the registers the asynchronous load is writing); the other variant
+      // issues the next load at the end of the chunk.
+      auto chunk_loop = [&](auto early_tag) {
+        constexpr bool EARLY = decltype(early_tag)::value;
+        uint32_t raw[32];
+        tmem_ld_32x32b_x32(tmem + ((uint32_t)(wq * 32) << 16) + (uint32_t)(acc * BN + half * 32), raw);
+#pragma unroll 1
+        for (int c0 = 0; c0 < BN; c0 += 64) {
+          const int cb = c0 + half * 32;     // first column of this thread's 32
+          const int kb = tc.k0 + cb;
+          const uint32_t next = tmem + ((uint32_t)(wq * 32) << 16) + (uint32_t)(acc * BN + cb + 64);
+          tmem_ld_wait();
+#pragma unroll
+          for (int j = 0; j < 32; j++) asm volatile("" : "+r"(raw[j]));  // uses stay after the wait
+          if (et == 0 && i == ALT_DBG_TILE) { DBG(8 + (c0 >> 6) * 4); }
+          if constexpr (!EARLY) {
+            if (wsl) {
+              float tot[32];
+              split_total(wsl, a.splits, BN, cb, row, tot);
+#pragma unroll
+              for (int j = 0; j < 32; j++) raw[j] = __float_as_uint(tot[j]);
+            }
+          }
+          float v[32];
+          {
+            const float4 *s4 = reinterpret_cast<const float4 *>(sScale + cb);
+            const float4 *b4 = reinterpret_cast<const float4 *>(sBias + cb);
+#pragma unroll
+            for (int j = 0; j < 8; j++) {
+              const float4 x = s4[j], y = b4[j];
+              v[4 * j + 0] = fmaf(__uint_as_float(raw[4 * j + 0]), x.x, y.x);
+              v[4 * j + 1] = fmaf(__uint_as_float(raw[4 * j + 1]), x.y, y.y);
+              v[4 * j + 2] = fmaf(__uint_as_float(raw[4 * j + 2]), x.z, y.z);
+              v[4 * j + 3] = fmaf(__uint_as_float(raw[4 * j + 3]), x.w, y.w);
+            }
+          }
+          if constexpr (EARLY) {
+            if (c0 + 64 < BN) tmem_ld_32x32b_x32(next, raw);
+          }
+          if (c0 + 64 >= BN) {  // accumulator buffer drained: MMA may reuse it
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) {
+              if constexpr (CG == 2) mbar_arrive_cluster(&tempty[acc], 0);  // the leader's MMA waits
+              else mbar_arrive(&tempty[acc]);
+            }
+          }
+          if constexpr (!EARLY) {
+            if (a.epi.residual && vrow) {
+              float rv[32];  // local memory, touched only when a residual exists
+              residual_chunk(a.epi, a.is_conv, a.K, n, p, q, kb, rv);
+#pragma unroll
+              for (int j = 0; j < 32; j++) v[j] += rv[j];
+            }
+          }
+          // activation folded into the bf16 conversion (cvt .relu)
+          uint32_t pk[16];
+          if (act == 1) {
+#pragma unroll
+            for (int j = 0; j < 16; j++) pk[j] = pack_bf16x2_relu(v[2 * j], v[2 * j + 1]);
+          } else if (act == 2) {
+#pragma unroll
+            for (int j = 0; j < 16; j++) pk[j] = pack_bf16x2_relu(fminf(v[2 * j], 6.f), fminf(v[2 * j + 1], 6.f));
+          } else {
+#pragma unroll
+            for (int j = 0; j < 16; j++) pk[j] = pack_bf16x2(v[2 * j], v[2 * j + 1]);
+          }
+          if (et == 0 && i == ALT_DBG_TILE) { DBG(9 + (c0 >> 6) * 4); }
+          if (a.out_mode == 2) {
+            // direct 16-byte stores: 8 channels are contiguous in y
+            if (vrow) {
+#pragma unroll
+              for (int c = 0; c < 4; c++) {
+                const int k = kb + 8 * c;
+                if (k < a.K) {
+                  uint16_t *dst = y + yrow + __ldg(a.yr.rd[1] + k);
+                  asm volatile("st.global.v4.b32 [%0], {%1, %2, %3, %4};" ::"l"(dst), "r"(pk[4 * c]),
+                               "r"(pk[4 * c + 1]), "r"(pk[4 * c + 2]), "r"(pk[4 * c + 3])
+                               : "memory");
+                }
+              }
+            }
+          } else if (a.out_mode == 1) {
+            // Each warp stores its own 32-row x 32-channel sub-tile: private
+            // double-buffered staging, swizzled rows, one TMA store per slab;
+            // no CTA-wide barrier.  Buffer `buf` is free once the store issued
+            // two chunks ago has read it (<= 1 store group in flight per warp).
+            const uint32_t buf = (uint32_t)((c0 >> 6) & 1) * 2048u;
+            if (lane == 0) bulk_wait_read1();
+            __syncwarp();
+#pragma unroll
+            for (int c = 0; c < 4; c++)
+              asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(wbuf + buf + soff[c]), "r"(pk[4 * c]),
+                           "r"(pk[4 * c + 1]), "r"(pk[4 * c + 2]), "r"(pk[4 * c + 3])
+                           : "memory");
+            if (et == 0 && i == ALT_DBG_TILE) { DBG(10 + (c0 >> 6) * 4); }
+            fence_async_smem();
+            __syncwarp();
+            if (lane == 0) {
+              const int nslab = 32 / sw_o;
+              for (int j = 0; j < nslab; j++) {
+                if (kb + j * sw_o >= a.K) break;  // channels past K: nothing to store
+                const int g = kb / sw_o + j;
+                const int gt = g / a.O.divg, gr = g - gt * a.O.divg;
+                int32_t co[5];
+#pragma unroll
+                for (int d = 0; d < 5; d++) co[d] = cbase[d] + a.O.coef[d][V_GT] * gt + a.O.coef[d][V_GR] * gr;
+                tma_store_5d(&tmY, sOut + (warp - 2) * 4096 + buf + j * 32 * pitch, co[0], co[1], co[2], co[3],
+                             co[4]);
+              }
+              bulk_commit();
+              if (et == 0 && i == ALT_DBG_TILE) { DBG(11 + (c0 >> 6) * 4); }
+            }
+          } else if constexpr (!EARLY) {
+            // generic layouts: every copy / pad position through the writer
+            if (vrow) write_chunk(a.yw, a.is_conv, a.K, y, n, p, q, kb, pk);
+          }
+          if constexpr (!EARLY) {
+            if (c0 + 64 < BN) tmem_ld_32x32b_x32(next, raw);
+          }
+        }
+      };
+      if (a.out_mode != 0 && !a.epi.residual && !wsl) chunk_loop(std::true_type{});
+      else chunk_loop(std::false_type{});
     }
     if (et == 0) { DBG(5); }
-    if (lane == 0 && a.out_mode) bulk_wait0();
+    if (lane == 0 && a.out_mode == 1) bulk_wait0();
   }
   tc_fence_before();
   __syncthreads();
@@ -738,6 +890,22 @@ static bool encode_view(const View &v, const void *base, int esize, int sw, CUte
 
 alt_status make_reader(Layout *L, Reader *r);
 alt_status make_writer(Layout *L, Writer *w);
+
+// out_mode 2 needs every 8-channel group contiguous and 16-byte aligned:
+// the output-channel dim (logical 1) innermost with a run that 8 divides,
+// every other stride a multiple of 8 elements
+static bool direct_store_ok(const LView &L) {
+  if (!L.ok || L.lrank < 2) return false;
+  int pc = -1;
+  for (int p = 0; p < L.prank; p++) {
+    if (L.pshape[p] == 1) continue;
+    if (L.owner[p] == 1 && L.coef[p] == 1) pc = p;
+  }
+  if (pc < 0 || L.pstride[pc] != 1 || L.pshape[pc] % 8 || L.off[1] != 0) return false;
+  for (int p = 0; p < L.prank; p++)
+    if (p != pc && L.pshape[p] > 1 && L.pstride[p] % 8) return false;
+  return true;
+}
 alt_status make_epi(const OpEpilogue &e, EpiParams *p);
 
 // ---- optional per-CTA timestamps (env ALT_TC_DEBUG=1; developer tool)
@@ -858,15 +1026,14 @@ static cudaError_t launch_plan(const TcPlan &pl, void *y, cudaStream_t stream) {
   uint16_t *yy = static_cast<uint16_t *>(y);
   if (pl.cg == 2) {
     if (pl.BN == 128) return launch_tc<128, 8, 2>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
-    return launch_tc<256, 6, 2>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+    return launch_tc<256, 5, 2>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
   }
   if (pl.BN == 64) return launch_tc<64, 8, 1>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
   if (pl.BN == 128) {
     if (pl.stages == 4) return launch_tc<128, 4, 1>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
     return launch_tc<128, 6, 1>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
   }
-  if (pl.stages == 3) return launch_tc<256, 3, 1>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
-  return launch_tc<256, 4, 1>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+  return launch_tc<256, 3, 1>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
 }
 
 // common driver for conv and GEMM
@@ -906,6 +1073,7 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       k[i++] = cfg->block_n; k[i++] = cfg->tile_n; k[i++] = cfg->tile_h; k[i++] = cfg->tile_w;
       k[i++] = cfg->stages;
       k[i++] = cfg->cta_pair;
+      k[i++] = cfg->split_k;
     }
     int dev = 0;
     cudaGetDevice(&dev);
@@ -992,7 +1160,18 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       // unfold duplicates) and a >= 8-channel contiguous run, else the writer
       a.out_mode = 0;
       memset(&pl.ty, 0, sizeof(pl.ty));
-      if (!(P.yl->flags & (ALT_HAS_PAD | ALT_HAS_UNFOLD))) {
+      static const int store_mode = [] {
+        const char *e = getenv("ALT_TC_STORE");
+        // default TMA stores (measured faster than direct 16-byte stores)
+        return e && e[0] == 'd' ? 2 : (e && e[0] == 'g' ? 0 : 1);
+      }();
+      if (store_mode == 2 && !(P.yl->flags & (ALT_HAS_PAD | ALT_HAS_UNFOLD)) && P.K % 8 == 0 &&
+          (reinterpret_cast<uintptr_t>(P.y) & 15) == 0 && direct_store_ok(P.vy)) {
+        alt_status st2 = make_reader(P.yl, &a.yr);
+        if (st2 != ALT_OK) return st2;
+        a.out_mode = 2;
+      }
+      if (a.out_mode == 0 && store_mode != 0 && !(P.yl->flags & (ALT_HAS_PAD | ALT_HAS_UNFOLD))) {
         char why2[160];
         for (int so = 32; so >= 8 && !a.out_mode; so /= 2) {
           View vy;
@@ -1020,6 +1199,32 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       a.spi = 64 / sw;
       a.num_iters = (a.total_slabs + a.spi - 1) / a.spi;
       a.sw = sw;
+      // split-K when the output tiles leave SMs idle (small M x N, long K)
+      {
+        const int64_t units = a.num_tiles;
+        const int64_t slots = num_sms() / cg;
+        int64_t sk = 1;
+        if (cfg && cfg->split_k > 0) sk = cfg->split_k;
+        // auto: no split (measured: the serial partial reduction costs more
+        // than the idle SMs it recovers on the ResNet-50 set; tuned per layer)
+        sk = std::max<int64_t>(1, std::min<int64_t>(sk, a.num_iters));
+        a.splits = (int32_t)sk;
+        a.ws = nullptr;
+        a.cnt = nullptr;
+        if (sk > 1) {
+          if ((int64_t)a.num_tiles * sk > 0x7fffffff) { set_error("tc: too many tiles"); return ALT_E_UNSUPPORTED; }
+          // per-plan workspace (lives as long as the process: captured graphs
+          // may replay the plan after the cache forgets it)
+          const size_t wsb = (size_t)units * cg * sk * 128 * BN * sizeof(float);
+          if (cudaMalloc(&a.ws, wsb) != cudaSuccess || cudaMalloc(&a.cnt, (size_t)units * cg * 4) != cudaSuccess ||
+              cudaMemset(a.cnt, 0, (size_t)units * cg * 4) != cudaSuccess) {
+            cudaGetLastError();
+            set_error("tc: split-K workspace: out of memory");
+            return ALT_E_NOMEM;
+          }
+          a.num_tiles = (int32_t)(units * sk);
+        }
+      }
       alt_status st;
       if ((st = make_epi(P.epi, &a.epi)) != ALT_OK) return st;
       // the kernel always applies scale * acc + bias: absent ones become the
@@ -1035,9 +1240,8 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       pl.grid = (int)std::min<int64_t>((int64_t)a.num_tiles * cg, num_sms() / cg * cg);
       pl.BN = BN;
       pl.cg = cg;
-      pl.stages = cg == 2 ? (BN == 128 ? 8 : 6) : (BN == 64 ? 8 : (BN == 128 ? 6 : 4));
+      pl.stages = cg == 2 ? (BN == 128 ? 8 : 5) : (BN == 64 ? 8 : (BN == 128 ? 6 : 3));
       if (cfg && BN == 128 && cfg->stages == 4) pl.stages = 4;
-      if (cfg && BN == 256 && cfg->stages == 3) pl.stages = 3;
       alt_kernel_cfg u{};
       u.path = ALT_PATH_TC;
       u.block_m = 128 * cg;
@@ -1046,6 +1250,7 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       u.block_k = 64;
       u.stages = pl.stages;
       u.tile_n = c.tn; u.tile_h = c.th; u.tile_w = c.tw;
+      u.split_k = a.splits;
       pl.used = u;
       cudaError_t e = launch_plan(pl, P.y, stream);
       count_launch();

@@ -1,0 +1,6 @@
+#!/bin/bash
+make -C paper_conf_eurosys_xuxpwwwdxcwc23_b200 -j8 >/dev/null 2>&1
+timeout 600 python -m pytest tests/test_gpu_conv.py -q -x -k "split" 2>&1 | tail -3
+timeout 600 python scripts/exp_split.py l4.3x3,l4.3x3s2,l4.1x1c,l4.1x1b,l4.1x1a,l3.3x3,l3.1x1c,l3.1x1b,l2.1x1b,l1.1x1b 2>&1
+timeout 300 python bench.py --steps 20 --warmup 3 --no-cpu-baseline 2>&1 | tail -1 | python -c "
+import json,sys; d=json.loads(sys.stdin.read()); print(d['value'], d['ms_per_step']); [print(l) for l in d['per_layer']]"

@@ -222,3 +222,40 @@ def test_tc_gemm(case):
     name, ap, bp, cp = case
     run_gemm("tcg" + name, 384, 192, 256, ap, bp, cp, torch.bfloat16, epi=True, cfg={"path": alt.PATH_TC},
              expect_path=alt.PATH_TC)
+
+
+# ------------------------------------------------------------- split-K --
+@pytest.mark.parametrize("sk,bn,pair", [(2, 256, 1), (3, 128, 1), (5, 64, 2), (0, 256, 0)])
+def test_tc_split_k(sk, bn, pair):
+    """split-K (alt_kernel_cfg.split_k; 0 = auto = none): partial tiles summed in split order by the last CTA, fused
+    epilogue with residual, parity with the oracle."""
+    cfg = {"path": alt.PATH_TC, "split_k": sk, "block_n": bn, "cta_pair": pair}
+    xp, wp, yp = LY.nchwxc(256, 64), LY.kcrs_yk_xc(512, 256, 256, 64), LY.nchwxc(512, 64)
+    _, plan = run_conv("tcsk", 2, 256, 7, 7, 512, 3, 3, 1, 1, xp, wp, yp, torch.bfloat16, epi=True,
+                       res_p=LY.nchwxc(512, 64), act=1, cfg=cfg, expect_path=alt.PATH_TC)
+    assert plan["split_k"] == (sk or 1)  # auto: no split (DESIGN.md)
+
+
+def test_tc_split_k_deterministic():
+    """the reduction order is fixed: repeated launches agree bit for bit"""
+    p = alt.conv_params(2, 256, 7, 7, 512, 3, 3, 1, 1)
+    x = synth.activations("skdx", (2, 256, 7, 7))
+    w = synth.weights("skdw", (512, 256, 3, 3))
+    xp, wp, yp = LY.nchwxc(256, 64), LY.kcrs_yk_xc(512, 256, 256, 64), LY.nchwxc(512, 64)
+    _, _, xd = make_operand("skdx", xp, x, torch.bfloat16)
+    _, _, wd = make_operand("skdw", wp, w, torch.bfloat16)
+    Lx, Lw, Ly = alt.Layout(x.shape, xp), alt.Layout(w.shape, wp), alt.Layout((2, 512, 7, 7), yp)
+    outs = []
+    for _ in range(4):
+        y = torch.zeros(Ly.phys_shape, dtype=torch.bfloat16, device="cuda")
+        alt.conv2d(p, Lx, xd, Lw, wd, Ly, y, cfg={"path": alt.PATH_TC, "split_k": 7})
+        outs.append(y)
+    torch.cuda.synchronize()
+    for y in outs[1:]:
+        assert np.array_equal(words(y), words(outs[0]))
+
+
+def test_tc_gemm_split_k():
+    _, plan = run_gemm("gsk", 200, 256, 2048, [], LY.transpose2(), [], torch.bfloat16, epi=True,
+                       cfg={"path": alt.PATH_TC, "split_k": 4}, expect_path=alt.PATH_TC)
+    assert plan["split_k"] == 4
