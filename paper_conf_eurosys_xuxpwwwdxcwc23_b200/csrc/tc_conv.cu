@@ -49,6 +49,7 @@ enum Var { V_N0 = 0, V_PT, V_PR, V_QT, V_QR, V_GT, V_GR, V_R, V_S, V_ONE, NVAR }
 struct OperandMap {
   int32_t coef[5][NVAR];
   int32_t divp, divq, divg;
+  FastDiv fp, fq, fg;  // the same divisors as multiply-shift (no integer division on the device)
   int32_t slab_bytes;
   int32_t oob0;  // dim-0 coordinate that makes a box all zeros
   int32_t sw;    // slab width (channels)
@@ -63,6 +64,7 @@ struct TcArgs {
   int32_t mt_h, mt_w;    // # tiles along h, w (n is the slowest)
   int32_t num_n_tiles, num_tiles;
   int32_t S, Gc;
+  FastDiv f_nnt, f_mtw, f_mth, f_spl, f_Gc, f_S;  // num_n_tiles, mt_w, mt_h, splits, Gc, S
   int32_t total_slabs, spi, num_iters;
   int32_t sw;
   Writer yw;
@@ -79,6 +81,11 @@ struct TcArgs {
 constexpr int kThreads = 320;  // producer, MMA, 8 epilogue warps
 constexpr int kStageBytesA = 128 * 64 * 2;
 constexpr int kOutStage = 128 * 64 * 2;  // one 64-column bf16 chunk of the tile
+
+// accumulator buffers in TMEM (512 columns): the MMA of tile i + NACC - 1
+// may run while the epilogue drains tile i
+template <int BN>
+struct Nacc { static constexpr int value = BN >= 256 ? 2 : 4; };
 
 template <int BN, int STAGES, int CG = 1>
 struct TcSmem {
@@ -189,10 +196,12 @@ struct TileCoord { int n0, p0, q0, k0; };
 // work unit `tile` -> this CTA's 128-row M tile and the unit's N tile; with a
 // CTA pair (CG = 2) a unit is two consecutive M tiles, one per CTA rank
 __device__ __forceinline__ TileCoord tile_coord(const TcArgs &a, int tile, int BN, int CG, int rank) {
-  const int mt = (tile / a.num_n_tiles) * CG + rank, nt = tile % a.num_n_tiles;
-  const int tw_i = mt % a.mt_w;
-  const int th_i = (mt / a.mt_w) % a.mt_h;
-  const int tn_i = mt / (a.mt_w * a.mt_h);
+  const int mq = (int)a.f_nnt.div((uint32_t)tile);
+  const int mt = mq * CG + rank, nt = tile - mq * a.num_n_tiles;
+  const int mw = (int)a.f_mtw.div((uint32_t)mt);
+  const int tw_i = mt - mw * a.mt_w;
+  const int tn_i = (int)a.f_mth.div((uint32_t)mw);
+  const int th_i = mw - tn_i * a.mt_h;
   return {tn_i * a.tile_n, th_i * a.tile_h, tw_i * a.tile_w, nt * BN};
 }
 
@@ -210,13 +219,13 @@ __global__ void __launch_bounds__(kThreads, 1)
   unsigned char *sA = smem;
   unsigned char *sB = smem + STAGES * kStageBytesA;
   unsigned char *sOut = smem + L::kOut;
-  float *sScale = reinterpret_cast<float *>(smem + L::kSB);
-  float *sBias = sScale + BN;
+  const uint32_t sSB = sm100::smem_u32(smem + L::kSB);  // scale [BN] then bias [BN] (fp32)
   uint64_t *full = reinterpret_cast<uint64_t *>(smem + L::kBar);
   uint64_t *empty = full + STAGES;
   uint64_t *tfull = empty + STAGES;   // [2]
-  uint64_t *tempty = tfull + 2;       // [2]
-  uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(tempty + 2);
+  constexpr int NACC = Nacc<BN>::value;
+  uint64_t *tempty = tfull + NACC;    // [NACC]
+  uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(tempty + NACC);
   volatile int32_t *last_flag = reinterpret_cast<volatile int32_t *>(tmem_slot + 1);
 
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
@@ -229,18 +238,22 @@ __global__ void __launch_bounds__(kThreads, 1)
       mbar_init(&full[s], 1);
       mbar_init(&empty[s], 1);
     }
-    for (int s = 0; s < 2; s++) {
+    for (int s = 0; s < NACC; s++) {
       mbar_init(&tfull[s], 1);
       mbar_init(&tempty[s], 8 * CG);  // every epilogue warp of the pair
     }
     fence_mbar_init();
   }
-  if (warp == 1) tmem_alloc<2 * BN, CG>(tmem_slot);
+  if (warp == 1) tmem_alloc<NACC * BN, CG>(tmem_slot);
   tc_fence_before();
   __syncthreads();
   if constexpr (CG == 2) cluster_sync();  // peer barriers initialised before any remote arrive
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
+  // programmatic dependent launch: the prologue above overlapped the previous
+  // kernel's tail; no global memory is touched before it has completed
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
   if (threadIdx.x == 0) { DBG(1); }
 
   if (warp == 0) {
@@ -254,21 +267,24 @@ __global__ void __launch_bounds__(kThreads, 1)
     unsigned char *sbase = isA ? sA : sB;
     const int sbytes = isA ? kStageBytesA : L::kB;
     const bool active = j < a.spi;
-    int it = 0;
-    for (int tile = unit0; tile < a.num_tiles; tile += unit_step) {
-      const int mn = tile / a.splits, sp = tile - mn * a.splits;
+    int it = 0, ti = 0;
+    for (int tile = unit0; tile < a.num_tiles; tile += unit_step, ti++) {
+      const int mn = (int)a.f_spl.div((uint32_t)tile), sp = tile - mn * a.splits;
       const TileCoord tc = tile_coord(a, mn, BN, CG, rank);
-      const int k_begin = sp * a.num_iters / a.splits, k_end = (sp + 1) * a.num_iters / a.splits;
+      const int k_begin = a.splits == 1 ? 0 : sp * a.num_iters / a.splits;
+      const int k_end = a.splits == 1 ? a.num_iters : (sp + 1) * a.num_iters / a.splits;
       int32_t v[NVAR];
       // B rows of this CTA: its 1/CG share of the unit's BN output channels
       const int pp = isA ? tc.p0 : 0, qq = isA ? tc.q0 : tc.k0 + rank * (BN / CG);
       v[V_N0] = isA ? tc.n0 : 0;
-      v[V_PT] = pp / om.divp; v[V_PR] = pp % om.divp;
-      v[V_QT] = qq / om.divq; v[V_QR] = qq % om.divq;
+      v[V_PT] = (int)om.fp.div((uint32_t)pp); v[V_PR] = pp - v[V_PT] * om.divp;
+      v[V_QT] = (int)om.fq.div((uint32_t)qq); v[V_QR] = qq - v[V_QT] * om.divq;
       v[V_ONE] = 1;
       for (int kit = k_begin; kit < k_end; kit++, it++) {
         const int stage = it % STAGES, round = it / STAGES;
+        if (lane == 0 && ti == ALT_DBG_TILE && kit == k_begin) { DBG(24); }
         if (round > 0) mbar_wait(&empty[stage], (round - 1) & 1);
+        if (lane == 0 && ti == ALT_DBG_TILE && kit == k_begin) { DBG(25); }
         // the leader's full barrier counts the bytes of both CTAs of a pair
         if (lane == 0 && rank == 0) mbar_expect_tx(&full[stage], CG * (kStageBytesA + L::kB));
         __syncwarp();
@@ -276,9 +292,9 @@ __global__ void __launch_bounds__(kThreads, 1)
           const int slab = kit * a.spi + j;
           const bool valid = slab < a.total_slabs;
           const int sl = valid ? slab : 0;
-          const int tap = sl / a.Gc, g = sl % a.Gc;
-          v[V_R] = tap / a.S; v[V_S] = tap % a.S;
-          v[V_GT] = g / om.divg; v[V_GR] = g % om.divg;
+          const int tap = (int)a.f_Gc.div((uint32_t)sl), g = sl - tap * a.Gc;
+          v[V_R] = (int)a.f_S.div((uint32_t)tap); v[V_S] = tap - v[V_R] * a.S;
+          v[V_GT] = (int)om.fg.div((uint32_t)g); v[V_GR] = g - v[V_GT] * om.divg;
           int32_t c[5];
           coords(om, v, c);
           if (!valid) c[0] = om.oob0;
@@ -303,15 +319,19 @@ __global__ void __launch_bounds__(kThreads, 1)
       const uint32_t lboA = sw == 8 ? aS : 16u, lboB = sw == 8 ? bS : 16u;
       int it = 0, i = 0;
       for (int tile = unit0; tile < a.num_tiles; tile += unit_step, i++) {
-        const int acc = i & 1, use = i >> 1;
+        const int acc = i % NACC, use = i / NACC;
+        if (i == ALT_DBG_TILE) { DBG(26); }
         if (use > 0) mbar_wait(&tempty[acc], (use - 1) & 1);
+        if (i == ALT_DBG_TILE) { DBG(27); }
         tc_fence_after();
         const uint32_t d = tmem + (uint32_t)(acc * BN);
-        const int sp = tile % a.splits;
-        const int k_begin = sp * a.num_iters / a.splits, k_end = (sp + 1) * a.num_iters / a.splits;
+        const int sp = tile - (int)a.f_spl.div((uint32_t)tile) * a.splits;
+        const int k_begin = a.splits == 1 ? 0 : sp * a.num_iters / a.splits;
+        const int k_end = a.splits == 1 ? a.num_iters : (sp + 1) * a.num_iters / a.splits;
         for (int kit = k_begin; kit < k_end; kit++, it++) {
           const int stage = it % STAGES, round = it / STAGES;
           mbar_wait(&full[stage], round & 1);
+          if (i == ALT_DBG_TILE && kit == k_begin) { DBG(28); }
           tc_fence_after();
           const uint32_t baseA = smem_u32(sA + stage * kStageBytesA), baseB = smem_u32(sB + stage * L::kB);
 #pragma unroll
@@ -330,6 +350,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
         if constexpr (CG == 2) mma_commit_2cta(&tfull[acc], 0x3);
         else mma_commit(&tfull[acc]);
+        if (i == ALT_DBG_TILE) { DBG(29); }
         if (i == 0) { DBG(3); }
       }
     }
@@ -346,14 +367,12 @@ __global__ void __launch_bounds__(kThreads, 1)
     const int pitch = sw_o * 2;            // bytes per row in a staging slab
     const int swz = pitch == 128 ? 3 : (pitch == 64 ? 2 : (pitch == 32 ? 1 : 0));
     // this thread's four 16-byte pieces inside a (swizzled) staging buffer
-    uint32_t soff[4];
-#pragma unroll
-    for (int c = 0; c < 4; c++) {
+    auto soff = [&](int c) -> uint32_t {
       const int ch = c * 8;
-      uint32_t off = (uint32_t)(lane * pitch + (ch % sw_o) * 2);
+      uint32_t off = (uint32_t)(lane * pitch + (ch & (sw_o - 1)) * 2);
       off ^= ((off >> 7) & ((1u << swz) - 1u)) << 4;
-      soff[c] = (uint32_t)((ch / sw_o) * 32 * pitch) + off;
-    }
+      return (uint32_t)((ch / sw_o) * 32 * pitch) + off;
+    };
     const uint32_t wbuf = smem_u32(sOut) + (uint32_t)((warp - 2) * 4096);
     const int act = a.epi.act;
     // scale / bias of a tile's BN channels, one per thread, fetched one tile
@@ -361,40 +380,36 @@ __global__ void __launch_bounds__(kThreads, 1)
     auto fetch_sb = [&](int tile, float &fs, float &fb) {
       fs = 1.f; fb = 0.f;
       if (tile < a.num_tiles && et < BN) {
-        const int k = min(tile_coord(a, tile / a.splits, BN, CG, rank).k0 + et, a.K - 1);
+        const int k = min(tile_coord(a, (int)a.f_spl.div((uint32_t)tile), BN, CG, rank).k0 + et, a.K - 1);
         fs = __ldg(a.epi.scale + k);
         fb = __ldg(a.epi.bias + k);
       }
     };
     float pf_s, pf_b;
     fetch_sb(unit0, pf_s, pf_b);
+    // this thread's row and its warp's 32-row sub-box origin inside a tile
+    // (tile rows are (n, h, w) with w fastest): divisions once per thread
+    const int rn = row / tn, rp = (row / a.tile_w) % a.tile_h, rq = row % a.tile_w;
+    const int r0 = wq * 32;
+    const int sn0 = r0 / tn, sp0 = (r0 / a.tile_w) % a.tile_h, sq0 = r0 % a.tile_w;
     int i = 0;
     for (int tile = unit0; tile < a.num_tiles; tile += unit_step, i++) {
-      const int acc = i & 1, use = i >> 1;
-      const int mn = tile / a.splits, ksp = tile - mn * a.splits;
+      const int acc = i % NACC, use = i / NACC;
+      const int mn = (int)a.f_spl.div((uint32_t)tile), ksp = tile - mn * a.splits;
       const TileCoord tc = tile_coord(a, mn, BN, CG, rank);
       named_bar(2, 256);  // every epilogue warp is done with the previous tile's values
-      if (et < BN) { sScale[et] = pf_s; sBias[et] = pf_b; }
+      if (et < BN) {  // explicit shared-space stores (the aligned base is a generic pointer)
+        asm volatile("st.shared.f32 [%0], %1;" ::"r"(sSB + 4u * et), "f"(pf_s) : "memory");
+        asm volatile("st.shared.f32 [%0], %1;" ::"r"(sSB + 4u * (BN + et)), "f"(pf_b) : "memory");
+      }
       named_bar(2, 256);
+      if (et == 0 && i == ALT_DBG_TILE) { DBG(30); }
       fetch_sb(tile + unit_step, pf_s, pf_b);
-      const int n = tc.n0 + row / tn, p = tc.p0 + (row / a.tile_w) % a.tile_h, q = tc.q0 + row % a.tile_w;
+      const int n = tc.n0 + rn, p = tc.p0 + rp, q = tc.q0 + rq;
       const bool vrow = n < a.N && p < a.Ho && q < a.Wo;
       int64_t yrow = 0;  // out_mode 2: offset of this thread's output row
       if (a.out_mode == 2 && vrow)
         yrow = a.is_conv ? __ldg(a.yr.rd[0] + n) + __ldg(a.yr.rd[2] + p) + __ldg(a.yr.rd[3] + q) : __ldg(a.yr.rd[0] + q);
-      // TMA-store coordinates of this warp's 32-row sub-box, less the
-      // channel-slab terms (added per store)
-      int32_t cbase[5];
-      if (a.out_mode == 1 && lane == 0) {
-        const int r0 = wq * 32;
-        const int sn = tc.n0 + r0 / tn, sp = tc.p0 + (r0 / a.tile_w) % a.tile_h, sq = tc.q0 + r0 % a.tile_w;
-        int32_t vo[NVAR];
-        vo[V_N0] = sn;
-        vo[V_PT] = sp / a.O.divp; vo[V_PR] = sp % a.O.divp;
-        vo[V_QT] = sq / a.O.divq; vo[V_QR] = sq % a.O.divq;
-        vo[V_GT] = 0; vo[V_GR] = 0; vo[V_R] = 0; vo[V_S] = 0; vo[V_ONE] = 1;
-        coords(a.O, vo, cbase);
-      }
       mbar_wait(&tfull[acc], use & 1);
       if (et == 0 && i == ALT_DBG_TILE) { DBG(2); }
       tc_fence_after();
@@ -460,11 +475,15 @@ __global__ void __launch_bounds__(kThreads, 1)
           }
           float v[32];
           {
-            const float4 *s4 = reinterpret_cast<const float4 *>(sScale + cb);
-            const float4 *b4 = reinterpret_cast<const float4 *>(sBias + cb);
 #pragma unroll
             for (int j = 0; j < 8; j++) {
-              const float4 x = s4[j], y = b4[j];
+              float4 x, y;
+              asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];"
+                           : "=f"(x.x), "=f"(x.y), "=f"(x.z), "=f"(x.w)
+                           : "r"(sSB + 4u * (cb + 4 * j)));
+              asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];"
+                           : "=f"(y.x), "=f"(y.y), "=f"(y.z), "=f"(y.w)
+                           : "r"(sSB + 4u * (BN + cb + 4 * j)));
               v[4 * j + 0] = fmaf(__uint_as_float(raw[4 * j + 0]), x.x, y.x);
               v[4 * j + 1] = fmaf(__uint_as_float(raw[4 * j + 1]), x.y, y.y);
               v[4 * j + 2] = fmaf(__uint_as_float(raw[4 * j + 2]), x.z, y.z);
@@ -527,18 +546,29 @@ __global__ void __launch_bounds__(kThreads, 1)
             __syncwarp();
 #pragma unroll
             for (int c = 0; c < 4; c++)
-              asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(wbuf + buf + soff[c]), "r"(pk[4 * c]),
+              asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(wbuf + buf + soff(c)), "r"(pk[4 * c]),
                            "r"(pk[4 * c + 1]), "r"(pk[4 * c + 2]), "r"(pk[4 * c + 3])
                            : "memory");
             if (et == 0 && i == ALT_DBG_TILE) { DBG(10 + (c0 >> 6) * 4); }
             fence_async_smem();
             __syncwarp();
             if (lane == 0) {
+              // TMA-store coordinates of this warp's 32-row sub-box
+              int32_t cbase[5];
+              {
+                const int sn = tc.n0 + sn0, sp = tc.p0 + sp0, sq = tc.q0 + sq0;
+                int32_t vo[NVAR];
+                vo[V_N0] = sn;
+                vo[V_PT] = (int)a.O.fp.div((uint32_t)sp); vo[V_PR] = sp - vo[V_PT] * a.O.divp;
+                vo[V_QT] = (int)a.O.fq.div((uint32_t)sq); vo[V_QR] = sq - vo[V_QT] * a.O.divq;
+                vo[V_GT] = 0; vo[V_GR] = 0; vo[V_R] = 0; vo[V_S] = 0; vo[V_ONE] = 1;
+                coords(a.O, vo, cbase);
+              }
               const int nslab = 32 / sw_o;
               for (int j = 0; j < nslab; j++) {
                 if (kb + j * sw_o >= a.K) break;  // channels past K: nothing to store
                 const int g = kb / sw_o + j;
-                const int gt = g / a.O.divg, gr = g - gt * a.O.divg;
+                const int gt = (int)a.O.fg.div((uint32_t)g), gr = g - gt * a.O.divg;
                 int32_t co[5];
 #pragma unroll
                 for (int d = 0; d < 5; d++) co[d] = cbase[d] + a.O.coef[d][V_GT] * gt + a.O.coef[d][V_GR] * gr;
@@ -559,6 +589,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       };
       if (a.out_mode != 0 && !a.epi.residual && !wsl) chunk_loop(std::true_type{});
       else chunk_loop(std::false_type{});
+      if (et == 0 && i == ALT_DBG_TILE) { DBG(31); }
     }
     if (et == 0) { DBG(5); }
     if (lane == 0 && a.out_mode == 1) bulk_wait0();
@@ -566,7 +597,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   tc_fence_before();
   __syncthreads();
   if constexpr (CG == 2) cluster_sync();  // the pair's MMAs and epilogues are done
-  if (warp == 1) tmem_dealloc<2 * BN, CG>(tmem);
+  if (warp == 1) tmem_dealloc<NACC * BN, CG>(tmem);
   if (threadIdx.x == 32) { DBG(6); }
 }
 
@@ -880,6 +911,9 @@ static bool encode_view(const View &v, const void *base, int esize, int sw, CUte
   om->divp = v.divp;
   om->divq = v.divq;
   om->divg = v.divg;
+  om->fp = FastDiv((uint32_t)v.divp);
+  om->fq = FastDiv((uint32_t)v.divq);
+  om->fg = FastDiv((uint32_t)v.divg);
   int64_t rows = 1;
   for (int i = 1; i < v.rank; i++) rows *= (int64_t)((v.d[i].box + v.d[i].estride - 1) / v.d[i].estride);
   om->slab_bytes = (int32_t)(rows * row_bytes);
@@ -979,23 +1013,32 @@ static cudaError_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const
     if (CG == 2) cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 0);
     attr_set = true;
   }
-  if constexpr (CG == 1) {
-    kern<<<grid, kThreads, smem, s>>>(ta, tb, ty, a, y);
-  } else {
-    cudaLaunchConfig_t lc{};
-    lc.gridDim = dim3((unsigned)grid);
-    lc.blockDim = dim3(kThreads);
-    lc.dynamicSmemBytes = smem;
-    lc.stream = s;
-    cudaLaunchAttribute at[1];
-    at[0].id = cudaLaunchAttributeClusterDimension;
-    at[0].val.clusterDim.x = 2;
-    at[0].val.clusterDim.y = 1;
-    at[0].val.clusterDim.z = 1;
-    lc.attrs = at;
-    lc.numAttrs = 1;
-    cudaLaunchKernelEx(&lc, kern, ta, tb, ty, a, y);
+  static const bool pdl = [] {
+    const char *e = getenv("ALT_PDL");
+    return !(e && e[0] == '0');
+  }();
+  cudaLaunchConfig_t lc{};
+  lc.gridDim = dim3((unsigned)grid);
+  lc.blockDim = dim3(kThreads);
+  lc.dynamicSmemBytes = smem;
+  lc.stream = s;
+  cudaLaunchAttribute at[2];
+  int na = 0;
+  if (CG == 2) {
+    at[na].id = cudaLaunchAttributeClusterDimension;
+    at[na].val.clusterDim.x = 2;
+    at[na].val.clusterDim.y = 1;
+    at[na].val.clusterDim.z = 1;
+    na++;
   }
+  if (pdl) {  // may start while the previous kernel in the stream drains
+    at[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[na].val.programmaticStreamSerializationAllowed = 1;
+    na++;
+  }
+  lc.attrs = at;
+  lc.numAttrs = na;
+  cudaLaunchKernelEx(&lc, kern, ta, tb, ty, a, y);
   return cudaGetLastError();
 }
 
@@ -1225,6 +1268,12 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
           a.num_tiles = (int32_t)(units * sk);
         }
       }
+      a.f_nnt = FastDiv((uint32_t)a.num_n_tiles);
+      a.f_mtw = FastDiv((uint32_t)a.mt_w);
+      a.f_mth = FastDiv((uint32_t)a.mt_h);
+      a.f_spl = FastDiv((uint32_t)a.splits);
+      a.f_Gc = FastDiv((uint32_t)a.Gc);
+      a.f_S = FastDiv((uint32_t)a.S);
       alt_status st;
       if ((st = make_epi(P.epi, &a.epi)) != ALT_OK) return st;
       // the kernel always applies scale * acc + bias: absent ones become the

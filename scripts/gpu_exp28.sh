@@ -1,0 +1,9 @@
+#!/bin/bash
+make -C paper_conf_eurosys_xuxpwwwdxcwc23_b200 -j8 >/dev/null 2>&1
+timeout 900 python -m pytest tests/ -m gpu -q -x 2>&1 | tail -3
+EPI_K=64,256 timeout 300 python scripts/exp_epi.py 2>&1
+for p in 1 0; do
+echo "== PDL $p"
+ALT_PDL=$p timeout 300 python bench.py --steps 20 --warmup 3 --no-cpu-baseline 2>&1 | tail -1 | python -c "
+import json,sys; d=json.loads(sys.stdin.read()); print(d['value'], d['ms_per_step'], d['roofline']['achieved']); [print(l['layer'], l['us'], l['tflops']) for l in d['per_layer']]"
+done

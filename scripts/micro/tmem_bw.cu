@@ -33,6 +33,18 @@ __global__ void k(int iters, unsigned long long *out, uint32_t *sink) {
       tmem_ld_wait();
 #pragma unroll
       for (int c = 0; c < 4; c++) x ^= r[c][lane];
+    } else if (MODE == 3 || MODE == 4) {
+      // MODE 3: load, then independent ALU work, then use; MODE 4: ALU work only
+      uint32_t r[32];
+      if (MODE == 3) tmem_ld_32x32b_x32(base + colbase + (it & 3) * 32, r);
+      float f = __uint_as_float(x) + 1.0f;
+#pragma unroll
+      for (int k = 0; k < 64; k++) f = fmaf(f, 1.0001f, 0.5f);
+      x ^= __float_as_uint(f);
+      if (MODE == 3) {
+        tmem_ld_wait();
+        x ^= r[lane] + r[(lane + 7) & 31];
+      }
     } else {
       uint32_t r[64];
       tmem_ld_32x32b_x64(base + colbase + (it & 1) * 64, r);
@@ -55,14 +67,15 @@ int main() {
   cudaMalloc(&d, 148 * 8);
   cudaMalloc(&s, 4);
   const int iters = 4096;
-  for (int mode = 0; mode < 3; mode++)
+  for (int mode = 0; mode < 5; mode++)
     for (int warps = 4; warps <= 8; warps += 4) {
-      void (*kern)(int, unsigned long long *, uint32_t *) = mode == 0 ? k<0> : (mode == 1 ? k<1> : k<2>);
+      void (*kern)(int, unsigned long long *, uint32_t *) =
+          mode == 0 ? k<0> : (mode == 1 ? k<1> : (mode == 2 ? k<2> : (mode == 3 ? k<3> : k<4>)));
       kern<<<148, warps * 32>>>(iters, d, s);
       cudaError_t e = cudaDeviceSynchronize();
       unsigned long long h[148];
       cudaMemcpy(h, d, sizeof(h), cudaMemcpyDeviceToHost);
-      const double bytes_per_iter = (mode == 0 ? 4096.0 : (mode == 1 ? 16384.0 : 8192.0)) * warps;
+      const double bytes_per_iter = (mode == 0 || mode == 3 ? 4096.0 : (mode == 1 ? 16384.0 : (mode == 2 ? 8192.0 : 0.0))) * warps;
       printf("mode %d warps %d: %s  %.1f cycles/iter  %.1f B/clk per SM\n", mode, warps, cudaGetErrorString(e),
              (double)h[0] / iters, bytes_per_iter * iters / h[0]);
     }
