@@ -289,24 +289,32 @@ def main():
           for _ in range(args.steps)]
     plans = []
     # The K timed steps are captured once into a CUDA graph (launch plans are
-    # cached by the library, so capture records only kernel + event nodes) and
-    # replayed: the timed region is pure device work.
-    graph = None
+    # cached by the library, so capture records only kernel nodes) and
+    # replayed: the timed region is pure device work.  A second graph with an
+    # event pair around every layer gives the per-layer breakdown (event nodes
+    # between kernels cost the programmatic-launch overlap, so that pass is
+    # not the headline).
+    def capture(with_events):
+        g = torch.cuda.CUDAGraph()
+        cap = torch.cuda.Stream()
+        cap.wait_stream(stream)
+        with torch.cuda.stream(cap):
+            with torch.cuda.graph(g, stream=cap):
+                for k in range(args.steps):
+                    S.step(ev[k] if with_events else None)
+        stream.wait_stream(cap)
+        return g
+
+    graph = graph_ev = None
     launches0 = alt.launch_count()
     if not args.eager:
         try:
-            graph = torch.cuda.CUDAGraph()
-            cap = torch.cuda.Stream()
-            cap.wait_stream(stream)
-            with torch.cuda.stream(cap):
-                with torch.cuda.graph(graph, stream=cap):
-                    for k in range(args.steps):
-                        S.step(ev[k])
-            stream.wait_stream(cap)
+            graph = capture(False)
+            launches = alt.launch_count() - launches0
+            graph_ev = capture(True)
         except Exception as e:  # fall back to eager launches
             print(f"graph capture failed ({e}); timing eager launches", file=sys.stderr)
-            graph = None
-    launches = alt.launch_count() - launches0
+            graph = graph_ev = None
     with Clocks(local) as clk:
         barrier(ws)
         torch.cuda.synchronize()
@@ -318,7 +326,7 @@ def main():
             graph.replay()
         else:
             for k in range(args.steps):
-                S.step(ev[k])
+                S.step()
         t1.record(stream)
         torch.cuda.synchronize()
         barrier(ws)
@@ -326,6 +334,13 @@ def main():
             launches = alt.launch_count() - launches0
     ms = t0.elapsed_time(t1) / args.steps
     ms = max_over_ranks(ms, ws)
+    # per-layer pass
+    if graph_ev is not None:
+        graph_ev.replay()
+    else:
+        for k in range(args.steps):
+            S.step(ev[k])
+    torch.cuda.synchronize()
     conv_ms = sum(ev[k][i][0].elapsed_time(ev[k][i][1]) for k in range(args.steps) for i in range(nL)) / args.steps
     for l in S.layers:
         alt.conv2d(l["p"], l["lx"], l["x"], l["lw"], l["w"], l["ly"], l["y"], scale=l["sc"], bias=l["bi"],

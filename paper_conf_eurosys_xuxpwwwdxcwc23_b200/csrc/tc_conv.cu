@@ -87,6 +87,16 @@ constexpr int kOutStage = 128 * 64 * 2;  // one 64-column bf16 chunk of the tile
 template <int BN>
 struct Nacc { static constexpr int value = BN >= 256 ? 2 : 4; };
 
+// Reduction-slab coordinate table: for every slab (filter tap x channel
+// slab) of the reduction, the part of the A / B box coordinates that depends
+// on the slab (5 ints each, A at [0..4], B at [8..12] of a 64-byte row).
+// Built once per CTA in the prologue, so the producer's per-stage work is
+// one shared load + 5 adds per box instead of the divisions and the 5 x 10
+// coefficient products of coords() (the single producer thread's issue
+// latency bounds the stage rate).
+constexpr int kTabSlabs = 288;
+constexpr int kTabBytes = kTabSlabs * 64;
+
 template <int BN, int STAGES, int CG = 1>
 struct TcSmem {
   static constexpr int kB = (BN / CG) * 64 * 2;  // this CTA's share of the B tile
@@ -94,7 +104,8 @@ struct TcSmem {
   static constexpr int kOut = kRing;                       // 2 staging buffers for TMA stores
   static constexpr int kSB = kOut + 2 * kOutStage;         // scale / bias of the tile (2 x BN floats)
   static constexpr int kBar = kSB + 2 * BN * 4;             // barriers
-  static constexpr int kBytes = kBar + 256 + 1008 /*1024-B alignment slack*/;
+  static constexpr int kTab = kBar + 256;                   // slab coordinate table
+  static constexpr int kBytes = kTab + kTabBytes + 1008 /*1024-B alignment slack*/;
 };
 
 __device__ __forceinline__ uint64_t gtimer() {
@@ -245,6 +256,28 @@ __global__ void __launch_bounds__(kThreads, 1)
     fence_mbar_init();
   }
   if (warp == 1) tmem_alloc<NACC * BN, CG>(tmem_slot);
+  // slab table (see kTabSlabs): slab -> (tap r, s; channel slab g = (gt, gr))
+  int32_t *tab = reinterpret_cast<int32_t *>(smem + L::kTab);
+  const int padded_slabs = a.num_iters * a.spi;
+  const bool use_tab = padded_slabs <= kTabSlabs;
+  if (use_tab) {
+    for (int sl = threadIdx.x; sl < padded_slabs; sl += kThreads) {
+      const bool valid = sl < a.total_slabs;
+      const int s0 = valid ? sl : 0;
+      const int tap = (int)a.f_Gc.div((uint32_t)s0), g = s0 - tap * a.Gc;
+      const int r = (int)a.f_S.div((uint32_t)tap), sx = tap - r * a.S;
+#pragma unroll
+      for (int o = 0; o < 2; o++) {
+        const OperandMap &om = o == 0 ? a.A : a.B;
+        const int gt = (int)om.fg.div((uint32_t)g), gr = g - gt * om.divg;
+#pragma unroll
+        for (int d = 0; d < 5; d++)
+          tab[sl * 16 + o * 8 + d] = om.coef[d][V_R] * r + om.coef[d][V_S] * sx + om.coef[d][V_GT] * gt +
+                                     om.coef[d][V_GR] * gr;
+        if (!valid) tab[sl * 16 + o * 8] = om.oob0;  // all-zero box (dim 0 has no tile term)
+      }
+    }
+  }
   tc_fence_before();
   __syncthreads();
   if constexpr (CG == 2) cluster_sync();  // peer barriers initialised before any remote arrive
@@ -280,6 +313,40 @@ __global__ void __launch_bounds__(kThreads, 1)
       v[V_PT] = (int)om.fp.div((uint32_t)pp); v[V_PR] = pp - v[V_PT] * om.divp;
       v[V_QT] = (int)om.fq.div((uint32_t)qq); v[V_QR] = qq - v[V_QT] * om.divq;
       v[V_ONE] = 1;
+      if (use_tab) {
+        // the tile's part of the box coordinates, once per tile
+        int32_t base[5];
+        {
+          int32_t vt[NVAR];
+#pragma unroll
+          for (int k = 0; k < NVAR; k++) vt[k] = v[k];
+          vt[V_R] = 0; vt[V_S] = 0; vt[V_GT] = 0; vt[V_GR] = 0;
+          coords(om, vt, base);
+        }
+        const uint32_t trow = smem_u32(tab) + (uint32_t)((isA ? 0 : 8) * 4 + j * 64);
+        int stage = it % STAGES;
+        uint32_t ph = (uint32_t)((it / STAGES) & 1);
+        for (int kit = k_begin; kit < k_end; kit++, it++) {
+          if (it >= STAGES) mbar_wait(&empty[stage], ph ^ 1);
+          if (lane == 0 && rank == 0) mbar_expect_tx(&full[stage], CG * (kStageBytesA + L::kB));
+          __syncwarp();
+          if (active) {
+            const uint32_t ta = trow + (uint32_t)(kit * a.spi * 64);
+            int32_t o0, o1, o2, o3, o4;
+            asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];" : "=r"(o0), "=r"(o1), "=r"(o2), "=r"(o3) : "r"(ta));
+            asm volatile("ld.shared.b32 %0, [%1];" : "=r"(o4) : "r"(ta + 16));
+            unsigned char *dst = sbase + stage * sbytes + j * om.slab_bytes;
+            if constexpr (CG == 2)
+              tma_load_5d_2cta(dst, tmap, &full[stage], base[0] + o0, base[1] + o1, base[2] + o2, base[3] + o3,
+                               base[4] + o4);
+            else
+              tma_load_5d(dst, tmap, &full[stage], base[0] + o0, base[1] + o1, base[2] + o2, base[3] + o3,
+                          base[4] + o4);
+          }
+          if (++stage == STAGES) { stage = 0; ph ^= 1u; }
+        }
+        continue;
+      }
       for (int kit = k_begin; kit < k_end; kit++, it++) {
         const int stage = it % STAGES, round = it / STAGES;
         if (lane == 0 && ti == ALT_DBG_TILE && kit == k_begin) { DBG(24); }
@@ -317,6 +384,17 @@ __global__ void __launch_bounds__(kThreads, 1)
       const uint32_t sbo = sw == 8 ? 128u : (uint32_t)(8 * sw * 2);
       const uint32_t aS = (uint32_t)a.A.slab_bytes, bS = (uint32_t)a.B.slab_bytes;
       const uint32_t lboA = sw == 8 ? aS : 16u, lboB = sw == 8 ? bS : 16u;
+      // descriptors of stage 0's four K=16 steps; stage s adds s * stage bytes
+      // to the start-address field (addr >> 4 in bits 0-13, no carry out)
+      uint64_t dA[4], dB[4];
+#pragma unroll
+      for (int kk = 0; kk < 4; kk++) {
+        const int kc = kk * 16;
+        const int slab = kc / sw;
+        const uint32_t off = (uint32_t)((kc % sw) * 2);
+        dA[kk] = smem_desc(smem_u32(sA) + slab * aS + off, lboA, sbo, layout);
+        dB[kk] = smem_desc(smem_u32(sB) + slab * bS + off, lboB, sbo, layout);
+      }
       int it = 0, i = 0;
       for (int tile = unit0; tile < a.num_tiles; tile += unit_step, i++) {
         const int acc = i % NACC, use = i / NACC;
@@ -328,25 +406,22 @@ __global__ void __launch_bounds__(kThreads, 1)
         const int sp = tile - (int)a.f_spl.div((uint32_t)tile) * a.splits;
         const int k_begin = a.splits == 1 ? 0 : sp * a.num_iters / a.splits;
         const int k_end = a.splits == 1 ? a.num_iters : (sp + 1) * a.num_iters / a.splits;
+        int stage = it % STAGES;
+        uint32_t ph = (uint32_t)((it / STAGES) & 1);
         for (int kit = k_begin; kit < k_end; kit++, it++) {
-          const int stage = it % STAGES, round = it / STAGES;
-          mbar_wait(&full[stage], round & 1);
+          mbar_wait(&full[stage], ph);
           if (i == ALT_DBG_TILE && kit == k_begin) { DBG(28); }
           tc_fence_after();
-          const uint32_t baseA = smem_u32(sA + stage * kStageBytesA), baseB = smem_u32(sB + stage * L::kB);
+          const uint64_t oA = (uint64_t)((stage * kStageBytesA) >> 4), oB = (uint64_t)((stage * L::kB) >> 4);
 #pragma unroll
           for (int kk = 0; kk < 4; kk++) {
-            const int kc = kk * 16;
-            const int slab = kc / sw;
-            const uint32_t off = (uint32_t)((kc % sw) * 2);
-            const uint64_t ad = smem_desc(baseA + slab * aS + off, lboA, sbo, layout);
-            const uint64_t bd = smem_desc(baseB + slab * bS + off, lboB, sbo, layout);
-            const bool accum = kit != k_begin || kk != 0;
-            if constexpr (CG == 2) mma_bf16_2cta(d, ad, bd, idesc, accum);
-            else mma_bf16(d, ad, bd, idesc, accum);
+            const uint32_t accum = (kit != k_begin || kk != 0) ? 1u : 0u;
+            if constexpr (CG == 2) mma_bf16_2cta(d, dA[kk] + oA, dB[kk] + oB, idesc, accum);
+            else mma_bf16(d, dA[kk] + oA, dB[kk] + oB, idesc, accum);
           }
           if constexpr (CG == 2) mma_commit_2cta(&empty[stage], 0x3);  // frees the stage in both CTAs
           else mma_commit(&empty[stage]);
+          if (++stage == STAGES) { stage = 0; ph ^= 1u; }
         }
         if constexpr (CG == 2) mma_commit_2cta(&tfull[acc], 0x3);
         else mma_commit(&tfull[acc]);
@@ -392,6 +467,9 @@ __global__ void __launch_bounds__(kThreads, 1)
     const int rn = row / tn, rp = (row / a.tile_w) % a.tile_h, rq = row % a.tile_w;
     const int r0 = wq * 32;
     const int sn0 = r0 / tn, sp0 = (r0 / a.tile_w) % a.tile_h, sq0 = r0 % a.tile_w;
+    int32_t ocg[5], ocr[5];  // store coordinates per channel slab (tile, in-tile)
+#pragma unroll
+    for (int d = 0; d < 5; d++) { ocg[d] = a.O.coef[d][V_GT]; ocr[d] = a.O.coef[d][V_GR]; }
     int i = 0;
     for (int tile = unit0; tile < a.num_tiles; tile += unit_step, i++) {
       const int acc = i % NACC, use = i / NACC;
@@ -407,6 +485,18 @@ __global__ void __launch_bounds__(kThreads, 1)
       fetch_sb(tile + unit_step, pf_s, pf_b);
       const int n = tc.n0 + rn, p = tc.p0 + rp, q = tc.q0 + rq;
       const bool vrow = n < a.N && p < a.Ho && q < a.Wo;
+      // TMA-store coordinates of this warp's 32-row sub-box (tile part),
+      // computed while the MMA may still be running
+      int32_t cbase[5] = {0, 0, 0, 0, 0};
+      if (a.out_mode == 1 && lane == 0) {
+        const int sn = tc.n0 + sn0, sp = tc.p0 + sp0, sq = tc.q0 + sq0;
+        int32_t vo[NVAR];
+        vo[V_N0] = sn;
+        vo[V_PT] = (int)a.O.fp.div((uint32_t)sp); vo[V_PR] = sp - vo[V_PT] * a.O.divp;
+        vo[V_QT] = (int)a.O.fq.div((uint32_t)sq); vo[V_QR] = sq - vo[V_QT] * a.O.divq;
+        vo[V_GT] = 0; vo[V_GR] = 0; vo[V_R] = 0; vo[V_S] = 0; vo[V_ONE] = 1;
+        coords(a.O, vo, cbase);
+      }
       int64_t yrow = 0;  // out_mode 2: offset of this thread's output row
       if (a.out_mode == 2 && vrow)
         yrow = a.is_conv ? __ldg(a.yr.rd[0] + n) + __ldg(a.yr.rd[2] + p) + __ldg(a.yr.rd[3] + q) : __ldg(a.yr.rd[0] + q);
@@ -553,17 +643,6 @@ __global__ void __launch_bounds__(kThreads, 1)
             fence_async_smem();
             __syncwarp();
             if (lane == 0) {
-              // TMA-store coordinates of this warp's 32-row sub-box
-              int32_t cbase[5];
-              {
-                const int sn = tc.n0 + sn0, sp = tc.p0 + sp0, sq = tc.q0 + sq0;
-                int32_t vo[NVAR];
-                vo[V_N0] = sn;
-                vo[V_PT] = (int)a.O.fp.div((uint32_t)sp); vo[V_PR] = sp - vo[V_PT] * a.O.divp;
-                vo[V_QT] = (int)a.O.fq.div((uint32_t)sq); vo[V_QR] = sq - vo[V_QT] * a.O.divq;
-                vo[V_GT] = 0; vo[V_GR] = 0; vo[V_R] = 0; vo[V_S] = 0; vo[V_ONE] = 1;
-                coords(a.O, vo, cbase);
-              }
               const int nslab = 32 / sw_o;
               for (int j = 0; j < nslab; j++) {
                 if (kb + j * sw_o >= a.K) break;  // channels past K: nothing to store
@@ -571,7 +650,7 @@ __global__ void __launch_bounds__(kThreads, 1)
                 const int gt = (int)a.O.fg.div((uint32_t)g), gr = g - gt * a.O.divg;
                 int32_t co[5];
 #pragma unroll
-                for (int d = 0; d < 5; d++) co[d] = cbase[d] + a.O.coef[d][V_GT] * gt + a.O.coef[d][V_GR] * gr;
+                for (int d = 0; d < 5; d++) co[d] = cbase[d] + ocg[d] * gt + ocr[d] * gr;
                 tma_store_5d(&tmY, sOut + (warp - 2) * 4096 + buf + j * 32 * pitch, co[0], co[1], co[2], co[3],
                              co[4]);
               }
@@ -1068,13 +1147,13 @@ static std::unordered_map<TcKey, TcPlan, TcKeyHash> g_tc_cache;
 static cudaError_t launch_plan(const TcPlan &pl, void *y, cudaStream_t stream) {
   uint16_t *yy = static_cast<uint16_t *>(y);
   if (pl.cg == 2) {
-    if (pl.BN == 128) return launch_tc<128, 8, 2>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+    if (pl.BN == 128) return launch_tc<128, 7, 2>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
     return launch_tc<256, 5, 2>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
   }
-  if (pl.BN == 64) return launch_tc<64, 8, 1>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+  if (pl.BN == 64) return launch_tc<64, 7, 1>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
   if (pl.BN == 128) {
     if (pl.stages == 4) return launch_tc<128, 4, 1>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
-    return launch_tc<128, 6, 1>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+    return launch_tc<128, 5, 1>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
   }
   return launch_tc<256, 3, 1>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
 }
@@ -1289,7 +1368,7 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       pl.grid = (int)std::min<int64_t>((int64_t)a.num_tiles * cg, num_sms() / cg * cg);
       pl.BN = BN;
       pl.cg = cg;
-      pl.stages = cg == 2 ? (BN == 128 ? 8 : 5) : (BN == 64 ? 8 : (BN == 128 ? 6 : 3));
+      pl.stages = cg == 2 ? (BN == 128 ? 7 : 5) : (BN == 64 ? 7 : (BN == 128 ? 5 : 3));
       if (cfg && BN == 128 && cfg->stages == 4) pl.stages = 4;
       alt_kernel_cfg u{};
       u.path = ALT_PATH_TC;
