@@ -18,7 +18,9 @@ from typing import Iterable, Sequence
 import torch
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-_LIB_PATH = os.path.join(_HERE, "libalt.so")
+# ALT_LIB_VARIANT=<name> loads libalt_<name>.so from this directory (developer A/B
+# comparisons of kernel variants; never a CPU path)
+_LIB_PATH = os.path.join(_HERE, "libalt%s.so" % ("_" + os.environ["ALT_LIB_VARIANT"] if os.environ.get("ALT_LIB_VARIANT") else ""))
 if not os.path.exists(_LIB_PATH):
     raise ImportError(f"{_LIB_PATH} is missing: run __graft_entry__.build() (make -C "
                       f"{_HERE}); there is no CPU fallback")

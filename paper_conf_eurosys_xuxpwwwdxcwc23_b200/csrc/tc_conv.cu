@@ -71,6 +71,7 @@ struct TcArgs {
   Reader yr;             // out_mode 2: owner offsets of y
   EpiParams epi;
   uint64_t *dbg;         // optional per-CTA timestamps (ALT_TC_DEBUG)
+  int32_t epi_dbg;       // developer knob (ALT_TC_EPI_DBG): 1 skip output stores, 2 skip the whole drain
   // split-K: work unit = (output tile, reduction range); partial fp32 tiles
   // in ws[cta_tile][split][BN/32][128][32], arrivals counted in cnt[cta_tile]
   int32_t splits;
@@ -467,6 +468,12 @@ __global__ void __launch_bounds__(kThreads, 1)
     const int rn = row / tn, rp = (row / a.tile_w) % a.tile_h, rq = row % a.tile_w;
     const int r0 = wq * 32;
     const int sn0 = r0 / tn, sp0 = (r0 / a.tile_w) % a.tile_h, sq0 = r0 % a.tile_w;
+    // per-thread constants of the store path (no divisions in the chunk loop)
+    uint32_t so[4];
+#pragma unroll
+    for (int c = 0; c < 4; c++) so[c] = soff(c);
+    const int lg_sw = sw_o == 32 ? 5 : (sw_o == 16 ? 4 : 3);  // sw_o is 8, 16 or 32
+    const int nslab = 32 >> lg_sw;
     int32_t ocg[5], ocr[5];  // store coordinates per channel slab (tile, in-tile)
 #pragma unroll
     for (int d = 0; d < 5; d++) { ocg[d] = a.O.coef[d][V_GT]; ocr[d] = a.O.coef[d][V_GR]; }
@@ -542,6 +549,15 @@ __global__ void __launch_bounds__(kThreads, 1)
       // function calls while a load is in flight (a call would save / restore
       // the registers the asynchronous load is writing); the other variant
       // issues the next load at the end of the chunk.
+      if (a.epi_dbg == 2) {
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) {
+          if constexpr (CG == 2) mbar_arrive_cluster(&tempty[acc], 0);
+          else mbar_arrive(&tempty[acc]);
+        }
+        continue;
+      }
       auto chunk_loop = [&](auto early_tag) {
         constexpr bool EARLY = decltype(early_tag)::value;
         uint32_t raw[32];
@@ -612,7 +628,9 @@ __global__ void __launch_bounds__(kThreads, 1)
             for (int j = 0; j < 16; j++) pk[j] = pack_bf16x2(v[2 * j], v[2 * j + 1]);
           }
           if (et == 0 && i == ALT_DBG_TILE) { DBG(9 + (c0 >> 6) * 4); }
-          if (a.out_mode == 2) {
+          if (a.epi_dbg == 1) {
+            if (pk[0] == 0x7fff1234u) y[0] = 0;  // keep the values live
+          } else if (a.out_mode == 2) {
             // direct 16-byte stores: 8 channels are contiguous in y
             if (vrow) {
 #pragma unroll
@@ -636,22 +654,21 @@ __global__ void __launch_bounds__(kThreads, 1)
             __syncwarp();
 #pragma unroll
             for (int c = 0; c < 4; c++)
-              asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(wbuf + buf + soff(c)), "r"(pk[4 * c]),
+              asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(wbuf + buf + so[c]), "r"(pk[4 * c]),
                            "r"(pk[4 * c + 1]), "r"(pk[4 * c + 2]), "r"(pk[4 * c + 3])
                            : "memory");
             if (et == 0 && i == ALT_DBG_TILE) { DBG(10 + (c0 >> 6) * 4); }
             fence_async_smem();
             __syncwarp();
             if (lane == 0) {
-              const int nslab = 32 / sw_o;
               for (int j = 0; j < nslab; j++) {
-                if (kb + j * sw_o >= a.K) break;  // channels past K: nothing to store
-                const int g = kb / sw_o + j;
+                if (kb + (j << lg_sw) >= a.K) break;  // channels past K: nothing to store
+                const int g = (kb >> lg_sw) + j;
                 const int gt = (int)a.O.fg.div((uint32_t)g), gr = g - gt * a.O.divg;
                 int32_t co[5];
 #pragma unroll
                 for (int d = 0; d < 5; d++) co[d] = cbase[d] + ocg[d] * gt + ocr[d] * gr;
-                tma_store_5d(&tmY, sOut + (warp - 2) * 4096 + buf + j * 32 * pitch, co[0], co[1], co[2], co[3],
+                tma_store_5d(&tmY, sOut + (warp - 2) * 4096 + buf + j * (32 << (lg_sw + 1)), co[0], co[1], co[2], co[3],
                              co[4]);
               }
               bulk_commit();
@@ -1365,6 +1382,10 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       }
       if ((st = make_writer(P.yl, &a.yw)) != ALT_OK) return st;
       a.dbg = debug_buffer();
+      {
+        static const int epi_dbg = [] { const char *e = getenv("ALT_TC_EPI_DBG"); return e ? atoi(e) : 0; }();
+        a.epi_dbg = epi_dbg;
+      }
       pl.grid = (int)std::min<int64_t>((int64_t)a.num_tiles * cg, num_sms() / cg * cg);
       pl.BN = BN;
       pl.cg = cg;
