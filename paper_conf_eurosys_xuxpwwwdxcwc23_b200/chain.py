@@ -41,7 +41,9 @@ def block_n(K: int) -> int:
 
 def wgt_prims(L: nets.ConvShape):
     if L.groups > 1:
-        return []
+        # depthwise: R S K (8 consecutive channels contiguous per tap, read as
+        # one 16-byte vector by the depthwise kernel)
+        return [("reorder", [1, 2, 3, 0])]
     if L.C % 8:
         return LY.kcrs_wfold(L.K, L.C, L.S)
     x = 8 if L.C % 8 else chan_tile(L.C)

@@ -46,5 +46,10 @@ alt_status tc_gemm(const GemmProblem &P, const alt_kernel_cfg *cfg, cudaStream_t
                    alt_kernel_cfg *used);
 alt_status dw_conv(const ConvProblem &P, cudaStream_t stream, alt_kernel_cfg *used);
 alt_status pool2d(const ConvProblem &P, int kind, cudaStream_t stream);
+// separable layout whose channel dim (logical 1) runs in 16-byte-aligned
+// groups of 8 contiguous elements (pads allowed when allow_pad: owner offsets)
+bool chan_vec8(const Layout &L, bool allow_pad);
+// device-resident ones / zeros (>= K floats, 16-byte aligned, process lifetime)
+alt_status identity_vectors(int64_t K, const float **ones, const float **zeros);
 
 }  // namespace alt

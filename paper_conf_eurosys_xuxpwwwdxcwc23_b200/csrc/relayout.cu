@@ -17,6 +17,9 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdlib>
+#include <mutex>
+#include <vector>
 #include <cstdio>
 
 #include "common.cuh"
@@ -340,6 +343,251 @@ static bool fill_pair(Layout *S, Layout *D, const SepDev &ss, const SepDev &ds, 
   return true;
 }
 
+
+// ------------------------------------------------------------------ K_ROW --
+// dst's innermost physical dims hold only the src-contiguous logical dim b
+// (any pad / unfold / split of it) and one dim p0 of logical dim a (dst
+// innermost, X elements).  For every combination of the other ("outer") dst
+// dims the CTA stages the X src rows it needs — a index rev_a(outer_a + j),
+// the window of b the block touches, read coalesced (16-byte vectors) along
+// b — into shared memory as [X][window], then writes the contiguous dst block
+// of that outer index as 16-byte vectors made of whole X-runs, each X-run's
+// b index looked up through rev_b(outer_b + suffix_b(pos)).  Serves the conv
+// input templates (pad + unfold + NCHW[x]c, Fig. 5 / §5.1), padded-channel
+// and window-folded image layouts.
+struct RowPlan {
+  int32_t a, b;            // logical dims of p0 / of the suffix
+  int32_t X, Lb;           // extent of p0, logical extent of b
+  int32_t LbS;             // staged row pitch (elements, multiple of 16 B)
+  int32_t span;            // staged window length (elements, multiple of V)
+  int32_t npos;            // dst positions per outer index (excluding p0)
+  int32_t nout;            // outer dims (innermost last)
+  FastDiv odiv[kMaxP];
+  int32_t oowner[kMaxP], orad[kMaxP];
+  uint32_t nouter;         // number of outer indices
+  int32_t per_iter;        // outer indices staged per CTA iteration
+  int32_t lrank;
+  const int32_t *rev[kMaxL];   // dst reverse tables
+  const int64_t *rd[kMaxL];    // src owner offsets
+  const int32_t *sbc;          // [npos] suffix part of b's combo
+  const int32_t *blo;          // [footprint_b] window start per outer b combo
+  int32_t vec_load;            // src rows loadable as 16-byte vectors along b
+};
+
+template <typename T>
+__global__ void __launch_bounds__(256) k_relayout_row(RowPlan R, const T *__restrict__ src, T *__restrict__ dst) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  T *rows = reinterpret_cast<T *>(smem_raw);  // [per_iter][X][LbS]
+  __shared__ int64_t s_base[64];              // per staged outer index: src offset of (a, b) = (0, 0)
+  __shared__ int32_t s_acombo[64];            // outer part of a's combo, or -1 for an all-zero block
+  __shared__ int32_t s_bcombo[64], s_lo[64];  // outer part of b's combo, window start
+  constexpr int V = 16 / sizeof(T);
+  const int X = R.X, LbS = R.LbS, span = R.span;
+  const int blk = R.npos * X;                 // dst elements per outer index
+  const int rows_per = X * LbS;
+  for (uint32_t o0 = blockIdx.x * R.per_iter; o0 < R.nouter; o0 += gridDim.x * R.per_iter) {
+    const int cnt = (int)min((uint32_t)R.per_iter, R.nouter - o0);
+    __syncthreads();
+    if (threadIdx.x < cnt) {
+      uint32_t rem = o0 + threadIdx.x;
+      int32_t combo[kMaxL];
+#pragma unroll
+      for (int d = 0; d < kMaxL; d++) combo[d] = 0;
+      for (int k = R.nout - 1; k >= 0; k--) {
+        uint32_t q, r;
+        R.odiv[k].divmod(rem, q, r);
+        combo[R.oowner[k]] += (int32_t)r * R.orad[k];
+        rem = q;
+      }
+      int64_t base = 0;
+      bool ok = true;
+      for (int d = 0; d < R.lrank; d++) {
+        if (d == R.a || d == R.b) continue;
+        const int32_t i = __ldg(R.rev[d] + combo[d]);
+        if (i < 0) { ok = false; break; }
+        base += __ldg(R.rd[d] + i);
+      }
+      s_base[threadIdx.x] = base;
+      s_acombo[threadIdx.x] = ok ? combo[R.a] : -1;
+      s_bcombo[threadIdx.x] = combo[R.b];
+      s_lo[threadIdx.x] = __ldg(R.blo + combo[R.b]);
+    }
+    __syncthreads();
+    // stage: element (o, j, bi) -> rows[o][j][bi - lo]; bi fastest (coalesced)
+    if (R.vec_load) {
+      const int nv = span / V;
+      for (int e = threadIdx.x; e < cnt * X * nv; e += blockDim.x) {
+        const int bv = e % nv, t = e / nv, j = t % X, o = t / X;
+        const int ac = s_acombo[o];
+        const int b0 = s_lo[o] + bv * V;
+        const int32_t ai = (ac < 0 || b0 >= R.Lb) ? -1 : __ldg(R.rev[R.a] + ac + j);
+        uint4 u = make_uint4(0u, 0u, 0u, 0u);
+        if (ai >= 0) u = __ldg(reinterpret_cast<const uint4 *>(src + s_base[o] + __ldg(R.rd[R.a] + ai) + b0));
+        *reinterpret_cast<uint4 *>(rows + (size_t)o * rows_per + (size_t)j * LbS + bv * V) = u;
+      }
+    } else {
+      for (int e = threadIdx.x; e < cnt * X * span; e += blockDim.x) {
+        const int bl = e % span, t = e / span, j = t % X, o = t / X;
+        const int ac = s_acombo[o];
+        const int bi = s_lo[o] + bl;
+        const int32_t ai = (ac < 0 || bi >= R.Lb) ? -1 : __ldg(R.rev[R.a] + ac + j);
+        rows[(size_t)o * rows_per + (size_t)j * LbS + bl] =
+            ai < 0 ? T(0) : src[s_base[o] + __ldg(R.rd[R.a] + ai) + bi];
+      }
+    }
+    __syncthreads();
+    // write: 16-byte vectors of the contiguous dst blocks of the cnt outer indices
+    T *dblk = dst + (int64_t)o0 * blk;
+    const int nvec = cnt * blk / V;
+    for (int v = threadIdx.x; v < nvec; v += blockDim.x) {
+      const int e0 = v * V;
+      const int o = e0 / blk, w = e0 - o * blk;
+      const T *rb = rows + (size_t)o * rows_per;
+      const int bc = s_bcombo[o], lo = s_lo[o];
+      T val[V];
+      if (X >= V) {
+        const int pos = w / X, j0 = w - pos * X;
+        const int32_t bi = __ldg(R.rev[R.b] + bc + __ldg(R.sbc + pos));
+#pragma unroll
+        for (int k = 0; k < V; k++) val[k] = bi < 0 ? T(0) : rb[(size_t)(j0 + k) * LbS + (bi - lo)];
+      } else {
+        const int pos0 = w / X;
+#pragma unroll
+        for (int k = 0; k < V; k++) {
+          const int pos = pos0 + k / X, j = k % X;
+          const int32_t bi = __ldg(R.rev[R.b] + bc + __ldg(R.sbc + pos));
+          val[k] = bi < 0 ? T(0) : rb[(size_t)j * LbS + (bi - lo)];
+        }
+      }
+      *reinterpret_cast<uint4 *>(dblk + e0) = *reinterpret_cast<const uint4 *>(val);
+    }
+  }
+}
+
+// host side of K_ROW: returns false (nothing launched) when not applicable
+static bool row_launch(Layout *S, const void *src, Layout *D, void *dst, int wb, const SepDev &ss,
+                       const SepDev &ds, cudaStream_t stream, int nsm, alt_status *st) {
+  const int V = 16 / wb;
+  if (D->pnumel >= (1ll << 31)) return false;
+  if ((reinterpret_cast<uintptr_t>(dst) & 15) || D->pnumel % V) return false;
+  const int p0 = D->prank - 1;
+  const int a = D->pdim_owner[p0];
+  const int b = S->pdim_owner[S->prank - 1];
+  if (a == b || D->pdim_rad[p0] != 1) return false;
+  const int64_t Lb = S->lshape[b];
+  for (int64_t i = 0; i < Lb; i++) if (S->rd[b][i] != i) return false;  // b contiguous in src
+  // suffix: dims just above p0 owned by b
+  int ps = p0;
+  while (ps - 1 >= 0 && D->pdim_owner[ps - 1] == b) ps--;
+  if (ps == p0) return false;
+  const int64_t X = D->pshape[p0];
+  if (X < V ? (V % X != 0) : (X % V != 0)) return false;
+  int64_t npos = 1;
+  for (int p = ps; p < p0; p++) npos *= D->pshape[p];
+  if (npos * X % V || npos > (1 << 20)) return false;
+  // suffix part of b's combo per position
+  std::vector<int32_t> sbc((size_t)npos);
+  for (int64_t pos = 0; pos < npos; pos++) {
+    int64_t rem = pos, combo = 0;
+    for (int p = p0 - 1; p >= ps; p--) {
+      combo += (rem % D->pshape[p]) * D->pdim_rad[p];
+      rem /= D->pshape[p];
+    }
+    sbc[(size_t)pos] = (int32_t)combo;
+  }
+  // every outer combo of b (mixed radix over b's outer dims): the b window
+  // its block touches, start aligned down to a vector
+  std::vector<int> bouter;
+  for (int p = 0; p < ps; p++) if (D->pdim_owner[p] == b) bouter.push_back(p);
+  const int64_t fb = (int64_t)D->rev[b].size();
+  std::vector<int32_t> blo((size_t)fb, 0);
+  int64_t span = 0;
+  {
+    int64_t nob = 1;
+    for (int p : bouter) nob *= D->pshape[p];
+    for (int64_t k = 0; k < nob; k++) {
+      int64_t rem = k, ob = 0;
+      for (int t = (int)bouter.size() - 1; t >= 0; t--) {
+        const int p = bouter[t];
+        ob += (rem % D->pshape[p]) * D->pdim_rad[p];
+        rem /= D->pshape[p];
+      }
+      int64_t lo = INT64_MAX, hi = -1;
+      for (int64_t pos = 0; pos < npos; pos++) {
+        const int32_t bi = D->rev[b][ob + sbc[(size_t)pos]];
+        if (bi >= 0) { lo = std::min<int64_t>(lo, bi); hi = std::max<int64_t>(hi, bi); }
+      }
+      if (hi < 0) lo = hi = 0;
+      lo = lo / V * V;
+      blo[(size_t)ob] = (int32_t)lo;
+      span = std::max<int64_t>(span, hi - lo + 1);
+    }
+  }
+  span = (span + V - 1) / V * V;
+  int64_t LbS = span;
+  if ((LbS * wb) % 128 == 0) LbS += V;  // rows j and j + 1 on different banks
+  const size_t blk_smem = (size_t)X * LbS * wb;
+  if (blk_smem > 32768) return false;
+  RowPlan R{};
+  R.a = a; R.b = b; R.X = (int32_t)X; R.Lb = (int32_t)Lb; R.npos = (int32_t)npos;
+  R.LbS = (int32_t)LbS; R.span = (int32_t)span;
+  R.lrank = D->lrank;
+  int k = 0;
+  int64_t nouter = 1;
+  for (int p = 0; p < ps; p++) {
+    R.odiv[k] = FastDiv((uint32_t)D->pshape[p]);
+    R.oowner[k] = D->pdim_owner[p];
+    R.orad[k] = D->pdim_rad[p];
+    nouter *= D->pshape[p];
+    k++;
+  }
+  R.nout = k;
+  R.nouter = (uint32_t)nouter;
+  for (int d = 0; d < D->lrank; d++) { R.rev[d] = ds.rev[d]; R.rd[d] = ss.rd[d]; }
+  // device copies of the two tables, cached per (layout pair, device)
+  static std::mutex mu;
+  struct Ent { uint64_t s, d; int dev; int32_t *ptr; };
+  static std::vector<Ent> cache;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  int32_t *dt = nullptr;
+  {
+    std::lock_guard<std::mutex> g(mu);
+    for (auto &e : cache) if (e.s == S->serial && e.d == D->serial && e.dev == dev) dt = e.ptr;
+    if (!dt) {
+      std::vector<int32_t> h(sbc);
+      h.insert(h.end(), blo.begin(), blo.end());
+      if (cudaMalloc(&dt, h.size() * 4) != cudaSuccess) { cudaGetLastError(); return false; }
+      if (cudaMemcpy(dt, h.data(), h.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess) { cudaGetLastError(); return false; }
+      cache.push_back({S->serial, D->serial, dev, dt});
+    }
+  }
+  R.sbc = dt;
+  R.blo = dt + npos;
+  bool vl = Lb % V == 0 && (reinterpret_cast<uintptr_t>(src) & 15) == 0;
+  for (int d = 0; d < S->lrank && vl; d++) {
+    if (d == b) continue;
+    for (int64_t o : S->rd[d]) if (o >= 0 && o % V) { vl = false; break; }
+  }
+  R.vec_load = vl ? 1 : 0;
+  int per = (int)std::max<int64_t>(1, std::min<int64_t>(64, 16384 / (int64_t)blk_smem));
+  R.per_iter = per;
+  const size_t smem = (size_t)per * blk_smem;
+  const int64_t iters = (nouter + per - 1) / per;
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(iters, (int64_t)nsm * 8));
+  if (wb == 2) {
+    cudaFuncSetAttribute(k_relayout_row<uint16_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    k_relayout_row<uint16_t><<<grid, 256, smem, stream>>>(R, (const uint16_t *)src, (uint16_t *)dst);
+  } else {
+    cudaFuncSetAttribute(k_relayout_row<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    k_relayout_row<uint32_t><<<grid, 256, smem, stream>>>(R, (const uint32_t *)src, (uint32_t *)dst);
+  }
+  count_launch();
+  *st = cudaGetLastError() == cudaSuccess ? ALT_OK : ALT_E_CUDA;
+  if (*st != ALT_OK) set_error("relayout (row) launch failed");
+  return true;
+}
+
 // ===================================================== strided permutation ==
 // Fast path for layouts built from split / reorder only (no pad, no unfold):
 // both are permutations of a common refinement of the logical digits, so the
@@ -647,6 +895,11 @@ alt_status relayout_launch(Layout *S, const void *src, Layout *D, void *dst, int
     for (int d = 0; d < D->lrank; d++)
       for (int32_t v : D->rev[d])
         if (v >= 0 && S->rd[d][v] < 0) { set_error("alt_relayout: source layout has no copy of an element dst needs"); return ALT_E_LOSSY; }
+    {
+      alt_status rst = ALT_OK;
+      static const bool no_row = getenv("ALT_RELAYOUT_NOROW") != nullptr;  // developer A/B knob
+      if (!no_row && row_launch(S, src, D, dst, wb, ss, ds, stream, nsm, &rst)) return rst;
+    }
     SepPair P{};
     if (fill_pair(S, D, ss, ds, &P)) {
       const int p0 = D->prank - 1;

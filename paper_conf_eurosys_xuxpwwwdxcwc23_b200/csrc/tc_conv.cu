@@ -58,6 +58,7 @@ struct OperandMap {
 struct TcArgs {
   OperandMap A, B, O;
   int32_t out_mode;      // 1: TMA-store epilogue, 2: direct 16-byte stores, 0: generic writer
+  int32_t res_vec;       // residual read as 16-byte vectors of 8 channels (epi.res tables)
   int32_t is_conv;
   int32_t N, K, Ho, Wo;  // output: conv y[N,K,Ho,Wo]; GEMM: N=1, Ho=1, Wo=M, K=cols
   int32_t tile_n, tile_h, tile_w;
@@ -507,6 +508,25 @@ __global__ void __launch_bounds__(kThreads, 1)
       int64_t yrow = 0;  // out_mode 2: offset of this thread's output row
       if (a.out_mode == 2 && vrow)
         yrow = a.is_conv ? __ldg(a.yr.rd[0] + n) + __ldg(a.yr.rd[2] + p) + __ldg(a.yr.rd[3] + q) : __ldg(a.yr.rd[0] + q);
+      // residual rows (res_vec): this thread's 32 channels of a chunk are four
+      // 16-byte vectors; chunk 0's are requested before the MMA completes,
+      // chunk c + 1's while chunk c is converted
+      int64_t rrow = -1;
+      if (a.res_vec && vrow)
+        rrow = a.is_conv ? __ldg(a.epi.res.rd[0] + n) + __ldg(a.epi.res.rd[2] + p) + __ldg(a.epi.res.rd[3] + q)
+                         : __ldg(a.epi.res.rd[0] + q);
+      uint4 rq[4];
+      auto load_res = [&](int cbx) {
+        const uint16_t *res = static_cast<const uint16_t *>(a.epi.residual);
+#pragma unroll
+        for (int c = 0; c < 4; c++) {
+          const int k = tc.k0 + cbx + 8 * c;
+          rq[c] = make_uint4(0u, 0u, 0u, 0u);
+          if (rrow >= 0 && k < a.K)
+            rq[c] = __ldg(reinterpret_cast<const uint4 *>(res + rrow + __ldg(a.epi.res.rd[1] + k)));
+        }
+      };
+      if (a.res_vec) load_res(half * 32);
       mbar_wait(&tfull[acc], use & 1);
       if (et == 0 && i == ALT_DBG_TILE) { DBG(2); }
       tc_fence_after();
@@ -558,8 +578,9 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
         continue;
       }
-      auto chunk_loop = [&](auto early_tag) {
+      auto chunk_loop = [&](auto early_tag, auto res_tag) {
         constexpr bool EARLY = decltype(early_tag)::value;
+        constexpr bool RESV = decltype(res_tag)::value;  // 16-byte residual vectors
         uint32_t raw[32];
         tmem_ld_32x32b_x32(tmem + ((uint32_t)(wq * 32) << 16) + (uint32_t)(acc * BN + half * 32), raw);
 #pragma unroll 1
@@ -596,6 +617,18 @@ __global__ void __launch_bounds__(kThreads, 1)
               v[4 * j + 3] = fmaf(__uint_as_float(raw[4 * j + 3]), x.w, y.w);
             }
           }
+          if constexpr (RESV) {
+#pragma unroll
+            for (int c = 0; c < 4; c++) {
+              const uint32_t w4[4] = {rq[c].x, rq[c].y, rq[c].z, rq[c].w};
+#pragma unroll
+              for (int h = 0; h < 4; h++) {
+                v[8 * c + 2 * h] += __uint_as_float(w4[h] << 16);
+                v[8 * c + 2 * h + 1] += __uint_as_float(w4[h] & 0xffff0000u);
+              }
+            }
+            if (c0 + 64 < BN) load_res(cb + 64);
+          }
           if constexpr (EARLY) {
             if (c0 + 64 < BN) tmem_ld_32x32b_x32(next, raw);
           }
@@ -608,7 +641,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             }
           }
           if constexpr (!EARLY) {
-            if (a.epi.residual && vrow) {
+            if (a.epi.residual && !a.res_vec && vrow) {
               float rv[32];  // local memory, touched only when a residual exists
               residual_chunk(a.epi, a.is_conv, a.K, n, p, q, kb, rv);
 #pragma unroll
@@ -683,8 +716,10 @@ __global__ void __launch_bounds__(kThreads, 1)
           }
         }
       };
-      if (a.out_mode != 0 && !a.epi.residual && !wsl) chunk_loop(std::true_type{});
-      else chunk_loop(std::false_type{});
+      if (a.out_mode != 0 && !a.epi.residual && !wsl) chunk_loop(std::true_type{}, std::false_type{});
+      else if (a.out_mode != 0 && a.res_vec && !wsl) chunk_loop(std::true_type{}, std::true_type{});
+      else if (a.res_vec) chunk_loop(std::false_type{}, std::true_type{});
+      else chunk_loop(std::false_type{}, std::false_type{});
       if (et == 0 && i == ALT_DBG_TILE) { DBG(31); }
     }
     if (et == 0) { DBG(5); }
@@ -1059,7 +1094,7 @@ extern "C" int alt__debug_tc(uint64_t *host, int64_t n) {
 namespace alt {
 
 // per-device ones / zeros vectors (never freed: process lifetime)
-static alt_status identity_epilogue(int64_t K, const float **ones, const float **zeros) {
+alt_status identity_vectors(int64_t K, const float **ones, const float **zeros) {
   static std::mutex mu;
   struct Buf { int dev; int64_t cap; float *ones, *zeros; };
   static std::vector<Buf> bufs;
@@ -1372,11 +1407,13 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       a.f_S = FastDiv((uint32_t)a.S);
       alt_status st;
       if ((st = make_epi(P.epi, &a.epi)) != ALT_OK) return st;
+      a.res_vec = P.epi.residual && a.epi.res.sep && chan_vec8(*P.epi.residual_l, true) &&
+                  (reinterpret_cast<uintptr_t>(P.epi.residual) & 15) == 0 ? 1 : 0;
       // the kernel always applies scale * acc + bias: absent ones become the
       // identity (device-resident ones / zeros, grown on demand)
       if (!a.epi.scale || !a.epi.bias) {
         const float *ones = nullptr, *zeros = nullptr;
-        if ((st = identity_epilogue(P.K, &ones, &zeros)) != ALT_OK) return st;
+        if ((st = identity_vectors(P.K, &ones, &zeros)) != ALT_OK) return st;
         if (!a.epi.scale) a.epi.scale = ones;
         if (!a.epi.bias) a.epi.bias = zeros;
       }

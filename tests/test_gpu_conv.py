@@ -93,6 +93,23 @@ def test_depthwise_and_grouped(dtype):
     run_conv("grp", 2, 16, 9, 9, 32, 3, 3, 1, 1, [], [], [], dtype, groups=4)
 
 
+DW_CASES = [  # (name, N, C, H, W, R, V, pad, x/y layout, residual layout)
+    ("dw_rsk_c64", 2, 64, 14, 13, 3, 1, 1, LY.nchwxc(64, 64), LY.nchwxc(64, 64)),
+    ("dw_rsk_s2", 3, 48, 15, 15, 3, 2, 1, LY.nchwxc(48, 16), None),
+    ("dw_rsk_5x5", 1, 32, 12, 9, 5, 1, 2, LY.nchwxc(32, 8), LY.nchwxc(32, 32)),
+    ("dw_rsk_1x1", 2, 24, 7, 7, 1, 1, 0, LY.nchwxc(24, 8), None),
+]
+
+
+@pytest.mark.parametrize("case", DW_CASES, ids=[c[0] for c in DW_CASES])
+def test_depthwise_vector_weights(case):
+    """Depthwise fast path: weights stored R S K (8 consecutive k contiguous
+    per tap), 16-byte residual vectors, every channel-run ordering."""
+    name, N, C, H, W, R, V, pad, xp, rp = case
+    run_conv(name, N, C, H, W, C, R, R, V, pad, xp, [("reorder", [1, 2, 3, 0])], xp, torch.bfloat16,
+             groups=C, epi=True, act=2, res_p=rp, expect_path=alt.PATH_DW)
+
+
 @pytest.mark.parametrize("dtype", [torch.float32, torch.bfloat16])
 def test_layout_independence_I2(dtype):
     outs = []
