@@ -251,8 +251,10 @@ typedef struct { int64_t M, N, K; } alt_matmul_params;
 #define ALT_TUNE_MAX_VALS 8
 typedef struct {
   /* candidate values per template parameter; nvals[i] == 0 = default set.
-   * conv:  0 it (x channel tile), 1 ot (y channel tile), 2 it' (w c tile),
-   *        3 ot' (w k tile), 4 tile_h, 5 tile_w, 6 block_n, 7 pad_x (0/1)
+   * conv:  0 it (x channel tile; the w c tile it' = it), 1 ot (y channel
+   *        tile), 2 (reserved), 3 cta_pair (0 auto, 2 single CTA), 4 tile_h,
+   *        5 tile_w, 6 block_n (the w k tile ot' = min(block_n, K)),
+   *        7 pad_x (0/1: materialise the conv zero padding in x)
    * gemm:  0 mt, 1 kt, 2 nt, 6 block_n */
   int64_t vals[8][ALT_TUNE_MAX_VALS];
   int32_t nvals[8];

@@ -157,6 +157,7 @@ __device__ __forceinline__ void tma_store_5d(const CUtensorMap *m, const void *s
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait_read1() { asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
 
 // Out-of-line slow paths of the epilogue (kept out of the hot loop body).
 // residual values of one row's 32 channels, read through the residual layout
@@ -218,7 +219,9 @@ __device__ __forceinline__ TileCoord tile_coord(const TcArgs &a, int tile, int B
   return {tn_i * a.tile_n, th_i * a.tile_h, tw_i * a.tile_w, nt * BN};
 }
 
-template <int BN, int STAGES, int CG>
+// RV: epilogue reads the residual as 16-byte vectors (a separate
+// instantiation keeps the residual-free epilogue's register allocation)
+template <int BN, int STAGES, int CG, bool RV>
 __global__ void __launch_bounds__(kThreads, 1)
     k_tc_conv(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
               const __grid_constant__ CUtensorMap tmY, const __grid_constant__ TcArgs a, uint16_t *__restrict__ y) {
@@ -512,7 +515,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       // 16-byte vectors; chunk 0's are requested before the MMA completes,
       // chunk c + 1's while chunk c is converted
       int64_t rrow = -1;
-      if (a.res_vec && vrow)
+      if (RV && vrow)
         rrow = a.is_conv ? __ldg(a.epi.res.rd[0] + n) + __ldg(a.epi.res.rd[2] + p) + __ldg(a.epi.res.rd[3] + q)
                          : __ldg(a.epi.res.rd[0] + q);
       uint4 rq[4];
@@ -526,7 +529,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             rq[c] = __ldg(reinterpret_cast<const uint4 *>(res + rrow + __ldg(a.epi.res.rd[1] + k)));
         }
       };
-      if (a.res_vec) load_res(half * 32);
+      if constexpr (RV) load_res(half * 32);
       mbar_wait(&tfull[acc], use & 1);
       if (et == 0 && i == ALT_DBG_TILE) { DBG(2); }
       tc_fence_after();
@@ -641,7 +644,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             }
           }
           if constexpr (!EARLY) {
-            if (a.epi.residual && !a.res_vec && vrow) {
+            if (!RV && a.epi.residual && vrow) {
               float rv[32];  // local memory, touched only when a residual exists
               residual_chunk(a.epi, a.is_conv, a.K, n, p, q, kb, rv);
 #pragma unroll
@@ -716,14 +719,17 @@ __global__ void __launch_bounds__(kThreads, 1)
           }
         }
       };
-      if (a.out_mode != 0 && !a.epi.residual && !wsl) chunk_loop(std::true_type{}, std::false_type{});
-      else if (a.out_mode != 0 && a.res_vec && !wsl) chunk_loop(std::true_type{}, std::true_type{});
-      else if (a.res_vec) chunk_loop(std::false_type{}, std::true_type{});
-      else chunk_loop(std::false_type{}, std::false_type{});
+      if constexpr (RV) {
+        if (a.out_mode != 0 && !wsl) chunk_loop(std::true_type{}, std::true_type{});
+        else chunk_loop(std::false_type{}, std::true_type{});
+      } else {
+        if (a.out_mode != 0 && !a.epi.residual && !wsl) chunk_loop(std::true_type{}, std::false_type{});
+        else chunk_loop(std::false_type{}, std::false_type{});
+      }
       if (et == 0 && i == ALT_DBG_TILE) { DBG(31); }
     }
     if (et == 0) { DBG(5); }
-    if (lane == 0 && a.out_mode == 1) bulk_wait0();
+    if (lane == 0 && a.out_mode == 1) bulk_wait_read0();  // smem reads done; the global writes complete with the grid
   }
   tc_fence_before();
   __syncthreads();
@@ -1131,11 +1137,11 @@ static int num_sms() {
   return n;
 }
 
-template <int BN, int STAGES, int CG_>
+template <int BN, int STAGES, int CG_, bool RV>
 static cudaError_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUtensorMap &ty, const TcArgs &a,
                              uint16_t *y, int grid, cudaStream_t s) {
   constexpr int CG = CG_;
-  auto kern = k_tc_conv<BN, STAGES, CG>;
+  auto kern = k_tc_conv<BN, STAGES, CG, RV>;
   const int smem = TcSmem<BN, STAGES, CG>::kBytes;
   static_assert(TcSmem<BN, STAGES, CG>::kBytes <= 232448, "smem budget");
   static bool attr_set = false;  // once per instantiation (not capture-safe to repeat)
@@ -1196,18 +1202,22 @@ struct TcPlan {
 static std::mutex g_tc_mu;
 static std::unordered_map<TcKey, TcPlan, TcKeyHash> g_tc_cache;
 
+template <bool RV>
+static cudaError_t launch_plan_rv(const TcPlan &pl, uint16_t *yy, cudaStream_t stream) {
+  if (pl.cg == 2) {
+    if (pl.BN == 128) return launch_tc<128, 7, 2, RV>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+    return launch_tc<256, 5, 2, RV>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+  }
+  if (pl.BN == 64) return launch_tc<64, 7, 1, RV>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+  if (pl.BN == 128) {
+    if (pl.stages == 4) return launch_tc<128, 4, 1, RV>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+    return launch_tc<128, 5, 1, RV>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+  }
+  return launch_tc<256, 3, 1, RV>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+}
 static cudaError_t launch_plan(const TcPlan &pl, void *y, cudaStream_t stream) {
   uint16_t *yy = static_cast<uint16_t *>(y);
-  if (pl.cg == 2) {
-    if (pl.BN == 128) return launch_tc<128, 7, 2>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
-    return launch_tc<256, 5, 2>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
-  }
-  if (pl.BN == 64) return launch_tc<64, 7, 1>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
-  if (pl.BN == 128) {
-    if (pl.stages == 4) return launch_tc<128, 4, 1>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
-    return launch_tc<128, 5, 1>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
-  }
-  return launch_tc<256, 3, 1>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+  return pl.a.res_vec ? launch_plan_rv<true>(pl, yy, stream) : launch_plan_rv<false>(pl, yy, stream);
 }
 
 // common driver for conv and GEMM

@@ -8,8 +8,8 @@ from scripts.exptime import timeit
 
 N = 32
 names = sys.argv[1].split(",")
-cfgs = [(256, 0, 1), (256, 0, 0), (256, 0, 2), (256, 0, 3), (128, 1, 1), (128, 1, 2), (128, 1, 3), (128, 2, 1),
-        (128, 2, 2), (64, 2, 1), (64, 2, 2), (64, 2, 4)]
+cfgs = [(256, 0, 1), (256, 0, 2), (256, 0, 3), (256, 2, 1), (256, 2, 2), (256, 2, 4), (256, 2, 5), (256, 2, 6),
+        (128, 1, 1), (128, 1, 2), (128, 2, 1), (128, 2, 2), (128, 2, 3), (128, 2, 4), (64, 2, 1), (64, 2, 2), (64, 2, 4)]
 for L in nets.RESNET50:
     if L.name not in names:
         continue
