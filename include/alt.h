@@ -252,7 +252,7 @@ typedef struct { int64_t M, N, K; } alt_matmul_params;
 typedef struct {
   /* candidate values per template parameter; nvals[i] == 0 = default set.
    * conv:  0 it (x channel tile; the w c tile it' = it), 1 ot (y channel
-   *        tile), 2 (reserved), 3 cta_pair (0 auto, 2 single CTA), 4 tile_h,
+   *        tile), 2 split_k, 3 cta_pair (0 auto, 2 single CTA), 4 tile_h,
    *        5 tile_w, 6 block_n (the w k tile ot' = min(block_n, K)),
    *        7 pad_x (0/1: materialise the conv zero padding in x)
    * gemm:  0 mt, 1 kt, 2 nt, 6 block_n */

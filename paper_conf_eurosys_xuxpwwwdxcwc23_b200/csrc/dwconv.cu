@@ -155,6 +155,81 @@ __global__ void __launch_bounds__(256, 2) k_dw_vec8(DwArgs a, const uint16_t *__
   }
 }
 
+// Fast 3x3 form (vector weights, vector output, aligned scale / bias,
+// vector or no residual): every tap's x and w vectors are requested before
+// any arithmetic (18 independent 16-byte loads in flight per thread; the
+// padded taps load a valid address and are zeroed), so the kernel is not
+// bound by one load latency per tap.  Same (r, s) accumulation order.
+__global__ void __launch_bounds__(256, 2) k_dw3x3_fast(DwArgs a, const uint16_t *__restrict__ x,
+                                                       const uint16_t *__restrict__ w, uint16_t *__restrict__ y) {
+  for (uint32_t idx = blockIdx.x * blockDim.x + threadIdx.x; idx < a.total; idx += gridDim.x * blockDim.x) {
+    const DwItem it = dw_item(a, idx);
+    const int64_t base = __ldg(a.xrd[0] + it.n) + __ldg(a.xrd[1] + it.c0);
+    int64_t ro[3], co[3];
+    bool vr[3], vc[3];
+#pragma unroll
+    for (int r = 0; r < 3; r++) {
+      const int ih = it.p * a.Vh - a.ph + r;
+      vr[r] = ih >= 0 && ih < a.H;
+      ro[r] = __ldg(a.xrd[2] + (vr[r] ? ih : 0));
+    }
+#pragma unroll
+    for (int s2 = 0; s2 < 3; s2++) {
+      const int iw = it.q * a.Vw - a.pw + s2;
+      vc[s2] = iw >= 0 && iw < a.W;
+      co[s2] = __ldg(a.xrd[3] + (vc[s2] ? iw : 0));
+    }
+    const int64_t wk = __ldg(a.wrd[0] + it.c0);
+    int64_t wro[3], wco[3];
+#pragma unroll
+    for (int r = 0; r < 3; r++) { wro[r] = __ldg(a.wrd[2] + r); wco[r] = __ldg(a.wrd[3] + r); }
+    uint4 xv[9], wv[9];
+#pragma unroll
+    for (int r = 0; r < 3; r++)
+#pragma unroll
+      for (int s2 = 0; s2 < 3; s2++) {
+        xv[r * 3 + s2] = __ldg(reinterpret_cast<const uint4 *>(x + base + ro[r] + co[s2]));
+        wv[r * 3 + s2] = __ldg(reinterpret_cast<const uint4 *>(w + wk + wro[r] + wco[s2]));
+      }
+    uint4 rv = make_uint4(0u, 0u, 0u, 0u);
+    if (a.res_vec) {
+      const int64_t o = __ldg(a.epi.res.rd[0] + it.n) + __ldg(a.epi.res.rd[1] + it.c0) +
+                        __ldg(a.epi.res.rd[2] + it.p) + __ldg(a.epi.res.rd[3] + it.q);
+      rv = __ldg(reinterpret_cast<const uint4 *>(static_cast<const uint16_t *>(a.epi.residual) + o));
+    }
+    const float4 *scp = reinterpret_cast<const float4 *>(a.epi.scale + it.c0);
+    const float4 *bip = reinterpret_cast<const float4 *>(a.epi.bias + it.c0);
+    const float4 s0 = __ldg(scp), s1 = __ldg(scp + 1), b0 = __ldg(bip), b1 = __ldg(bip + 1);
+    const int64_t yo = __ldg(a.yrd[0] + it.n) + __ldg(a.yrd[1] + it.c0) + __ldg(a.yrd[2] + it.p) +
+                       __ldg(a.yrd[3] + it.q);
+    float acc[8];
+#pragma unroll
+    for (int j = 0; j < 8; j++) acc[j] = 0.f;
+#pragma unroll
+    for (int t = 0; t < 9; t++) {
+      if (!(vr[t / 3] && vc[t % 3])) continue;
+      float f[8], g[8];
+      unpack8(xv[t], f);
+      unpack8(wv[t], g);
+#pragma unroll
+      for (int j = 0; j < 8; j++) acc[j] = fmaf(f[j], g[j], acc[j]);
+    }
+    float res[8];
+    unpack8(rv, res);
+    const float ss[8] = {s0.x, s0.y, s0.z, s0.w, s1.x, s1.y, s1.z, s1.w};
+    const float bb[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+    float v[8];
+#pragma unroll
+    for (int j = 0; j < 8; j++) v[j] = apply_act(fmaf(acc[j], ss[j], bb[j]) + res[j], a.epi.act);
+    uint4 u;
+    u.x = (uint32_t)f32_to_bf16_rne(v[0]) | ((uint32_t)f32_to_bf16_rne(v[1]) << 16);
+    u.y = (uint32_t)f32_to_bf16_rne(v[2]) | ((uint32_t)f32_to_bf16_rne(v[3]) << 16);
+    u.z = (uint32_t)f32_to_bf16_rne(v[4]) | ((uint32_t)f32_to_bf16_rne(v[5]) << 16);
+    u.w = (uint32_t)f32_to_bf16_rne(v[6]) | ((uint32_t)f32_to_bf16_rne(v[7]) << 16);
+    *reinterpret_cast<uint4 *>(y + yo) = u;
+  }
+}
+
 // channel runs of 8 contiguous, 16-byte aligned vectors, one copy per element
 bool chan_vec8(const Layout &L, bool allow_pad) {
   if (!L.separable) return false;
@@ -261,7 +336,9 @@ alt_status dw_conv(const ConvProblem &P, cudaStream_t stream, alt_kernel_cfg *us
   const auto *x = static_cast<const uint16_t *>(P.x);
   const auto *w = static_cast<const uint16_t *>(P.w);
   auto *y = static_cast<uint16_t *>(P.y);
-  if (r3) k_dw_vec8<3, 3><<<grid, 256, 0, stream>>>(a, x, w, y);
+  const bool fast = r3 && a.w_vec && a.vec_out && a.sb_vec && (!P.epi.residual || a.res_vec);
+  if (fast) k_dw3x3_fast<<<grid, 256, 0, stream>>>(a, x, w, y);
+  else if (r3) k_dw_vec8<3, 3><<<grid, 256, 0, stream>>>(a, x, w, y);
   else if (r1) k_dw_vec8<1, 1><<<grid, 256, 0, stream>>>(a, x, w, y);
   else k_dw_vec8<5, 5><<<grid, 256, 0, stream>>>(a, x, w, y);
   count_launch();
@@ -301,6 +378,33 @@ __global__ void __launch_bounds__(256) k_pool_vec8(PoolArgs a, const uint16_t *_
 #pragma unroll
     for (int j = 0; j < 8; j++) acc[j] = a.kind == 0 ? -INFINITY : 0.f;
     int cnt = 0;
+    if (a.R == 3 && a.S == 3) {
+      // all nine window vectors requested before any arithmetic (padded taps
+      // load a valid address and are skipped), same (r, s) order
+      int64_t ro[3], co[3];
+      bool vr[3], vc[3];
+#pragma unroll
+      for (int r = 0; r < 3; r++) {
+        const int ih = it.p * a.Vh - a.ph + r;
+        vr[r] = ih >= 0 && ih < a.H;
+        ro[r] = __ldg(a.xrd[2] + (vr[r] ? ih : 0));
+        const int iw = it.q * a.Vw - a.pw + r;
+        vc[r] = iw >= 0 && iw < a.W;
+        co[r] = __ldg(a.xrd[3] + (vc[r] ? iw : 0));
+      }
+      uint4 xv[9];
+#pragma unroll
+      for (int t = 0; t < 9; t++) xv[t] = __ldg(reinterpret_cast<const uint4 *>(x + base + ro[t / 3] + co[t % 3]));
+#pragma unroll
+      for (int t = 0; t < 9; t++) {
+        if (!(vr[t / 3] && vc[t % 3])) continue;
+        float f[8];
+        unpack8(xv[t], f);
+#pragma unroll
+        for (int j = 0; j < 8; j++) acc[j] = a.kind == 0 ? fmaxf(acc[j], f[j]) : acc[j] + f[j];
+        cnt++;
+      }
+    } else
     for (int r = 0; r < a.R; r++) {
       const int ih = it.p * a.Vh - a.ph + r;
       if (ih < 0 || ih >= a.H) continue;

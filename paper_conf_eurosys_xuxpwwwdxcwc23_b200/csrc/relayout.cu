@@ -372,6 +372,9 @@ struct RowPlan {
   const int32_t *sbc;          // [npos] suffix part of b's combo
   const int32_t *blo;          // [footprint_b] window start per outer b combo
   int32_t vec_load;            // src rows loadable as 16-byte vectors along b
+  int32_t lgX;                 // log2 X
+  FastDiv f_nv, f_span, f_vpb;  // span / V, span, blk / V
+  int32_t bstatic;             // b has no outer dims: sbc holds the b index itself (or -1)
 };
 
 template <typename T>
@@ -413,11 +416,13 @@ __global__ void __launch_bounds__(256) k_relayout_row(RowPlan R, const T *__rest
       s_lo[threadIdx.x] = __ldg(R.blo + combo[R.b]);
     }
     __syncthreads();
-    // stage: element (o, j, bi) -> rows[o][j][bi - lo]; bi fastest (coalesced)
+    // stage: element (o, j, bi) -> rows[o][j][bi - lo]; flat over (row, vector)
+    // so every thread has work for any window length; b fastest (coalesced)
     if (R.vec_load) {
       const int nv = span / V;
       for (int e = threadIdx.x; e < cnt * X * nv; e += blockDim.x) {
-        const int bv = e % nv, t = e / nv, j = t % X, o = t / X;
+        const int row = (int)R.f_nv.div((uint32_t)e), bv = e - row * nv;
+        const int o = row >> R.lgX, j = row & (X - 1);
         const int ac = s_acombo[o];
         const int b0 = s_lo[o] + bv * V;
         const int32_t ai = (ac < 0 || b0 >= R.Lb) ? -1 : __ldg(R.rev[R.a] + ac + j);
@@ -427,7 +432,8 @@ __global__ void __launch_bounds__(256) k_relayout_row(RowPlan R, const T *__rest
       }
     } else {
       for (int e = threadIdx.x; e < cnt * X * span; e += blockDim.x) {
-        const int bl = e % span, t = e / span, j = t % X, o = t / X;
+        const int row = (int)R.f_span.div((uint32_t)e), bl = e - row * span;
+        const int o = row >> R.lgX, j = row & (X - 1);
         const int ac = s_acombo[o];
         const int bi = s_lo[o] + bl;
         const int32_t ai = (ac < 0 || bi >= R.Lb) ? -1 : __ldg(R.rev[R.a] + ac + j);
@@ -436,30 +442,30 @@ __global__ void __launch_bounds__(256) k_relayout_row(RowPlan R, const T *__rest
       }
     }
     __syncthreads();
-    // write: 16-byte vectors of the contiguous dst blocks of the cnt outer indices
+    // write: 16-byte vectors of the contiguous dst blocks of the cnt outer
+    // indices (they are consecutive, so the cnt blocks are one dst range)
     T *dblk = dst + (int64_t)o0 * blk;
-    const int nvec = cnt * blk / V;
-    for (int v = threadIdx.x; v < nvec; v += blockDim.x) {
-      const int e0 = v * V;
-      const int o = e0 / blk, w = e0 - o * blk;
+    const int vpb = blk / V;  // vectors per block
+    for (int v = threadIdx.x; v < cnt * vpb; v += blockDim.x) {
+      const int o = (int)R.f_vpb.div((uint32_t)v), w = (v - o * vpb) * V;
       const T *rb = rows + (size_t)o * rows_per;
       const int bc = s_bcombo[o], lo = s_lo[o];
       T val[V];
       if (X >= V) {
-        const int pos = w / X, j0 = w - pos * X;
-        const int32_t bi = __ldg(R.rev[R.b] + bc + __ldg(R.sbc + pos));
+        const int pos = w >> R.lgX, j0 = w & (X - 1);
+        const int32_t bi = R.bstatic ? __ldg(R.sbc + pos) : __ldg(R.rev[R.b] + bc + __ldg(R.sbc + pos));
 #pragma unroll
         for (int k = 0; k < V; k++) val[k] = bi < 0 ? T(0) : rb[(size_t)(j0 + k) * LbS + (bi - lo)];
       } else {
-        const int pos0 = w / X;
+        const int pos0 = w >> R.lgX;
 #pragma unroll
         for (int k = 0; k < V; k++) {
-          const int pos = pos0 + k / X, j = k % X;
-          const int32_t bi = __ldg(R.rev[R.b] + bc + __ldg(R.sbc + pos));
+          const int pos = pos0 + (k >> R.lgX), j = k & (X - 1);
+          const int32_t bi = R.bstatic ? __ldg(R.sbc + pos) : __ldg(R.rev[R.b] + bc + __ldg(R.sbc + pos));
           val[k] = bi < 0 ? T(0) : rb[(size_t)j * LbS + (bi - lo)];
         }
       }
-      *reinterpret_cast<uint4 *>(dblk + e0) = *reinterpret_cast<const uint4 *>(val);
+      *reinterpret_cast<uint4 *>(dblk + (int64_t)v * V) = *reinterpret_cast<const uint4 *>(val);
     }
   }
 }
@@ -482,6 +488,7 @@ static bool row_launch(Layout *S, const void *src, Layout *D, void *dst, int wb,
   if (ps == p0) return false;
   const int64_t X = D->pshape[p0];
   if (X < V ? (V % X != 0) : (X % V != 0)) return false;
+  if (X & (X - 1)) return false;  // power of two (shift / mask decode)
   int64_t npos = 1;
   for (int p = ps; p < p0; p++) npos *= D->pshape[p];
   if (npos * X % V || npos > (1 << 20)) return false;
@@ -556,6 +563,8 @@ static bool row_launch(Layout *S, const void *src, Layout *D, void *dst, int wb,
     for (auto &e : cache) if (e.s == S->serial && e.d == D->serial && e.dev == dev) dt = e.ptr;
     if (!dt) {
       std::vector<int32_t> h(sbc);
+      if (bouter.empty())  // static b map: store the b index itself
+        for (size_t q = 0; q < h.size(); q++) h[q] = D->rev[b][h[q]] < 0 ? -1 : D->rev[b][h[q]];
       h.insert(h.end(), blo.begin(), blo.end());
       if (cudaMalloc(&dt, h.size() * 4) != cudaSuccess) { cudaGetLastError(); return false; }
       if (cudaMemcpy(dt, h.data(), h.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess) { cudaGetLastError(); return false; }
@@ -564,6 +573,12 @@ static bool row_launch(Layout *S, const void *src, Layout *D, void *dst, int wb,
   }
   R.sbc = dt;
   R.blo = dt + npos;
+  R.lgX = 0;
+  while ((1ll << R.lgX) < X) R.lgX++;
+  R.bstatic = bouter.empty() ? 1 : 0;
+  R.f_nv = FastDiv((uint32_t)(span / V));
+  R.f_span = FastDiv((uint32_t)span);
+  R.f_vpb = FastDiv((uint32_t)(npos * X / V));
   bool vl = Lb % V == 0 && (reinterpret_cast<uintptr_t>(src) & 15) == 0;
   for (int d = 0; d < S->lrank && vl; d++) {
     if (d == b) continue;

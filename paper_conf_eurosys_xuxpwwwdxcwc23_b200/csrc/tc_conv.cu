@@ -187,19 +187,30 @@ static __device__ __noinline__ void write_chunk(const Writer &w, int is_conv, in
 }
 
 // split-K: the tile's value = sum of the splits' partials in split order
-// (all read back from the workspace, this CTA's own included), so the result
-// does not depend on which CTA finishes last.  Out of line: the split path
-// is rare and must not cost the common path registers.
-static __device__ __noinline__ void split_total(const float *wt, int splits, int BN, int cb, int row, float *out) {
+// (this CTA's own split taken from its accumulator, the others read back
+// from the workspace), so the result does not depend on which CTA finishes
+// last.  Workspace layout per CTA tile and split: [BN/32][8][128] float4
+// (32-column chunk, float4 slot, row): a warp's 32 rows are 512 contiguous
+// bytes, so partial stores and loads are fully coalesced.  Out of line: the
+// split path is rare and must not cost the common path registers.
+static __device__ __noinline__ void split_total(const float *wt, int splits, int own, int BN, int cb, int row,
+                                                const uint32_t *mine, float *out) {
   float t[32];
 #pragma unroll
   for (int j = 0; j < 32; j++) t[j] = 0.f;
   for (int s = 0; s < splits; s++) {
-    const float4 *src = reinterpret_cast<const float4 *>(wt + (size_t)s * (128 * BN) + ((size_t)(cb >> 5) * 128 + row) * 32);
+    if (s == own) {
+#pragma unroll
+      for (int j = 0; j < 32; j++) t[j] += __uint_as_float(mine[j]);
+      continue;
+    }
+    const float4 *src = reinterpret_cast<const float4 *>(wt + (size_t)s * (128 * BN)) + (size_t)(cb >> 5) * 8 * 128 + row;
+    float4 f[8];
+#pragma unroll
+    for (int j = 0; j < 8; j++) f[j] = __ldcg(src + j * 128);
 #pragma unroll
     for (int j = 0; j < 8; j++) {
-      const float4 f = __ldcg(src + j);
-      t[4 * j] += f.x; t[4 * j + 1] += f.y; t[4 * j + 2] += f.z; t[4 * j + 3] += f.w;
+      t[4 * j] += f[j].x; t[4 * j + 1] += f[j].y; t[4 * j + 2] += f[j].z; t[4 * j + 3] += f[j].w;
     }
   }
 #pragma unroll
@@ -544,14 +555,17 @@ __global__ void __launch_bounds__(kThreads, 1)
           uint32_t raw[32];
           tmem_ld_32x32b_x32(tmem + ((uint32_t)(wq * 32) << 16) + (uint32_t)(acc * BN + cb), raw);
           tmem_ld_wait();
-          uint4 *dst = reinterpret_cast<uint4 *>(mine + ((size_t)(cb >> 5) * 128 + row) * 32);
+          uint4 *dst = reinterpret_cast<uint4 *>(mine) + (size_t)(cb >> 5) * 8 * 128 + row;
 #pragma unroll
-          for (int j = 0; j < 8; j++) dst[j] = make_uint4(raw[4 * j], raw[4 * j + 1], raw[4 * j + 2], raw[4 * j + 3]);
+          for (int j = 0; j < 8; j++)
+            __stcg(dst + j * 128, make_uint4(raw[4 * j], raw[4 * j + 1], raw[4 * j + 2], raw[4 * j + 3]));
         }
         __threadfence();
+        if (et == 0 && i == ALT_DBG_TILE) { DBG(4); }
         named_bar(1, 256);
         if (et == 0) *last_flag = atomicAdd(a.cnt + cta_tile, 1) == a.splits - 1;
         named_bar(1, 256);
+        if (et == 0 && i == ALT_DBG_TILE) { DBG(7); }
         if (!*last_flag) {  // another CTA finishes this tile: free the accumulator
           tc_fence_before();
           __syncwarp();
@@ -598,7 +612,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           if constexpr (!EARLY) {
             if (wsl) {
               float tot[32];
-              split_total(wsl, a.splits, BN, cb, row, tot);
+              split_total(wsl, a.splits, ksp, BN, cb, row, raw, tot);
 #pragma unroll
               for (int j = 0; j < 32; j++) raw[j] = __float_as_uint(tot[j]);
             }

@@ -207,6 +207,7 @@ extern "C" alt_status alt_tune(alt_op_kind op, const void *op_params, alt_dtype 
     std::vector<int64_t> ths = vals_or(space, 4, {0});  // 0 = kernel heuristic
     std::vector<int64_t> tws = vals_or(space, 5, {0});
     std::vector<int64_t> pairs = vals_or(space, 3, {0});  // cta_pair: 0 auto (pair when BN >= 128), 2 single CTA
+    std::vector<int64_t> sks = vals_or(space, 2, {1});    // split-K factor
     for (int64_t it : its) {
       if (it > Cp || Cp % it || it % 8) continue;
       if (space && space->fix_x) { if (it != its[0]) continue; }
@@ -220,6 +221,7 @@ extern "C" alt_status alt_tune(alt_op_kind op, const void *op_params, alt_dtype 
             for (int64_t th : ths) {
               for (int64_t tw : tws) {
                for (int64_t pr : pairs) {
+                for (int64_t sk : sks) {
                 if (measured >= max_points) break;
                 if (pr == 1 && bn < 128) continue;
                 Seq xs = act_layout(p.C, Cp, it, pad ? p.pad_h : 0);
@@ -238,6 +240,7 @@ extern "C" alt_status alt_tune(alt_op_kind op, const void *op_params, alt_dtype 
                 cfg.path = ALT_PATH_AUTO;
                 cfg.block_n = (int32_t)bn;
                 cfg.cta_pair = (int32_t)pr;
+                cfg.split_k = (int32_t)sk;
                 if (th && tw) {
                   cfg.tile_h = (int32_t)th;
                   cfg.tile_w = (int32_t)tw;
@@ -252,6 +255,7 @@ extern "C" alt_status alt_tune(alt_op_kind op, const void *op_params, alt_dtype 
                 alt_kernel_cfg used{};
                 alt_last_plan(&used);
                 record(Lx.h ? &xs : nullptr, &ws, &ys, used, us);
+                }
                }
               }
             }

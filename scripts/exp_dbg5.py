@@ -1,5 +1,5 @@
 """Per-CTA timeline of one conv layer (build EXTRA=-DALT_DBG_TILE=t, env ALT_TC_DEBUG=1).
-usage: exp_dbg5.py LAYER [block_n] [cta_pair]"""
+usage: exp_dbg5.py LAYER [block_n] [cta_pair] [split_k]"""
 import os, sys, ctypes
 os.environ["ALT_TC_DEBUG"] = "1"
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
@@ -9,7 +9,7 @@ import paper_conf_eurosys_xuxpwwwdxcwc23_b200 as alt
 from paper_conf_eurosys_xuxpwwwdxcwc23_b200 import _alt
 lib = _alt._lib
 lib.alt__debug_tc.argtypes = [ctypes.c_void_p, ctypes.c_int64]
-names = {0: "start", 1: "setup done", 3: "mma: tile0 committed", 5: "epi: all done", 6: "end",
+names = {4: "epi: partial written", 7: "epi: last decided", 0: "start", 1: "setup done", 3: "mma: tile0 committed", 5: "epi: all done", 6: "end",
          24: "prod: before empty wait", 25: "prod: after empty wait", 26: "mma: before tempty", 27: "mma: after tempty",
          28: "mma: first full", 29: "mma: commit tfull", 2: "epi: tfull", 30: "epi: sb staged", 8: "epi: c0 ld",
          9: "epi: c0 math", 10: "epi: c0 smem", 11: "epi: c0 store", 31: "epi: tile end"}
@@ -19,6 +19,7 @@ for name in sys.argv[1].split(","):
     cfg = dict(l["cfg"])
     if len(sys.argv) > 2: cfg["block_n"] = int(sys.argv[2])
     if len(sys.argv) > 3: cfg["cta_pair"] = int(sys.argv[3])
+    if len(sys.argv) > 4: cfg["split_k"] = int(sys.argv[4])
     f = lambda: alt.conv2d(l["p"], l["lx"], l["x"], l["lw"], l["w"], l["ly"], l["y"], scale=l["sc"], bias=l["bi"], act="relu", cfg=cfg)
     for _ in range(3):
         f()

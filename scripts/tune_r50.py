@@ -16,7 +16,8 @@ for L in nets.RESNET50:
     if L.C % 8:
         continue
     p = alt.conv_params(N, L.C, L.H, L.W, L.K, L.R, L.S, L.stride, L.pad)
-    space = {0: [64, 32, 16], 1: [64, 32], 3: [0, 2], 6: [256, 128, 64], 7: [0, 1] if L.R > 1 else [0]}
+    space = {0: [64, 32, 16], 1: [64, 32], 2: [1, 2, 4], 3: [0, 2], 6: [256, 128, 64],
+             7: [0, 1] if L.R > 1 else [0]}
     t0 = time.time()
     r = alt.tune("conv2d", p, alt.ALT_BF16, space, max_points=512, warmup=3, reps=10)
     tunecache.store("conv2d", L, N, r)
