@@ -11,13 +11,18 @@ conversion ops (complex -> complex edges) — here they are fused.
 """
 from __future__ import annotations
 
+import json
 import math
+import os
 
 import torch
 
 from . import _alt as A
 from . import layouts as LY
 from . import nets, synth
+
+
+_TUNE_PATH = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "chain_tune.json")
 
 
 def chan_tile(C: int) -> int:
@@ -98,6 +103,19 @@ class Chain:
             bi = synth.bn_bias(name + "b" + L.name, L.K).to(dev)
             gen_w[i] = (wl, w, sc, bi)
         self.weights = gen_w
+        # tuned kernel configurations (loop tuning with the layouts fixed by
+        # propagation), from chain_tune.json when present
+        self.name = name
+        self.cfgs = {}
+        self.cfgs_loaded = False
+        try:
+            with open(_TUNE_PATH) as f:
+                ent = json.load(f).get(self.tune_key())
+            if ent:
+                self.cfgs = {int(k): v for k, v in ent.items()}
+                self.cfgs_loaded = True
+        except (OSError, ValueError):
+            pass
         torch.cuda.synchronize(dev) if dev.type == "cuda" else None
         self.flops = sum(op[1].flops(N) for op in ops if op[0] == "conv")
 
@@ -129,6 +147,87 @@ class Chain:
         src_edge, conversion = A.plan_chain(kinds, edges, lays)
         return sum(conversion), 0
 
+    # -------------------------------------------------------------- tuning
+    def tune_key(self):
+        return f"{self.name}|N{self.N}"
+
+    def tune(self, reps=10, warmup=3, store=True, log=None):
+        """Per conv op, time candidate kernel configurations (BLOCK_N, CTA
+        pair, split-K, output-pixel tile) on the device with every layout
+        fixed by propagation (Alg. 1: the downstream layouts are decided, the
+        loop schedule is tuned), keep the fastest; stored in chain_tune.json."""
+        import itertools
+        self.run()
+        torch.cuda.synchronize()
+        best = {}
+        for i, op in enumerate(self.ops):
+            if op[0] != "conv" or op[1].groups > 1:
+                continue
+            L, src, res, relu, dst = op[1], op[2], op[3], op[4], op[5]
+            wl, w, sc, bi = self.weights[i]
+            p = A.conv_params(self.N, L.C, L.H, L.W, L.K, L.R, L.S, L.stride, L.pad, L.groups)
+            kw = dict(residual=self.buf[res], residual_l=self.layouts[res]) if res is not None else {}
+            act = ("relu6" if self._relu6 else "relu") if relu else None
+            Ho, Wo = L.out_hw()
+            tiles = [None] + [(128 // (th * tw), th, tw) for th in (1, 2, 4) for tw in (4, 8, 16, 32)
+                              if tw <= 2 * Wo and th <= 2 * Ho and 128 // (th * tw) <= max(self.N, 1)]
+            cands = []
+            M = self.N * Ho * Wo
+            for bn, pair, sk, t in itertools.product((64, 128, 256), (0, 2), (1, 2, 4), tiles):
+                if bn > 64 and bn >= 2 * L.K:
+                    continue
+                # split-K only where the output tiles leave SMs idle (bounded workspace)
+                if sk > 1 and -(-M // 128) * -(-L.K // bn) > 296:
+                    continue
+                c = {"path": A.PATH_TC, "block_n": bn, "cta_pair": pair, "split_k": sk}
+                if t is not None:
+                    c.update(tile_n=t[0], tile_h=t[1], tile_w=t[2])
+                cands.append(c)
+            res_t = []
+            for c in cands:
+                f = lambda c=c: A.conv2d(p, self.layouts[src], self.buf[src], wl, w, self.layouts[dst],
+                                         self.buf[dst], scale=sc, bias=bi, act=act, cfg=c, **kw)
+                try:
+                    for _ in range(warmup):
+                        f()
+                    torch.cuda.synchronize()
+                    # device time without host launch overhead: `reps` launches
+                    # captured in a CUDA graph (the plan is cached, so capture
+                    # records kernel nodes only)
+                    g = torch.cuda.CUDAGraph()
+                    cs = torch.cuda.Stream()
+                    cs.wait_stream(torch.cuda.current_stream())
+                    with torch.cuda.stream(cs), torch.cuda.graph(g, stream=cs):
+                        for _ in range(reps):
+                            f()
+                    torch.cuda.current_stream().wait_stream(cs)
+                    g.replay()
+                    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    e0.record()
+                    g.replay()
+                    e1.record()
+                    torch.cuda.synchronize()
+                    res_t.append((e0.elapsed_time(e1) / reps * 1e3, c))
+                except (A.AltError, RuntimeError):
+                    torch.cuda.synchronize()
+                    continue
+            if res_t:
+                res_t.sort(key=lambda t: t[0])
+                best[i] = res_t[0][1]
+                if log:
+                    log(f"op {i} {L.name}: {res_t[0][0]:.1f} us of {len(res_t)} cfgs {res_t[0][1]}")
+        self.cfgs = best
+        if store:
+            try:
+                with open(_TUNE_PATH) as f:
+                    allc = json.load(f)
+            except (OSError, ValueError):
+                allc = {}
+            allc[self.tune_key()] = {str(k): v for k, v in best.items()}
+            with open(_TUNE_PATH, "w") as f:
+                json.dump(allc, f, indent=0, sort_keys=True)
+        return best
+
     # ------------------------------------------------------------- running
     def run(self, stream=None):
         """One forward pass: the input pad op converts the image into conv1's
@@ -144,7 +243,7 @@ class Chain:
                     kw = dict(residual=self.buf[res], residual_l=self.layouts[res])
                 act = ("relu6" if self._relu6 else "relu") if relu else None
                 A.conv2d(p, self.layouts[src], self.buf[src], wl, w, self.layouts[dst], self.buf[dst],
-                         scale=sc, bias=bi, act=act, stream=stream, **kw)
+                         scale=sc, bias=bi, act=act, stream=stream, cfg=self.cfgs.get(i), **kw)
             else:
                 _, k, s, pd, src, dst = op
                 n, c, h, w_ = self.shapes[src]

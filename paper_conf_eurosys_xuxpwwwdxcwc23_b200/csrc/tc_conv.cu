@@ -119,7 +119,7 @@ __device__ __forceinline__ uint64_t gtimer() {
 #define ALT_DBG_TILE 0  // which of a CTA's tiles the epilogue timestamps follow
 #endif
 #define DBG(slot) \
-  if (a.dbg) a.dbg[(size_t)blockIdx.x * 32 + (slot)] = gtimer()
+  if (a.dbg) a.dbg[(size_t)blockIdx.x * 40 + (slot)] = gtimer()
 
 __device__ __forceinline__ void coords(const OperandMap &m, const int32_t (&v)[NVAR], int32_t (&c)[5]) {
 #pragma unroll
@@ -301,6 +301,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   const uint32_t tmem = *tmem_slot;
   // programmatic dependent launch: the prologue above overlapped the previous
   // kernel's tail; no global memory is touched before it has completed
+  if (threadIdx.x == 0) { DBG(32); }
   asm volatile("griddepcontrol.wait;" ::: "memory");
   asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
   if (threadIdx.x == 0) { DBG(1); }
@@ -1100,7 +1101,7 @@ static uint64_t *debug_buffer() {
   if (!init) {
     init = true;
     const char *e = getenv("ALT_TC_DEBUG");
-    if (e && e[0] == '1' && cudaMalloc(&buf, (size_t)32 * 8 << 20) != cudaSuccess) buf = nullptr;
+    if (e && e[0] == '1' && cudaMalloc(&buf, (size_t)40 * 8 << 20) != cudaSuccess) buf = nullptr;
   }
   return buf;
 }
@@ -1414,6 +1415,18 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
           // per-plan workspace (lives as long as the process: captured graphs
           // may replay the plan after the cache forgets it)
           const size_t wsb = (size_t)units * cg * sk * 128 * BN * sizeof(float);
+          // bounded: plans (and their workspaces) live for the process, so a
+          // tuner sweeping many split points must not exhaust the device
+          static std::mutex ws_mu;
+          static size_t ws_total = 0;
+          {
+            std::lock_guard<std::mutex> g(ws_mu);
+            if (ws_total + wsb > ((size_t)4 << 30)) {
+              set_error("tc: split-K workspace budget (4 GiB per process) exhausted");
+              return ALT_E_NOMEM;
+            }
+            ws_total += wsb;
+          }
           if (cudaMalloc(&a.ws, wsb) != cudaSuccess || cudaMalloc(&a.cnt, (size_t)units * cg * 4) != cudaSuccess ||
               cudaMemset(a.cnt, 0, (size_t)units * cg * 4) != cudaSuccess) {
             cudaGetLastError();

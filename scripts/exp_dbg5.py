@@ -9,7 +9,7 @@ import paper_conf_eurosys_xuxpwwwdxcwc23_b200 as alt
 from paper_conf_eurosys_xuxpwwwdxcwc23_b200 import _alt
 lib = _alt._lib
 lib.alt__debug_tc.argtypes = [ctypes.c_void_p, ctypes.c_int64]
-names = {4: "epi: partial written", 7: "epi: last decided", 0: "start", 1: "setup done", 3: "mma: tile0 committed", 5: "epi: all done", 6: "end",
+names = {32: "prologue done (before griddep wait)", 4: "epi: partial written", 7: "epi: last decided", 0: "start", 1: "setup done", 3: "mma: tile0 committed", 5: "epi: all done", 6: "end",
          24: "prod: before empty wait", 25: "prod: after empty wait", 26: "mma: before tempty", 27: "mma: after tempty",
          28: "mma: first full", 29: "mma: commit tfull", 2: "epi: tfull", 30: "epi: sb staged", 8: "epi: c0 ld",
          9: "epi: c0 math", 10: "epi: c0 smem", 11: "epi: c0 store", 31: "epi: tile end"}
@@ -24,10 +24,15 @@ for name in sys.argv[1].split(","):
     for _ in range(3):
         f()
     torch.cuda.synchronize()
+    if os.environ.get("ISOLATED"):  # one launch on an idle GPU
+        lib.alt__debug_tc.restype = ctypes.c_int
+        torch.cuda._sleep(1000000)
+        f()
+        torch.cuda.synchronize()
     ncta = 148
-    buf = np.zeros(ncta * 32, np.uint64)
-    lib.alt__debug_tc(buf.ctypes.data, ncta * 32)
-    t = buf.reshape(ncta, 32).astype(np.int64)
+    buf = np.zeros(ncta * 40, np.uint64)
+    lib.alt__debug_tc(buf.ctypes.data, ncta * 40)
+    t = buf.reshape(ncta, 40).astype(np.int64)
     t0 = t[:, 0][t[:, 0] > 0].min()
     rel = np.where(t > 0, (t - t0) / 1000.0, np.nan)
     print(name, alt.last_plan())
