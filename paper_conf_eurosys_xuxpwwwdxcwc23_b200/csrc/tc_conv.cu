@@ -80,7 +80,18 @@ struct TcArgs {
   int32_t *cnt;
 };
 
-constexpr int kThreads = 320;  // producer, MMA, 8 epilogue warps
+#ifndef ALT_EPI_WARPS
+#define ALT_EPI_WARPS 8
+#endif
+// epilogue warps: 4 TMEM lane quarters x kParts column parts.  The drain is
+// latency-bound (TMEM load -> FMA -> pack -> smem -> TMA store per 32-column
+// chunk).  16 warps (ALT_EPI_WARPS=16) were measured slower: the 576-thread
+// CTA is capped at 96 registers and the epilogue spills.
+constexpr int kEpiWarps = ALT_EPI_WARPS;
+constexpr int kParts = kEpiWarps / 4;
+constexpr int kStep = 32 * kParts;     // columns per chunk round
+constexpr int kEpiThreads = 32 * kEpiWarps;
+constexpr int kThreads = 64 + kEpiThreads;  // producer, MMA, epilogue warps
 constexpr int kStageBytesA = 128 * 64 * 2;
 constexpr int kOutStage = 128 * 64 * 2;  // one 64-column bf16 chunk of the tile
 
@@ -96,7 +107,7 @@ struct Nacc { static constexpr int value = BN >= 256 ? 2 : 4; };
 // one shared load + 5 adds per box instead of the divisions and the 5 x 10
 // coefficient products of coords() (the single producer thread's issue
 // latency bounds the stage rate).
-constexpr int kTabSlabs = 288;
+constexpr int kTabSlabs = kEpiWarps == 8 ? 288 : 240;
 constexpr int kTabBytes = kTabSlabs * 64;
 
 template <int BN, int STAGES, int CG = 1>
@@ -104,7 +115,7 @@ struct TcSmem {
   static constexpr int kB = (BN / CG) * 64 * 2;  // this CTA's share of the B tile
   static constexpr int kRing = STAGES * (kStageBytesA + kB);
   static constexpr int kOut = kRing;                       // 2 staging buffers for TMA stores
-  static constexpr int kSB = kOut + 2 * kOutStage;         // scale / bias of the tile (2 x BN floats)
+  static constexpr int kSB = kOut + kEpiWarps * 4096;      // scale / bias of the tile (2 x BN floats)
   static constexpr int kBar = kSB + 2 * BN * 4;             // barriers
   static constexpr int kTab = kBar + 256;                   // slab coordinate table
   static constexpr int kBytes = kTab + kTabBytes + 1008 /*1024-B alignment slack*/;
@@ -267,7 +278,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
     for (int s = 0; s < NACC; s++) {
       mbar_init(&tfull[s], 1);
-      mbar_init(&tempty[s], 8 * CG);  // every epilogue warp of the pair
+      mbar_init(&tempty[s], kEpiWarps * CG);  // every epilogue warp of the pair
     }
     fence_mbar_init();
   }
@@ -452,7 +463,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     // column half (w - 2) / 4 of every 64-column chunk.
     const int et = threadIdx.x - 64;       // 0..255
     const int wq = warp & 3;
-    const int half = (warp - 2) >> 2;
+    const int half = (warp - 2) >> 2;      // column part (0 .. kParts - 1)
     const int row = wq * 32 + lane;        // accumulator row = tile row
     const int tn = a.tile_h * a.tile_w;
     const int sw_o = a.out_mode == 1 ? a.O.sw : 32;
@@ -498,12 +509,12 @@ __global__ void __launch_bounds__(kThreads, 1)
       const int acc = i % NACC, use = i / NACC;
       const int mn = (int)a.f_spl.div((uint32_t)tile), ksp = tile - mn * a.splits;
       const TileCoord tc = tile_coord(a, mn, BN, CG, rank);
-      named_bar(2, 256);  // every epilogue warp is done with the previous tile's values
+      named_bar(2, kEpiThreads);  // every epilogue warp is done with the previous tile's values
       if (et < BN) {  // explicit shared-space stores (the aligned base is a generic pointer)
         asm volatile("st.shared.f32 [%0], %1;" ::"r"(sSB + 4u * et), "f"(pf_s) : "memory");
         asm volatile("st.shared.f32 [%0], %1;" ::"r"(sSB + 4u * (BN + et)), "f"(pf_b) : "memory");
       }
-      named_bar(2, 256);
+      named_bar(2, kEpiThreads);
       if (et == 0 && i == ALT_DBG_TILE) { DBG(30); }
       fetch_sb(tile + unit_step, pf_s, pf_b);
       const int n = tc.n0 + rn, p = tc.p0 + rp, q = tc.q0 + rq;
@@ -551,8 +562,9 @@ __global__ void __launch_bounds__(kThreads, 1)
         float *wt = a.ws + cta_tile * (size_t)a.splits * (128 * BN);
         float *mine = wt + (size_t)ksp * (128 * BN);
 #pragma unroll 1
-        for (int c0 = 0; c0 < BN; c0 += 64) {
+        for (int c0 = 0; c0 < BN; c0 += kStep) {
           const int cb = c0 + half * 32;
+          if (cb >= BN) continue;
           uint32_t raw[32];
           tmem_ld_32x32b_x32(tmem + ((uint32_t)(wq * 32) << 16) + (uint32_t)(acc * BN + cb), raw);
           tmem_ld_wait();
@@ -563,9 +575,9 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
         __threadfence();
         if (et == 0 && i == ALT_DBG_TILE) { DBG(4); }
-        named_bar(1, 256);
+        named_bar(1, kEpiThreads);
         if (et == 0) *last_flag = atomicAdd(a.cnt + cta_tile, 1) == a.splits - 1;
-        named_bar(1, 256);
+        named_bar(1, kEpiThreads);
         if (et == 0 && i == ALT_DBG_TILE) { DBG(7); }
         if (!*last_flag) {  // another CTA finishes this tile: free the accumulator
           tc_fence_before();
@@ -599,17 +611,26 @@ __global__ void __launch_bounds__(kThreads, 1)
       auto chunk_loop = [&](auto early_tag, auto res_tag) {
         constexpr bool EARLY = decltype(early_tag)::value;
         constexpr bool RESV = decltype(res_tag)::value;  // 16-byte residual vectors
+        if (half * 32 >= BN) {  // this warp's column part is past BLOCK_N: nothing to drain
+          tc_fence_before();
+          __syncwarp();
+          if (lane == 0) {
+            if constexpr (CG == 2) mbar_arrive_cluster(&tempty[acc], 0);
+            else mbar_arrive(&tempty[acc]);
+          }
+          return;
+        }
         uint32_t raw[32];
         tmem_ld_32x32b_x32(tmem + ((uint32_t)(wq * 32) << 16) + (uint32_t)(acc * BN + half * 32), raw);
 #pragma unroll 1
-        for (int c0 = 0; c0 < BN; c0 += 64) {
+        for (int c0 = 0; c0 < BN; c0 += kStep) {
           const int cb = c0 + half * 32;     // first column of this thread's 32
           const int kb = tc.k0 + cb;
-          const uint32_t next = tmem + ((uint32_t)(wq * 32) << 16) + (uint32_t)(acc * BN + cb + 64);
+          const uint32_t next = tmem + ((uint32_t)(wq * 32) << 16) + (uint32_t)(acc * BN + cb + kStep);
           tmem_ld_wait();
 #pragma unroll
           for (int j = 0; j < 32; j++) asm volatile("" : "+r"(raw[j]));  // uses stay after the wait
-          if (et == 0 && i == ALT_DBG_TILE) { DBG(8 + (c0 >> 6) * 4); }
+          if (et == 0 && i == ALT_DBG_TILE) { DBG(8 + (c0 / kStep) * 4); }
           if constexpr (!EARLY) {
             if (wsl) {
               float tot[32];
@@ -645,12 +666,12 @@ __global__ void __launch_bounds__(kThreads, 1)
                 v[8 * c + 2 * h + 1] += __uint_as_float(w4[h] & 0xffff0000u);
               }
             }
-            if (c0 + 64 < BN) load_res(cb + 64);
+            if (c0 + kStep < BN) load_res(cb + kStep);
           }
           if constexpr (EARLY) {
-            if (c0 + 64 < BN) tmem_ld_32x32b_x32(next, raw);
+            if (c0 + kStep < BN) tmem_ld_32x32b_x32(next, raw);
           }
-          if (c0 + 64 >= BN) {  // accumulator buffer drained: MMA may reuse it
+          if (c0 + kStep >= BN) {  // accumulator buffer drained: MMA may reuse it
             tc_fence_before();
             __syncwarp();
             if (lane == 0) {
@@ -678,7 +699,7 @@ __global__ void __launch_bounds__(kThreads, 1)
 #pragma unroll
             for (int j = 0; j < 16; j++) pk[j] = pack_bf16x2(v[2 * j], v[2 * j + 1]);
           }
-          if (et == 0 && i == ALT_DBG_TILE) { DBG(9 + (c0 >> 6) * 4); }
+          if (et == 0 && i == ALT_DBG_TILE) { DBG(9 + (c0 / kStep) * 4); }
           if (a.epi_dbg == 1) {
             if (pk[0] == 0x7fff1234u) y[0] = 0;  // keep the values live
           } else if (a.out_mode == 2) {
@@ -700,7 +721,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             // double-buffered staging, swizzled rows, one TMA store per slab;
             // no CTA-wide barrier.  Buffer `buf` is free once the store issued
             // two chunks ago has read it (<= 1 store group in flight per warp).
-            const uint32_t buf = (uint32_t)((c0 >> 6) & 1) * 2048u;
+            const uint32_t buf = (uint32_t)((c0 / kStep) & 1) * 2048u;
             if (lane == 0) bulk_wait_read1();
             __syncwarp();
 #pragma unroll
@@ -708,7 +729,7 @@ __global__ void __launch_bounds__(kThreads, 1)
               asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(wbuf + buf + so[c]), "r"(pk[4 * c]),
                            "r"(pk[4 * c + 1]), "r"(pk[4 * c + 2]), "r"(pk[4 * c + 3])
                            : "memory");
-            if (et == 0 && i == ALT_DBG_TILE) { DBG(10 + (c0 >> 6) * 4); }
+            if (et == 0 && i == ALT_DBG_TILE) { DBG(10 + (c0 / kStep) * 4); }
             fence_async_smem();
             __syncwarp();
             if (lane == 0) {
@@ -723,14 +744,14 @@ __global__ void __launch_bounds__(kThreads, 1)
                              co[4]);
               }
               bulk_commit();
-              if (et == 0 && i == ALT_DBG_TILE) { DBG(11 + (c0 >> 6) * 4); }
+              if (et == 0 && i == ALT_DBG_TILE) { DBG(11 + (c0 / kStep) * 4); }
             }
           } else if constexpr (!EARLY) {
             // generic layouts: every copy / pad position through the writer
             if (vrow) write_chunk(a.yw, a.is_conv, a.K, y, n, p, q, kb, pk);
           }
           if constexpr (!EARLY) {
-            if (c0 + 64 < BN) tmem_ld_32x32b_x32(next, raw);
+            if (c0 + kStep < BN) tmem_ld_32x32b_x32(next, raw);
           }
         }
       };
@@ -1217,18 +1238,21 @@ struct TcPlan {
 static std::mutex g_tc_mu;
 static std::unordered_map<TcKey, TcPlan, TcKeyHash> g_tc_cache;
 
+// smem-ring depth per (BLOCK_N, CTA group): the deepest ring that fits 227 KB
+// next to the kEpiWarps staging buffers and the slab table
+constexpr int stages_for(int BN, int CG) {
+  return kEpiWarps == 8 ? (CG == 2 ? (BN == 128 ? 7 : 5) : (BN == 64 ? 7 : (BN == 128 ? 5 : 3)))
+                        : (CG == 2 ? (BN == 128 ? 5 : 4) : (BN == 64 ? 5 : (BN == 128 ? 4 : 3)));
+}
 template <bool RV>
 static cudaError_t launch_plan_rv(const TcPlan &pl, uint16_t *yy, cudaStream_t stream) {
   if (pl.cg == 2) {
-    if (pl.BN == 128) return launch_tc<128, 7, 2, RV>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
-    return launch_tc<256, 5, 2, RV>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+    if (pl.BN == 128) return launch_tc<128, stages_for(128, 2), 2, RV>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+    return launch_tc<256, stages_for(256, 2), 2, RV>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
   }
-  if (pl.BN == 64) return launch_tc<64, 7, 1, RV>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
-  if (pl.BN == 128) {
-    if (pl.stages == 4) return launch_tc<128, 4, 1, RV>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
-    return launch_tc<128, 5, 1, RV>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
-  }
-  return launch_tc<256, 3, 1, RV>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+  if (pl.BN == 64) return launch_tc<64, stages_for(64, 1), 1, RV>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+  if (pl.BN == 128) return launch_tc<128, stages_for(128, 1), 1, RV>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+  return launch_tc<256, stages_for(256, 1), 1, RV>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
 }
 static cudaError_t launch_plan(const TcPlan &pl, void *y, cudaStream_t stream) {
   uint16_t *yy = static_cast<uint16_t *>(y);
@@ -1463,8 +1487,7 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       pl.grid = (int)std::min<int64_t>((int64_t)a.num_tiles * cg, num_sms() / cg * cg);
       pl.BN = BN;
       pl.cg = cg;
-      pl.stages = cg == 2 ? (BN == 128 ? 7 : 5) : (BN == 64 ? 7 : (BN == 128 ? 5 : 3));
-      if (cfg && BN == 128 && cfg->stages == 4) pl.stages = 4;
+      pl.stages = stages_for(BN, cg);
       alt_kernel_cfg u{};
       u.path = ALT_PATH_TC;
       u.block_m = 128 * cg;
