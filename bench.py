@@ -353,9 +353,18 @@ def main():
                    act="relu", cfg=l["cfg"])
         plans.append(alt.last_plan())
     per_layer = []
+    bf16_peak, hbm_peak, peak_src = peaks()
+    t_roof_sum = t_meas_sum = 0.0
     for i, l in enumerate(S.layers):
         t = statistics.median(ev[k][i][0].elapsed_time(ev[k][i][1]) for k in range(args.steps))
+        # per-layer roofline time: max(FLOPs / tensor peak, algorithmic bytes / HBM peak)
+        t_tc = l["L"].flops(S.N) / (bf16_peak * 1e12)
+        t_hbm = l["L"].min_bytes(S.N) / (hbm_peak * 1e9)
+        t_roof_sum += max(t_tc, t_hbm)
+        t_meas_sum += t * 1e-3
         per_layer.append({"layer": l["L"].name, "us": round(t * 1e3, 2),
+                          "bound": "tensor" if t_tc >= t_hbm else "hbm",
+                          "roofline_frac": round(max(t_tc, t_hbm) / (t * 1e-3), 3),
                           "tflops": round(l["L"].flops(S.N) / (t * 1e-3) / 1e12, 1),
                           "path": plans[i]["path"], "tile": [plans[i]["tile_n"], plans[i]["tile_h"],
                                                              plans[i]["tile_w"]],
@@ -378,7 +387,6 @@ def main():
     e_ms = max_over_ranks(e0.elapsed_time(e1) / e_steps, ws)
     h2d, d2h = S.io_bytes()
 
-    bf16_peak, hbm_peak, peak_src = peaks()
     achieved = S.flops / (conv_ms * 1e-3) / 1e12
     line = {"metric": METRIC, "value": round(value, 2), "unit": "TFLOP/s", "n_gpus": ws,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 4),
@@ -389,8 +397,11 @@ def main():
                          "peak_source": f"{peak_src} bf16 dense (burst)", "unit": "TFLOP/s",
                          "frac": round(achieved / bf16_peak, 4),
                          "traffic": None, "algorithmic_bytes_per_step": S.alg_bytes,
+                         "set_roofline_time_frac": round(t_roof_sum / t_meas_sum, 4),
                          "note": "achieved = sum of layer FLOPs / sum of per-launch CUDA-event times; "
-                                 "13 of 23 layers are HBM-bound at batch 32 (SURVEY §8d)"},
+                                 "13 of 23 layers are HBM-bound at batch 32 (SURVEY §8d); "
+                                 "set_roofline_time_frac = sum over layers of max(FLOPs/tensor peak, "
+                                 "bytes/HBM peak) / sum of measured layer times"},
             "e2e": {"value": round(S.flops * ws / (e_ms * 1e-3) / 1e12, 3), "unit": "TFLOP/s",
                     "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
                     "ms_per_step": round(e_ms, 3)},
