@@ -196,6 +196,13 @@ typedef struct {
                           is cut into s ranges whose fp32 partial tiles are
                           summed in split order by the last CTA to finish
                           (deterministic); for grids smaller than the GPU */
+  int32_t split_cluster; /* 1: the split_k (2 or 4) ranges of a tile run as one
+                          thread-block cluster and are summed in split order
+                          through distributed shared memory, each CTA
+                          finishing 1/split of the tile's rows (no workspace;
+                          one CTA per tile part, block_n 128 / 256, no
+                          residual, a TMA-store output layout; otherwise
+                          ALT_E_UNSUPPORTED) */
 } alt_kernel_cfg;
 
 alt_status alt_conv2d(const alt_conv2d_params *p, alt_layout x_l, const void *x,
@@ -252,7 +259,8 @@ typedef struct { int64_t M, N, K; } alt_matmul_params;
 typedef struct {
   /* candidate values per template parameter; nvals[i] == 0 = default set.
    * conv:  0 it (x channel tile; the w c tile it' = it), 1 ot (y channel
-   *        tile), 2 split_k, 3 cta_pair (0 auto, 2 single CTA), 4 tile_h,
+   *        tile), 2 split_k (negative: -s = split_cluster form with s ranges),
+   *        3 cta_pair (0 auto, 2 single CTA), 4 tile_h,
    *        5 tile_w, 6 block_n (the w k tile ot' = min(block_n, K)),
    *        7 pad_x (0/1: materialise the conv zero padding in x)
    * gemm:  0 mt, 1 kt, 2 nt, 6 block_n */

@@ -63,7 +63,8 @@ class _Epi(ctypes.Structure):
 
 class KernelCfg(ctypes.Structure):
     _fields_ = [(n, ctypes.c_int32) for n in ("path", "block_m", "block_n", "block_k", "stages",
-                                              "cta_pair", "tile_n", "tile_h", "tile_w", "split_k")]
+                                              "cta_pair", "tile_n", "tile_h", "tile_w", "split_k",
+                                              "split_cluster")]
 
     def as_dict(self):
         return {n: getattr(self, n) for n, _ in self._fields_ if n != "_pad"}

@@ -173,13 +173,17 @@ class Chain:
                               if tw <= 2 * Wo and th <= 2 * Ho and 128 // (th * tw) <= max(self.N, 1)]
             cands = []
             M = self.N * Ho * Wo
-            for bn, pair, sk, t in itertools.product((64, 128, 256), (0, 2), (1, 2, 4), tiles):
+            for bn, pair, sk, t in itertools.product((64, 128, 256), (0, 2), (1, 2, 4, -2, -4), tiles):
                 if bn > 64 and bn >= 2 * L.K:
                     continue
                 # split-K only where the output tiles leave SMs idle (bounded workspace)
-                if sk > 1 and -(-M // 128) * -(-L.K // bn) > 296:
+                if abs(sk) > 1 and -(-M // 128) * -(-L.K // bn) > 296:
                     continue
-                c = {"path": A.PATH_TC, "block_n": bn, "cta_pair": pair, "split_k": sk}
+                # cluster split-K (negative): one CTA per tile part, no residual
+                if sk < 0 and (pair != 2 or bn < 128 or res is not None):
+                    continue
+                c = {"path": A.PATH_TC, "block_n": bn, "cta_pair": pair, "split_k": abs(sk),
+                     "split_cluster": int(sk < 0)}
                 if t is not None:
                     c.update(tile_n=t[0], tile_h=t[1], tile_w=t[2])
                 cands.append(c)

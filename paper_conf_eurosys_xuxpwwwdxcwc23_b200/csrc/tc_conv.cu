@@ -242,8 +242,14 @@ __device__ __forceinline__ TileCoord tile_coord(const TcArgs &a, int tile, int B
 }
 
 // RV: epilogue reads the residual as 16-byte vectors (a separate
-// instantiation keeps the residual-free epilogue's register allocation)
-template <int BN, int STAGES, int CG, bool RV>
+// instantiation keeps the residual-free epilogue's register allocation).
+// SC > 1: cluster split-K — the SC reduction ranges of one output tile run as
+// the SC CTAs of a thread-block cluster (one tile per CTA, no workspace); each
+// CTA drains its fp32 partial into its own (then idle) smem ring, and after a
+// cluster barrier CTA r reduces rows [r * 128 / SC, (r + 1) * 128 / SC) of all
+// SC partials through distributed shared memory in split order, applies the
+// epilogue and stores them — the reduction and the epilogue are split SC ways.
+template <int BN, int STAGES, int CG, bool RV, int SC>
 __global__ void __launch_bounds__(kThreads, 1)
     k_tc_conv(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
               const __grid_constant__ CUtensorMap tmY, const __grid_constant__ TcArgs a, uint16_t *__restrict__ y) {
@@ -402,6 +408,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
       }
     }
+    if constexpr (SC > 1) { __syncwarp(); cluster_sync(); }  // partials of the cluster drained
   } else if (warp == 1) {
     if (lane == 0 && rank == 0) {
       // ------------------------------------------------------ MMA issuer
@@ -457,6 +464,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         if (i == 0) { DBG(3); }
       }
     }
+    if constexpr (SC > 1) { __syncwarp(); cluster_sync(); }  // partials of the cluster drained
   } else {
     // -------------------------------------------------------- epilogue
     // 8 warps: warp w reads TMEM lane quarter (w % 4) (hardware rule) and
@@ -556,8 +564,28 @@ __global__ void __launch_bounds__(kThreads, 1)
       mbar_wait(&tfull[acc], use & 1);
       if (et == 0 && i == ALT_DBG_TILE) { DBG(2); }
       tc_fence_after();
+      if constexpr (SC > 1) {
+        // cluster split-K, phase 1: this CTA's fp32 partial -> its own smem
+        // ring (every stage consumed: one tile per CTA), [BN/32][128 rows][32]
+        // with the 16-byte slots of a row XOR-swizzled by (row & 7)
+#pragma unroll 1
+        for (int c0 = 0; c0 < BN; c0 += kStep) {
+          const int cb = c0 + half * 32;
+          if (cb >= BN) continue;
+          uint32_t raw[32];
+          tmem_ld_32x32b_x32(tmem + ((uint32_t)(wq * 32) << 16) + (uint32_t)(acc * BN + cb), raw);
+          tmem_ld_wait();
+          const uint32_t base = smem_u32(smem) + (uint32_t)(((cb >> 5) * 128 + row) * 128);
+#pragma unroll
+          for (int j4 = 0; j4 < 8; j4++)
+            asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(base + (uint32_t)((j4 ^ (row & 7)) * 16)),
+                         "r"(raw[4 * j4]), "r"(raw[4 * j4 + 1]), "r"(raw[4 * j4 + 2]), "r"(raw[4 * j4 + 3])
+                         : "memory");
+        }
+        continue;  // one tile per CTA; phase 2 after the cluster barrier
+      }
       const float *wsl = nullptr;  // this CTA tile's partials (split-K)
-      if (a.splits > 1) {
+      if (SC == 1 && a.splits > 1) {
         const size_t cta_tile = (size_t)mn * CG + rank;
         float *wt = a.ws + cta_tile * (size_t)a.splits * (128 * BN);
         float *mine = wt + (size_t)ksp * (128 * BN);
@@ -764,12 +792,102 @@ __global__ void __launch_bounds__(kThreads, 1)
       }
       if (et == 0 && i == ALT_DBG_TILE) { DBG(31); }
     }
+    if constexpr (SC > 1) {
+      // cluster split-K, phase 2 (out_mode 1): CTA `crank` owns TMEM lane
+      // quarters [crank * 4 / SC, (crank + 1) * 4 / SC) of the tile; work item
+      // = (quarter, 32-column chunk), one per warp at a time; the SC partials
+      // are read through DSMEM and summed in split order
+      __syncwarp();
+      cluster_sync();
+      const int crank = (int)cluster_ctarank();
+      const TileCoord tc = tile_coord(a, (int)a.f_spl.div((uint32_t)unit0), BN, CG, rank);
+      constexpr int NQ = 4 / SC, NCH = BN / 32;
+      const int ew = warp - 2;
+      int cnt = 0;
+      for (int item = ew; item < NQ * NCH; item += kEpiWarps, cnt++) {
+        const int qq = crank * NQ + item / NCH, ch = item % NCH;
+        const int rr = qq * 32 + lane;  // tile row of this thread
+        const int cb = ch * 32, kb = tc.k0 + cb;
+        float t[32];
+#pragma unroll
+        for (int j = 0; j < 32; j++) t[j] = 0.f;
+        const uint32_t local = smem_u32(smem) + (uint32_t)((ch * 128 + rr) * 128);
+        for (int sp2 = 0; sp2 < SC; sp2++) {
+          uint32_t ra;
+          asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(ra) : "r"(local), "r"(sp2));
+#pragma unroll
+          for (int j4 = 0; j4 < 8; j4++) {
+            float f0, f1, f2, f3;
+            asm volatile("ld.shared::cluster.v4.f32 {%0, %1, %2, %3}, [%4];"
+                         : "=f"(f0), "=f"(f1), "=f"(f2), "=f"(f3)
+                         : "r"(ra + (uint32_t)((j4 ^ (rr & 7)) * 16)));
+            t[4 * j4] += f0; t[4 * j4 + 1] += f1; t[4 * j4 + 2] += f2; t[4 * j4 + 3] += f3;
+          }
+        }
+        float v[32];
+#pragma unroll
+        for (int j = 0; j < 8; j++) {
+          float4 x, yb;
+          asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];"
+                       : "=f"(x.x), "=f"(x.y), "=f"(x.z), "=f"(x.w) : "r"(sSB + 4u * (cb + 4 * j)));
+          asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];"
+                       : "=f"(yb.x), "=f"(yb.y), "=f"(yb.z), "=f"(yb.w) : "r"(sSB + 4u * (BN + cb + 4 * j)));
+          v[4 * j + 0] = fmaf(t[4 * j + 0], x.x, yb.x);
+          v[4 * j + 1] = fmaf(t[4 * j + 1], x.y, yb.y);
+          v[4 * j + 2] = fmaf(t[4 * j + 2], x.z, yb.z);
+          v[4 * j + 3] = fmaf(t[4 * j + 3], x.w, yb.w);
+        }
+        uint32_t pk[16];
+        if (act == 1) {
+#pragma unroll
+          for (int j = 0; j < 16; j++) pk[j] = pack_bf16x2_relu(v[2 * j], v[2 * j + 1]);
+        } else if (act == 2) {
+#pragma unroll
+          for (int j = 0; j < 16; j++) pk[j] = pack_bf16x2_relu(fminf(v[2 * j], 6.f), fminf(v[2 * j + 1], 6.f));
+        } else {
+#pragma unroll
+          for (int j = 0; j < 16; j++) pk[j] = pack_bf16x2(v[2 * j], v[2 * j + 1]);
+        }
+        const uint32_t buf = (uint32_t)(cnt & 1) * 2048u;
+        if (lane == 0) bulk_wait_read1();
+        __syncwarp();
+#pragma unroll
+        for (int c = 0; c < 4; c++)
+          asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(wbuf + buf + so[c]), "r"(pk[4 * c]),
+                       "r"(pk[4 * c + 1]), "r"(pk[4 * c + 2]), "r"(pk[4 * c + 3])
+                       : "memory");
+        fence_async_smem();
+        __syncwarp();
+        if (lane == 0) {
+          // store coordinates of this quarter's 32-row sub-box
+          const int r0 = qq * 32;
+          const int sn = tc.n0 + r0 / tn, spp = tc.p0 + (r0 / a.tile_w) % a.tile_h, sq = tc.q0 + r0 % a.tile_w;
+          int32_t vo[NVAR], cbq[5];
+          vo[V_N0] = sn;
+          vo[V_PT] = (int)a.O.fp.div((uint32_t)spp); vo[V_PR] = spp - vo[V_PT] * a.O.divp;
+          vo[V_QT] = (int)a.O.fq.div((uint32_t)sq); vo[V_QR] = sq - vo[V_QT] * a.O.divq;
+          vo[V_GT] = 0; vo[V_GR] = 0; vo[V_R] = 0; vo[V_S] = 0; vo[V_ONE] = 1;
+          coords(a.O, vo, cbq);
+          for (int j = 0; j < nslab; j++) {
+            if (kb + (j << lg_sw) >= a.K) break;
+            const int g = (kb >> lg_sw) + j;
+            const int gt = (int)a.O.fg.div((uint32_t)g), gr = g - gt * a.O.divg;
+            int32_t co[5];
+#pragma unroll
+            for (int d = 0; d < 5; d++) co[d] = cbq[d] + ocg[d] * gt + ocr[d] * gr;
+            tma_store_5d(&tmY, sOut + (warp - 2) * 4096 + buf + j * (32 << (lg_sw + 1)), co[0], co[1], co[2], co[3],
+                         co[4]);
+          }
+          bulk_commit();
+        }
+      }
+    }
     if (et == 0) { DBG(5); }
     if (lane == 0 && a.out_mode == 1) bulk_wait_read0();  // smem reads done; the global writes complete with the grid
   }
   tc_fence_before();
   __syncthreads();
-  if constexpr (CG == 2) cluster_sync();  // the pair's MMAs and epilogues are done
+  if constexpr (CG == 2 || SC > 1) cluster_sync();  // the pair's MMAs / the peers' DSMEM reads are done
   if (warp == 1) tmem_dealloc<NACC * BN, CG>(tmem);
   if (threadIdx.x == 32) { DBG(6); }
 }
@@ -1173,11 +1291,11 @@ static int num_sms() {
   return n;
 }
 
-template <int BN, int STAGES, int CG_, bool RV>
+template <int BN, int STAGES, int CG_, bool RV, int SC = 1>
 static cudaError_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUtensorMap &ty, const TcArgs &a,
                              uint16_t *y, int grid, cudaStream_t s) {
   constexpr int CG = CG_;
-  auto kern = k_tc_conv<BN, STAGES, CG, RV>;
+  auto kern = k_tc_conv<BN, STAGES, CG, RV, SC>;
   const int smem = TcSmem<BN, STAGES, CG>::kBytes;
   static_assert(TcSmem<BN, STAGES, CG>::kBytes <= 232448, "smem budget");
   static bool attr_set = false;  // once per instantiation (not capture-safe to repeat)
@@ -1197,9 +1315,9 @@ static cudaError_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const
   lc.stream = s;
   cudaLaunchAttribute at[2];
   int na = 0;
-  if (CG == 2) {
+  if (CG * SC > 1) {
     at[na].id = cudaLaunchAttributeClusterDimension;
-    at[na].val.clusterDim.x = 2;
+    at[na].val.clusterDim.x = CG * SC;
     at[na].val.clusterDim.y = 1;
     at[na].val.clusterDim.z = 1;
     na++;
@@ -1233,6 +1351,7 @@ struct TcPlan {
   TcArgs a;
   int grid;
   int BN, stages, cg;
+  int sc;  // cluster split-K factor (1 = off)
   alt_kernel_cfg used;
 };
 static std::mutex g_tc_mu;
@@ -1256,6 +1375,13 @@ static cudaError_t launch_plan_rv(const TcPlan &pl, uint16_t *yy, cudaStream_t s
 }
 static cudaError_t launch_plan(const TcPlan &pl, void *y, cudaStream_t stream) {
   uint16_t *yy = static_cast<uint16_t *>(y);
+  if (pl.sc > 1) {  // cluster split-K: one CTA, no residual vectors (planner-checked)
+    if (pl.BN == 128)
+      return pl.sc == 2 ? launch_tc<128, stages_for(128, 1), 1, false, 2>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream)
+                        : launch_tc<128, stages_for(128, 1), 1, false, 4>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+    return pl.sc == 2 ? launch_tc<256, stages_for(256, 1), 1, false, 2>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream)
+                      : launch_tc<256, stages_for(256, 1), 1, false, 4>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+  }
   return pl.a.res_vec ? launch_plan_rv<true>(pl, yy, stream) : launch_plan_rv<false>(pl, yy, stream);
 }
 
@@ -1297,6 +1423,7 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       k[i++] = cfg->stages;
       k[i++] = cfg->cta_pair;
       k[i++] = cfg->split_k;
+      k[i++] = cfg->split_cluster;
     }
     int dev = 0;
     cudaGetDevice(&dev);
@@ -1434,7 +1561,17 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
         a.splits = (int32_t)sk;
         a.ws = nullptr;
         a.cnt = nullptr;
-        if (sk > 1) {
+        // cluster split-K: the sk ranges of a tile as one cluster, reduced
+        // through DSMEM (single CTA, TMA-store output, no residual, sk 2 / 4)
+        pl.sc = 1;
+        if (cfg && cfg->split_cluster && sk > 1) {
+          if (cg != 1 || (sk != 2 && sk != 4) || BN < 128 || a.out_mode != 1 || P.epi.residual) {
+            set_error("tc: cluster split-K needs one CTA, block_n 128/256, split 2/4, a TMA-store output and no residual");
+            return ALT_E_UNSUPPORTED;
+          }
+          pl.sc = (int)sk;
+          a.num_tiles = (int32_t)(units * sk);
+        } else if (sk > 1) {
           if ((int64_t)a.num_tiles * sk > 0x7fffffff) { set_error("tc: too many tiles"); return ALT_E_UNSUPPORTED; }
           // per-plan workspace (lives as long as the process: captured graphs
           // may replay the plan after the cache forgets it)
@@ -1484,7 +1621,8 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
         static const int epi_dbg = [] { const char *e = getenv("ALT_TC_EPI_DBG"); return e ? atoi(e) : 0; }();
         a.epi_dbg = epi_dbg;
       }
-      pl.grid = (int)std::min<int64_t>((int64_t)a.num_tiles * cg, num_sms() / cg * cg);
+      pl.grid = pl.sc > 1 ? a.num_tiles  // one tile per CTA
+                          : (int)std::min<int64_t>((int64_t)a.num_tiles * cg, num_sms() / cg * cg);
       pl.BN = BN;
       pl.cg = cg;
       pl.stages = stages_for(BN, cg);
@@ -1497,6 +1635,7 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       u.stages = pl.stages;
       u.tile_n = c.tn; u.tile_h = c.th; u.tile_w = c.tw;
       u.split_k = a.splits;
+      u.split_cluster = pl.sc > 1 ? 1 : 0;
       pl.used = u;
       cudaError_t e = launch_plan(pl, P.y, stream);
       count_launch();

@@ -240,7 +240,8 @@ extern "C" alt_status alt_tune(alt_op_kind op, const void *op_params, alt_dtype 
                 cfg.path = ALT_PATH_AUTO;
                 cfg.block_n = (int32_t)bn;
                 cfg.cta_pair = (int32_t)pr;
-                cfg.split_k = (int32_t)sk;
+                cfg.split_k = (int32_t)(sk < 0 ? -sk : sk);  // negative: the cluster (DSMEM) form
+                cfg.split_cluster = sk < 0 ? 1 : 0;
                 if (th && tw) {
                   cfg.tile_h = (int32_t)th;
                   cfg.tile_w = (int32_t)tw;

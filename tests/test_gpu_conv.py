@@ -276,3 +276,40 @@ def test_tc_gemm_split_k():
     _, plan = run_gemm("gsk", 200, 256, 2048, [], LY.transpose2(), [], torch.bfloat16, epi=True,
                        cfg={"path": alt.PATH_TC, "split_k": 4}, expect_path=alt.PATH_TC)
     assert plan["split_k"] == 4
+
+
+# ------------------------------------------------------ cluster split-K --
+@pytest.mark.parametrize("sk,bn,shape", [(2, 256, (2, 256, 7, 7, 512)), (4, 128, (2, 256, 7, 7, 512)),
+                                         (4, 256, (3, 128, 9, 11, 256)), (2, 128, (1, 64, 14, 14, 128))])
+def test_tc_split_cluster(sk, bn, shape):
+    """cluster split-K (alt_kernel_cfg.split_cluster): the split ranges of a tile run as one thread-block
+    cluster and are summed through distributed shared memory; fused BN + ReLU, ragged M tiles."""
+    N, C, H, W, K = shape
+    cfg = {"path": alt.PATH_TC, "split_k": sk, "block_n": bn, "cta_pair": 2, "split_cluster": 1}
+    xp, wp, yp = LY.nchwxc(C, 64), LY.kcrs_yk_xc(K, C, min(K, 256), 64), LY.nchwxc(K, 64)
+    _, plan = run_conv("tcsc%d%d" % (sk, bn), N, C, H, W, K, 3, 3, 1, 1, xp, wp, yp, torch.bfloat16, epi=True,
+                       act=1, cfg=cfg, expect_path=alt.PATH_TC)
+    assert plan["split_k"] == sk and plan["split_cluster"] == 1
+
+
+def test_tc_split_cluster_deterministic_and_unsupported():
+    p = alt.conv_params(2, 256, 7, 7, 512, 3, 3, 1, 1)
+    x = synth.activations("scdx", (2, 256, 7, 7))
+    w = synth.weights("scdw", (512, 256, 3, 3))
+    xp, wp, yp = LY.nchwxc(256, 64), LY.kcrs_yk_xc(512, 256, 256, 64), LY.nchwxc(512, 64)
+    _, _, xd = make_operand("scdx", xp, x, torch.bfloat16)
+    _, _, wd = make_operand("scdw", wp, w, torch.bfloat16)
+    Lx, Lw, Ly = alt.Layout(x.shape, xp), alt.Layout(w.shape, wp), alt.Layout((2, 512, 7, 7), yp)
+    cfg = {"path": alt.PATH_TC, "split_k": 4, "block_n": 256, "cta_pair": 2, "split_cluster": 1}
+    outs = []
+    for _ in range(3):
+        y = torch.zeros(Ly.phys_shape, dtype=torch.bfloat16, device="cuda")
+        alt.conv2d(p, Lx, xd, Lw, wd, Ly, y, cfg=cfg)
+        outs.append(y)
+    torch.cuda.synchronize()
+    for y in outs[1:]:
+        assert np.array_equal(words(y), words(outs[0]))
+    # a residual is not served by the cluster form: the call fails loudly
+    with pytest.raises(alt.AltError) as e:
+        alt.conv2d(p, Lx, xd, Lw, wd, Ly, outs[0], residual=outs[1], residual_l=Ly, cfg=cfg)
+    assert e.value.code == alt._alt.ALT_E_UNSUPPORTED
