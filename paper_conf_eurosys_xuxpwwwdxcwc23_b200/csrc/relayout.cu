@@ -377,7 +377,13 @@ struct RowPlan {
   int32_t bstatic;             // b has no outer dims: sbc holds the b index itself (or -1)
 };
 
-template <typename T>
+// RB = 0: rows staged as [X][window] (any X).  RB = 8 / 16 (X * sizeof(T)
+// bytes, vector loads): each thread loads one 16-byte b-vector of all X rows
+// and transposes it in registers, so the stage holds [window][X] — every
+// X-run of the dst is one 8 / 16-byte shared load in the write phase.  Runs
+// are stored at slot b ^ ((b / V) & (V - 1)) within each V-run group, which
+// spreads a warp's stores (lane stride V runs) over the banks.
+template <typename T, int RB>
 __global__ void __launch_bounds__(256) k_relayout_row(RowPlan R, const T *__restrict__ src, T *__restrict__ dst) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   T *rows = reinterpret_cast<T *>(smem_raw);  // [per_iter][X][LbS]
@@ -418,7 +424,46 @@ __global__ void __launch_bounds__(256) k_relayout_row(RowPlan R, const T *__rest
     __syncthreads();
     // stage: element (o, j, bi) -> rows[o][j][bi - lo]; flat over (row, vector)
     // so every thread has work for any window length; b fastest (coalesced)
-    if (R.vec_load) {
+    if constexpr (RB > 0) {
+      constexpr int XR = RB / sizeof(T);  // == X
+      const int nv = span / V;
+      for (int e = threadIdx.x; e < cnt * nv; e += blockDim.x) {
+        const int o = (int)R.f_nv.div((uint32_t)e), bv = e - o * nv;
+        const int ac = s_acombo[o];
+        const int b0 = s_lo[o] + bv * V;
+        uint4 u[XR];
+#pragma unroll
+        for (int j = 0; j < XR; j++) {
+          const int32_t ai = (ac < 0 || b0 >= R.Lb) ? -1 : __ldg(R.rev[R.a] + ac + j);
+          u[j] = make_uint4(0u, 0u, 0u, 0u);
+          if (ai >= 0) u[j] = __ldg(reinterpret_cast<const uint4 *>(src + s_base[o] + __ldg(R.rd[R.a] + ai) + b0));
+        }
+        unsigned char *ob = reinterpret_cast<unsigned char *>(rows + (size_t)o * rows_per);
+#pragma unroll
+        for (int k = 0; k < V; k++) {
+          const int bl = bv * V + k;
+          const int slot = bl ^ ((bl / V) & (V - 1));
+          uint32_t w[RB / 4];
+          if constexpr (sizeof(T) == 2) {
+            // run k = element k of every row j: 16-bit transpose with byte_perm
+            const uint32_t sel = (k & 1) ? 0x7632u : 0x5410u;
+#pragma unroll
+            for (int jp = 0; jp < XR / 2; jp++) {
+              const uint32_t *a0 = reinterpret_cast<const uint32_t *>(&u[2 * jp]);
+              const uint32_t *a1 = reinterpret_cast<const uint32_t *>(&u[2 * jp + 1]);
+              w[jp] = __byte_perm(a0[k >> 1], a1[k >> 1], sel);
+            }
+          } else {
+#pragma unroll
+            for (int j = 0; j < XR; j++) w[j] = reinterpret_cast<const uint32_t *>(&u[j])[k];
+          }
+          if constexpr (RB == 16)
+            *reinterpret_cast<uint4 *>(ob + (size_t)slot * 16) = make_uint4(w[0], w[1], w[2], w[3]);
+          else
+            *reinterpret_cast<uint2 *>(ob + (size_t)slot * 8) = make_uint2(w[0], w[1]);
+        }
+      }
+    } else if (R.vec_load) {
       const int nv = span / V;
       for (int e = threadIdx.x; e < cnt * X * nv; e += blockDim.x) {
         const int row = (int)R.f_nv.div((uint32_t)e), bv = e - row * nv;
@@ -451,7 +496,29 @@ __global__ void __launch_bounds__(256) k_relayout_row(RowPlan R, const T *__rest
       const T *rb = rows + (size_t)o * rows_per;
       const int bc = s_bcombo[o], lo = s_lo[o];
       T val[V];
-      if (X >= V) {
+      if constexpr (RB > 0) {
+        const unsigned char *ob = reinterpret_cast<const unsigned char *>(rb);
+        constexpr int RUNS = 16 / RB;  // X-runs per 16-byte dst vector
+        uint32_t wv[4];
+#pragma unroll
+        for (int r = 0; r < RUNS; r++) {
+          const int pos = (w >> R.lgX) + r;
+          const int32_t bi = R.bstatic ? __ldg(R.sbc + pos) : __ldg(R.rev[R.b] + bc + __ldg(R.sbc + pos));
+          const int bl = bi - lo;
+          const int slot = bl ^ ((bl / V) & (V - 1));
+          if constexpr (RB == 16) {
+            uint4 q = make_uint4(0u, 0u, 0u, 0u);
+            if (bi >= 0) q = *reinterpret_cast<const uint4 *>(ob + (size_t)slot * 16);
+            wv[0] = q.x; wv[1] = q.y; wv[2] = q.z; wv[3] = q.w;
+          } else {
+            uint2 q = make_uint2(0u, 0u);
+            if (bi >= 0) q = *reinterpret_cast<const uint2 *>(ob + (size_t)slot * 8);
+            wv[2 * r] = q.x; wv[2 * r + 1] = q.y;
+          }
+        }
+        *reinterpret_cast<uint4 *>(dblk + (int64_t)v * V) = make_uint4(wv[0], wv[1], wv[2], wv[3]);
+        continue;
+      } else if (X >= V) {
         const int pos = w >> R.lgX, j0 = w & (X - 1);
         const int32_t bi = R.bstatic ? __ldg(R.sbc + pos) : __ldg(R.rev[R.b] + bc + __ldg(R.sbc + pos));
 #pragma unroll
@@ -533,6 +600,17 @@ static bool row_launch(Layout *S, const void *src, Layout *D, void *dst, int wb,
   span = (span + V - 1) / V * V;
   int64_t LbS = span;
   if ((LbS * wb) % 128 == 0) LbS += V;  // rows j and j + 1 on different banks
+  // transposed staging when an X-run is 8 or 16 bytes and rows load as vectors
+  bool vl0 = Lb % V == 0 && (reinterpret_cast<uintptr_t>(src) & 15) == 0;
+  for (int d = 0; d < S->lrank && vl0; d++) {
+    if (d == b) continue;
+    for (int64_t o : S->rd[d]) if (o >= 0 && o % V) { vl0 = false; break; }
+  }
+  static const bool no_tr = getenv("ALT_RELAYOUT_NOTR") != nullptr;  // developer A/B knob
+  // (measured: a win for 8-byte runs, e.g. the window-folded image 5.5x; for
+  // 16-byte runs the [X][window] form's wider stage parallelism is faster)
+  const int RB = (!no_tr && vl0 && X * wb == 8) ? 8 : 0;
+  if (RB) LbS = span;  // [window][X] runs, no row padding
   const size_t blk_smem = (size_t)X * LbS * wb;
   if (blk_smem > 32768) return false;
   RowPlan R{};
@@ -590,13 +668,19 @@ static bool row_launch(Layout *S, const void *src, Layout *D, void *dst, int wb,
   const size_t smem = (size_t)per * blk_smem;
   const int64_t iters = (nouter + per - 1) / per;
   const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(iters, (int64_t)nsm * 8));
+#define ROW_LAUNCH(T, RBV)                                                                               \
+  do {                                                                                                   \
+    cudaFuncSetAttribute(k_relayout_row<T, RBV>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem); \
+    k_relayout_row<T, RBV><<<grid, 256, smem, stream>>>(R, (const T *)src, (T *)dst);                    \
+  } while (0)
   if (wb == 2) {
-    cudaFuncSetAttribute(k_relayout_row<uint16_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    k_relayout_row<uint16_t><<<grid, 256, smem, stream>>>(R, (const uint16_t *)src, (uint16_t *)dst);
+    if (RB == 8) ROW_LAUNCH(uint16_t, 8);
+    else ROW_LAUNCH(uint16_t, 0);
   } else {
-    cudaFuncSetAttribute(k_relayout_row<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    k_relayout_row<uint32_t><<<grid, 256, smem, stream>>>(R, (const uint32_t *)src, (uint32_t *)dst);
+    if (RB == 8) ROW_LAUNCH(uint32_t, 8);
+    else ROW_LAUNCH(uint32_t, 0);
   }
+#undef ROW_LAUNCH
   count_launch();
   *st = cudaGetLastError() == cudaSuccess ? ALT_OK : ALT_E_CUDA;
   if (*st != ALT_OK) set_error("relayout (row) launch failed");
