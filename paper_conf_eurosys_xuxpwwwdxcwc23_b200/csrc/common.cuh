@@ -4,10 +4,36 @@
 #include <cuda_runtime.h>
 
 #include <cstdint>
+#include <utility>
 
 #include "layout.h"
 
 namespace alt {
+
+// Programmatic dependent launch for the CUDA-core kernels of a chain: the
+// kernel may be scheduled while the previous kernel in the stream drains
+// (its launch latency, and the next tensor-core kernel's prologue, overlap
+// work); pdl_wait() at the top of the kernel orders every global access after
+// the previous grid's completion.  Without the attribute both are no-ops.
+__device__ __forceinline__ void pdl_wait() {
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_pdl(void (*kern)(KArgs...), int grid, int block, size_t smem, cudaStream_t s,
+                              Args &&...args) {
+  cudaLaunchConfig_t lc{};
+  lc.gridDim = dim3((unsigned)grid);
+  lc.blockDim = dim3((unsigned)block);
+  lc.dynamicSmemBytes = smem;
+  lc.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  lc.attrs = at;
+  lc.numAttrs = 1;
+  return cudaLaunchKernelEx(&lc, kern, std::forward<Args>(args)...);
+}
 
 // Unsigned 32-bit division by a run-time constant (Granlund-Montgomery):
 // q = mulhi(n, mul) >> shr, valid for n, d < 2^31.

@@ -69,6 +69,7 @@ __device__ __forceinline__ DwItem dw_item(const DwArgs &a, uint32_t idx) {
 template <int R, int S>
 __global__ void __launch_bounds__(256, 2) k_dw_vec8(DwArgs a, const uint16_t *__restrict__ x,
                                                  const uint16_t *__restrict__ w, uint16_t *__restrict__ y) {
+  pdl_wait();
   for (uint32_t idx = blockIdx.x * blockDim.x + threadIdx.x; idx < a.total; idx += gridDim.x * blockDim.x) {
     const DwItem it = dw_item(a, idx);
     float acc[8];
@@ -162,6 +163,7 @@ __global__ void __launch_bounds__(256, 2) k_dw_vec8(DwArgs a, const uint16_t *__
 // bound by one load latency per tap.  Same (r, s) accumulation order.
 __global__ void __launch_bounds__(256, 2) k_dw3x3_fast(DwArgs a, const uint16_t *__restrict__ x,
                                                        const uint16_t *__restrict__ w, uint16_t *__restrict__ y) {
+  pdl_wait();
   for (uint32_t idx = blockIdx.x * blockDim.x + threadIdx.x; idx < a.total; idx += gridDim.x * blockDim.x) {
     const DwItem it = dw_item(a, idx);
     const int64_t base = __ldg(a.xrd[0] + it.n) + __ldg(a.xrd[1] + it.c0);
@@ -337,10 +339,10 @@ alt_status dw_conv(const ConvProblem &P, cudaStream_t stream, alt_kernel_cfg *us
   const auto *w = static_cast<const uint16_t *>(P.w);
   auto *y = static_cast<uint16_t *>(P.y);
   const bool fast = r3 && a.w_vec && a.vec_out && a.sb_vec && (!P.epi.residual || a.res_vec);
-  if (fast) k_dw3x3_fast<<<grid, 256, 0, stream>>>(a, x, w, y);
-  else if (r3) k_dw_vec8<3, 3><<<grid, 256, 0, stream>>>(a, x, w, y);
-  else if (r1) k_dw_vec8<1, 1><<<grid, 256, 0, stream>>>(a, x, w, y);
-  else k_dw_vec8<5, 5><<<grid, 256, 0, stream>>>(a, x, w, y);
+  if (fast) launch_pdl(k_dw3x3_fast, grid, 256, 0, stream, a, x, w, y);
+  else if (r3) launch_pdl(k_dw_vec8<3, 3>, grid, 256, 0, stream, a, x, w, y);
+  else if (r1) launch_pdl(k_dw_vec8<1, 1>, grid, 256, 0, stream, a, x, w, y);
+  else launch_pdl(k_dw_vec8<5, 5>, grid, 256, 0, stream, a, x, w, y);
   count_launch();
   if (cudaGetLastError() != cudaSuccess) { set_error("dw launch failed"); return ALT_E_CUDA; }
   alt_kernel_cfg u{};
@@ -368,6 +370,7 @@ struct PoolArgs {
 // average sums in (r, s) order in fp32 like the scalar kernel
 __global__ void __launch_bounds__(256) k_pool_vec8(PoolArgs a, const uint16_t *__restrict__ x,
                                                    uint16_t *__restrict__ y) {
+  pdl_wait();
   DwArgs d{};  // work-item decode shared with the depthwise kernel
   d.cvec = a.cvec; d.nrun = a.nrun; d.Wo = a.Wo; d.Ho = a.Ho;
   d.f_cvec = a.f_cvec; d.f_wo = a.f_wo; d.f_ho = a.f_ho; d.f_nrun = a.f_nrun;
@@ -501,7 +504,7 @@ alt_status pool2d(const ConvProblem &P, int kind, cudaStream_t stream) {
     a.f_cvec = FastDiv((uint32_t)a.cvec); a.f_wo = FastDiv((uint32_t)a.Wo);
     a.f_ho = FastDiv((uint32_t)a.Ho); a.f_nrun = FastDiv((uint32_t)a.nrun);
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((a.total + 255) / 256, 148 * 16));
-    k_pool_vec8<<<grid, 256, 0, stream>>>(a, static_cast<const uint16_t *>(P.x), static_cast<uint16_t *>(P.y));
+    launch_pdl(k_pool_vec8, grid, 256, 0, stream, a, static_cast<const uint16_t *>(P.x), static_cast<uint16_t *>(P.y));
     count_launch();
     if (cudaGetLastError() != cudaSuccess) { set_error("pool launch failed"); return ALT_E_CUDA; }
     return ALT_OK;

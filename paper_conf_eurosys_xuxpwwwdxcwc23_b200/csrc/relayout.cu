@@ -391,6 +391,7 @@ __global__ void __launch_bounds__(256) k_relayout_row(RowPlan R, const T *__rest
   __shared__ int32_t s_acombo[64];            // outer part of a's combo, or -1 for an all-zero block
   __shared__ int32_t s_bcombo[64], s_lo[64];  // outer part of b's combo, window start
   constexpr int V = 16 / sizeof(T);
+  pdl_wait();
   const int X = R.X, LbS = R.LbS, span = R.span;
   const int blk = R.npos * X;                 // dst elements per outer index
   const int rows_per = X * LbS;
@@ -671,7 +672,7 @@ static bool row_launch(Layout *S, const void *src, Layout *D, void *dst, int wb,
 #define ROW_LAUNCH(T, RBV)                                                                               \
   do {                                                                                                   \
     cudaFuncSetAttribute(k_relayout_row<T, RBV>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem); \
-    k_relayout_row<T, RBV><<<grid, 256, smem, stream>>>(R, (const T *)src, (T *)dst);                    \
+    launch_pdl(k_relayout_row<T, RBV>, grid, 256, smem, stream, R, (const T *)src, (T *)dst);           \
   } while (0)
   if (wb == 2) {
     if (RB == 8) ROW_LAUNCH(uint16_t, 8);
@@ -830,9 +831,11 @@ __global__ void __launch_bounds__(256) k_perm_trans(PermDims P, const T *__restr
     __syncthreads();
     if constexpr (TY >= 4 * V) {
       // wide Y: tile rows x; 16-byte loads along y, column-walk stores
-      for (int e = threadIdx.x; e < TX * (TY / V); e += blockDim.x) {
-        const int x = e / (TY / V), y = (e % (TY / V)) * V;
-        if (x >= nx || y >= ny) continue;
+      // loops cover the tile's valid nx x ny region only (tiny extents, e.g.
+      // 16 x 9 weight tiles, would otherwise scan mostly-empty slots)
+      const int nyv = (ny + V - 1) / V, nxv = (nx + V - 1) / V;
+      for (int e = threadIdx.x; e < nx * nyv; e += blockDim.x) {
+        const int x = e / nyv, y = (e - x * nyv) * V;
         const T *s = src + sb + (int64_t)x * P.sx + y;
         if (y + V <= ny && ((reinterpret_cast<uintptr_t>(s) & 15) == 0)) {
           *reinterpret_cast<uint4 *>(&tile[at(x, y)]) = ld16(s);
@@ -841,9 +844,8 @@ __global__ void __launch_bounds__(256) k_perm_trans(PermDims P, const T *__restr
         }
       }
       __syncthreads();
-      for (int e = threadIdx.x; e < TY * (TX / V); e += blockDim.x) {
-        const int y = e / (TX / V), x = (e % (TX / V)) * V;
-        if (y >= ny || x >= nx) continue;
+      for (int e = threadIdx.x; e < ny * nxv; e += blockDim.x) {
+        const int y = e / nxv, x = (e - y * nxv) * V;
         T *d = dst + db + (int64_t)y * P.dy + x;
         if (x + V <= nx && ((reinterpret_cast<uintptr_t>(d) & 15) == 0)) {
           T v[V];
@@ -858,9 +860,9 @@ __global__ void __launch_bounds__(256) k_perm_trans(PermDims P, const T *__restr
       // narrow Y (a few vectors per src run): tile rows y; neighbouring
       // threads load neighbouring x (coalesced when the runs are adjacent) and
       // scatter into rows y, stores are 16-byte vectors along x
-      for (int e = threadIdx.x; e < TX * (TY / V); e += blockDim.x) {
-        const int x = e % TX, y = (e / TX) * V;
-        if (x >= nx || y >= ny) continue;
+      const int nyv = (ny + V - 1) / V, nxv = (nx + V - 1) / V;
+      for (int e = threadIdx.x; e < nx * nyv; e += blockDim.x) {
+        const int yv = e / nx, x = e - yv * nx, y = yv * V;
         const T *s = src + sb + (int64_t)x * P.sx + y;
         if (y + V <= ny && ((reinterpret_cast<uintptr_t>(s) & 15) == 0)) {
           const uint4 u = ld16(s);
@@ -872,9 +874,8 @@ __global__ void __launch_bounds__(256) k_perm_trans(PermDims P, const T *__restr
         }
       }
       __syncthreads();
-      for (int e = threadIdx.x; e < TY * (TX / V); e += blockDim.x) {
-        const int y = e / (TX / V), x = (e % (TX / V)) * V;
-        if (y >= ny || x >= nx) continue;
+      for (int e = threadIdx.x; e < ny * nxv; e += blockDim.x) {
+        const int y = e / nxv, x = (e - y * nxv) * V;
         T *d = dst + db + (int64_t)y * P.dy + x;
         if (x + V <= nx && ((reinterpret_cast<uintptr_t>(d) & 15) == 0)) {
           *reinterpret_cast<uint4 *>(d) = *reinterpret_cast<const uint4 *>(&tile[y * TX + x]);
