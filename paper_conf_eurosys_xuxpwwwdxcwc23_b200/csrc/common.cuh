@@ -4,6 +4,7 @@
 #include <cuda_runtime.h>
 
 #include <cstdint>
+#include <cstdlib>
 #include <utility>
 
 #include "layout.h"
@@ -27,11 +28,12 @@ inline cudaError_t launch_pdl(void (*kern)(KArgs...), int grid, int block, size_
   lc.blockDim = dim3((unsigned)block);
   lc.dynamicSmemBytes = smem;
   lc.stream = s;
+  static const bool on = [] { const char *e = getenv("ALT_PDL_CC"); return !(e && e[0] == '0'); }();
   cudaLaunchAttribute at[1];
   at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
   at[0].val.programmaticStreamSerializationAllowed = 1;
   lc.attrs = at;
-  lc.numAttrs = 1;
+  lc.numAttrs = on ? 1 : 0;
   return cudaLaunchKernelEx(&lc, kern, std::forward<Args>(args)...);
 }
 

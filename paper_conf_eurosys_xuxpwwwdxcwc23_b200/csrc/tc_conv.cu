@@ -510,6 +510,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     const int lg_sw = sw_o == 32 ? 5 : (sw_o == 16 ? 4 : 3);  // sw_o is 8, 16 or 32
     const int nslab = 32 >> lg_sw;
     int32_t ocg[5], ocr[5];  // store coordinates per channel slab (tile, in-tile)
+    uint32_t sbuf_ctr = 0;   // TMA-store staging buffer parity (per warp, across tiles)
 #pragma unroll
     for (int d = 0; d < 5; d++) { ocg[d] = a.O.coef[d][V_GT]; ocr[d] = a.O.coef[d][V_GR]; }
     int i = 0;
@@ -749,7 +750,10 @@ __global__ void __launch_bounds__(kThreads, 1)
             // double-buffered staging, swizzled rows, one TMA store per slab;
             // no CTA-wide barrier.  Buffer `buf` is free once the store issued
             // two chunks ago has read it (<= 1 store group in flight per warp).
-            const uint32_t buf = (uint32_t)((c0 / kStep) & 1) * 2048u;
+            // alternate the two buffers across every chunk this warp stores
+            // (not per tile: with BLOCK_N 64 a tile is one chunk, and the
+            // previous tile's store may still be reading the other buffer)
+            const uint32_t buf = (uint32_t)(sbuf_ctr++ & 1u) * 2048u;
             if (lane == 0) bulk_wait_read1();
             __syncwarp();
 #pragma unroll
@@ -848,7 +852,7 @@ __global__ void __launch_bounds__(kThreads, 1)
 #pragma unroll
           for (int j = 0; j < 16; j++) pk[j] = pack_bf16x2(v[2 * j], v[2 * j + 1]);
         }
-        const uint32_t buf = (uint32_t)(cnt & 1) * 2048u;
+        const uint32_t buf = (uint32_t)(sbuf_ctr++ & 1u) * 2048u;
         if (lane == 0) bulk_wait_read1();
         __syncwarp();
 #pragma unroll

@@ -313,3 +313,34 @@ def test_tc_split_cluster_deterministic_and_unsupported():
     with pytest.raises(alt.AltError) as e:
         alt.conv2d(p, Lx, xd, Lw, wd, Ly, outs[0], residual=outs[1], residual_l=Ly, cfg=cfg)
     assert e.value.code == alt._alt.ALT_E_UNSUPPORTED
+
+
+# ------------------------------------------- TMA-store staging reuse --
+@pytest.mark.parametrize("C,K,R", [(16, 32, 3), (16, 64, 1), (3, 32, 3)])
+def test_tc_many_short_tiles_tma_store(C, K, R):
+    """Regression: BLOCK_N 64 tiles are one epilogue chunk each; with a short
+    mainloop (few input channels) a CTA stores tile after tile, and the
+    staging buffers must alternate across tiles (the previous tile's TMA store
+    may still be reading).  Batch 16 at 112x112 = 784+ tiles per launch; the
+    first images are the first tile of every CTA."""
+    N, H = 16, 112
+    x = synth.activations("ms%d%d" % (C, K), (N, C, H, H))
+    w = synth.weights("msw%d%d" % (C, K), (K, C, R, R))
+    if C % 8:
+        xp, wp = LY.conv_input_wfold(C, R, 1, R // 2), LY.kcrs_wfold(K, C, R)
+    else:
+        xp, wp = LY.nchwxc(C, C), LY.kcrs_yk_xc(K, C, K, C)
+    yp = LY.nchwxc(K, 32)
+    Ox, _, xd = make_operand("msx", xp, x, torch.bfloat16)
+    Ow, wph, wd = make_operand("msw", wp, w, torch.bfloat16)
+    Lx, Lw, Ly = alt.Layout(x.shape, xp), alt.Layout(w.shape, wp), alt.Layout((N, K, H, H), yp)
+    y = torch.full(Ly.phys_shape, 3.0, dtype=torch.bfloat16, device="cuda")
+    alt.conv2d(alt.conv_params(N, C, H, H, K, R, R, 1, R // 2), Lx, xd, Lw, wd, Ly, y,
+               cfg={"path": alt.PATH_TC, "block_n": 64})
+    torch.cuda.synchronize()
+    assert alt.last_plan()["path"] == alt.PATH_TC
+    pd = dict(N=1, C=C, H=H, W=H, K=K, R=R, S=R, stride_h=1, stride_w=1, pad_h=R // 2, pad_w=R // 2)
+    Ox1, Oy1 = oracle.Layout((1, C, H, H), xp), oracle.Layout((1, K, H, H), yp)
+    for n in (0, 1, N - 1):
+        ref = oracle.conv2d(pd, Ox1, words(xd[n:n + 1]), Ow, wph)
+        assert_parity(Oy1.read_f64(words(y[n:n + 1])), ref, torch.bfloat16)
