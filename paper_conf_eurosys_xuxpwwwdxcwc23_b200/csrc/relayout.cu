@@ -831,11 +831,9 @@ __global__ void __launch_bounds__(256) k_perm_trans(PermDims P, const T *__restr
     __syncthreads();
     if constexpr (TY >= 4 * V) {
       // wide Y: tile rows x; 16-byte loads along y, column-walk stores
-      // loops cover the tile's valid nx x ny region only (tiny extents, e.g.
-      // 16 x 9 weight tiles, would otherwise scan mostly-empty slots)
-      const int nyv = (ny + V - 1) / V, nxv = (nx + V - 1) / V;
-      for (int e = threadIdx.x; e < nx * nyv; e += blockDim.x) {
-        const int x = e / nyv, y = (e - x * nyv) * V;
+      for (int e = threadIdx.x; e < TX * (TY / V); e += blockDim.x) {
+        const int x = e / (TY / V), y = (e % (TY / V)) * V;
+        if (x >= nx || y >= ny) continue;
         const T *s = src + sb + (int64_t)x * P.sx + y;
         if (y + V <= ny && ((reinterpret_cast<uintptr_t>(s) & 15) == 0)) {
           *reinterpret_cast<uint4 *>(&tile[at(x, y)]) = ld16(s);
@@ -844,8 +842,9 @@ __global__ void __launch_bounds__(256) k_perm_trans(PermDims P, const T *__restr
         }
       }
       __syncthreads();
-      for (int e = threadIdx.x; e < ny * nxv; e += blockDim.x) {
-        const int y = e / nxv, x = (e - y * nxv) * V;
+      for (int e = threadIdx.x; e < TY * (TX / V); e += blockDim.x) {
+        const int y = e / (TX / V), x = (e % (TX / V)) * V;
+        if (y >= ny || x >= nx) continue;
         T *d = dst + db + (int64_t)y * P.dy + x;
         if (x + V <= nx && ((reinterpret_cast<uintptr_t>(d) & 15) == 0)) {
           T v[V];
@@ -860,9 +859,9 @@ __global__ void __launch_bounds__(256) k_perm_trans(PermDims P, const T *__restr
       // narrow Y (a few vectors per src run): tile rows y; neighbouring
       // threads load neighbouring x (coalesced when the runs are adjacent) and
       // scatter into rows y, stores are 16-byte vectors along x
-      const int nyv = (ny + V - 1) / V, nxv = (nx + V - 1) / V;
-      for (int e = threadIdx.x; e < nx * nyv; e += blockDim.x) {
-        const int yv = e / nx, x = e - yv * nx, y = yv * V;
+      for (int e = threadIdx.x; e < TX * (TY / V); e += blockDim.x) {
+        const int x = e % TX, y = (e / TX) * V;
+        if (x >= nx || y >= ny) continue;
         const T *s = src + sb + (int64_t)x * P.sx + y;
         if (y + V <= ny && ((reinterpret_cast<uintptr_t>(s) & 15) == 0)) {
           const uint4 u = ld16(s);
@@ -874,8 +873,9 @@ __global__ void __launch_bounds__(256) k_perm_trans(PermDims P, const T *__restr
         }
       }
       __syncthreads();
-      for (int e = threadIdx.x; e < ny * nxv; e += blockDim.x) {
-        const int y = e / nxv, x = (e - y * nxv) * V;
+      for (int e = threadIdx.x; e < TY * (TX / V); e += blockDim.x) {
+        const int y = e / (TX / V), x = (e % (TX / V)) * V;
+        if (y >= ny || x >= nx) continue;
         T *d = dst + db + (int64_t)y * P.dy + x;
         if (x + V <= nx && ((reinterpret_cast<uintptr_t>(d) & 15) == 0)) {
           *reinterpret_cast<uint4 *>(d) = *reinterpret_cast<const uint4 *>(&tile[y * TX + x]);
@@ -883,6 +883,56 @@ __global__ void __launch_bounds__(256) k_perm_trans(PermDims P, const T *__restr
           for (int j = 0; j < V && x + j < nx; j++) d[j] = tile[y * TX + x + j];
         }
       }
+    }
+  }
+}
+
+
+// register transpose: one thread moves a V x V block (V = 16 / sizeof(T)):
+// V 16-byte loads along Y (src-contiguous) from V consecutive X rows, a
+// V x V transpose in registers (byte_perm for 16-bit words), V 16-byte stores
+// along X (dst-contiguous).  Neighbouring threads take neighbouring Y blocks,
+// so both the loads (per X row) and the stores (per Y row, when dst rows of
+// consecutive y are adjacent, e.g. NCHW -> NCHW[V]c) coalesce; no shared
+// memory and no barriers.  Needs ex % V == ey % V == 0 and V-aligned strides.
+template <typename T>
+__global__ void __launch_bounds__(256) k_perm_rt(PermDims P, const T *__restrict__ src, T *__restrict__ dst,
+                                               uint32_t nblk) {
+  pdl_wait();  // launched with launch_pdl: no global access before the previous grid completes
+  constexpr int V = 16 / sizeof(T);
+  const uint32_t byn = (uint32_t)(P.ey / V), bxn = (uint32_t)(P.ex / V);
+  for (uint32_t t = blockIdx.x * blockDim.x + threadIdx.x; t < nblk; t += gridDim.x * blockDim.x) {
+    uint32_t rem = t;
+    const uint32_t by = rem % byn;
+    rem /= byn;
+    const uint32_t bx = rem % bxn;
+    rem /= bxn;
+    int64_t sb = 0, db = 0;
+    for (int k = P.nd - 1; k >= 0; k--) {
+      uint32_t q, r;
+      P.ext[k].divmod(rem, q, r);
+      sb += (int64_t)r * P.sstr[k];
+      db += (int64_t)r * P.dstr[k];
+      rem = q;
+    }
+    const int64_t x0 = (int64_t)bx * V, y0 = (int64_t)by * V;
+    uint4 u[V];
+#pragma unroll
+    for (int j = 0; j < V; j++) u[j] = ld16(src + sb + (x0 + j) * P.sx + y0);
+#pragma unroll
+    for (int k = 0; k < V; k++) {
+      uint32_t w[4];
+      if constexpr (sizeof(T) == 2) {
+        const uint32_t sel = (k & 1) ? 0x7632u : 0x5410u;
+#pragma unroll
+        for (int jp = 0; jp < 4; jp++)
+          w[jp] = __byte_perm(reinterpret_cast<const uint32_t *>(&u[2 * jp])[k >> 1],
+                              reinterpret_cast<const uint32_t *>(&u[2 * jp + 1])[k >> 1], sel);
+      } else {
+#pragma unroll
+        for (int j = 0; j < 4; j++) w[j] = reinterpret_cast<const uint32_t *>(&u[j])[k];
+      }
+      *reinterpret_cast<uint4 *>(dst + db + (y0 + k) * P.dy + x0) = make_uint4(w[0], w[1], w[2], w[3]);
     }
   }
 }
@@ -925,6 +975,24 @@ static bool perm_launch(Layout *S, const void *src, Layout *D, void *dst, int wb
   } else {
     P.ey = r[iy].ext;
     P.dy = r[iy].dstr;
+    static const bool no_rt = getenv("ALT_RELAYOUT_NORT") != nullptr;  // developer A/B knob
+    // only where the stores coalesce too: a thread's V stores are adjacent
+    // (dst X extent = one vector, e.g. NCHW -> NCHW[V]c) or there is a single
+    // Y block (lanes step along X, e.g. NCHW[V]c -> NCHW); measured, the other
+    // shapes are faster through the shared-memory tile
+    bool rt = !no_rt && P.ex % V == 0 && P.ey % V == 0 && P.sx % V == 0 && P.dy % V == 0 &&
+              (P.dy == V || P.ey == V);
+    for (int k = 0; k < nd && rt; k++) rt = P.sstr[k] % V == 0 && P.dstr[k] % V == 0;
+    const int64_t nblk = rt ? D->pnumel / (V * V) : 0;
+    if (rt && nblk < (1ll << 31)) {
+      const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((nblk + 255) / 256, (int64_t)nsm * 16));
+      if (wb == 2) launch_pdl(k_perm_rt<uint16_t>, grid, 256, 0, stream, P, (const uint16_t *)src, (uint16_t *)dst, (uint32_t)nblk);
+      else launch_pdl(k_perm_rt<uint32_t>, grid, 256, 0, stream, P, (const uint32_t *)src, (uint32_t *)dst, (uint32_t)nblk);
+      count_launch();
+      *st = cudaGetLastError() == cudaSuccess ? ALT_OK : ALT_E_CUDA;
+      if (*st != ALT_OK) set_error("relayout (register transpose) launch failed");
+      return true;
+    }
     // tile shape: TX x TY elements (16 KB), the pair wasting
     // the fewest elements on ragged edges (larger square-ish tiles on ties)
     const int64_t area = 16384 / wb;  // 16 KB of shared memory per tile
