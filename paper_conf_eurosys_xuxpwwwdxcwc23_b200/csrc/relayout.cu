@@ -895,18 +895,40 @@ __global__ void __launch_bounds__(256) k_perm_trans(PermDims P, const T *__restr
 // so both the loads (per X row) and the stores (per Y row, when dst rows of
 // consecutive y are adjacent, e.g. NCHW -> NCHW[V]c) coalesce; no shared
 // memory and no barriers.  Needs ex % V == ey % V == 0 and V-aligned strides.
+// Lane mapping: a warp covers LX x-blocks by LY y-blocks (LX * LY = 32,
+// y-blocks fastest), so a load instruction reads LY * 16 contiguous bytes of
+// each of the lanes' src rows and a store instruction writes LX * 16
+// contiguous bytes of each dst row.
 template <typename T>
 __global__ void __launch_bounds__(256) k_perm_rt(PermDims P, const T *__restrict__ src, T *__restrict__ dst,
-                                               uint32_t nblk) {
+                                               uint32_t nblk, int lgLY) {
   pdl_wait();  // launched with launch_pdl: no global access before the previous grid completes
   constexpr int V = 16 / sizeof(T);
+  // lgLY < 0: flat mapping (y-blocks, then x-blocks, then batch, fastest
+  // first) — used when a thread's V stores are adjacent (dy == V) or there is
+  // one y-block (ey == V) and the warp tiling does not divide the extents
+  const int lg = lgLY < 0 ? 0 : lgLY;
+  const uint32_t LY = 1u << lg, LX = 32u >> lg;
   const uint32_t byn = (uint32_t)(P.ey / V), bxn = (uint32_t)(P.ex / V);
+  const uint32_t gyn = byn / LY, gxn = bxn / LX;  // warp tiles along y / x
   for (uint32_t t = blockIdx.x * blockDim.x + threadIdx.x; t < nblk; t += gridDim.x * blockDim.x) {
-    uint32_t rem = t;
-    const uint32_t by = rem % byn;
-    rem /= byn;
-    const uint32_t bx = rem % bxn;
-    rem /= bxn;
+    uint32_t rem, by, bx;
+    if (lgLY < 0) {
+      rem = t;
+      by = rem % byn;
+      rem /= byn;
+      bx = rem % bxn;
+      rem /= bxn;
+    } else {
+      const uint32_t lane = t & 31u;
+      rem = t >> 5;
+      const uint32_t gy = rem % gyn;
+      rem /= gyn;
+      const uint32_t gx = rem % gxn;
+      rem /= gxn;
+      by = gy * LY + (lane & (LY - 1));
+      bx = gx * LX + (lane >> lg);
+    }
     int64_t sb = 0, db = 0;
     for (int k = P.nd - 1; k >= 0; k--) {
       uint32_t q, r;
@@ -976,18 +998,27 @@ static bool perm_launch(Layout *S, const void *src, Layout *D, void *dst, int wb
     P.ey = r[iy].ext;
     P.dy = r[iy].dstr;
     static const bool no_rt = getenv("ALT_RELAYOUT_NORT") != nullptr;  // developer A/B knob
-    // only where the stores coalesce too: a thread's V stores are adjacent
-    // (dst X extent = one vector, e.g. NCHW -> NCHW[V]c) or there is a single
-    // Y block (lanes step along X, e.g. NCHW[V]c -> NCHW); measured, the other
-    // shapes are faster through the shared-memory tile
-    bool rt = !no_rt && P.ex % V == 0 && P.ey % V == 0 && P.sx % V == 0 && P.dy % V == 0 &&
-              (P.dy == V || P.ey == V);
+    // both the loads (LY y-blocks per src row) and the stores (LX x-blocks
+    // per dst row) coalesce for any V-divisible extents (lane mapping below)
+    bool rt = !no_rt && P.ex % V == 0 && P.ey % V == 0 && P.sx % V == 0 && P.dy % V == 0;
     for (int k = 0; k < nd && rt; k++) rt = P.sstr[k] % V == 0 && P.dstr[k] % V == 0;
+    // lanes per y-row: as many y-blocks as there are (<= 32), the rest along x
+    int lgLY = 5;
+    if (rt) {
+      const int64_t byn = P.ey / V, bxn = P.ex / V;
+      while (lgLY > 0 && (byn % (1ll << lgLY) != 0 || bxn % (32ll >> lgLY) != 0)) lgLY--;
+      if (byn % (1ll << lgLY) != 0 || bxn % (32ll >> lgLY) != 0) {
+        if (P.dy == V || P.ey == V) lgLY = -1;  // flat mapping still coalesces
+        else rt = false;
+      } else if (P.dy == V && lgLY == 5) {
+        lgLY = -1;  // same lanes as the 32 x 1 tiling, cheaper decode
+      }
+    }
     const int64_t nblk = rt ? D->pnumel / (V * V) : 0;
     if (rt && nblk < (1ll << 31)) {
       const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((nblk + 255) / 256, (int64_t)nsm * 16));
-      if (wb == 2) launch_pdl(k_perm_rt<uint16_t>, grid, 256, 0, stream, P, (const uint16_t *)src, (uint16_t *)dst, (uint32_t)nblk);
-      else launch_pdl(k_perm_rt<uint32_t>, grid, 256, 0, stream, P, (const uint32_t *)src, (uint32_t *)dst, (uint32_t)nblk);
+      if (wb == 2) launch_pdl(k_perm_rt<uint16_t>, grid, 256, 0, stream, P, (const uint16_t *)src, (uint16_t *)dst, (uint32_t)nblk, lgLY);
+      else launch_pdl(k_perm_rt<uint32_t>, grid, 256, 0, stream, P, (const uint32_t *)src, (uint32_t *)dst, (uint32_t)nblk, lgLY);
       count_launch();
       *st = cudaGetLastError() == cudaSuccess ? ALT_OK : ALT_E_CUDA;
       if (*st != ALT_OK) set_error("relayout (register transpose) launch failed");
