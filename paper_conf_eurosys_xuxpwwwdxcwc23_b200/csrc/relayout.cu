@@ -910,7 +910,7 @@ __global__ void __launch_bounds__(256) k_perm_rt(PermDims P, const T *__restrict
   const int lg = lgLY < 0 ? 0 : lgLY;
   const uint32_t LY = 1u << lg, LX = 32u >> lg;
   const uint32_t byn = (uint32_t)(P.ey / V), bxn = (uint32_t)(P.ex / V);
-  const uint32_t gyn = byn / LY, gxn = bxn / LX;  // warp tiles along y / x
+  const uint32_t gyn = (byn + LY - 1) / LY, gxn = bxn / LX;  // warp tiles along y (ragged) / x
   for (uint32_t t = blockIdx.x * blockDim.x + threadIdx.x; t < nblk; t += gridDim.x * blockDim.x) {
     uint32_t rem, by, bx;
     if (lgLY < 0) {
@@ -928,6 +928,7 @@ __global__ void __launch_bounds__(256) k_perm_rt(PermDims P, const T *__restrict
       rem /= gxn;
       by = gy * LY + (lane & (LY - 1));
       bx = gx * LX + (lane >> lg);
+      if (by >= byn) continue;  // ragged last y tile
     }
     int64_t sb = 0, db = 0;
     for (int k = P.nd - 1; k >= 0; k--) {
@@ -1006,15 +1007,22 @@ static bool perm_launch(Layout *S, const void *src, Layout *D, void *dst, int wb
     int lgLY = 5;
     if (rt) {
       const int64_t byn = P.ey / V, bxn = P.ex / V;
-      while (lgLY > 0 && (byn % (1ll << lgLY) != 0 || bxn % (32ll >> lgLY) != 0)) lgLY--;
-      if (byn % (1ll << lgLY) != 0 || bxn % (32ll >> lgLY) != 0) {
-        if (P.dy == V || P.ey == V) lgLY = -1;  // flat mapping still coalesces
-        else rt = false;
-      } else if (P.dy == V && lgLY == 5) {
-        lgLY = -1;  // same lanes as the 32 x 1 tiling, cheaper decode
+      // LX x-blocks (<= 8, dividing bxn) per dst row and LY = 32 / LX y-blocks
+      // per src row: both sides move >= 64 contiguous bytes per instruction
+      int LX = 1;
+      while (LX < 8 && bxn % (LX * 2) == 0) LX *= 2;
+      lgLY = 5;
+      while ((32 >> lgLY) < LX) lgLY--;
+      if ((1ll << lgLY) > byn * 2 || LX == 1) {  // most y lanes idle / one x-block
+        if (P.dy == V || P.ey == V) lgLY = -1;   // flat mapping coalesces here
+        else if (LX == 1) rt = false;
       }
     }
-    const int64_t nblk = rt ? D->pnumel / (V * V) : 0;
+    int64_t nblk = rt ? D->pnumel / (V * V) : 0;
+    if (rt && lgLY >= 0) {  // threads = 32 x warp tiles x batch (the last y tile may be ragged)
+      const int64_t byn = P.ey / V, bxn = P.ex / V, LY = 1ll << lgLY, LX = 32 >> lgLY;
+      nblk = 32 * ((byn + LY - 1) / LY) * (bxn / LX) * (D->pnumel / (P.ex * P.ey));
+    }
     if (rt && nblk < (1ll << 31)) {
       const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((nblk + 255) / 256, (int64_t)nsm * 16));
       if (wb == 2) launch_pdl(k_perm_rt<uint16_t>, grid, 256, 0, stream, P, (const uint16_t *)src, (uint16_t *)dst, (uint32_t)nblk, lgLY);
