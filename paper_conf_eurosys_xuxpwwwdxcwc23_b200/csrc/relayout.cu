@@ -538,6 +538,70 @@ __global__ void __launch_bounds__(256) k_relayout_row(RowPlan R, const T *__rest
   }
 }
 
+
+// K_ROW, identity suffix (dst positions = the b indices in order, e.g. the
+// padded-channel image layout N C/8 H W 8c) with 16-byte X-runs: no staging —
+// a thread loads one 16-byte b-vector of each of the X rows (pad rows are
+// zeros), transposes it in registers and stores the V runs, which are
+// adjacent in dst.  Neighbouring threads take neighbouring b-vectors.
+template <typename T>
+__global__ void __launch_bounds__(256) k_relayout_row_ident(RowPlan R, const T *__restrict__ src,
+                                                            T *__restrict__ dst, uint32_t nthr) {
+  pdl_wait();
+  constexpr int V = 16 / sizeof(T);
+  constexpr int X = V;  // 16-byte runs
+  const uint32_t nv = (uint32_t)(R.Lb / V);
+  for (uint32_t t = blockIdx.x * blockDim.x + threadIdx.x; t < nthr; t += gridDim.x * blockDim.x) {
+    const uint32_t o = t / nv, bv = t - o * nv;
+    uint32_t rem = o;
+    int32_t combo[kMaxL];
+#pragma unroll
+    for (int d = 0; d < kMaxL; d++) combo[d] = 0;
+    for (int k = R.nout - 1; k >= 0; k--) {
+      uint32_t q, r;
+      R.odiv[k].divmod(rem, q, r);
+      combo[R.oowner[k]] += (int32_t)r * R.orad[k];
+      rem = q;
+    }
+    int64_t base = 0;
+    bool ok = true;
+    for (int d = 0; d < R.lrank; d++) {
+      if (d == R.a || d == R.b) continue;
+      const int32_t i = __ldg(R.rev[d] + combo[d]);
+      if (i < 0) { ok = false; break; }
+      base += __ldg(R.rd[d] + i);
+    }
+    uint4 u[X];
+#pragma unroll
+    for (int j = 0; j < X; j++) {
+      const int32_t ai = ok ? __ldg(R.rev[R.a] + combo[R.a] + j) : -1;
+      u[j] = ai < 0 ? make_uint4(0u, 0u, 0u, 0u)
+                    : __ldg(reinterpret_cast<const uint4 *>(src + base + __ldg(R.rd[R.a] + ai) + (int64_t)bv * V));
+    }
+    T *d = dst + (int64_t)o * (R.npos * X) + (int64_t)bv * V * X;
+#pragma unroll
+    for (int k = 0; k < V; k++) {
+      uint32_t w[4];
+      if constexpr (sizeof(T) == 2) {
+        const uint32_t sel = (k & 1) ? 0x7632u : 0x5410u;
+#pragma unroll
+        for (int jp = 0; jp < 4; jp++)
+          w[jp] = __byte_perm(reinterpret_cast<const uint32_t *>(&u[2 * jp])[k >> 1],
+                              reinterpret_cast<const uint32_t *>(&u[2 * jp + 1])[k >> 1], sel);
+      } else {
+#pragma unroll
+        for (int j = 0; j < 4; j++) w[j] = reinterpret_cast<const uint32_t *>(&u[j])[k];
+      }
+      *reinterpret_cast<uint4 *>(d + k * X) = make_uint4(w[0], w[1], w[2], w[3]);
+    }
+  }
+}
+
+// position q of the suffix holds b index q (no pad / unfold of b)
+static bool bmap_static_is(const Layout *D, int b, const std::vector<int32_t> &sbc, int64_t q) {
+  return D->rev[b][sbc[(size_t)q]] == q;
+}
+
 // host side of K_ROW: returns false (nothing launched) when not applicable
 static bool row_launch(Layout *S, const void *src, Layout *D, void *dst, int wb, const SepDev &ss,
                        const SepDev &ds, cudaStream_t stream, int nsm, alt_status *st) {
@@ -664,6 +728,24 @@ static bool row_launch(Layout *S, const void *src, Layout *D, void *dst, int wb,
     for (int64_t o : S->rd[d]) if (o >= 0 && o % V) { vl = false; break; }
   }
   R.vec_load = vl ? 1 : 0;
+  // identity suffix with 16-byte runs: the staging-free register-transpose form
+  {
+    bool ident = R.bstatic && npos == Lb && X * wb == 16 && vl0;
+    for (int64_t q = 0; q < npos && ident; q++) ident = bmap_static_is(D, b, sbc, q);
+    static const bool no_id = getenv("ALT_RELAYOUT_NOID") != nullptr;  // developer A/B knob
+    if (ident && !no_id) {
+      const int64_t nthr = nouter * (Lb / V);
+      if (nthr < (1ll << 31)) {
+        const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((nthr + 255) / 256, (int64_t)nsm * 16));
+        if (wb == 2) launch_pdl(k_relayout_row_ident<uint16_t>, grid, 256, 0, stream, R, (const uint16_t *)src, (uint16_t *)dst, (uint32_t)nthr);
+        else launch_pdl(k_relayout_row_ident<uint32_t>, grid, 256, 0, stream, R, (const uint32_t *)src, (uint32_t *)dst, (uint32_t)nthr);
+        count_launch();
+        *st = cudaGetLastError() == cudaSuccess ? ALT_OK : ALT_E_CUDA;
+        if (*st != ALT_OK) set_error("relayout (row, identity) launch failed");
+        return true;
+      }
+    }
+  }
   int per = (int)std::max<int64_t>(1, std::min<int64_t>(64, 16384 / (int64_t)blk_smem));
   R.per_iter = per;
   const size_t smem = (size_t)per * blk_smem;
