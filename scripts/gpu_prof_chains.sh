@@ -13,7 +13,7 @@ prof.start(); ch.run(); torch.cuda.synchronize(); prof.stop()
 PY
 for w in mv2 r18; do
   timeout 900 ncu --set full --clock-control none --profile-from-start off -o $O/$w python /tmp/one_chain.py $w > $O/$w.log 2>&1; echo "$w rc=$?"
-  python scripts/ncu_table.py $O/$w.ncu-rep $O/${w}_table.txt > /dev/null 2>&1; tail -2 $O/${w}_table.txt
+  python scripts/ncu_table.py $O/$w.ncu-rep $O/${w}_table.txt > /dev/null 2>&1; tail -2 $O/${w}_table.txt; rm -f $O/$w.ncu-rep
 done
 cat > /tmp/relayout_set.py <<'PY'
 import sys, torch
@@ -33,4 +33,4 @@ for S, src, D, dst in items: alt.relayout(S, src, D, dst)
 torch.cuda.synchronize(); prof.stop()
 PY
 timeout 900 ncu --set full --clock-control none --profile-from-start off -o $O/relayout python /tmp/relayout_set.py > $O/relayout.log 2>&1; echo "relayout rc=$?"
-python scripts/ncu_table.py $O/relayout.ncu-rep $O/relayout_table.txt > /dev/null 2>&1; cat $O/relayout_table.txt
+python scripts/ncu_table.py $O/relayout.ncu-rep $O/relayout_table.txt > /dev/null 2>&1; cat $O/relayout_table.txt; rm -f $O/relayout.ncu-rep
