@@ -9,7 +9,7 @@ import paper_conf_eurosys_xuxpwwwdxcwc23_b200 as alt
 from paper_conf_eurosys_xuxpwwwdxcwc23_b200 import _alt
 lib = _alt._lib
 lib.alt__debug_tc.argtypes = [ctypes.c_void_p, ctypes.c_int64]
-names = {32: "prologue done (before griddep wait)", 4: "epi: partial written", 7: "epi: last decided", 0: "start", 1: "setup done", 3: "mma: tile0 committed", 5: "epi: all done", 6: "end",
+names = {33: "pro: barriers init", 34: "pro: tmem alloc (warp 1)", 35: "pro: slab table", 32: "prologue done (before griddep wait)", 4: "epi: partial written", 7: "epi: last decided", 0: "start", 1: "setup done", 3: "mma: tile0 committed", 5: "epi: all done", 6: "end",
          24: "prod: before empty wait", 25: "prod: after empty wait", 26: "mma: before tempty", 27: "mma: after tempty",
          28: "mma: first full", 29: "mma: commit tfull", 2: "epi: tfull", 30: "epi: sb staged", 8: "epi: c0 ld",
          9: "epi: c0 math", 10: "epi: c0 smem", 11: "epi: c0 store", 31: "epi: tile end"}
