@@ -143,3 +143,13 @@ def test_plan_chain_matches_oracle():
     # non-trivial advanced primitive stops propagation with a conversion
     unf = [("pad", 2, 1, 1), ("unfold", 2, 10, 8)]
     _plan_case(["complex", "elementwise"], [(None, 0, S, 0), (0, 1, S, 0), (1, None, S, 0)], {1: unf})
+
+
+def test_zero_extent_layouts_are_rejected():
+    """a layout needs every logical extent >= 1 (empty batches are handled
+    by the operators themselves: N = 0 / M = 0 calls are no-ops)"""
+    import paper_conf_eurosys_xuxpwwwdxcwc23_b200 as alt
+    for shp in [(0, 16, 4, 4), (5, 0)]:
+        with pytest.raises(alt.AltError) as e:
+            alt.Layout(shp, [])
+        assert e.value.code == alt._alt.ALT_E_INVALID
