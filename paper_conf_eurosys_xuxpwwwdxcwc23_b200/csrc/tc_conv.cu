@@ -287,8 +287,10 @@ __global__ void __launch_bounds__(kThreads, 1)
       mbar_init(&tempty[s], kEpiWarps * CG);  // every epilogue warp of the pair
     }
     fence_mbar_init();
+    DBG(33);
   }
   if (warp == 1) tmem_alloc<NACC * BN, CG>(tmem_slot);
+  if (threadIdx.x == 32) { DBG(34); }
   // slab table (see kTabSlabs): slab -> (tap r, s; channel slab g = (gt, gr))
   int32_t *tab = reinterpret_cast<int32_t *>(smem + L::kTab);
   const int padded_slabs = a.num_iters * a.spi;
@@ -311,6 +313,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       }
     }
   }
+  if (threadIdx.x == 0) { DBG(35); }
   tc_fence_before();
   __syncthreads();
   if constexpr (CG == 2) cluster_sync();  // peer barriers initialised before any remote arrive

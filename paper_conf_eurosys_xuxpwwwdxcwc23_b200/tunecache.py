@@ -49,3 +49,21 @@ def store(op: str, L, N: int, result: dict, dtype: str = "bf16"):
     with open(_PATH, "w") as f:
         for v in c.values():
             f.write(json.dumps(v) + "\n")
+
+
+def gemm_key(M: int, N: int, K: int, dtype: str = "bf16") -> str:
+    return f"matmul|M{M}|N{N}|K{K}|{dtype}"
+
+
+def lookup_gemm(M: int, N: int, K: int, dtype: str = "bf16"):
+    """kernel configuration for a GEMM on the bench's tiled layouts, or None"""
+    e = _load().get(gemm_key(M, N, K, dtype))
+    return None if e is None else e["cfg"]
+
+
+def store_gemm(M: int, N: int, K: int, cfg: dict, us: float, dtype: str = "bf16"):
+    c = _load()
+    c[gemm_key(M, N, K, dtype)] = {"key": gemm_key(M, N, K, dtype), "cfg": cfg, "us": us}
+    with open(_PATH, "w") as f:
+        for v in c.values():
+            f.write(json.dumps(v) + "\n")
