@@ -98,7 +98,9 @@ constexpr int kOutStage = 128 * 64 * 2;  // one 64-column bf16 chunk of the tile
 // accumulator buffers in TMEM (512 columns): the MMA of tile i + NACC - 1
 // may run while the epilogue drains tile i
 template <int BN>
-struct Nacc { static constexpr int value = BN >= 256 ? 2 : 4; };
+struct Nacc { static constexpr int value = BN >= 192 ? 2 : 4; };
+// TMEM allocations are powers of two >= 32 columns
+constexpr int tmem_cols(int c) { return c <= 32 ? 32 : (c <= 64 ? 64 : (c <= 128 ? 128 : (c <= 256 ? 256 : 512))); }
 
 // Reduction-slab coordinate table: for every slab (filter tap x channel
 // slab) of the reduction, the part of the A / B box coordinates that depends
@@ -289,7 +291,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     fence_mbar_init();
     DBG(33);
   }
-  if (warp == 1) tmem_alloc<NACC * BN, CG>(tmem_slot);
+  if (warp == 1) tmem_alloc<tmem_cols(NACC * BN), CG>(tmem_slot);
   if (threadIdx.x == 32) { DBG(34); }
   // slab table (see kTabSlabs): slab -> (tap r, s; channel slab g = (gt, gr))
   int32_t *tab = reinterpret_cast<int32_t *>(smem + L::kTab);
@@ -895,7 +897,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   tc_fence_before();
   __syncthreads();
   if constexpr (CG == 2 || SC > 1) cluster_sync();  // the pair's MMAs / the peers' DSMEM reads are done
-  if (warp == 1) tmem_dealloc<NACC * BN, CG>(tmem);
+  if (warp == 1) tmem_dealloc<tmem_cols(NACC * BN), CG>(tmem);
   if (threadIdx.x == 32) { DBG(6); }
 }
 
@@ -1367,13 +1369,14 @@ static std::unordered_map<TcKey, TcPlan, TcKeyHash> g_tc_cache;
 // smem-ring depth per (BLOCK_N, CTA group): the deepest ring that fits 227 KB
 // next to the kEpiWarps staging buffers and the slab table
 constexpr int stages_for(int BN, int CG) {
-  return kEpiWarps == 8 ? (CG == 2 ? (BN == 128 ? 7 : 5) : (BN == 64 ? 7 : (BN == 128 ? 5 : 3)))
+  return kEpiWarps == 8 ? (CG == 2 ? (BN == 128 ? 7 : 5) : (BN == 64 ? 7 : (BN == 128 ? 5 : 3)))  // BN 192: pair, 5
                         : (CG == 2 ? (BN == 128 ? 5 : 4) : (BN == 64 ? 5 : (BN == 128 ? 4 : 3)));
 }
 template <bool RV>
 static cudaError_t launch_plan_rv(const TcPlan &pl, uint16_t *yy, cudaStream_t stream) {
   if (pl.cg == 2) {
     if (pl.BN == 128) return launch_tc<128, stages_for(128, 2), 2, RV>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+    if (pl.BN == 192) return launch_tc<192, stages_for(192, 2), 2, RV>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
     return launch_tc<256, stages_for(256, 2), 2, RV>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
   }
   if (pl.BN == 64) return launch_tc<64, stages_for(64, 1), 1, RV>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
@@ -1476,11 +1479,12 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
     });
   }
   int BN = cfg && cfg->block_n ? cfg->block_n : (P.K > 128 ? 256 : (P.K > 64 ? 128 : 64));
-  if (BN != 64 && BN != 128 && BN != 256) { set_error("tc: block_n must be 64/128/256"); return ALT_E_UNSUPPORTED; }
+  if (BN != 64 && BN != 128 && BN != 192 && BN != 256) { set_error("tc: block_n must be 64/128/192/256"); return ALT_E_UNSUPPORTED; }
   // CTA pair (tcgen05 cta_group::2, M = 256): cfg->cta_pair 1 = pair,
   // 2 = single CTA, 0 = pair when BLOCK_N >= 128
   const int cg = (cfg && cfg->cta_pair == 2) ? 1 : ((cfg && cfg->cta_pair == 1) || BN >= 128 ? 2 : 1);
   if (cg == 2 && BN < 128) { set_error("tc: a CTA pair needs block_n >= 128"); return ALT_E_UNSUPPORTED; }
+  if (BN == 192 && cg != 2) { set_error("tc: block_n 192 runs as a CTA pair (96 B rows per CTA)"); return ALT_E_UNSUPPORTED; }
   for (const Cand &c : cands) {
     RoleInfo ra[kMaxL], rb[kMaxL], ry[kMaxL];
     memcpy(ra, P.ra, sizeof(ra));

@@ -9,24 +9,30 @@ from scripts.exptime import timeit
 M = 8192
 for name, K, N in nets.BERT_GEMMS:
     La = alt.Layout((M, K), LY.gemm_a_tiled(M, K, 128, 64))
-    Lb = alt.Layout((K, N), LY.gemm_b_tiled_nk(K, N, 256, 64))
     Lc = alt.Layout((M, N), LY.gemm_c_tiled(M, N, 128, 64))
-    a, b, c = La.empty(torch.bfloat16).normal_(), Lb.empty(torch.bfloat16).normal_(), Lc.empty(torch.bfloat16)
+    a, c = La.empty(torch.bfloat16).normal_(), Lc.empty(torch.bfloat16)
     res = []
-    for bn, pair, sk, scl in itertools.product((128, 256), (0, 2), (1, 2, 3), (0, 1)):
-        if scl and (pair != 2 or sk == 1 or sk == 3):
+    # joint layout + loop point: the B tile nt of the layout N/nt K/64 nt 64 and the kernel's BLOCK_N
+    for nt in (256, 192):
+        if N % nt:
             continue
-        cfg = {"path": 1, "block_n": bn, "cta_pair": pair, "split_k": sk, "split_cluster": scl}
-        try:
-            us = timeit(lambda: alt.matmul(M, N, K, La, a, Lb, b, Lc, c, cfg=cfg))
-            res.append((us, cfg))
-        except alt.AltError:
-            pass
+        Lb = alt.Layout((K, N), LY.gemm_b_tiled_nk(K, N, nt, 64))
+        b = Lb.empty(torch.bfloat16).normal_()
+        bns = (128, 256) if nt == 256 else (192,)
+        for bn, pair, sk, scl in itertools.product(bns, (0, 2), (1, 2, 3), (0, 1)):
+            if scl and (pair != 2 or sk == 1 or sk == 3):
+                continue
+            cfg = {"path": 1, "block_n": bn, "cta_pair": pair, "split_k": sk, "split_cluster": scl}
+            try:
+                us = timeit(lambda: alt.matmul(M, N, K, La, a, Lb, b, Lc, c, cfg=cfg))
+                res.append((us, dict(cfg, b_nt=nt)))
+            except alt.AltError:
+                pass
     res.sort(key=lambda r: r[0])
     best_us, best = res[0]
     tunecache.store_gemm(M, N, K, best, best_us)
     print(f"{name}: best {best_us:.2f} us {2 * M * N * K / best_us / 1e6:.0f} TFLOP/s {best}; "
-          f"runner-up {[(round(u, 2), c['block_n'], c['cta_pair'], c['split_k'], c['split_cluster']) for u, c in res[1:4]]}",
+          f"runner-up {[(round(u, 2), c['b_nt'], c['block_n'], c['cta_pair'], c['split_k'], c['split_cluster']) for u, c in res[1:4]]}",
           flush=True)
 if len(sys.argv) > 1:
     import shutil

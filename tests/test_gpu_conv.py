@@ -344,3 +344,11 @@ def test_tc_many_short_tiles_tma_store(C, K, R):
     for n in (0, 1, N - 1):
         ref = oracle.conv2d(pd, Ox1, words(xd[n:n + 1]), Ow, wph)
         assert_parity(Oy1.read_f64(words(y[n:n + 1])), ref, torch.bfloat16)
+
+
+@pytest.mark.parametrize("M,N,K", [(1024, 768, 256), (300, 384, 136)])
+def test_tc_gemm_block_n_192(M, N, K):
+    """BLOCK_N 192 (CTA pair, 96 B rows per CTA) on B tiled N/192 K/64"""
+    _, plan = run_gemm("g192_%d" % N, M, N, K, [], LY.gemm_b_tiled_nk(K, N, 192, 8), [], torch.bfloat16, epi=True,
+                       cfg={"path": alt.PATH_TC, "block_n": 192}, expect_path=alt.PATH_TC)
+    assert plan["block_n"] == 192 and plan["cta_pair"] == 1

@@ -111,7 +111,10 @@ def test_bert_gemm_m8192_bench_config(gemm):
     from paper_conf_eurosys_xuxpwwwdxcwc23_b200 import synth
     A = synth.activations("fsA" + name, (M, K)).to(torch.bfloat16)
     B = synth.weights("fsB" + name, (K, N)).to(torch.bfloat16)
-    ap, bp, cp = LY.gemm_a_tiled(M, K, 128, 64), LY.gemm_b_tiled_nk(K, N, 256, 64), LY.gemm_c_tiled(M, N, 128, 64)
+    from paper_conf_eurosys_xuxpwwwdxcwc23_b200 import tunecache
+    cfg = dict(tunecache.lookup_gemm(M, N, K) or {"path": 1, "block_n": 256})
+    nt = cfg.pop("b_nt", 256)
+    ap, bp, cp = LY.gemm_a_tiled(M, K, 128, 64), LY.gemm_b_tiled_nk(K, N, nt, 64), LY.gemm_c_tiled(M, N, 128, 64)
     La, Lb, Lc = alt.Layout((M, K), ap), alt.Layout((K, N), bp), alt.Layout((M, N), cp)
     Oa, Ob, Oc = oracle.Layout((M, K), ap), oracle.Layout((K, N), bp), oracle.Layout((M, N), cp)
     aw = Oa.materialize(words(A).reshape(M, K))
@@ -119,8 +122,7 @@ def test_bert_gemm_m8192_bench_config(gemm):
     a = torch.from_numpy(aw.view(np.int16)).view(torch.bfloat16).cuda()
     b = torch.from_numpy(bw.view(np.int16)).view(torch.bfloat16).cuda()
     c = Lc.empty(torch.bfloat16)
-    from paper_conf_eurosys_xuxpwwwdxcwc23_b200 import tunecache
-    alt.matmul(M, N, K, La, a, Lb, b, Lc, c, cfg=tunecache.lookup_gemm(M, N, K) or {"path": 1, "block_n": 256})
+    alt.matmul(M, N, K, La, a, Lb, b, Lc, c, cfg=cfg)
     torch.cuda.synchronize()
     got = Oc.read_f64(words(c))
     for m0, m1 in ((0, 256), (M - 256, M)):
