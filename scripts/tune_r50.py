@@ -46,7 +46,7 @@ for L in nets.RESNET50:
     p = alt.conv_params(N, L.C, L.H, L.W, L.K, L.R, L.S, L.stride, L.pad)
     Ho, Wo = L.out_hw()
     tws = [0] + [t for t in (4, 8, 16, 32) if t <= 2 * Wo]
-    space = {0: [64, 32], 1: [64], 2: [1, 2, 4, -2, -4], 3: [0, 2], 4: [1, 2, 4], 5: tws, 6: [256, 128, 64],
+    space = {0: [64, 32], 1: [64, 32], 2: [1, 2, 4, -2, -4], 3: [0, 2], 4: [1, 2, 4], 5: tws, 6: [256, 128, 64],
              7: [0, 1] if L.R > 1 else [0]}
     t0 = time.time()
     r = alt.tune("conv2d", p, alt.ALT_BF16, space, max_points=4096, warmup=3, reps=10)
