@@ -196,7 +196,11 @@ typedef struct {
                           is cut into s ranges whose fp32 partial tiles are
                           summed in split order by the last CTA to finish
                           (deterministic); for grids smaller than the GPU */
-  int32_t split_cluster; /* 1: the split_k (2 or 4) ranges of a tile run as one
+  int32_t split_cluster; /* 2: "tail split" — whole waves of output tiles run
+                          unsplit and only the tiles of the last, partial wave
+                          are split split_k ways (workspace form); removes
+                          most of the wave-quantisation loss.
+                          1: the split_k (2 or 4) ranges of a tile run as one
                           thread-block cluster and are summed in split order
                           through distributed shared memory, each CTA
                           finishing 1/split of the tile's rows (no workspace;

@@ -76,6 +76,8 @@ struct TcArgs {
   // split-K: work unit = (output tile, reduction range); partial fp32 tiles
   // in ws[cta_tile][split][BN/32][128][32], arrivals counted in cnt[cta_tile]
   int32_t splits;
+  int32_t full_units;    // units [0, full_units) run unsplit; later output tiles are split
+                         // `splits` ways (0 = every tile split; tail mode: the last wave only)
   float *ws;
   int32_t *cnt;
 };
@@ -230,6 +232,24 @@ static __device__ __noinline__ void split_total(const float *wt, int splits, int
   for (int j = 0; j < 32; j++) out[j] = t[j];
 }
 
+// work unit -> (output tile mn, split index sp, reduction range [kb, ke))
+struct UnitInfo { int mn, sp, kb, ke; bool split; };
+__device__ __forceinline__ UnitInfo unit_info(const TcArgs &a, int tile) {
+  UnitInfo u;
+  if (tile < a.full_units) {
+    u.mn = tile; u.sp = 0; u.kb = 0; u.ke = a.num_iters; u.split = false;
+    return u;
+  }
+  const int t = tile - a.full_units;
+  const int q = (int)a.f_spl.div((uint32_t)t);
+  u.mn = a.full_units + q;
+  u.sp = t - q * a.splits;
+  u.split = a.splits > 1;
+  u.kb = u.split ? u.sp * a.num_iters / a.splits : 0;
+  u.ke = u.split ? (u.sp + 1) * a.num_iters / a.splits : a.num_iters;
+  return u;
+}
+
 struct TileCoord { int n0, p0, q0, k0; };
 // work unit `tile` -> this CTA's 128-row M tile and the unit's N tile; with a
 // CTA pair (CG = 2) a unit is two consecutive M tiles, one per CTA rank
@@ -341,10 +361,9 @@ __global__ void __launch_bounds__(kThreads, 1)
     const bool active = j < a.spi;
     int it = 0, ti = 0;
     for (int tile = unit0; tile < a.num_tiles; tile += unit_step, ti++) {
-      const int mn = (int)a.f_spl.div((uint32_t)tile), sp = tile - mn * a.splits;
-      const TileCoord tc = tile_coord(a, mn, BN, CG, rank);
-      const int k_begin = a.splits == 1 ? 0 : sp * a.num_iters / a.splits;
-      const int k_end = a.splits == 1 ? a.num_iters : (sp + 1) * a.num_iters / a.splits;
+      const UnitInfo ui = unit_info(a, tile);
+      const TileCoord tc = tile_coord(a, ui.mn, BN, CG, rank);
+      const int k_begin = ui.kb, k_end = ui.ke;
       int32_t v[NVAR];
       // B rows of this CTA: its 1/CG share of the unit's BN output channels
       const int pp = isA ? tc.p0 : 0, qq = isA ? tc.q0 : tc.k0 + rank * (BN / CG);
@@ -443,9 +462,8 @@ __global__ void __launch_bounds__(kThreads, 1)
         if (i == ALT_DBG_TILE) { DBG(27); }
         tc_fence_after();
         const uint32_t d = tmem + (uint32_t)(acc * BN);
-        const int sp = tile - (int)a.f_spl.div((uint32_t)tile) * a.splits;
-        const int k_begin = a.splits == 1 ? 0 : sp * a.num_iters / a.splits;
-        const int k_end = a.splits == 1 ? a.num_iters : (sp + 1) * a.num_iters / a.splits;
+        const UnitInfo ui = unit_info(a, tile);
+        const int k_begin = ui.kb, k_end = ui.ke;
         int stage = it % STAGES;
         uint32_t ph = (uint32_t)((it / STAGES) & 1);
         for (int kit = k_begin; kit < k_end; kit++, it++) {
@@ -496,7 +514,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     auto fetch_sb = [&](int tile, float &fs, float &fb) {
       fs = 1.f; fb = 0.f;
       if (tile < a.num_tiles && et < BN) {
-        const int k = min(tile_coord(a, (int)a.f_spl.div((uint32_t)tile), BN, CG, rank).k0 + et, a.K - 1);
+        const int k = min(tile_coord(a, unit_info(a, tile).mn, BN, CG, rank).k0 + et, a.K - 1);
         fs = __ldg(a.epi.scale + k);
         fb = __ldg(a.epi.bias + k);
       }
@@ -521,7 +539,8 @@ __global__ void __launch_bounds__(kThreads, 1)
     int i = 0;
     for (int tile = unit0; tile < a.num_tiles; tile += unit_step, i++) {
       const int acc = i % NACC, use = i / NACC;
-      const int mn = (int)a.f_spl.div((uint32_t)tile), ksp = tile - mn * a.splits;
+      const UnitInfo ui = unit_info(a, tile);
+      const int mn = ui.mn, ksp = ui.sp;
       const TileCoord tc = tile_coord(a, mn, BN, CG, rank);
       named_bar(2, kEpiThreads);  // every epilogue warp is done with the previous tile's values
       if (et < BN) {  // explicit shared-space stores (the aligned base is a generic pointer)
@@ -591,8 +610,8 @@ __global__ void __launch_bounds__(kThreads, 1)
         continue;  // one tile per CTA; phase 2 after the cluster barrier
       }
       const float *wsl = nullptr;  // this CTA tile's partials (split-K)
-      if (SC == 1 && a.splits > 1) {
-        const size_t cta_tile = (size_t)mn * CG + rank;
+      if (SC == 1 && ui.split) {
+        const size_t cta_tile = (size_t)(mn - a.full_units) * CG + rank;
         float *wt = a.ws + cta_tile * (size_t)a.splits * (128 * BN);
         float *mine = wt + (size_t)ksp * (128 * BN);
 #pragma unroll 1
@@ -809,7 +828,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       __syncwarp();
       cluster_sync();
       const int crank = (int)cluster_ctarank();
-      const TileCoord tc = tile_coord(a, (int)a.f_spl.div((uint32_t)unit0), BN, CG, rank);
+      const TileCoord tc = tile_coord(a, unit_info(a, unit0).mn, BN, CG, rank);
       constexpr int NQ = 4 / SC, NCH = BN / 32;
       const int ew = warp - 2;
       int cnt = 0;
@@ -1570,12 +1589,22 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
         // than the idle SMs it recovers on the ResNet-50 set; tuned per layer)
         sk = std::max<int64_t>(1, std::min<int64_t>(sk, a.num_iters));
         a.splits = (int32_t)sk;
+        a.full_units = 0;
         a.ws = nullptr;
         a.cnt = nullptr;
+        // tail split (split_cluster == 2): whole waves run unsplit, only the
+        // output tiles of the last, partial wave are split sk ways
+        int64_t split_units = units;
+        if (cfg && cfg->split_cluster == 2 && sk > 1) {
+          const int64_t tail = units % slots;
+          split_units = units > slots ? tail : units;
+          a.full_units = (int32_t)(units - split_units);
+          if (split_units == 0) { sk = 1; a.splits = 1; }
+        }
         // cluster split-K: the sk ranges of a tile as one cluster, reduced
         // through DSMEM (single CTA, TMA-store output, no residual, sk 2 / 4)
         pl.sc = 1;
-        if (cfg && cfg->split_cluster && sk > 1) {
+        if (cfg && cfg->split_cluster == 1 && sk > 1) {
           if (cg != 1 || (sk != 2 && sk != 4) || BN < 128 || a.out_mode != 1 || P.epi.residual) {
             set_error("tc: cluster split-K needs one CTA, block_n 128/256, split 2/4, a TMA-store output and no residual");
             return ALT_E_UNSUPPORTED;
@@ -1586,7 +1615,7 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
           if ((int64_t)a.num_tiles * sk > 0x7fffffff) { set_error("tc: too many tiles"); return ALT_E_UNSUPPORTED; }
           // per-plan workspace (lives as long as the process: captured graphs
           // may replay the plan after the cache forgets it)
-          const size_t wsb = (size_t)units * cg * sk * 128 * BN * sizeof(float);
+          const size_t wsb = (size_t)split_units * cg * sk * 128 * BN * sizeof(float);
           // bounded: plans (and their workspaces) live for the process, so a
           // tuner sweeping many split points must not exhaust the device
           static std::mutex ws_mu;
@@ -1599,13 +1628,13 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
             }
             ws_total += wsb;
           }
-          if (cudaMalloc(&a.ws, wsb) != cudaSuccess || cudaMalloc(&a.cnt, (size_t)units * cg * 4) != cudaSuccess ||
-              cudaMemset(a.cnt, 0, (size_t)units * cg * 4) != cudaSuccess) {
+          if (cudaMalloc(&a.ws, wsb) != cudaSuccess || cudaMalloc(&a.cnt, (size_t)split_units * cg * 4) != cudaSuccess ||
+              cudaMemset(a.cnt, 0, (size_t)split_units * cg * 4) != cudaSuccess) {
             cudaGetLastError();
             set_error("tc: split-K workspace: out of memory");
             return ALT_E_NOMEM;
           }
-          a.num_tiles = (int32_t)(units * sk);
+          a.num_tiles = (int32_t)(a.full_units + split_units * sk);
         }
       }
       a.f_nnt = FastDiv((uint32_t)a.num_n_tiles);
@@ -1646,7 +1675,7 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       u.stages = pl.stages;
       u.tile_n = c.tn; u.tile_h = c.th; u.tile_w = c.tw;
       u.split_k = a.splits;
-      u.split_cluster = pl.sc > 1 ? 1 : 0;
+      u.split_cluster = pl.sc > 1 ? 1 : (a.full_units > 0 && a.splits > 1 ? 2 : 0);
       pl.used = u;
       cudaError_t e = launch_plan(pl, P.y, stream);
       count_launch();

@@ -19,8 +19,10 @@ for name, K, N in nets.BERT_GEMMS:
         Lb = alt.Layout((K, N), LY.gemm_b_tiled_nk(K, N, nt, 64))
         b = Lb.empty(torch.bfloat16).normal_()
         bns = (128, 256) if nt == 256 else (192,)
-        for bn, pair, sk, scl in itertools.product(bns, (0, 2), (1, 2, 3), (0, 1)):
-            if scl and (pair != 2 or sk == 1 or sk == 3):
+        for bn, pair, sk, scl in itertools.product(bns, (0, 2), (1, 2, 3, 4), (0, 1, 2)):
+            if scl == 1 and (pair != 2 or sk == 1 or sk == 3):
+                continue
+            if scl == 2 and sk == 1:
                 continue
             cfg = {"path": 1, "block_n": bn, "cta_pair": pair, "split_k": sk, "split_cluster": scl}
             try:

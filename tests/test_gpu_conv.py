@@ -352,3 +352,19 @@ def test_tc_gemm_block_n_192(M, N, K):
     _, plan = run_gemm("g192_%d" % N, M, N, K, [], LY.gemm_b_tiled_nk(K, N, 192, 8), [], torch.bfloat16, epi=True,
                        cfg={"path": alt.PATH_TC, "block_n": 192}, expect_path=alt.PATH_TC)
     assert plan["block_n"] == 192 and plan["cta_pair"] == 1
+
+
+@pytest.mark.parametrize("sk", [2, 3])
+def test_tc_tail_split(sk):
+    """tail split (split_cluster = 2): whole waves of tiles unsplit, the last
+    partial wave's tiles split sk ways; GEMM with 2.3 waves of CTA pairs and a
+    conv with residual, against the oracle"""
+    M = 128 * 2 * 170   # 170 pair tiles x 1 N tile: 2 full waves of 74 pairs + a tail of 22
+    _, plan = run_gemm("tail%d" % sk, M, 256, 512, [], LY.transpose2(), [], torch.bfloat16, epi=True,
+                       cfg={"path": alt.PATH_TC, "block_n": 256, "split_k": sk, "split_cluster": 2},
+                       expect_path=alt.PATH_TC)
+    assert plan["split_k"] == sk and plan["split_cluster"] == 2
+    xp, wp, yp = LY.nchwxc(256, 64), LY.kcrs_yk_xc(512, 256, 256, 64), LY.nchwxc(512, 64)
+    run_conv("tailc%d" % sk, 8, 256, 14, 14, 512, 3, 3, 1, 1, xp, wp, yp, torch.bfloat16, epi=True,
+             res_p=LY.nchwxc(512, 64), act=1, cfg={"path": alt.PATH_TC, "block_n": 256, "split_k": sk,
+                                                   "split_cluster": 2}, expect_path=alt.PATH_TC)
