@@ -80,6 +80,9 @@ struct TcArgs {
                          // `splits` ways (0 = every tile split; tail mode: the last wave only)
   float *ws;
   int32_t *cnt;
+  int32_t coop;          // split tiles reduced cooperatively: each of the splits CTAs
+                         // finishes 1 / splits of the tile's rows (all pieces co-resident)
+  int32_t *done;         // per split tile: CTAs finished (resets cnt / done for the next launch)
 };
 
 #ifndef ALT_EPI_WARPS
@@ -610,6 +613,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         continue;  // one tile per CTA; phase 2 after the cluster barrier
       }
       const float *wsl = nullptr;  // this CTA tile's partials (split-K)
+      int coop_rows = -1;          // cooperative split: 1 = this warp finishes its rows, 0 = another CTA does
       if (SC == 1 && ui.split) {
         const size_t cta_tile = (size_t)(mn - a.full_units) * CG + rank;
         float *wt = a.ws + cta_tile * (size_t)a.splits * (128 * BN);
@@ -629,6 +633,28 @@ __global__ void __launch_bounds__(kThreads, 1)
         __threadfence();
         if (et == 0 && i == ALT_DBG_TILE) { DBG(4); }
         named_bar(1, kEpiThreads);
+        if (a.coop) {
+          // every piece of the tile is resident (planner-checked): wait for all
+          // partials, release the accumulator, then finish the rows of the
+          // lane quarters this split owns (quarter q -> split q * splits / 4)
+          if (et == 0) {
+            atomicAdd(a.cnt + cta_tile, 1);
+            int seen = 0;
+            do {
+              asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(seen) : "l"(a.cnt + cta_tile) : "memory");
+              if (seen < a.splits) __nanosleep(64);
+            } while (seen < a.splits);
+          }
+          named_bar(1, kEpiThreads);
+          tc_fence_before();
+          __syncwarp();
+          if (lane == 0) {
+            if constexpr (CG == 2) mbar_arrive_cluster(&tempty[acc], 0);
+            else mbar_arrive(&tempty[acc]);
+          }
+          coop_rows = (wq * a.splits) / 4 == ksp;
+          wsl = wt;
+        } else {
         if (et == 0) *last_flag = atomicAdd(a.cnt + cta_tile, 1) == a.splits - 1;
         named_bar(1, kEpiThreads);
         if (et == 0 && i == ALT_DBG_TILE) { DBG(7); }
@@ -644,6 +670,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         __threadfence();
         if (et == 0) a.cnt[cta_tile] = 0;  // ready for the next launch
         wsl = wt;
+        }
       }
       // TMEM reads are software-pipelined (TMEM read is 32 B/clk per SM):
       // on the plain path (TMA-store output, no residual, no split) chunk
@@ -664,7 +691,9 @@ __global__ void __launch_bounds__(kThreads, 1)
       auto chunk_loop = [&](auto early_tag, auto res_tag) {
         constexpr bool EARLY = decltype(early_tag)::value;
         constexpr bool RESV = decltype(res_tag)::value;  // 16-byte residual vectors
+        if (coop_rows == 0) return;  // cooperative split: another CTA finishes these rows
         if (half * 32 >= BN) {  // this warp's column part is past BLOCK_N: nothing to drain
+          if (coop_rows >= 0) return;  // accumulator already released
           tc_fence_before();
           __syncwarp();
           if (lane == 0) {
@@ -687,7 +716,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           if constexpr (!EARLY) {
             if (wsl) {
               float tot[32];
-              split_total(wsl, a.splits, ksp, BN, cb, row, raw, tot);
+              split_total(wsl, a.splits, coop_rows >= 0 ? -1 : ksp, BN, cb, row, raw, tot);
 #pragma unroll
               for (int j = 0; j < 32; j++) raw[j] = __float_as_uint(tot[j]);
             }
@@ -724,7 +753,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           if constexpr (EARLY) {
             if (c0 + kStep < BN) tmem_ld_32x32b_x32(next, raw);
           }
-          if (c0 + kStep >= BN) {  // accumulator buffer drained: MMA may reuse it
+          if (c0 + kStep >= BN && coop_rows < 0) {  // accumulator buffer drained: MMA may reuse it
             tc_fence_before();
             __syncwarp();
             if (lane == 0) {
@@ -817,6 +846,18 @@ __global__ void __launch_bounds__(kThreads, 1)
       } else {
         if (a.out_mode != 0 && !a.epi.residual && !wsl) chunk_loop(std::true_type{}, std::false_type{});
         else chunk_loop(std::false_type{}, std::false_type{});
+      }
+      if (coop_rows >= 0) {
+        // cooperative split: the last CTA of the tile to finish resets the
+        // counters for the next launch (every CTA is past its wait by then)
+        named_bar(1, kEpiThreads);
+        if (et == 0) {
+          const size_t cta_tile = (size_t)(mn - a.full_units) * CG + rank;
+          if (atomicAdd(a.done + cta_tile, 1) == a.splits - 1) {
+            a.cnt[cta_tile] = 0;
+            a.done[cta_tile] = 0;
+          }
+        }
       }
       if (et == 0 && i == ALT_DBG_TILE) { DBG(31); }
     }
@@ -1628,8 +1669,15 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
             }
             ws_total += wsb;
           }
+          // cooperative reduction (tail split, 2 / 4 splits, every piece in one
+          // round of the persistent grid so all pieces of a tile are resident)
+          a.coop = (cfg && cfg->split_cluster == 2 && (sk == 2 || sk == 4) &&
+                    split_units * sk <= slots) ? 1 : 0;
+          a.done = nullptr;
           if (cudaMalloc(&a.ws, wsb) != cudaSuccess || cudaMalloc(&a.cnt, (size_t)split_units * cg * 4) != cudaSuccess ||
-              cudaMemset(a.cnt, 0, (size_t)split_units * cg * 4) != cudaSuccess) {
+              cudaMemset(a.cnt, 0, (size_t)split_units * cg * 4) != cudaSuccess ||
+              (a.coop && (cudaMalloc(&a.done, (size_t)split_units * cg * 4) != cudaSuccess ||
+                          cudaMemset(a.done, 0, (size_t)split_units * cg * 4) != cudaSuccess))) {
             cudaGetLastError();
             set_error("tc: split-K workspace: out of memory");
             return ALT_E_NOMEM;
