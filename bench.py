@@ -249,10 +249,10 @@ def main():
     ap.add_argument("--batch", type=int, default=32, help="images per GPU")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--eager", action="store_true", help="time eager launches instead of a CUDA graph")
-    ap.add_argument("--workload", default="r50", choices=["r50", "r18", "mv2", "bert", "relayout"],
+    ap.add_argument("--workload", default="r50", choices=["r50", "r18", "mv2", "bert", "relayout", "fig12"],
                     help="r50 = BASELINE config 2 (the driver's default); r18 = config 5 "
                          "(batch-sharded chain, global batch 256); mv2 = config 4; bert = config 3; "
-                         "relayout = the D6 bandwidth set")
+                         "relayout = the D6 bandwidth set; fig12 = the paper's propagation study")
     args = ap.parse_args()
     if args.workload != "r50":
         import bench_workloads

@@ -9,6 +9,11 @@
   bert      config 3: BERT-base GEMMs at seq 512 (M = 8192 = 16 sequences) on
             tiled layouts
   relayout  the D6 set of layout conversions, HBM GB/s per case
+  fig12     the paper's Fig. 12 propagation study: pad ->
+            C2D 3x3 -> C2D 1x1 at 512 channels (7x7, 14x14), layouts chosen by
+            forward propagation (ALT-FP), backward propagation (ALT-BP) or
+            independent tuning with the conversion fused into the 3x3's
+            epilogue (ALT) or run standalone
 
 Each prints one JSON line like bench.py's.
 """
@@ -169,8 +174,126 @@ def run(args):
         out = _line(args, ws, tot_bytes / (tot_ms * 1e-3) / 1e9, "GB/s", tot_ms, {
             "workload": "D6 relayout set (ResNet tensors at batch 256, BERT A, KCRS weights)",
             "parallelism": f"dp{ws}"}, {"scaling": "weak", "hbm_peak_gbs": peak, "cases": cases})
+    elif args.workload == "fig12":
+        out = fig12(args, ws)
     if rank == 0 and out is not None:
         print(json.dumps(out))
     if ws > 1:
         import torch.distributed as dist
         dist.destroy_process_group()
+
+
+# ------------------------------------------------------------------ Fig. 12 -
+def fig12(args, ws):
+    """Fig. 12: subgraph pad -> C2D 3x3 (512 -> 512, s1, p1) ->
+    C2D 1x1 (512 -> K1) at 7x7 (K1 = 512) and 14x14 (K1 = 2048).  Every
+    (layout, kernel configuration) point is timed on the device (CUDA graph
+    of repeated launches); the policies combine them as the paper describes:
+      ALT-FP  tune the 3x3 (its x and y layouts), the 1x1 reads the 3x3's y
+      ALT-BP  tune the 1x1 (its x layout), the 3x3 must write that layout
+      ALT     tune both independently; the 1x1's layout is written by the
+              3x3's fused epilogue (this build's conversion) or converted by
+              a standalone relayout (the paper's conversion op)"""
+    import itertools
+    import paper_conf_eurosys_xuxpwwwdxcwc23_b200 as alt
+    from paper_conf_eurosys_xuxpwwwdxcwc23_b200 import layouts as LY
+    from paper_conf_eurosys_xuxpwwwdxcwc23_b200 import synth
+    dev = torch.device("cuda", 0)
+    C = 512
+    tiles = (64, 32, 16)
+    cfgs = [{"path": 1, "block_n": bn, "cta_pair": pr, "split_k": sk, "split_cluster": scl}
+            for bn, pr, (sk, scl) in itertools.product((128, 256), (0, 2), ((1, 0), (2, 0), (2, 1), (4, 1)))
+            if not (scl and pr != 2)]
+
+    def tmin(fn_for_cfg):
+        best = None
+        for c in cfgs:
+            try:
+                t = _time(lambda: fn_for_cfg(c), 10, 2, 1) * 1e3
+            except Exception:
+                torch.cuda.synchronize()
+                continue
+            if best is None or t < best[0]:
+                best = (t, c)
+        return best
+
+    subs = []
+    for (name, H, K1) in (("Sg#1 7x7", 7, 512), ("Sg#2 14x14", 14, 2048)):
+        for N in (1, 32):
+            x0 = synth.activations(f"f12x{H}", (N, C, H, H)).to(torch.bfloat16).to(dev)
+            Lx0 = alt.Layout((N, C, H, H), [])
+            w3 = synth.weights("f12w3", (C, C, 3, 3)).to(torch.bfloat16).to(dev)
+            w1 = synth.weights(f"f12w1{K1}", (K1, C, 1, 1)).to(torch.bfloat16).to(dev)
+            p3, p1 = alt.conv_params(N, C, H, H, C, 3, 3, 1, 1), alt.conv_params(N, C, H, H, K1, 1, 1, 1, 0)
+            L3 = {}
+            for it in tiles:  # 3x3 input layouts written by the pad op (padding materialised or not)
+                for pad in (0, 1):
+                    L = alt.Layout((N, C, H, H), LY.nchwxc(C, it, pad_hw=pad))
+                    buf = L.empty(torch.bfloat16, dev)
+                    alt.relayout(Lx0, x0, L, buf)
+                    L3[(it, pad)] = (L, buf)
+            Lmid = {t: alt.Layout((N, C, H, H), LY.nchwxc(C, t)) for t in tiles}
+            mid = {t: Lmid[t].empty(torch.bfloat16, dev) for t in tiles}
+            Ly1 = alt.Layout((N, K1, H, H), LY.nchwxc(K1, 64))
+            y1 = Ly1.empty(torch.bfloat16, dev)
+            W3, W1 = {}, {}
+            for it in tiles:
+                for bn in (128, 256):
+                    lw = alt.Layout((C, C, 3, 3), LY.kcrs_yk_xc(C, C, bn, it))
+                    wt = lw.empty(torch.bfloat16, dev)
+                    alt.relayout(alt.Layout((C, C, 3, 3), []), w3, lw, wt)
+                    W3[(it, bn)] = (lw, wt)
+                    lw1 = alt.Layout((K1, C, 1, 1), LY.kcrs_yk_xc(K1, C, bn, it))
+                    wt1 = lw1.empty(torch.bfloat16, dev)
+                    alt.relayout(alt.Layout((K1, C, 1, 1), []), w1, lw1, wt1)
+                    W1[(it, bn)] = (lw1, wt1)
+            torch.cuda.synchronize()
+            # pad op (plain NCHW -> the 3x3's input layout)
+            t_pad = {k: _time(lambda k=k: alt.relayout(Lx0, x0, L3[k][0], L3[k][1]), 10, 2, 1) * 1e3 for k in L3}
+            # C2D 3x3 for every (x layout, y layout); C2D 1x1 for every x layout
+            t3 = {}
+            for (it, pad), ot in itertools.product(L3.keys(), tiles):
+                Lx, xb = L3[(it, pad)]
+                t3[(it, pad, ot)] = tmin(lambda c, Lx=Lx, xb=xb, it=it, ot=ot: alt.conv2d(
+                    p3, Lx, xb, W3[(it, c["block_n"])][0], W3[(it, c["block_n"])][1], Lmid[ot], mid[ot], cfg=c))
+            t1 = {ot: tmin(lambda c, ot=ot: alt.conv2d(p1, Lmid[ot], mid[ot], W1[(ot, c["block_n"])][0],
+                                                        W1[(ot, c["block_n"])][1], Ly1, y1, cfg=c)) for ot in tiles}
+            t3 = {k: v for k, v in t3.items() if v is not None}
+            t1 = {k: v for k, v in t1.items() if v is not None}
+            conv = {(a, b): _time(lambda a=a, b=b: alt.relayout(Lmid[a], mid[a], Lmid[b], mid[b]), 10, 2, 1) * 1e3
+                    for a in tiles for b in tiles if a != b}
+            k3 = lambda k: t3[k][0] + t_pad[k[:2]]  # noqa: E731
+            # ALT-FP: best 3x3 point, the 1x1 reads its y layout
+            fp3 = min(t3, key=k3)
+            fp = (k3(fp3), t1[fp3[2]][0])
+            # ALT-BP: best 1x1 point, the 3x3 must write that layout
+            ot1 = min(t1, key=lambda o: t1[o][0])
+            bp3 = min((k for k in t3 if k[2] == ot1), key=k3)
+            bp = (k3(bp3), t1[ot1][0])
+            # ALT: independent; fused conversion = the 3x3 (its own x) writes the 1x1's layout
+            alt_f3 = min((k for k in t3 if k[:2] == fp3[:2] and k[2] == ot1), key=k3)
+            altf = (k3(alt_f3), t1[ot1][0])
+            conv_us = conv.get((fp3[2], ot1), 0.0)
+            alts = (k3(fp3), conv_us, t1[ot1][0])
+            subs.append({"subgraph": name, "batch": N, "K1": K1,
+                         "ALT-FP": {"c2d3x3_us": round(fp[0], 2), "c2d1x1_us": round(fp[1], 2),
+                                    "total_us": round(sum(fp), 2), "layouts": {"x3": fp3[:2], "y3=x1": fp3[2]}},
+                         "ALT-BP": {"c2d3x3_us": round(bp[0], 2), "c2d1x1_us": round(bp[1], 2),
+                                    "total_us": round(sum(bp), 2), "layouts": {"x3": bp3[:2], "y3=x1": ot1}},
+                         "ALT (fused conversion)": {"c2d3x3_us": round(altf[0], 2), "c2d1x1_us": round(altf[1], 2),
+                                                    "total_us": round(sum(altf), 2),
+                                                    "layouts": {"x3": alt_f3[:2], "y3": ot1, "x1": ot1}},
+                         "ALT (standalone conversion)": {"c2d3x3_us": round(alts[0], 2),
+                                                         "conversion_us": round(alts[1], 2),
+                                                         "c2d1x1_us": round(alts[2], 2),
+                                                         "total_us": round(sum(alts), 2),
+                                                         "layouts": {"x3": fp3[:2], "y3": fp3[2], "x1": ot1}}})
+    value = sum(s_["ALT (fused conversion)"]["total_us"] for s_ in subs)
+    line = _line(args, ws, value, "us", value * 1e-3,
+                 {"workload": "Fig. 12 propagation study: pad -> C2D 3x3 512 -> C2D 1x1 (7x7 -> 512, "
+                              "14x14 -> 2048), batch 1 and 32, layouts NCHW[x]c x in {64,32,16} with "
+                              "optional materialised padding", "parallelism": "dp1"},
+                 {"scaling": "weak", "higher_is_better": False, "subgraphs": subs,
+                  "note": "value = sum over subgraphs of the ALT (independent tuning, fused conversion) "
+                          "totals; pad op time included in the C2D 3x3 column"})
+    return line
