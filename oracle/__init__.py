@@ -231,8 +231,9 @@ def conv2d_f64(p: dict, x: np.ndarray, w: np.ndarray, scale=None, bias=None,
     Vh, Vw = p.get("stride_h", 1), p.get("stride_w", 1)
     ph, pw = p.get("pad_h", 0), p.get("pad_w", 0)
     g = p.get("groups", 1)
-    Ho, Wo = (H + 2 * ph - R) // Vh + 1, (W + 2 * pw - S) // Vw + 1
-    pr = np.array([N, C, H, W, K, R, S, Vh, Vw, ph, pw, g], np.int64)
+    dh, dw = p.get("dil_h", 1), p.get("dil_w", 1)
+    Ho, Wo = (H + 2 * ph - dh * (R - 1) - 1) // Vh + 1, (W + 2 * pw - dw * (S - 1) - 1) // Vw + 1
+    pr = np.array([N, C, H, W, K, R, S, Vh, Vw, ph, pw, g, dh, dw], np.int64)
     x, w = _f64(x), _f64(w)
     assert x.shape == (N, C, H, W) and w.shape == (K, C // g, R, S)
     y = np.zeros((N, K, Ho, Wo), np.float64)
@@ -260,7 +261,8 @@ def conv2d_points(p: dict, x_l: Layout, x: np.ndarray, w_l: Layout, w: np.ndarra
     """O3 + O6 evaluated at chosen outputs (n,k,p,q), reading through F."""
     N, C, H, W, K, R, S = (p[k] for k in "NCHWKRS")
     pr = np.array([N, C, H, W, K, R, S, p.get("stride_h", 1), p.get("stride_w", 1),
-                   p.get("pad_h", 0), p.get("pad_w", 0), p.get("groups", 1)], np.int64)
+                   p.get("pad_h", 0), p.get("pad_w", 0), p.get("groups", 1), p.get("dil_h", 1),
+                   p.get("dil_w", 1)], np.int64)
     x = np.ascontiguousarray(x)
     w = np.ascontiguousarray(w)
     if x.dtype == np.float32:

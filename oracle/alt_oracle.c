@@ -432,17 +432,19 @@ static double epilogue(double acc, const double *scale, const double *bias,
 /* ------------------------------------------------------------------ O3 --- */
 /* Direct (textbook) conv2d on fp64 row-major logical arrays:
  *   y[n,k,p,q] = sum_{c<C/g} sum_{r<R} sum_{s<S}
- *                x[n, g(k) C/g + c, p V_h - pad_h + r, q V_w - pad_w + s] w[k,c,r,s]
- * x = 0 outside [0,H) x [0,W); g(k) = floor(k groups / K).  The sum runs in
+ *                x[n, g(k) C/g + c, p V_h - pad_h + d_h r, q V_w - pad_w + d_w s] w[k,c,r,s]
+ * x = 0 outside [0,H) x [0,W); g(k) = floor(k groups / K); dilation d (DIL,
+ * the paper's single-operator set P:1546-1549; d = 1 is plain C2D);
+ * Ho = floor((H + 2 pad_h - d_h (R - 1) - 1) / V_h) + 1.  The sum runs in
  * (c, r, s) ascending order.  Images n0 <= n < n1 are computed (the rest of
- * y is left untouched).  p[] = {N,C,H,W,K,R,S,Vh,Vw,ph,pw,groups}. */
+ * y is left untouched).  p[] = {N,C,H,W,K,R,S,Vh,Vw,ph,pw,groups,dh,dw}. */
 void orc_conv2d_f64(const long long *p, const double *x, const double *w,
                     const double *scale, const double *bias, const double *res,
                     int act, long long n0, long long n1, double *y) {
   long long N = p[0], C = p[1], H = p[2], W = p[3], K = p[4], R = p[5], S = p[6];
-  long long Vh = p[7], Vw = p[8], ph = p[9], pw = p[10], G = p[11];
+  long long Vh = p[7], Vw = p[8], ph = p[9], pw = p[10], G = p[11], dh = p[12], dw = p[13];
   (void)N;
-  long long Ho = (H + 2 * ph - R) / Vh + 1, Wo = (W + 2 * pw - S) / Vw + 1;
+  long long Ho = (H + 2 * ph - dh * (R - 1) - 1) / Vh + 1, Wo = (W + 2 * pw - dw * (S - 1) - 1) / Vw + 1;
   long long Cg = C / G;
 #pragma omp parallel for collapse(2) schedule(dynamic)
   for (long long n = n0; n < n1; n++)
@@ -454,7 +456,7 @@ void orc_conv2d_f64(const long long *p, const double *x, const double *w,
           for (long long c = 0; c < Cg; c++)
             for (long long r = 0; r < R; r++)
               for (long long s = 0; s < S; s++) {
-                long long ih = oh * Vh - ph + r, iw = ow * Vw - pw + s;
+                long long ih = oh * Vh - ph + dh * r, iw = ow * Vw - pw + dw * s;
                 if (ih < 0 || ih >= H || iw < 0 || iw >= W) continue;
                 acc += x[((n * C + g * Cg + c) * H + ih) * W + iw] *
                        w[((k * Cg + c) * R + r) * S + s];
@@ -474,7 +476,7 @@ int orc_conv2d_points(const long long *p, const orc_layout *XL, const void *x,
                       const orc_layout *RL, const void *res, int act,
                       long long npts, const long long *pts, double *out) {
   long long C = p[1], H = p[2], W = p[3], K = p[4], R = p[5], S = p[6];
-  long long Vh = p[7], Vw = p[8], ph = p[9], pw = p[10], G = p[11];
+  long long Vh = p[7], Vw = p[8], ph = p[9], pw = p[10], G = p[11], dh = p[12], dw = p[13];
   long long Cg = C / G;
   int lossy = 0;
 #pragma omp parallel for schedule(dynamic) reduction(| : lossy)
@@ -486,7 +488,7 @@ int orc_conv2d_points(const long long *p, const orc_layout *XL, const void *x,
     for (long long c = 0; c < Cg; c++)
       for (long long r = 0; r < R; r++)
         for (long long s = 0; s < S; s++) {
-          long long ih = oh * Vh - ph + r, iw = ow * Vw - pw + s;
+          long long ih = oh * Vh - ph + dh * r, iw = ow * Vw - pw + dw * s;
           if (ih < 0 || ih >= H || iw < 0 || iw >= W) continue;
           li[0] = n; li[1] = g * Cg + c; li[2] = ih; li[3] = iw;
           if (!orc_F(XL, li, pc)) { lossy = 1; continue; }

@@ -230,3 +230,58 @@ def test_pool_vs_torch_float64():
         got = oracle.pool2d_f64(x, k, k, s, p, "avg")
         ref = torch.nn.functional.avg_pool2d(torch.from_numpy(x), k, s, p, count_include_pad=False).numpy()
         np.testing.assert_allclose(got, ref, rtol=1e-12, atol=1e-14)
+
+
+# ------------------------------------------------------------ dilation (DIL) --
+DIL_CASES = [  # (params, dil_h, dil_w): the paper's DIL operator
+    (_params(2, 6, 11, 10, 4, 3, 3, 1, 2), 2, 2),
+    (_params(1, 4, 13, 9, 3, 3, 2, 2, 1), 3, 2),
+    (_params(2, 8, 9, 9, 8, 3, 3, 1, 2, groups=4), 2, 1),
+]
+
+
+def _dil(p, dh, dw):
+    q = dict(p)
+    q["dil_h"], q["dil_w"] = dh, dw
+    return q
+
+
+@pytest.mark.parametrize("case", DIL_CASES)
+def test_dilated_conv_vs_torch_float64(case):
+    """O3 with dilation against the library routine (torch float64)"""
+    p, dh, dw = case
+    q = _dil(p, dh, dw)
+    rng = np.random.default_rng(11)
+    x = rng.uniform(-1, 1, (p["N"], p["C"], p["H"], p["W"]))
+    w = rng.uniform(-1, 1, (p["K"], p["C"] // p["groups"], p["R"], p["S"]))
+    y = oracle.conv2d_f64(q, x, w)
+    ref = torch.nn.functional.conv2d(torch.from_numpy(x), torch.from_numpy(w), stride=(p["stride_h"], p["stride_w"]),
+                                     padding=(p["pad_h"], p["pad_w"]), groups=p["groups"], dilation=(dh, dw)).numpy()
+    assert y.shape == ref.shape
+    np.testing.assert_allclose(y, ref, rtol=1e-12, atol=1e-12)
+
+
+def test_dilated_conv_brute_force_and_special_cases():
+    """bit-exact pure-Python loops (same order); dilation 1 is plain C2D; a
+    dilated R x R filter equals the undilated (d(R-1)+1)^2 filter with zeros
+    between its taps (the definition of dilation)"""
+    p = _params(1, 3, 9, 8, 2, 3, 3, 1, 2)
+    rng = np.random.default_rng(12)
+    x = rng.uniform(-1, 1, (1, 3, 9, 8))
+    w = rng.uniform(-1, 1, (2, 3, 3, 3))
+    y = oracle.conv2d_f64(_dil(p, 2, 2), x, w)
+    Ho, Wo = (9 + 4 - 4 - 1) // 1 + 1, (8 + 4 - 4 - 1) // 1 + 1
+    b = np.zeros((1, 2, Ho, Wo))
+    for k, oh, ow in itertools.product(range(2), range(Ho), range(Wo)):
+        acc = 0.0
+        for c, r, s in itertools.product(range(3), range(3), range(3)):
+            ih, iw = oh - 2 + 2 * r, ow - 2 + 2 * s
+            if 0 <= ih < 9 and 0 <= iw < 8:
+                acc += x[0, c, ih, iw] * w[k, c, r, s]
+        b[0, k, oh, ow] = acc
+    assert np.array_equal(y, b)
+    assert np.array_equal(oracle.conv2d_f64(_dil(p, 1, 1), x, w), oracle.conv2d_f64(p, x, w))
+    wz = np.zeros((2, 3, 5, 5))
+    wz[:, :, ::2, ::2] = w
+    pz = _params(1, 3, 9, 8, 2, 5, 5, 1, 2)
+    np.testing.assert_allclose(y, oracle.conv2d_f64(pz, x, wz), rtol=1e-13, atol=1e-13)
