@@ -44,7 +44,7 @@ typedef enum {
   ALT_E_SHAPE = 2,        /* layout logical shape != operand shape; B > D      */
   ALT_E_NONDIVISIBLE = 3, /* split factors do not multiply to the extent      */
   ALT_E_LOSSY = 4,        /* a needed element has no copy in the source layout */
-  ALT_E_UNSUPPORTED = 5,  /* valid request without a kernel (e.g. dilation>1) */
+  ALT_E_UNSUPPORTED = 5,  /* valid request without a kernel on the forced path */
   ALT_E_CUDA = 6,         /* CUDA runtime / driver error                      */
   ALT_E_NOMEM = 7         /* host or device allocation failed                 */
 } alt_status;
@@ -149,7 +149,10 @@ alt_status alt_relayout(alt_layout src_l, const void *src, alt_layout dst_l,
  * with x = 0 outside [0,H)x[0,W) (semantic zero padding; if x_l itself holds
  * pad zeros the kernel may read them instead — identical results).
  * groups in {1, C (depthwise, K == C)}; other groups run on the generic
- * path; dil_h = dil_w = 1 (else ALT_E_UNSUPPORTED). */
+ * path; dil_h / dil_w > 1 (dilated conv, the paper's DIL operator): tap
+ * (r, s) reads x[p V - pad + dil_h r, q V - pad + dil_w s], Ho = (H + 2 pad -
+ * dil (R - 1) - 1) / V + 1; served by the SIMT path (ALT_E_UNSUPPORTED when
+ * the tensor-core or depthwise path is forced). */
 typedef struct {
   int64_t N, C, H, W, K, R, S;
   int32_t stride_h, stride_w, pad_h, pad_w, dil_h, dil_w, groups;

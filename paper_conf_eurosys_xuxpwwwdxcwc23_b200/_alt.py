@@ -272,13 +272,13 @@ def _cfg(cfg):
     return c
 
 
-def conv_params(N, C, H, W, K, R, S, stride=1, pad=0, groups=1) -> ConvParams:
+def conv_params(N, C, H, W, K, R, S, stride=1, pad=0, groups=1, dilation=1) -> ConvParams:
     p = ConvParams()
     p.N, p.C, p.H, p.W, p.K, p.R, p.S = N, C, H, W, K, R, S
     sh, sw = (stride, stride) if isinstance(stride, int) else stride
     ph, pw = (pad, pad) if isinstance(pad, int) else pad
     p.stride_h, p.stride_w, p.pad_h, p.pad_w = sh, sw, ph, pw
-    p.dil_h = p.dil_w = 1
+    p.dil_h, p.dil_w = (dilation, dilation) if isinstance(dilation, int) else dilation
     p.groups = groups
     return p
 

@@ -162,12 +162,13 @@ alt_status alt_conv2d(const alt_conv2d_params *p, alt_layout x_l, const void *x,
     set_error("alt_conv2d: bad geometry");
     return ALT_E_INVALID;
   }
-  if (p->dil_h > 1 || p->dil_w > 1) { set_error("alt_conv2d: dilation > 1 not supported (NEXT)"); return ALT_E_UNSUPPORTED; }
+  const int32_t dh = p->dil_h < 1 ? 1 : p->dil_h, dw = p->dil_w < 1 ? 1 : p->dil_w;
   const int32_t G = p->groups < 1 ? 1 : p->groups;
   if (p->C % G || p->K % G) { set_error("alt_conv2d: groups must divide C and K"); return ALT_E_INVALID; }
-  const int64_t Ho = (p->H + 2 * p->pad_h - p->R) / p->stride_h + 1;
-  const int64_t Wo = (p->W + 2 * p->pad_w - p->S) / p->stride_w + 1;
-  if (Ho < 1 || Wo < 1) { set_error("alt_conv2d: empty output"); return ALT_E_INVALID; }
+  const int64_t Ho = (p->H + 2 * p->pad_h - (int64_t)dh * (p->R - 1) - 1) / p->stride_h + 1;
+  const int64_t Wo = (p->W + 2 * p->pad_w - (int64_t)dw * (p->S - 1) - 1) / p->stride_w + 1;
+  if (p->H + 2 * p->pad_h < (int64_t)dh * (p->R - 1) + 1 || p->W + 2 * p->pad_w < (int64_t)dw * (p->S - 1) + 1 ||
+      Ho < 1 || Wo < 1) { set_error("alt_conv2d: empty output"); return ALT_E_INVALID; }
   const int64_t xs[4] = {p->N, p->C, p->H, p->W}, ws[4] = {p->K, p->C / G, p->R, p->S},
                 ys[4] = {p->N, p->K, Ho, Wo};
   if (p->N > 0 && (!shape_is(&x_l->impl, 4, xs) || !shape_is(&w_l->impl, 4, ws) || !shape_is(&y_l->impl, 4, ys))) {
@@ -180,6 +181,7 @@ alt_status alt_conv2d(const alt_conv2d_params *p, alt_layout x_l, const void *x,
   P.N = p->N; P.C = p->C; P.H = p->H; P.W = p->W; P.K = p->K; P.R = p->R; P.S = p->S;
   P.Ho = Ho; P.Wo = Wo;
   P.Vh = p->stride_h; P.Vw = p->stride_w; P.ph = p->pad_h; P.pw = p->pad_w; P.groups = G;
+  P.dh = dh; P.dw = dw;
   P.xl = &x_l->impl; P.wl = &w_l->impl; P.yl = &y_l->impl;
   P.x = x; P.w = w; P.y = y; P.dtype = dtype;
   alt_status st = fill_epi(epi, P.yl, &P.epi);
@@ -187,14 +189,21 @@ alt_status alt_conv2d(const alt_conv2d_params *p, alt_layout x_l, const void *x,
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   const int32_t path = cfg ? cfg->path : ALT_PATH_AUTO;
   alt_kernel_cfg used{};
-  if (path == ALT_PATH_TC || (path == ALT_PATH_AUTO && G == 1)) {
+  // dilation runs on the generic path (the tensor-core and depthwise kernels
+  // cut undilated windows)
+  const bool dil = dh > 1 || dw > 1;
+  if (dil && (path == ALT_PATH_TC || path == ALT_PATH_DW)) {
+    set_error("alt_conv2d: dilation > 1 runs on the SIMT path only");
+    return ALT_E_UNSUPPORTED;
+  }
+  if (!dil && (path == ALT_PATH_TC || (path == ALT_PATH_AUTO && G == 1))) {
     st = tc_conv(P, cfg, s, &used);
     if (st != ALT_E_UNSUPPORTED || path == ALT_PATH_TC) {
       if (st == ALT_OK) set_last_plan(used);
       return st;
     }
   }
-  if (path == ALT_PATH_DW || (path == ALT_PATH_AUTO && G == p->C && G == p->K)) {
+  if (!dil && (path == ALT_PATH_DW || (path == ALT_PATH_AUTO && G == p->C && G == p->K))) {
     st = dw_conv(P, s, &used);
     if (st != ALT_E_UNSUPPORTED || path == ALT_PATH_DW) {
       if (st == ALT_OK) set_last_plan(used);

@@ -18,6 +18,7 @@ struct OpEpilogue {
 struct ConvProblem {
   int64_t N, C, H, W, K, R, S, Ho, Wo;
   int32_t Vh, Vw, ph, pw, groups;
+  int32_t dh = 1, dw = 1;  // dilation (SIMT path)
   Layout *xl, *wl, *yl;
   const void *x, *w;
   void *y;

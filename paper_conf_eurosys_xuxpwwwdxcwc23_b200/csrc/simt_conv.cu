@@ -25,6 +25,7 @@ struct SimtArgs {
   // conv geometry
   int64_t N, C, H, W, K, R, S, Ho, Wo;
   int32_t Vh, Vw, ph, pw;
+  int32_t dh, dw;  // dilation
   Reader xr, wr;                // conv: x (n,c,h,w), w (k,c,r,s); gemm: A (m,k), B (k,n)
   Writer yw;
   EpiParams epi;
@@ -72,7 +73,7 @@ __global__ void __launch_bounds__(256) k_simt_igemm(SimtArgs a, const T *__restr
         if (a.is_conv) {
           const int64_t c = k / RS, rs = k - c * RS;
           const int64_t r = rs / a.S, s = rs - r * a.S;
-          const int64_t ih = row_h[mm] + r, iw = row_w[mm] + s;
+          const int64_t ih = row_h[mm] + r * a.dh, iw = row_w[mm] + s * a.dw;
           off = (ih >= 0 && ih < a.H && iw >= 0 && iw < a.W) ? a.xr.off4(rn, c, ih, iw) : -1;
         } else {
           off = a.xr.off2(rn, k);
@@ -167,10 +168,10 @@ __global__ void __launch_bounds__(256) k_simt_grouped(SimtArgs a, int64_t G, con
     float acc = 0.f;
     for (int64_t c = 0; c < Cg; c++)
       for (int64_t r = 0; r < a.R; r++) {
-        const int64_t ih = p * a.Vh - a.ph + r;
+        const int64_t ih = p * a.Vh - a.ph + r * a.dh;
         if (ih < 0 || ih >= a.H) continue;
         for (int64_t s = 0; s < a.S; s++) {
-          const int64_t iw = q * a.Vw - a.pw + s;
+          const int64_t iw = q * a.Vw - a.pw + s * a.dw;
           if (iw < 0 || iw >= a.W) continue;
           const int64_t xo = a.xr.off4(n, g * Cg + c, ih, iw);
           const int64_t wo = a.wr.off4(k, c, r, s);
@@ -235,6 +236,7 @@ alt_status simt_conv(const ConvProblem &P, cudaStream_t stream) {
   a.N = P.N; a.C = P.C; a.H = P.H; a.W = P.W; a.K = P.K; a.R = P.R; a.S = P.S;
   a.Ho = P.Ho; a.Wo = P.Wo;
   a.Vh = P.Vh; a.Vw = P.Vw; a.ph = P.ph; a.pw = P.pw;
+  a.dh = P.dh; a.dw = P.dw;
   a.M = P.N * P.Ho * P.Wo;
   a.Ncol = P.K;
   a.Kred = (P.C / P.groups) * P.R * P.S;

@@ -193,6 +193,7 @@ extern "C" alt_status alt_tune(alt_op_kind op, const void *op_params, alt_dtype 
   if (op == ALT_OP_CONV2D) {
     const alt_conv2d_params &p = *static_cast<const alt_conv2d_params *>(op_params);
     if (p.groups > 1) { set_error("alt_tune: grouped conv has no template (NEXT)"); scratch.release(s); return ALT_E_UNSUPPORTED; }
+    if (p.dil_h > 1 || p.dil_w > 1) { set_error("alt_tune: dilated conv has no template (NEXT)"); scratch.release(s); return ALT_E_UNSUPPORTED; }
     const int64_t Ho = (p.H + 2 * p.pad_h - p.R) / p.stride_h + 1, Wo = (p.W + 2 * p.pad_w - p.S) / p.stride_w + 1;
     const int64_t Cp = p.C % 8 ? (p.C + 7) / 8 * 8 : p.C;
     const int64_t xl[4] = {p.N, p.C, p.H, p.W}, wl[4] = {p.K, p.C, p.R, p.S}, yl[4] = {p.N, p.K, Ho, Wo};

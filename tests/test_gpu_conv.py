@@ -368,3 +368,37 @@ def test_tc_tail_split(sk):
     run_conv("tailc%d" % sk, 8, 256, 14, 14, 512, 3, 3, 1, 1, xp, wp, yp, torch.bfloat16, epi=True,
              res_p=LY.nchwxc(512, 64), act=1, cfg={"path": alt.PATH_TC, "block_n": 256, "split_k": sk,
                                                    "split_cluster": 2}, expect_path=alt.PATH_TC)
+
+
+# ------------------------------------------------------- dilation (DIL) --
+DIL = [  # name, N, C, H, W, K, R, V, pad, dil, groups, x, w, y
+    ("d2_nchw8c", 2, 16, 13, 11, 24, 3, 1, 2, 2, 1, LY.nchwxc(16, 8), LY.kcrs_yk_xc(24, 16, 8, 8), LY.nchwxc(24, 8)),
+    ("d3_s2_plain", 1, 8, 17, 15, 8, 3, 2, 3, 3, 1, [], [], []),
+    ("d2_grouped", 2, 16, 9, 9, 16, 3, 1, 2, 2, 4, LY.nhwc(), [], LY.nhwc()),
+]
+
+
+@pytest.mark.parametrize("case", DIL, ids=[c[0] for c in DIL])
+@pytest.mark.parametrize("dtype", [torch.float32, torch.bfloat16])
+def test_dilated_conv(case, dtype):
+    """dilated conv (the paper's DIL operator) on the generic path through any layouts"""
+    name, N, C, H, W, K, R, V, pad, d, g, xp, wp, yp = case
+    x = synth.activations(name + "x", (N, C, H, W))
+    w = synth.weights(name + "w", (K, C // g, R, R))
+    Ho = (H + 2 * pad - d * (R - 1) - 1) // V + 1
+    Wo = (W + 2 * pad - d * (R - 1) - 1) // V + 1
+    Ox, xph, xd = make_operand(name, xp, x, dtype)
+    Ow, wph, wd = make_operand(name + "w", wp, w, dtype)
+    Lx, Lw, Ly = alt.Layout(x.shape, xp), alt.Layout(w.shape, wp), alt.Layout((N, K, Ho, Wo), yp)
+    y = torch.full(Ly.phys_shape, 3.0, dtype=dtype, device="cuda")
+    p = alt.conv_params(N, C, H, W, K, R, R, V, pad, g, dilation=d)
+    alt.conv2d(p, Lx, xd, Lw, wd, Ly, y, act=1)
+    torch.cuda.synchronize()
+    assert alt.last_plan()["path"] == alt.PATH_SIMT
+    pd = dict(N=N, C=C, H=H, W=W, K=K, R=R, S=R, stride_h=V, stride_w=V, pad_h=pad, pad_w=pad, groups=g,
+              dil_h=d, dil_w=d)
+    ref = oracle.conv2d(pd, Ox, xph, Ow, wph, act=1)
+    assert_parity(read_output(oracle.Layout((N, K, Ho, Wo), yp), y, dtype), ref, dtype)
+    with pytest.raises(alt.AltError) as e:   # forced tensor-core path: no dilated kernel
+        alt.conv2d(p, Lx, xd, Lw, wd, Ly, y, cfg={"path": alt.PATH_TC})
+    assert e.value.code == alt._alt.ALT_E_UNSUPPORTED
