@@ -151,8 +151,9 @@ alt_status alt_relayout(alt_layout src_l, const void *src, alt_layout dst_l,
  * groups in {1, C (depthwise, K == C)}; other groups run on the generic
  * path; dil_h / dil_w > 1 (dilated conv, the paper's DIL operator): tap
  * (r, s) reads x[p V - pad + dil_h r, q V - pad + dil_w s], Ho = (H + 2 pad -
- * dil (R - 1) - 1) / V + 1; served by the SIMT path (ALT_E_UNSUPPORTED when
- * the tensor-core or depthwise path is forced). */
+ * dil (R - 1) - 1) / V + 1; served by the tensor-core path (the tap offset
+ * d r enters the TMA box coordinates) or the SIMT path (ALT_E_UNSUPPORTED when
+ * the depthwise path is forced). */
 typedef struct {
   int64_t N, C, H, W, K, R, S;
   int32_t stride_h, stride_w, pad_h, pad_w, dil_h, dil_w, groups;

@@ -189,14 +189,14 @@ alt_status alt_conv2d(const alt_conv2d_params *p, alt_layout x_l, const void *x,
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   const int32_t path = cfg ? cfg->path : ALT_PATH_AUTO;
   alt_kernel_cfg used{};
-  // dilation runs on the generic path (the tensor-core and depthwise kernels
-  // cut undilated windows)
+  // dilation: tensor-core path (tap offsets d r in the TMA box rule) or the
+  // generic path; the depthwise kernel cuts undilated windows
   const bool dil = dh > 1 || dw > 1;
-  if (dil && (path == ALT_PATH_TC || path == ALT_PATH_DW)) {
-    set_error("alt_conv2d: dilation > 1 runs on the SIMT path only");
+  if (dil && path == ALT_PATH_DW) {
+    set_error("alt_conv2d: dilation > 1 has no depthwise kernel (SIMT or tensor-core path)");
     return ALT_E_UNSUPPORTED;
   }
-  if (!dil && (path == ALT_PATH_TC || (path == ALT_PATH_AUTO && G == 1))) {
+  if (path == ALT_PATH_TC || (path == ALT_PATH_AUTO && G == 1)) {
     st = tc_conv(P, cfg, s, &used);
     if (st != ALT_E_UNSUPPORTED || path == ALT_PATH_TC) {
       if (st == ALT_OK) set_last_plan(used);

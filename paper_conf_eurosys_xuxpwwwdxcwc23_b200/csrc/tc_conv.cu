@@ -1751,8 +1751,10 @@ alt_status tc_conv(const ConvProblem &P, const alt_kernel_cfg *cfg, cudaStream_t
   // x logical (n, c, h, w); w logical (k, c, r, s); y logical (n, k, p, q)
   T.ra[0].role = R_N;
   T.ra[1].role = R_C;
-  T.ra[2] = RoleInfo{R_H, 1, P.Vh, P.ph, (int)P.R, 1};
-  T.ra[3] = RoleInfo{R_W, 1, P.Vw, P.pw, (int)P.S, 1};
+  // dilation d: tap r adds d r to the box coordinate (the TMA coordinate
+  // rule's V_R coefficient) and the window spans d (R - 1) + 1 rows
+  T.ra[2] = RoleInfo{R_H, 1, P.Vh, P.ph, (int)((P.R - 1) * P.dh + 1), P.dh};
+  T.ra[3] = RoleInfo{R_W, 1, P.Vw, P.pw, (int)((P.S - 1) * P.dw + 1), P.dw};
   T.rb[0] = RoleInfo{R_W, 1, 1, 0, 1, 0};
   T.rb[1].role = R_C;
   T.rb[2].role = R_TR;
@@ -1768,7 +1770,7 @@ alt_status tc_conv(const ConvProblem &P, const alt_kernel_cfg *cfg, cudaStream_t
   {
     LView xf, wf;
     int64_t Cf = 0;
-    if (fold_window(T.va, T.vb, P.S, P.Vw, P.pw, P.Wo, &xf, &wf, &Cf)) {
+    if (P.dw == 1 && fold_window(T.va, T.vb, P.S, P.Vw, P.pw, P.Wo, &xf, &wf, &Cf)) {
       T.va = xf; T.vb = wf;
       T.ra[3] = RoleInfo{R_W, 1, 1, 0, 1, 0};
       T.S = 1; T.C = Cf;

@@ -381,7 +381,8 @@ DIL = [  # name, N, C, H, W, K, R, V, pad, dil, groups, x, w, y
 @pytest.mark.parametrize("case", DIL, ids=[c[0] for c in DIL])
 @pytest.mark.parametrize("dtype", [torch.float32, torch.bfloat16])
 def test_dilated_conv(case, dtype):
-    """dilated conv (the paper's DIL operator) on the generic path through any layouts"""
+    """dilated conv (the paper's DIL operator) through any layouts, on the SIMT
+    path and (channel-tiled bf16 layouts) the tensor-core path"""
     name, N, C, H, W, K, R, V, pad, d, g, xp, wp, yp = case
     x = synth.activations(name + "x", (N, C, H, W))
     w = synth.weights(name + "w", (K, C // g, R, R))
@@ -392,13 +393,16 @@ def test_dilated_conv(case, dtype):
     Lx, Lw, Ly = alt.Layout(x.shape, xp), alt.Layout(w.shape, wp), alt.Layout((N, K, Ho, Wo), yp)
     y = torch.full(Ly.phys_shape, 3.0, dtype=dtype, device="cuda")
     p = alt.conv_params(N, C, H, W, K, R, R, V, pad, g, dilation=d)
-    alt.conv2d(p, Lx, xd, Lw, wd, Ly, y, act=1)
-    torch.cuda.synchronize()
-    assert alt.last_plan()["path"] == alt.PATH_SIMT
     pd = dict(N=N, C=C, H=H, W=W, K=K, R=R, S=R, stride_h=V, stride_w=V, pad_h=pad, pad_w=pad, groups=g,
               dil_h=d, dil_w=d)
     ref = oracle.conv2d(pd, Ox, xph, Ow, wph, act=1)
-    assert_parity(read_output(oracle.Layout((N, K, Ho, Wo), yp), y, dtype), ref, dtype)
-    with pytest.raises(alt.AltError) as e:   # forced tensor-core path: no dilated kernel
-        alt.conv2d(p, Lx, xd, Lw, wd, Ly, y, cfg={"path": alt.PATH_TC})
+    paths = [alt.PATH_SIMT] + ([alt.PATH_TC] if g == 1 and dtype == torch.bfloat16 and C % 8 == 0 and xp else [])
+    for path in paths:
+        y.fill_(3.0)
+        alt.conv2d(p, Lx, xd, Lw, wd, Ly, y, act=1, cfg={"path": path})
+        torch.cuda.synchronize()
+        assert alt.last_plan()["path"] == path
+        assert_parity(read_output(oracle.Layout((N, K, Ho, Wo), yp), y, dtype), ref, dtype)
+    with pytest.raises(alt.AltError) as e:   # forced depthwise path: no dilated kernel
+        alt.conv2d(p, Lx, xd, Lw, wd, Ly, y, cfg={"path": alt.PATH_DW})
     assert e.value.code == alt._alt.ALT_E_UNSUPPORTED
