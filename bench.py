@@ -191,6 +191,38 @@ class LayerSet:
                        bias=l["bi"], act="relu", cfg=l["cfg"])
             l["y_host"].copy_(l["y"], non_blocking=True)
 
+    def step_e2e_overlap(self, start_ev=None):
+        """the same work with the copies on their own streams: H2D of layer
+        i + 1 and D2H of layer i - 1 overlap layer i's conversion and conv
+        (per-layer events order every buffer reuse, also across steps)"""
+        import torch
+        alt = self.alt
+        comp = torch.cuda.current_stream()
+        if not hasattr(self, "s_in"):
+            self.s_in, self.s_out = torch.cuda.Stream(), torch.cuda.Stream()
+            self.ev = [{k: torch.cuda.Event() for k in ("in", "rl", "conv", "out")} for _ in self.layers]
+        if start_ev is not None:
+            self.s_in.wait_event(start_ev)
+            self.s_out.wait_event(start_ev)
+        for l, e in zip(self.layers, self.ev):
+            self.s_in.wait_event(e["rl"])            # previous step's relayout read x0d
+            with torch.cuda.stream(self.s_in):
+                l["x0d"].copy_(l["x_host"], non_blocking=True)
+            e["in"].record(self.s_in)
+            comp.wait_event(e["in"])
+            alt.relayout(l["lx0"], l["x0d"], l["lx"], l["x"])
+            e["rl"].record(comp)
+            comp.wait_event(e["out"])                # previous step's D2H read y
+            alt.conv2d(l["p"], l["lx"], l["x"], l["lw"], l["w"], l["ly"], l["y"], scale=l["sc"],
+                       bias=l["bi"], act="relu", cfg=l["cfg"])
+            e["conv"].record(comp)
+            self.s_out.wait_event(e["conv"])
+            with torch.cuda.stream(self.s_out):
+                l["y_host"].copy_(l["y"], non_blocking=True)
+            e["out"].record(self.s_out)
+        comp.wait_event(self.ev[-1]["out"])         # the step ends when its last result is on the host
+        comp.wait_stream(self.s_in)
+
     def io_bytes(self):
         h2d = sum(l["x_host"].numel() * 2 for l in self.layers)
         d2h = sum(l["y_host"].numel() * 2 for l in self.layers)
@@ -371,17 +403,18 @@ def main():
                           "block_n": plans[i]["block_n"]})
     value = S.flops * ws / (ms * 1e-3) / 1e12
 
-    # e2e through the public API with host buffers
+    # e2e through the public API with host buffers (copies overlapped with
+    # the conversions and convs on their own streams)
     for _ in range(2):
-        S.step_e2e()
+        S.step_e2e_overlap()
     torch.cuda.synchronize()
     barrier(ws)
     e0 = torch.cuda.Event(enable_timing=True)
     e1 = torch.cuda.Event(enable_timing=True)
     e_steps = max(1, min(args.steps, 5))
     e0.record(stream)
-    for _ in range(e_steps):
-        S.step_e2e()
+    for k in range(e_steps):
+        S.step_e2e_overlap(start_ev=e0 if k == 0 else None)
     e1.record(stream)
     torch.cuda.synchronize()
     e_ms = max_over_ranks(e0.elapsed_time(e1) / e_steps, ws)
@@ -404,7 +437,9 @@ def main():
                                  "bytes/HBM peak) / sum of measured layer times"},
             "e2e": {"value": round(S.flops * ws / (e_ms * 1e-3) / 1e12, 3), "unit": "TFLOP/s",
                     "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
-                    "ms_per_step": round(e_ms, 3)},
+                    "ms_per_step": round(e_ms, 3),
+                    "note": "per layer: pinned H2D of the NCHW input, conversion to the tuned layout, "
+                            "conv, D2H of the output; copies on their own streams overlap compute"},
             "gpu_launches": launches, "clocks": getattr(clk, "summary", None),
             "per_layer": per_layer}
     traffic_file = os.path.join(ROOT, "profiles", "traffic_r50.json")

@@ -52,6 +52,17 @@ def test_r50_layer_set_b32_bench_config():
             worst = max(worst, err)
             assert err <= BF16_TOL, (L.name, n, err)
     assert worst > 0.0  # bf16 outputs: an exact match would mean the check compared nothing
+    # the e2e path (copies on their own streams, events ordering every buffer
+    # reuse across steps) delivers the same outputs to the host
+    for l in S.layers:
+        l["y"].zero_()
+    for _ in range(2):
+        S.step_e2e_overlap()
+    torch.cuda.synchronize()
+    S.step()
+    torch.cuda.synchronize()
+    for l in S.layers:
+        assert np.array_equal(words(l["y_host"]), words(l["y"])), l["L"].name
 
 
 def _check_chain_images(ch: CH.Chain, relu6: bool, images):
