@@ -610,6 +610,7 @@ __global__ void __launch_bounds__(kThreads, 1)
                          "r"(raw[4 * j4]), "r"(raw[4 * j4 + 1]), "r"(raw[4 * j4 + 2]), "r"(raw[4 * j4 + 3])
                          : "memory");
         }
+        if (et == 0) { DBG(36); }
         continue;  // one tile per CTA; phase 2 after the cluster barrier
       }
       const float *wsl = nullptr;  // this CTA tile's partials (split-K)
@@ -868,6 +869,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       // are read through DSMEM and summed in split order
       __syncwarp();
       cluster_sync();
+      if (et == 0) { DBG(37); }
       const int crank = (int)cluster_ctarank();
       const TileCoord tc = tile_coord(a, unit_info(a, unit0).mn, BN, CG, rank);
       constexpr int NQ = 4 / SC, NCH = BN / 32;
@@ -881,18 +883,25 @@ __global__ void __launch_bounds__(kThreads, 1)
 #pragma unroll
         for (int j = 0; j < 32; j++) t[j] = 0.f;
         const uint32_t local = smem_u32(smem) + (uint32_t)((ch * 128 + rr) * 128);
+        // all eight 16-byte loads of a split are issued before any add (an
+        // add right after its load would stall the in-order issue and
+        // serialise the distributed-shared-memory round trips)
+#pragma unroll
         for (int sp2 = 0; sp2 < SC; sp2++) {
           uint32_t ra;
-          asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(ra) : "r"(local), "r"(sp2));
+          asm("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(ra) : "r"(local), "r"(sp2));
+          float4 f[8];
+#pragma unroll
+          for (int j4 = 0; j4 < 8; j4++)
+            asm volatile("ld.shared::cluster.v4.f32 {%0, %1, %2, %3}, [%4];"
+                         : "=f"(f[j4].x), "=f"(f[j4].y), "=f"(f[j4].z), "=f"(f[j4].w)
+                         : "r"(ra + (uint32_t)((j4 ^ (rr & 7)) * 16)));
 #pragma unroll
           for (int j4 = 0; j4 < 8; j4++) {
-            float f0, f1, f2, f3;
-            asm volatile("ld.shared::cluster.v4.f32 {%0, %1, %2, %3}, [%4];"
-                         : "=f"(f0), "=f"(f1), "=f"(f2), "=f"(f3)
-                         : "r"(ra + (uint32_t)((j4 ^ (rr & 7)) * 16)));
-            t[4 * j4] += f0; t[4 * j4 + 1] += f1; t[4 * j4 + 2] += f2; t[4 * j4 + 3] += f3;
+            t[4 * j4] += f[j4].x; t[4 * j4 + 1] += f[j4].y; t[4 * j4 + 2] += f[j4].z; t[4 * j4 + 3] += f[j4].w;
           }
         }
+        if (et == 0 && cnt == 0) { DBG(38); }
         float v[32];
 #pragma unroll
         for (int j = 0; j < 8; j++) {
@@ -949,6 +958,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           }
           bulk_commit();
         }
+        if (et == 0 && cnt == 0) { DBG(39); }
       }
     }
     if (et == 0) { DBG(5); }
