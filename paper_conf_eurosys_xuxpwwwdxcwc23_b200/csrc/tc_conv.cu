@@ -435,7 +435,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
       }
     }
-    if constexpr (SC > 1) { __syncwarp(); cluster_sync(); }  // partials of the cluster drained
+    if constexpr (SC > 1) { __syncwarp(); cluster_sync(); cluster_sync(); }  // rings free; partials pushed
   } else if (warp == 1) {
     if (lane == 0 && rank == 0) {
       // ------------------------------------------------------ MMA issuer
@@ -490,7 +490,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         if (i == 0) { DBG(3); }
       }
     }
-    if constexpr (SC > 1) { __syncwarp(); cluster_sync(); }  // partials of the cluster drained
+    if constexpr (SC > 1) { __syncwarp(); cluster_sync(); cluster_sync(); }  // rings free; partials pushed
   } else {
     // -------------------------------------------------------- epilogue
     // 8 warps: warp w reads TMEM lane quarter (w % 4) (hardware rule) and
@@ -593,22 +593,36 @@ __global__ void __launch_bounds__(kThreads, 1)
       if (et == 0 && i == ALT_DBG_TILE) { DBG(2); }
       tc_fence_after();
       if constexpr (SC > 1) {
-        // cluster split-K, phase 1: this CTA's fp32 partial -> its own smem
-        // ring (every stage consumed: one tile per CTA), [BN/32][128 rows][32]
-        // with the 16-byte slots of a row XOR-swizzled by (row & 7)
+        // cluster split-K, phase 1: this CTA's fp32 partial rows are pushed
+        // (fire-and-forget DSMEM stores) into the ring of the CTA that
+        // finishes them — lane quarter q belongs to split q * SC / 4 — as
+        // slice [my split][quarter within the owner][32-column chunk], each
+        // 32 rows x 128 B with the 16-byte slots XOR-swizzled by (row & 7);
+        // phase 2 then reduces from local shared memory only
+        // every CTA's MMAs must be complete (its ring consumed) before any
+        // peer writes into it: a cluster barrier after the accumulator is full
+        __syncwarp();
+        cluster_sync();
+        {
+          constexpr int NQ = 4 / SC;
+          const int my_split = (int)cluster_ctarank();
+          const int owner = (wq * SC) / 4, qi = wq - owner * NQ;
 #pragma unroll 1
-        for (int c0 = 0; c0 < BN; c0 += kStep) {
-          const int cb = c0 + half * 32;
-          if (cb >= BN) continue;
-          uint32_t raw[32];
-          tmem_ld_32x32b_x32(tmem + ((uint32_t)(wq * 32) << 16) + (uint32_t)(acc * BN + cb), raw);
-          tmem_ld_wait();
-          const uint32_t base = smem_u32(smem) + (uint32_t)(((cb >> 5) * 128 + row) * 128);
+          for (int c0 = 0; c0 < BN; c0 += kStep) {
+            const int cb = c0 + half * 32;
+            if (cb >= BN) continue;
+            uint32_t raw[32];
+            tmem_ld_32x32b_x32(tmem + ((uint32_t)(wq * 32) << 16) + (uint32_t)(acc * BN + cb), raw);
+            tmem_ld_wait();
+            const uint32_t slice = (uint32_t)(((my_split * NQ + qi) * (BN / 32) + (cb >> 5)) * 4096);
+            uint32_t ra;
+            asm("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(ra) : "r"(smem_u32(smem) + slice + lane * 128), "r"(owner));
 #pragma unroll
-          for (int j4 = 0; j4 < 8; j4++)
-            asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(base + (uint32_t)((j4 ^ (row & 7)) * 16)),
-                         "r"(raw[4 * j4]), "r"(raw[4 * j4 + 1]), "r"(raw[4 * j4 + 2]), "r"(raw[4 * j4 + 3])
-                         : "memory");
+            for (int j4 = 0; j4 < 8; j4++)
+              asm volatile("st.shared::cluster.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(ra + (uint32_t)((j4 ^ (lane & 7)) * 16)),
+                           "r"(raw[4 * j4]), "r"(raw[4 * j4 + 1]), "r"(raw[4 * j4 + 2]), "r"(raw[4 * j4 + 3])
+                           : "memory");
+          }
         }
         if (et == 0) { DBG(36); }
         continue;  // one tile per CTA; phase 2 after the cluster barrier
@@ -882,20 +896,17 @@ __global__ void __launch_bounds__(kThreads, 1)
         float t[32];
 #pragma unroll
         for (int j = 0; j < 32; j++) t[j] = 0.f;
-        const uint32_t local = smem_u32(smem) + (uint32_t)((ch * 128 + rr) * 128);
-        // all eight 16-byte loads of a split are issued before any add (an
-        // add right after its load would stall the in-order issue and
-        // serialise the distributed-shared-memory round trips)
+        // the SC slices of these rows were pushed here in phase 1: local reads
+        const int qi = qq - crank * NQ;
 #pragma unroll
         for (int sp2 = 0; sp2 < SC; sp2++) {
-          uint32_t ra;
-          asm("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(ra) : "r"(local), "r"(sp2));
+          const uint32_t ra = smem_u32(smem) + (uint32_t)(((sp2 * NQ + qi) * NCH + ch) * 4096 + lane * 128);
           float4 f[8];
 #pragma unroll
           for (int j4 = 0; j4 < 8; j4++)
-            asm volatile("ld.shared::cluster.v4.f32 {%0, %1, %2, %3}, [%4];"
+            asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];"
                          : "=f"(f[j4].x), "=f"(f[j4].y), "=f"(f[j4].z), "=f"(f[j4].w)
-                         : "r"(ra + (uint32_t)((j4 ^ (rr & 7)) * 16)));
+                         : "r"(ra + (uint32_t)((j4 ^ (lane & 7)) * 16)));
 #pragma unroll
           for (int j4 = 0; j4 < 8; j4++) {
             t[4 * j4] += f[j4].x; t[4 * j4 + 1] += f[j4].y; t[4 * j4 + 2] += f[j4].z; t[4 * j4 + 3] += f[j4].w;
