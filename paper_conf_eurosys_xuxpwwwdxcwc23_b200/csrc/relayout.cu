@@ -496,7 +496,7 @@ __global__ void __launch_bounds__(256) k_relayout_row(RowPlan R, const T *__rest
       const int o = (int)R.f_vpb.div((uint32_t)v), w = (v - o * vpb) * V;
       const T *rb = rows + (size_t)o * rows_per;
       const int bc = s_bcombo[o], lo = s_lo[o];
-      T val[V];
+      T val[V] = {};
       if constexpr (RB > 0) {
         const unsigned char *ob = reinterpret_cast<const unsigned char *>(rb);
         constexpr int RUNS = 16 / RB;  // X-runs per 16-byte dst vector

@@ -891,7 +891,6 @@ __global__ void __launch_bounds__(kThreads, 1)
       int cnt = 0;
       for (int item = ew; item < NQ * NCH; item += kEpiWarps, cnt++) {
         const int qq = crank * NQ + item / NCH, ch = item % NCH;
-        const int rr = qq * 32 + lane;  // tile row of this thread
         const int cb = ch * 32, kb = tc.k0 + cb;
         float t[32];
 #pragma unroll
