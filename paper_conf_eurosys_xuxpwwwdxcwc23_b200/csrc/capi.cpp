@@ -196,7 +196,8 @@ alt_status alt_conv2d(const alt_conv2d_params *p, alt_layout x_l, const void *x,
     set_error("alt_conv2d: dilation > 1 has no depthwise kernel (SIMT or tensor-core path)");
     return ALT_E_UNSUPPORTED;
   }
-  if (path == ALT_PATH_TC || (path == ALT_PATH_AUTO && G == 1)) {
+  const bool grp_tc = G > 1 && G < p->C && (p->C / G) % 8 == 0 && (p->K / G) % 8 == 0;
+  if (path == ALT_PATH_TC || (path == ALT_PATH_AUTO && (G == 1 || grp_tc))) {
     st = tc_conv(P, cfg, s, &used);
     if (st != ALT_E_UNSUPPORTED || path == ALT_PATH_TC) {
       if (st == ALT_OK) set_last_plan(used);

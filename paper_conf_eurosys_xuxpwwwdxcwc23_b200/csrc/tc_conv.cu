@@ -59,6 +59,9 @@ struct TcArgs {
   OperandMap A, B, O;
   int32_t out_mode;      // 1: TMA-store epilogue, 2: direct 16-byte stores, 0: generic writer
   int32_t res_vec;       // residual read as 16-byte vectors of 8 channels (epi.res tables)
+  // grouped conv: one launch per group; the group's input channel slabs start
+  // at slab a_goff of x, its weight rows at b_koff, its outputs at channel y_koff
+  int32_t a_goff, b_koff, y_koff;
   int32_t is_conv;
   int32_t N, K, Ho, Wo;  // output: conv y[N,K,Ho,Wo]; GEMM: N=1, Ho=1, Wo=M, K=cols
   int32_t tile_n, tile_h, tile_w;
@@ -180,13 +183,13 @@ __device__ __forceinline__ void bulk_wait_read0() { asm volatile("cp.async.bulk.
 // Out-of-line slow paths of the epilogue (kept out of the hot loop body).
 // residual values of one row's 32 channels, read through the residual layout
 static __device__ __noinline__ void residual_chunk(const EpiParams &e, int is_conv, int K, int n, int p, int q,
-                                                   int kb, float *out) {
+                                                   int kb, int koff, float *out) {
   const uint16_t *res = static_cast<const uint16_t *>(e.residual);
   for (int j = 0; j < 32; j++) {
     const int k = kb + j;
     float r = 0.f;
     if (k < K) {
-      const int64_t o = is_conv ? e.res.off4(n, k, p, q) : e.res.off2(q, k);
+      const int64_t o = is_conv ? e.res.off4(n, koff + k, p, q) : e.res.off2(q, koff + k);
       if (o >= 0) r = bf16_to_f32(__ldg(res + o));
     }
     out[j] = r;
@@ -194,13 +197,13 @@ static __device__ __noinline__ void residual_chunk(const EpiParams &e, int is_co
 }
 // one row's 32 channels through the generic writer (pads, unfold copies)
 static __device__ __noinline__ void write_chunk(const Writer &w, int is_conv, int K, uint16_t *y, int n, int p,
-                                                int q, int kb, const uint32_t *pk) {
+                                                int q, int kb, int koff, const uint32_t *pk) {
   for (int j = 0; j < 32; j++) {
     const int k = kb + j;
     if (k >= K) break;
     const uint16_t h = (uint16_t)(j & 1 ? pk[j >> 1] >> 16 : pk[j >> 1] & 0xffff);
-    if (is_conv) write4<uint16_t>(w, y, n, k, p, q, h);
-    else write2<uint16_t>(w, y, q, k, h);
+    if (is_conv) write4<uint16_t>(w, y, n, koff + k, p, q, h);
+    else write2<uint16_t>(w, y, q, koff + k, h);
   }
 }
 
@@ -329,7 +332,8 @@ __global__ void __launch_bounds__(kThreads, 1)
 #pragma unroll
       for (int o = 0; o < 2; o++) {
         const OperandMap &om = o == 0 ? a.A : a.B;
-        const int gt = (int)om.fg.div((uint32_t)g), gr = g - gt * om.divg;
+        const int ga = o == 0 ? g + a.a_goff : g;
+        const int gt = (int)om.fg.div((uint32_t)ga), gr = ga - gt * om.divg;
 #pragma unroll
         for (int d = 0; d < 5; d++)
           tab[sl * 16 + o * 8 + d] = om.coef[d][V_R] * r + om.coef[d][V_S] * sx + om.coef[d][V_GT] * gt +
@@ -369,7 +373,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       const int k_begin = ui.kb, k_end = ui.ke;
       int32_t v[NVAR];
       // B rows of this CTA: its 1/CG share of the unit's BN output channels
-      const int pp = isA ? tc.p0 : 0, qq = isA ? tc.q0 : tc.k0 + rank * (BN / CG);
+      const int pp = isA ? tc.p0 : 0, qq = isA ? tc.q0 : tc.k0 + rank * (BN / CG) + a.b_koff;
       v[V_N0] = isA ? tc.n0 : 0;
       v[V_PT] = (int)om.fp.div((uint32_t)pp); v[V_PR] = pp - v[V_PT] * om.divp;
       v[V_QT] = (int)om.fq.div((uint32_t)qq); v[V_QR] = qq - v[V_QT] * om.divq;
@@ -422,7 +426,8 @@ __global__ void __launch_bounds__(kThreads, 1)
           const int sl = valid ? slab : 0;
           const int tap = (int)a.f_Gc.div((uint32_t)sl), g = sl - tap * a.Gc;
           v[V_R] = (int)a.f_S.div((uint32_t)tap); v[V_S] = tap - v[V_R] * a.S;
-          v[V_GT] = (int)om.fg.div((uint32_t)g); v[V_GR] = g - v[V_GT] * om.divg;
+          const int ga = isA ? g + a.a_goff : g;
+          v[V_GT] = (int)om.fg.div((uint32_t)ga); v[V_GR] = ga - v[V_GT] * om.divg;
           int32_t c[5];
           coords(om, v, c);
           if (!valid) c[0] = om.oob0;
@@ -585,7 +590,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           const int k = tc.k0 + cbx + 8 * c;
           rq[c] = make_uint4(0u, 0u, 0u, 0u);
           if (rrow >= 0 && k < a.K)
-            rq[c] = __ldg(reinterpret_cast<const uint4 *>(res + rrow + __ldg(a.epi.res.rd[1] + k)));
+            rq[c] = __ldg(reinterpret_cast<const uint4 *>(res + rrow + __ldg(a.epi.res.rd[1] + a.y_koff + k)));
         }
       };
       if constexpr (RV) load_res(half * 32);
@@ -779,7 +784,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           if constexpr (!EARLY) {
             if (!RV && a.epi.residual && vrow) {
               float rv[32];  // local memory, touched only when a residual exists
-              residual_chunk(a.epi, a.is_conv, a.K, n, p, q, kb, rv);
+              residual_chunk(a.epi, a.is_conv, a.K, n, p, q, kb, a.y_koff, rv);
 #pragma unroll
               for (int j = 0; j < 32; j++) v[j] += rv[j];
             }
@@ -806,7 +811,7 @@ __global__ void __launch_bounds__(kThreads, 1)
               for (int c = 0; c < 4; c++) {
                 const int k = kb + 8 * c;
                 if (k < a.K) {
-                  uint16_t *dst = y + yrow + __ldg(a.yr.rd[1] + k);
+                  uint16_t *dst = y + yrow + __ldg(a.yr.rd[1] + a.y_koff + k);
                   asm volatile("st.global.v4.b32 [%0], {%1, %2, %3, %4};" ::"l"(dst), "r"(pk[4 * c]),
                                "r"(pk[4 * c + 1]), "r"(pk[4 * c + 2]), "r"(pk[4 * c + 3])
                                : "memory");
@@ -835,7 +840,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             if (lane == 0) {
               for (int j = 0; j < nslab; j++) {
                 if (kb + (j << lg_sw) >= a.K) break;  // channels past K: nothing to store
-                const int g = (kb >> lg_sw) + j;
+                const int g = ((kb + a.y_koff) >> lg_sw) + j;
                 const int gt = (int)a.O.fg.div((uint32_t)g), gr = g - gt * a.O.divg;
                 int32_t co[5];
 #pragma unroll
@@ -848,7 +853,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             }
           } else if constexpr (!EARLY) {
             // generic layouts: every copy / pad position through the writer
-            if (vrow) write_chunk(a.yw, a.is_conv, a.K, y, n, p, q, kb, pk);
+            if (vrow) write_chunk(a.yw, a.is_conv, a.K, y, n, p, q, kb, a.y_koff, pk);
           }
           if constexpr (!EARLY) {
             if (c0 + kStep < BN) tmem_ld_32x32b_x32(next, raw);
@@ -958,7 +963,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           coords(a.O, vo, cbq);
           for (int j = 0; j < nslab; j++) {
             if (kb + (j << lg_sw) >= a.K) break;
-            const int g = (kb >> lg_sw) + j;
+            const int g = ((kb + a.y_koff) >> lg_sw) + j;
             const int gt = (int)a.O.fg.div((uint32_t)g), gr = g - gt * a.O.divg;
             int32_t co[5];
 #pragma unroll
@@ -1486,6 +1491,7 @@ struct TcProblem {
   int64_t N, K, Ho, Wo;       // output geometry (GEMM: 1, cols, 1, M)
   int64_t R, S, C;            // taps and reduction channels
   OpEpilogue epi;
+  int64_t coff = 0, koff = 0; // grouped conv: this group's first input / output channel
 };
 
 static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t stream, alt_kernel_cfg *used,
@@ -1508,6 +1514,7 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
     k[i++] = (int64_t)(uintptr_t)P.epi.residual;
     k[i++] = P.epi.residual_l ? (int64_t)P.epi.residual_l->serial : 0;
     k[i++] = P.epi.act;
+    k[i++] = (P.coff << 32) | P.koff;
     if (cfg) {
       k[i++] = cfg->block_n; k[i++] = cfg->tile_n; k[i++] = cfg->tile_h; k[i++] = cfg->tile_w;
       k[i++] = cfg->stages;
@@ -1606,7 +1613,7 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
         // default TMA stores (measured faster than direct 16-byte stores)
         return e && e[0] == 'd' ? 2 : (e && e[0] == 'g' ? 0 : 1);
       }();
-      if (store_mode == 2 && !(P.yl->flags & (ALT_HAS_PAD | ALT_HAS_UNFOLD)) && P.K % 8 == 0 &&
+      if (store_mode == 2 && !(P.yl->flags & (ALT_HAS_PAD | ALT_HAS_UNFOLD)) && P.K % 8 == 0 && P.koff % 8 == 0 &&
           (reinterpret_cast<uintptr_t>(P.y) & 15) == 0 && direct_store_ok(P.vy)) {
         alt_status st2 = make_reader(P.yl, &a.yr);
         if (st2 != ALT_OK) return st2;
@@ -1615,6 +1622,7 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       if (a.out_mode == 0 && store_mode != 0 && !(P.yl->flags & (ALT_HAS_PAD | ALT_HAS_UNFOLD))) {
         char why2[160];
         for (int so = 32; so >= 8 && !a.out_mode; so /= 2) {
+          if (P.koff % so) continue;  // a group's first channel must start a store slab
           View vy;
           if (!build_view(P.vy, ry, so, &vy, why2)) continue;
           int64_t rowsY = 1;
@@ -1636,6 +1644,10 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       a.num_tiles = (int32_t)(((mtiles + cg - 1) / cg) * ntiles);  // work units
       a.S = (int32_t)P.S;
       a.Gc = (int32_t)((P.C + sw - 1) / sw);
+      if (P.coff % sw) { snprintf(why, 160, "group channel offset %% slab"); continue; }
+      a.a_goff = (int32_t)(P.coff / sw);
+      a.b_koff = (int32_t)P.koff;
+      a.y_koff = (int32_t)P.koff;
       a.total_slabs = (int32_t)(P.R * P.S * a.Gc);
       a.spi = 64 / sw;
       a.num_iters = (a.total_slabs + a.spi - 1) / a.spi;
@@ -1763,7 +1775,12 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
 
 alt_status tc_conv(const ConvProblem &P, const alt_kernel_cfg *cfg, cudaStream_t stream, alt_kernel_cfg *used) {
   if (P.dtype != ALT_BF16) { set_error("tc path: bf16 only"); return ALT_E_UNSUPPORTED; }
-  if (P.groups != 1) { set_error("tc path: groups == 1 only"); return ALT_E_UNSUPPORTED; }
+  const int64_t G = P.groups < 1 ? 1 : P.groups;
+  const int64_t Cg = P.C / G, Kg = P.K / G;
+  if (G > 1 && (Cg % 8 || Kg % 8 || G == P.C)) {
+    set_error("tc path: grouped conv needs C/groups and K/groups multiples of 8 (depthwise: the dw kernel)");
+    return ALT_E_UNSUPPORTED;
+  }
   TcProblem T{};
   T.is_conv = true;
   T.al = P.xl; T.bl = P.wl; T.yl = P.yl;
@@ -1783,21 +1800,34 @@ alt_status tc_conv(const ConvProblem &P, const alt_kernel_cfg *cfg, cudaStream_t
   T.ry[1].role = R_C;
   T.ry[2] = RoleInfo{R_H, 1, 1, 0, 1, 0};
   T.ry[3] = RoleInfo{R_W, 1, 1, 0, 1, 0};
-  T.N = P.N; T.K = P.K; T.Ho = P.Ho; T.Wo = P.Wo;
-  T.R = P.R; T.S = P.S; T.C = P.C;
+  T.N = P.N; T.K = Kg; T.Ho = P.Ho; T.Wo = P.Wo;
+  T.R = P.R; T.S = P.S; T.C = Cg;
   T.epi = P.epi;
   T.va = lview(*P.xl); T.vb = lview(*P.wl); T.vy = lview(*P.yl);
   {
     LView xf, wf;
     int64_t Cf = 0;
-    if (P.dw == 1 && fold_window(T.va, T.vb, P.S, P.Vw, P.pw, P.Wo, &xf, &wf, &Cf)) {
+    if (G == 1 && P.dw == 1 && fold_window(T.va, T.vb, P.S, P.Vw, P.pw, P.Wo, &xf, &wf, &Cf)) {
       T.va = xf; T.vb = wf;
       T.ra[3] = RoleInfo{R_W, 1, 1, 0, 1, 0};
       T.S = 1; T.C = Cf;
     }
   }
   if (P.N * P.Ho * P.Wo >= (1ll << 31)) { set_error("tc: too many output pixels"); return ALT_E_UNSUPPORTED; }
-  return tc_run(T, cfg, stream, used, 0, 0);
+  if (G == 1) return tc_run(T, cfg, stream, used, 0, 0);
+  // grouped conv: one launch per group (the paper's GRP operator), each a
+  // Cg -> Kg implicit GEMM reading its channel slabs of x, its weight rows
+  // and writing its output channels through the same layouts
+  for (int64_t g = 0; g < G; g++) {
+    TcProblem Tg = T;
+    Tg.coff = g * Cg;
+    Tg.koff = g * Kg;
+    if (T.epi.scale) Tg.epi.scale = T.epi.scale + g * Kg;
+    if (T.epi.bias) Tg.epi.bias = T.epi.bias + g * Kg;
+    const alt_status st = tc_run(Tg, cfg, stream, used, 0, 0);
+    if (st != ALT_OK) return st;
+  }
+  return ALT_OK;
 }
 
 alt_status tc_gemm(const GemmProblem &P, const alt_kernel_cfg *cfg, cudaStream_t stream, alt_kernel_cfg *used) {

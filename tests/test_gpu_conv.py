@@ -406,3 +406,24 @@ def test_dilated_conv(case, dtype):
     with pytest.raises(alt.AltError) as e:   # forced depthwise path: no dilated kernel
         alt.conv2d(p, Lx, xd, Lw, wd, Ly, y, cfg={"path": alt.PATH_DW})
     assert e.value.code == alt._alt.ALT_E_UNSUPPORTED
+
+
+# --------------------------------------------------- grouped conv (GRP) --
+GRP = [  # name, N, C, H, W, K, R, V, pad, groups, x, w, y, residual
+    ("g2_c64", 2, 64, 14, 14, 64, 3, 1, 1, 2, LY.nchwxc(64, 32), LY.kcrs_yk_xc(64, 32, 32, 32), LY.nchwxc(64, 32),
+     None),
+    ("g4_s2_res", 2, 128, 15, 13, 256, 3, 2, 1, 4, LY.nchwxc(128, 32), LY.kcrs_yk_xc(256, 32, 64, 32),
+     LY.nchwxc(256, 64), LY.nchwxc(256, 64)),
+    ("g8_1x1_ragged", 3, 64, 9, 7, 192, 1, 1, 0, 8, LY.nchwxc(64, 8), LY.kcrs_yk_xc(192, 8, 8, 8), LY.nchwxc(192, 8),
+     LY.nchwxc(192, 8)),
+]
+
+
+@pytest.mark.parametrize("case", GRP, ids=[c[0] for c in GRP])
+def test_grouped_conv_tensor_core(case):
+    """grouped conv (the paper's GRP operator) on the tensor-core path: one
+    launch per group reading its channel slabs, weight rows and writing its
+    output channels through the declared layouts"""
+    name, N, C, H, W, K, R, V, pad, g, xp, wp, yp, rp = case
+    _, plan = run_conv(name, N, C, H, W, K, R, R, V, pad, xp, wp, yp, torch.bfloat16, groups=g, epi=True,
+                       res_p=rp, act=1, cfg={"path": alt.PATH_AUTO}, expect_path=alt.PATH_TC)
