@@ -1,6 +1,6 @@
 #!/bin/bash
 # Round-1 evidence run: GPU tests, smoke, bench (default + other workloads), ncu launch list + one --set full capture.
-cd $GRAFT_REPO_ROOT; O=gpurun_out/r01f; mkdir -p $O
+cd $GRAFT_REPO_ROOT; O=gpurun_out/r01g; mkdir -p $O
 make -C paper_conf_eurosys_xuxpwwwdxcwc23_b200 -j8 >/dev/null 2>&1
 timeout 900 python -m pytest tests -m gpu -x -q > $O/pytest_gpu.log 2>&1; echo "pytest rc=$?"; tail -3 $O/pytest_gpu.log
 timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.log 2>&1; echo "smoke rc=$?"; tail -2 $O/smoke.log
