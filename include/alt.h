@@ -141,6 +141,28 @@ alt_status alt_layout_logical_to_phys(alt_layout l, const int64_t *logical_coord
 alt_status alt_relayout(alt_layout src_l, const void *src, alt_layout dst_l,
                         void *dst, alt_dtype dtype, alt_stream_t stream);
 
+/* ------------------------------------------------ store_at / decouple_at -- */
+/* The store_at primitive and its inverse ("fusing two tensors
+ * together by attaching one to another ... attach each element of the bias
+ * vector to each column of the weight matrix"; reading A26 in DESIGN.md):
+ *   Z = store_at(A, b, dim):  Z has A's logical shape with extent E_dim + 1
+ *   along dim; Z[i] = A[i] for i_dim < E_dim, Z[i] = b[i without dim] for
+ *   i_dim == E_dim.
+ * a is read through a_l (logical shape = A's), z written through z_l (logical
+ * shape = A's with dim extended by one; every physical position, pad / unfold
+ * overhang zeros included).  b is DENSE row-major over A's dims without dim
+ * (prod of those extents elements).  All pointers device, caller-owned; a bit
+ * copy of dtype-width elements (NaN payloads, -0 preserved).  Errors:
+ * ALT_E_INVALID (NULL / host pointer, dim out of range, bad dtype),
+ * ALT_E_SHAPE (z_l / a_l logical shapes inconsistent), ALT_E_LOSSY (a_l has
+ * no copy of an element), ALT_E_CUDA (launch failure). */
+alt_status alt_store_at(alt_layout a_l, const void *a, const void *b, int32_t dim,
+                        alt_layout z_l, void *z, alt_dtype dtype, alt_stream_t stream);
+/* (A, b) = decouple_at(Z, dim): the inverse; a written through a_l (all
+ * physical positions), b dense row-major.  Same errors as alt_store_at. */
+alt_status alt_decouple_at(alt_layout z_l, const void *z, int32_t dim, alt_layout a_l,
+                           void *a, void *b, alt_dtype dtype, alt_stream_t stream);
+
 /* ---------------------------------------------- operators on layouts -- */
 /* conv2d, P:498-514 (Fig. 3): logical x [N,C,H,W],
  * w [K, C/groups, R, S], y [N, K, Ho, Wo], Ho = (H + 2 pad_h - R)/stride_h + 1
@@ -227,6 +249,20 @@ alt_status alt_matmul(int64_t M, int64_t N, int64_t K, alt_layout a_l,
                       alt_layout c_l, void *c, alt_dtype dtype,
                       const alt_epilogue *epi, const alt_kernel_cfg *cfg,
                       alt_stream_t stream);
+
+/* GEMM consuming a store_at weight: z_l has logical shape
+ * [K + 1, N] = store_at(B, bias, 0), i.e. column n is (B[:, n], bias[n]):
+ *   C[m,n] = act(scale[n] * sum_{k<K} A[m,k] Z[k,n] + Z[K,n] + residual).
+ * The contraction reads rows k < K of Z through z_l (the same kernels as
+ * alt_matmul); the attached row Z[K, :] is the bias, widened to fp32 by one
+ * N-element gather launch on `stream` into stream-ordered scratch.  epi may
+ * carry scale / residual / act; epi->bias must be NULL (ALT_E_INVALID).
+ * Other errors as alt_matmul. */
+alt_status alt_matmul_store_at(int64_t M, int64_t N, int64_t K, alt_layout a_l,
+                               const void *a, alt_layout z_l, const void *z,
+                               alt_layout c_l, void *c, alt_dtype dtype,
+                               const alt_epilogue *epi, const alt_kernel_cfg *cfg,
+                               alt_stream_t stream);
 
 /* 2-D pooling on declared layouts (support op of the ResNet chains; not one
  * of the paper's operators).  Uses p's N, C, H, W, R, S (window),

@@ -8,8 +8,8 @@ network layer tables, the batch-sharded chain runner).
 """
 from ._alt import (ACT, ALT_BF16, ALT_F32, AltError, ConvParams, KernelCfg, Layout, PATH_AUTO,
                    PATH_DW, PATH_SIMT, PATH_TC, conv2d, conv_params, last_plan, launch_count,
-                   lib_path, matmul, plan_chain, pool2d, relayout, tune)
+                   decouple_at, lib_path, matmul, matmul_store_at, plan_chain, store_at, pool2d, relayout, tune)
 
 __all__ = ["ACT", "ALT_BF16", "ALT_F32", "AltError", "ConvParams", "KernelCfg", "Layout",
            "PATH_AUTO", "PATH_DW", "PATH_SIMT", "PATH_TC", "conv2d", "conv_params", "last_plan",
-           "launch_count", "lib_path", "matmul", "plan_chain", "pool2d", "relayout", "tune"]
+           "launch_count", "lib_path", "matmul", "matmul_store_at", "store_at", "decouple_at", "plan_chain", "pool2d", "relayout", "tune"]

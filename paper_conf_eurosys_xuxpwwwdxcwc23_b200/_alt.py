@@ -104,6 +104,9 @@ _lib.alt_launch_count.restype = ctypes.c_uint64
 _lib.alt_tune.argtypes = [ctypes.c_int, _p, ctypes.c_int, _p, _p, _p, _p]
 _lib.alt_plan_chain.argtypes = [_i32, _p, _i32, _p, _p, _p, _p, _p, _p, _p]
 _lib.alt_pool2d.argtypes = [_p, _p, _p, _p, _p, ctypes.c_int, ctypes.c_int32, _p]
+_lib.alt_store_at.argtypes = [_p, _p, _p, ctypes.c_int32, _p, _p, ctypes.c_int, _p]
+_lib.alt_decouple_at.argtypes = [_p, _p, ctypes.c_int32, _p, _p, _p, ctypes.c_int, _p]
+_lib.alt_matmul_store_at.argtypes = [_i64, _i64, _i64, _p, _p, _p, _p, _p, _p, ctypes.c_int, _p, _p, _p]
 for _f in ("alt_layout_create", "alt_layout_destroy", "alt_layout_query", "alt_layout_logical",
            "alt_layout_phys_to_logical", "alt_layout_logical_to_phys", "alt_relayout",
            "alt_conv2d", "alt_matmul", "alt_last_plan", "alt_tune", "alt_plan_chain", "alt_pool2d"):
@@ -305,6 +308,32 @@ def matmul(M, N, K, a_l: Layout, a, b_l: Layout, b, c_l: Layout, c, scale=None, 
     return c
 
 
+def store_at(a_l: Layout, a, b, dim: int, z_l: Layout, z, stream=None):
+    """alt_store_at: z (in z_l) = a with b attached as the last slice of dim."""
+    _check(_lib.alt_store_at(a_l.handle, _ptr(a), _ptr(b), int(dim), z_l.handle, _ptr(z), _dtype_code(z),
+                             _stream_ptr(stream)), "alt_store_at")
+    return z
+
+
+def decouple_at(z_l: Layout, z, dim: int, a_l: Layout, a, b, stream=None):
+    """alt_decouple_at: the inverse of store_at; a through a_l, b dense."""
+    _check(_lib.alt_decouple_at(z_l.handle, _ptr(z), int(dim), a_l.handle, _ptr(a), _ptr(b), _dtype_code(z),
+                                _stream_ptr(stream)), "alt_decouple_at")
+    return a, b
+
+
+def matmul_store_at(M, N, K, a_l: Layout, a, z_l: Layout, z, c_l: Layout, c, scale=None, residual=None,
+                    residual_l=None, act=0, cfg=None, stream=None):
+    """alt_matmul_store_at: C = act(scale * A Z[:K] + Z[K] + residual), Z = store_at(B, bias, 0)."""
+    e = _epi(scale, None, residual, residual_l, act)
+    k = _cfg(cfg)
+    _check(_lib.alt_matmul_store_at(int(M), int(N), int(K), a_l.handle, _ptr(a), z_l.handle, _ptr(z),
+                                    c_l.handle, _ptr(c), _dtype_code(a), ctypes.byref(e) if e else None,
+                                    ctypes.byref(k) if k else None, _stream_ptr(stream)),
+           "alt_matmul_store_at")
+    return c
+
+
 def pool2d(p: ConvParams, x_l: Layout, x, y_l: Layout, y, kind: str = "max", stream=None):
     """alt_pool2d: max / average pooling through declared layouts."""
     _check(_lib.alt_pool2d(ctypes.byref(p), x_l.handle, _ptr(x), y_l.handle, _ptr(y), _dtype_code(x),
@@ -364,4 +393,5 @@ def plan_chain(op_kind: Sequence[int], edges: Sequence[tuple], edge_layouts: Seq
 EXPORTED = ["alt_status_str", "alt_last_error", "alt_layout_create", "alt_layout_destroy",
             "alt_layout_query", "alt_layout_logical", "alt_layout_phys_to_logical",
             "alt_layout_logical_to_phys", "alt_relayout", "alt_conv2d", "alt_matmul",
-            "alt_last_plan", "alt_launch_count", "alt_tune", "alt_plan_chain", "alt_pool2d"]
+            "alt_last_plan", "alt_launch_count", "alt_tune", "alt_plan_chain", "alt_pool2d",
+            "alt_store_at", "alt_decouple_at", "alt_matmul_store_at"]

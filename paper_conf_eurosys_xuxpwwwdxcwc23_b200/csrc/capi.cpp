@@ -220,6 +220,8 @@ alt_status alt_conv2d(const alt_conv2d_params *p, alt_layout x_l, const void *x,
   return st;
 }
 
+static alt_status gemm_dispatch(GemmProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s);
+
 alt_status alt_matmul(int64_t M, int64_t N, int64_t K, alt_layout a_l, const void *a,
                       alt_layout b_l, const void *b, alt_layout c_l, void *c, alt_dtype dtype,
                       const alt_epilogue *epi, const alt_kernel_cfg *cfg, alt_stream_t stream) {
@@ -239,7 +241,11 @@ alt_status alt_matmul(int64_t M, int64_t N, int64_t K, alt_layout a_l, const voi
   P.a = a; P.b = b; P.c = c; P.dtype = dtype;
   alt_status st = fill_epi(epi, P.cl, &P.epi);
   if (st != ALT_OK) return st;
-  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  return gemm_dispatch(P, cfg, reinterpret_cast<cudaStream_t>(stream));
+}
+
+static alt_status gemm_dispatch(GemmProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s) {
+  alt_status st = ALT_OK;
   const int32_t path = cfg ? cfg->path : ALT_PATH_AUTO;
   alt_kernel_cfg used{};
   if (path == ALT_PATH_TC || path == ALT_PATH_AUTO) {
@@ -290,6 +296,90 @@ alt_status alt_last_plan(alt_kernel_cfg *cfg) {
   if (!cfg) return ALT_E_INVALID;
   *cfg = g_last_plan;
   return ALT_OK;
+}
+
+static int dtype_wb(alt_dtype d) { return d == ALT_BF16 ? 2 : d == ALT_F32 ? 4 : 0; }
+
+// Z's logical shape must be A's with dim extended by one
+static alt_status check_attach(const char *what, const Layout *A, const Layout *Z, int32_t dim) {
+  if (dim < 0 || dim >= A->lrank) { set_error("%s: dim %d out of range", what, dim); return ALT_E_INVALID; }
+  if (Z->lrank != A->lrank) { set_error("%s: logical ranks differ", what); return ALT_E_SHAPE; }
+  for (int d = 0; d < A->lrank; d++)
+    if (Z->lshape[d] != A->lshape[d] + (d == dim ? 1 : 0)) {
+      set_error("%s: z logical shape must be a's with dim %d extended by one (dim %d)", what, dim, d);
+      return ALT_E_SHAPE;
+    }
+  return ALT_OK;
+}
+
+alt_status alt_store_at(alt_layout a_l, const void *a, const void *b, int32_t dim, alt_layout z_l, void *z,
+                        alt_dtype dtype, alt_stream_t stream) {
+  if (!a_l || !z_l) { set_error("alt_store_at: NULL layout"); return ALT_E_INVALID; }
+  const int wb = dtype_wb(dtype);
+  if (!wb) { set_error("alt_store_at: bad dtype"); return ALT_E_INVALID; }
+  alt_status st = check_attach("alt_store_at", &a_l->impl, &z_l->impl, dim);
+  if (st != ALT_OK) return st;
+  if (!(a_l->impl.flags & ALT_LOSSLESS)) { set_error("alt_store_at: a's layout is lossy"); return ALT_E_LOSSY; }
+  if (z_l->impl.pnumel == 0) return ALT_OK;
+  if (!is_device_ptr(z) || (a_l->impl.lnumel && !is_device_ptr(a)) ||
+      (z_l->impl.lnumel / z_l->impl.lshape[dim] && !is_device_ptr(b))) {
+    set_error("alt_store_at: a / b / z must be device pointers");
+    return ALT_E_INVALID;
+  }
+  return store_at_launch(&a_l->impl, a, b, dim, &z_l->impl, z, wb, reinterpret_cast<cudaStream_t>(stream));
+}
+
+alt_status alt_decouple_at(alt_layout z_l, const void *z, int32_t dim, alt_layout a_l, void *a, void *b,
+                           alt_dtype dtype, alt_stream_t stream) {
+  if (!a_l || !z_l) { set_error("alt_decouple_at: NULL layout"); return ALT_E_INVALID; }
+  const int wb = dtype_wb(dtype);
+  if (!wb) { set_error("alt_decouple_at: bad dtype"); return ALT_E_INVALID; }
+  alt_status st = check_attach("alt_decouple_at", &a_l->impl, &z_l->impl, dim);
+  if (st != ALT_OK) return st;
+  if (!(z_l->impl.flags & ALT_LOSSLESS)) { set_error("alt_decouple_at: z's layout is lossy"); return ALT_E_LOSSY; }
+  if (z_l->impl.lnumel == 0) return ALT_OK;
+  if (!is_device_ptr(z) || !is_device_ptr(a) || !is_device_ptr(b)) {
+    set_error("alt_decouple_at: z / a / b must be device pointers");
+    return ALT_E_INVALID;
+  }
+  return decouple_at_launch(&z_l->impl, z, dim, &a_l->impl, a, b, wb, reinterpret_cast<cudaStream_t>(stream));
+}
+
+alt_status alt_matmul_store_at(int64_t M, int64_t N, int64_t K, alt_layout a_l, const void *a, alt_layout z_l,
+                               const void *z, alt_layout c_l, void *c, alt_dtype dtype, const alt_epilogue *epi,
+                               const alt_kernel_cfg *cfg, alt_stream_t stream) {
+  if (!a_l || !z_l || !c_l) { set_error("alt_matmul_store_at: NULL layout"); return ALT_E_INVALID; }
+  const int wb = dtype_wb(dtype);
+  if (!wb) { set_error("alt_matmul_store_at: bad dtype"); return ALT_E_INVALID; }
+  if (M < 0 || N < 1 || K < 1) { set_error("alt_matmul_store_at: bad sizes"); return ALT_E_INVALID; }
+  if (epi && epi->bias) { set_error("alt_matmul_store_at: the bias is the attached row of z; epi->bias must be NULL"); return ALT_E_INVALID; }
+  const int64_t as[2] = {M, K}, zs[2] = {K + 1, N}, cs[2] = {M, N};
+  if (M > 0 && (!shape_is(&a_l->impl, 2, as) || !shape_is(&z_l->impl, 2, zs) || !shape_is(&c_l->impl, 2, cs))) {
+    set_error("alt_matmul_store_at: layout logical shapes do not match A[M,K] / Z[K+1,N] / C[M,N]");
+    return ALT_E_SHAPE;
+  }
+  if (M == 0) return ALT_OK;
+  if (!is_device_ptr(a) || !is_device_ptr(z) || !is_device_ptr(c)) { set_error("alt_matmul_store_at: A/Z/C must be device pointers"); return ALT_E_INVALID; }
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  GemmProblem P{};
+  P.M = M; P.N = N; P.K = K;
+  P.al = &a_l->impl; P.bl = &z_l->impl; P.cl = &c_l->impl;  // rows k < K of Z are B
+  P.a = a; P.b = z; P.c = c; P.dtype = dtype;
+  alt_status st = fill_epi(epi, P.cl, &P.epi);
+  if (st != ALT_OK) return st;
+  float *bias = nullptr;
+  if (cudaMallocAsync(reinterpret_cast<void **>(&bias), (size_t)N * sizeof(float), s) != cudaSuccess) {
+    cudaGetLastError();
+    set_error("alt_matmul_store_at: scratch allocation failed");
+    return ALT_E_NOMEM;
+  }
+  st = attached_row_f32(&z_l->impl, z, 0, wb, bias, s);
+  if (st == ALT_OK) {
+    P.epi.bias = bias;
+    st = gemm_dispatch(P, cfg, s);
+  }
+  cudaFreeAsync(bias, s);
+  return st;
 }
 
 uint64_t alt_launch_count(void) { return g_launches.load(); }

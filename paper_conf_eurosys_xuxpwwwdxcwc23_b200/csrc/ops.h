@@ -47,6 +47,12 @@ alt_status tc_gemm(const GemmProblem &P, const alt_kernel_cfg *cfg, cudaStream_t
                    alt_kernel_cfg *used);
 alt_status dw_conv(const ConvProblem &P, cudaStream_t stream, alt_kernel_cfg *used);
 alt_status pool2d(const ConvProblem &P, int kind, cudaStream_t stream);
+// store_at.cu (reading A26)
+alt_status store_at_launch(Layout *A, const void *a, const void *b, int32_t dim, Layout *Z, void *z, int wb,
+                           cudaStream_t stream);
+alt_status decouple_at_launch(Layout *Z, const void *z, int32_t dim, Layout *A, void *a, void *b, int wb,
+                              cudaStream_t stream);
+alt_status attached_row_f32(Layout *Z, const void *z, int32_t dim, int wb, float *out, cudaStream_t stream);
 // separable layout whose channel dim (logical 1) runs in 16-byte-aligned
 // groups of 8 contiguous elements (pads allowed when allow_pad: owner offsets)
 bool chan_vec8(const Layout &L, bool allow_pad);

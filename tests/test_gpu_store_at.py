@@ -1,0 +1,136 @@
+"""GPU parity: store_at / decouple_at (reading A26) and the GEMM
+that reads its bias from the attached row (alt_matmul_store_at), through the
+C-ABI, against oracle O8 (oracle/store_at.py) + O2 (layout materialisation).
+
+store_at / decouple_at are bit copies: compared word for word.  The GEMM is
+compared with the fp64 oracle under the tolerances of tests/helpers.py (the
+attached bias is the dtype-rounded value, as the oracle is fed)."""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import paper_conf_eurosys_xuxpwwwdxcwc23_b200 as alt
+from oracle.store_at import decouple_at as o_decouple_at
+from oracle.store_at import gemm_store_at_f64, store_at as o_store_at
+from paper_conf_eurosys_xuxpwwwdxcwc23_b200 import synth
+
+from .helpers import assert_parity, from_words, make_operand, read_output, words
+
+pytestmark = pytest.mark.gpu
+
+# Z = store_at(B [K, N], bias [N], 0) stored [N, K + 1 (+ pad)]: each weight
+# column followed by its bias element (the paper's FC example)
+def z_col(K, pad):
+    return [("reorder", [1, 0])] + ([("pad", 1, 0, pad)] if pad else [])
+
+
+STORE_CASES = [
+    # name, A logical shape, dim, A prims, Z prims
+    ("fc col-attached", (136, 96), 0, [], z_col(136, 7)),
+    ("fc col-attached unpadded", (64, 40), 0, [("reorder", [1, 0])], z_col(64, 0)),
+    ("3d tiled dim1", (4, 30, 24), 1, [("split", 2, [3, 8])], [("split", 2, [3, 8]), ("reorder", [0, 2, 1, 3])]),
+    ("row attach dim1", (50, 33), 1, [("pad", 1, 0, 7)], []),
+]
+
+
+@pytest.mark.parametrize("dtype", [torch.bfloat16, torch.float32], ids=["bf16", "f32"])
+@pytest.mark.parametrize("case", STORE_CASES, ids=[c[0] for c in STORE_CASES])
+def test_store_at_bit_exact(case, dtype):
+    name, ashape, dim, ap, zp = case
+    A = synth.activations("sa_A" + name, ashape)
+    bshape = ashape[:dim] + ashape[dim + 1:]
+    b = synth.activations("sa_b" + name, bshape)
+    OA, _, ad = make_operand("sa_A", ap, A, dtype)
+    bw = words(b.to(dtype))
+    bd = from_words(bw, dtype)
+    zshape = ashape[:dim] + (ashape[dim] + 1,) + ashape[dim + 1:]
+    OZ = oracle.Layout(zshape, zp)
+    want = OZ.materialize(o_store_at(words(A.to(dtype)), bw, dim))
+    La, Lz = alt.Layout(ashape, ap), alt.Layout(zshape, zp)
+    z = torch.full(Lz.phys_shape, 7, dtype=dtype, device="cuda")  # pads must be overwritten with 0
+    alt.store_at(La, ad, bd, dim, Lz, z)
+    torch.cuda.synchronize()
+    assert np.array_equal(words(z).reshape(OZ.phys_shape), want.reshape(OZ.phys_shape))
+
+    # decouple_at back into A's layout (all positions, pad zeros) and dense b
+    a2 = torch.full(La.phys_shape, 7, dtype=dtype, device="cuda")
+    b2 = torch.full(bshape, 7, dtype=dtype, device="cuda")
+    alt.decouple_at(Lz, z, dim, La, a2, b2)
+    torch.cuda.synchronize()
+    Aw, bw2 = o_decouple_at(o_store_at(words(A.to(dtype)), bw, dim), dim)
+    assert np.array_equal(words(a2).reshape(OA.phys_shape), OA.materialize(Aw).reshape(OA.phys_shape))
+    assert np.array_equal(words(b2).reshape(bshape), bw2.reshape(bshape))
+
+
+def test_store_at_rejects_bad_arguments():
+    La, Lz = alt.Layout((8, 4), []), alt.Layout((9, 4), [])
+    a = torch.zeros(8, 4, dtype=torch.bfloat16, device="cuda")
+    b = torch.zeros(4, dtype=torch.bfloat16, device="cuda")
+    z = torch.zeros(9, 4, dtype=torch.bfloat16, device="cuda")
+    with pytest.raises(alt.AltError):
+        alt.store_at(La, a, b, 1, Lz, z)          # z is not a with dim 1 extended
+    with pytest.raises(alt.AltError):
+        alt.store_at(La, a, b, 2, Lz, z)          # dim out of range
+    with pytest.raises(alt.AltError):
+        alt.store_at(La, a.cpu(), b, 0, Lz, z)    # host pointer
+
+
+GEMM_CASES = [
+    # M, N, K, Z pad, path
+    (384, 192, 256, 7, "tc"),
+    (200, 96, 136, 7, "auto"),
+    (130, 72, 64, 0, "simt"),
+    (256, 256, 512, 7, "auto"),
+]
+
+
+@pytest.mark.parametrize("dtype", [torch.bfloat16, torch.float32], ids=["bf16", "f32"])
+@pytest.mark.parametrize("case", GEMM_CASES, ids=[f"{c[0]}x{c[1]}x{c[2]}p{c[3]}{c[4]}" for c in GEMM_CASES])
+def test_matmul_store_at_parity(case, dtype):
+    M, N, K, pad, path = case
+    if dtype == torch.float32 and path == "tc":
+        pytest.skip("tensor-core path is bf16")
+    A = synth.activations("msa_A", (M, K))
+    B = synth.weights("msa_B", (K, N))
+    bias = synth.bn_bias("msa_b", N)
+    scale = synth.bn_scale("msa_s", N)
+    res = synth.activations("msa_r", (M, N))
+    _, _, ad = make_operand("msa_A", [], A, dtype)
+    _, _, rd = make_operand("msa_r", [], res, dtype)
+    Lb = alt.Layout((K, N), [])
+    bd = B.to(dtype).cuda()
+    bb = bias.to(dtype).cuda()
+    Lz = alt.Layout((K + 1, N), z_col(K, pad))
+    z = torch.empty(Lz.phys_shape, dtype=dtype, device="cuda")
+    alt.store_at(Lb, bd, bb, 0, Lz, z)
+    La, Lc = alt.Layout((M, K), []), alt.Layout((M, N), [])
+    c = torch.empty((M, N), dtype=dtype, device="cuda")
+    cfg = {"path": {"tc": alt.PATH_TC, "simt": alt.PATH_SIMT, "auto": alt.PATH_AUTO}[path]}
+    alt.matmul_store_at(M, N, K, La, ad, Lz, z, Lc, c, scale=scale.cuda(), residual=rd, residual_l=Lc,
+                        act="relu", cfg=cfg)
+    torch.cuda.synchronize()
+    if path != "auto":
+        assert alt.last_plan()["path"] == cfg["path"]
+    f64 = lambda t: t.to(dtype).double().numpy()  # noqa: E731  (operands as the kernel sees them)
+    Z = o_store_at(f64(B), f64(bias), 0)
+    want = gemm_store_at_f64(f64(A), Z, scale=scale.double().numpy(), residual=f64(res), act="relu")
+    got = read_output(oracle.Layout((M, N), []), c, dtype)
+    assert_parity(got, want, dtype)
+
+
+def test_matmul_store_at_rejects_separate_bias():
+    M, N, K = 128, 64, 64
+    La, Lz, Lc = alt.Layout((M, K), []), alt.Layout((K + 1, N), []), alt.Layout((M, N), [])
+    a = torch.zeros(M, K, dtype=torch.bfloat16, device="cuda")
+    z = torch.zeros(K + 1, N, dtype=torch.bfloat16, device="cuda")
+    c = torch.zeros(M, N, dtype=torch.bfloat16, device="cuda")
+    bias = torch.zeros(N, device="cuda")
+    e = alt._alt._epi(None, bias, None, None, 0)
+    import ctypes
+    rc = alt._alt._lib.alt_matmul_store_at(M, N, K, La.handle, a.data_ptr(), Lz.handle, z.data_ptr(),
+                                           Lc.handle, c.data_ptr(), alt.ALT_BF16, ctypes.byref(e), None,
+                                           torch.cuda.current_stream().cuda_stream)
+    assert rc != 0
+    with pytest.raises(alt.AltError):  # Z must be [K + 1, N]
+        alt.matmul_store_at(M, N, K + 1, La, a, Lz, z, Lc, c)
