@@ -367,6 +367,19 @@ alt_status alt_matmul_store_at(int64_t M, int64_t N, int64_t K, alt_layout a_l, 
   P.a = a; P.b = z; P.c = c; P.dtype = dtype;
   alt_status st = fill_epi(epi, P.cl, &P.epi);
   if (st != ALT_OK) return st;
+  Layout *Z = &z_l->impl;
+  if (Z->separable) {
+    // the epilogue reads bias[n] = Z[K, n] in place: offset rd0[K] + rd1[n]
+    SepDev sz{};
+    const LayoutDesc *dz = nullptr;
+    if ((st = device_tables(Z, &sz, &dz)) != ALT_OK) return st;
+    P.epi.bias_att = z;
+    P.epi.bias_att_rd = sz.rd[1];
+    P.epi.bias_att_base = Z->rd[0][K];
+    P.epi.bias_att_bf16 = dtype == ALT_BF16;
+    return gemm_dispatch(P, cfg, s);
+  }
+  // non-separable Z: gather the attached row into fp32 scratch first
   float *bias = nullptr;
   if (cudaMallocAsync(reinterpret_cast<void **>(&bias), (size_t)N * sizeof(float), s) != cudaSuccess) {
     cudaGetLastError();

@@ -50,7 +50,22 @@ struct EpiParams {
   const void *residual;
   Reader res;
   int32_t act;
+  // bias attached to the weight by store_at: the bias of output
+  // channel k is batt[batt_base + batt_rd[k]] (bf16 or fp32), read in place
+  const void *batt;
+  const int64_t *batt_rd;
+  int64_t batt_base;
+  int32_t batt_bf16;
 };
+
+__device__ __forceinline__ float epi_bias(const EpiParams &e, int64_t k) {
+  if (e.batt) {
+    const int64_t o = e.batt_base + __ldg(e.batt_rd + k);
+    return e.batt_bf16 ? bf16_to_f32(__ldg(static_cast<const uint16_t *>(e.batt) + o))
+                       : __ldg(static_cast<const float *>(e.batt) + o);
+  }
+  return __ldg(e.bias + k);
+}
 
 __device__ __forceinline__ float apply_act(float v, int act) {
   if (act == 1) v = fmaxf(v, 0.f);

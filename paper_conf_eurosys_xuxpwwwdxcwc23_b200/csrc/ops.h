@@ -13,6 +13,11 @@ struct OpEpilogue {
   const void *residual = nullptr;
   Layout *residual_l = nullptr;
   int32_t act = 0;
+  // store_at-attached bias (alt_matmul_store_at): see EpiParams::batt
+  const void *bias_att = nullptr;
+  const int64_t *bias_att_rd = nullptr;
+  int64_t bias_att_base = 0;
+  int32_t bias_att_bf16 = 0;
 };
 
 struct ConvProblem {

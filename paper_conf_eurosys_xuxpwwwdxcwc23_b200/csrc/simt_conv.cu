@@ -130,7 +130,7 @@ __global__ void __launch_bounds__(256) k_simt_igemm(SimtArgs a, const T *__restr
       if (n >= a.Ncol) continue;
       float v = acc[i][j];
       if (a.epi.scale) v *= __ldg(a.epi.scale + n);
-      if (a.epi.bias) v += __ldg(a.epi.bias + n);
+      if (a.epi.bias || a.epi.batt) v += epi_bias(a.epi, n);
       if (a.is_conv) {
         const int64_t q = m % a.Wo, p = (m / a.Wo) % a.Ho;
         if (a.epi.residual) {
@@ -225,6 +225,10 @@ alt_status make_epi(const OpEpilogue &e, EpiParams *p) {
   p->bias = e.bias;
   p->residual = e.residual;
   p->act = e.act;
+  p->batt = e.bias_att;
+  p->batt_rd = e.bias_att_rd;
+  p->batt_base = e.bias_att_base;
+  p->batt_bf16 = e.bias_att_bf16;
   p->res = Reader{};
   if (e.residual) return make_reader(e.residual_l, &p->res);
   return ALT_OK;

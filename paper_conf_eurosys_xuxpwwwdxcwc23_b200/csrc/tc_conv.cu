@@ -524,7 +524,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       if (tile < a.num_tiles && et < BN) {
         const int k = min(tile_coord(a, unit_info(a, tile).mn, BN, CG, rank).k0 + et, a.K - 1);
         fs = __ldg(a.epi.scale + k);
-        fb = __ldg(a.epi.bias + k);
+        fb = epi_bias(a.epi, k);
       }
     };
     float pf_s, pf_b;
@@ -1511,6 +1511,7 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
                P.ra[d].win;
     }
     k[i++] = (int64_t)(uintptr_t)P.epi.scale; k[i++] = (int64_t)(uintptr_t)P.epi.bias;
+    k[i++] = (int64_t)(uintptr_t)P.epi.bias_att;
     k[i++] = (int64_t)(uintptr_t)P.epi.residual;
     k[i++] = P.epi.residual_l ? (int64_t)P.epi.residual_l->serial : 0;
     k[i++] = P.epi.act;

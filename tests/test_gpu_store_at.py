@@ -21,7 +21,11 @@ pytestmark = pytest.mark.gpu
 
 # Z = store_at(B [K, N], bias [N], 0) stored [N, K + 1 (+ pad)]: each weight
 # column followed by its bias element (the paper's FC example)
+# (pad -1: the same placement written as one fused dim — a non-separable
+# layout, served by the gather-then-GEMM form)
 def z_col(K, pad):
+    if pad < 0:
+        return [("reorder", [1, 0]), ("fuse", 0, 2)]
     return [("reorder", [1, 0])] + ([("pad", 1, 0, pad)] if pad else [])
 
 
@@ -82,6 +86,7 @@ GEMM_CASES = [
     (200, 96, 136, 7, "auto"),
     (130, 72, 64, 0, "simt"),
     (256, 256, 512, 7, "auto"),
+    (96, 40, 72, -1, "auto"),
 ]
 
 
