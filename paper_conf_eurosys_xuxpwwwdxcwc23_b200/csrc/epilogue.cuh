@@ -59,11 +59,13 @@ struct EpiParams {
 };
 
 __device__ __forceinline__ float epi_bias(const EpiParams &e, int64_t k) {
+#ifndef ALT_NO_BATT  // developer A/B knob: build without the attached-bias read
   if (e.batt) {
     const int64_t o = e.batt_base + __ldg(e.batt_rd + k);
     return e.batt_bf16 ? bf16_to_f32(__ldg(static_cast<const uint16_t *>(e.batt) + o))
                        : __ldg(static_cast<const float *>(e.batt) + o);
   }
+#endif
   return __ldg(e.bias + k);
 }
 

@@ -87,6 +87,7 @@ GEMM_CASES = [
     (130, 72, 64, 0, "simt"),
     (256, 256, 512, 7, "auto"),
     (96, 40, 72, -1, "auto"),
+    (512, 320, 768, 63, "tc"),   # the measured layout: 128-byte row pitch
 ]
 
 
