@@ -153,3 +153,30 @@ def test_zero_extent_layouts_are_rejected():
         with pytest.raises(alt.AltError) as e:
             alt.Layout(shp, [])
         assert e.value.code == alt._alt.ALT_E_INVALID
+
+
+def test_store_at_argument_errors_without_gpu():
+    """alt_store_at / alt_decouple_at / alt_matmul_store_at validate shapes,
+    dims, dtypes and the epilogue before touching any pointer (no GPU)."""
+    La, Lz, Lbad = alt.Layout((8, 4), []), alt.Layout((9, 4), []), alt.Layout((8, 5), [])
+    L = _alt._lib
+    codes = {
+        "null layout": L.alt_store_at(None, None, None, 0, Lz.handle, None, alt.ALT_BF16, None),
+        "dim range": L.alt_store_at(La.handle, None, None, 2, Lz.handle, None, alt.ALT_BF16, None),
+        "bad dtype": L.alt_store_at(La.handle, None, None, 0, Lz.handle, None, 9, None),
+        "wrong dim": L.alt_store_at(La.handle, None, None, 1, Lz.handle, None, alt.ALT_BF16, None),
+        "decouple shape": L.alt_decouple_at(Lz.handle, None, 0, Lbad.handle, None, None, alt.ALT_F32, None),
+        "gemm z shape": L.alt_matmul_store_at(16, 4, 9, alt.Layout((16, 9), []).handle, None, Lz.handle,
+                                              None, alt.Layout((16, 4), []).handle, None, alt.ALT_BF16,
+                                              None, None, None),
+        "host pointers": L.alt_store_at(La.handle, np.zeros(32, np.uint16).ctypes.data, np.zeros(4, np.uint16).ctypes.data,
+                                        0, Lz.handle, np.zeros(36, np.uint16).ctypes.data, alt.ALT_BF16, None),
+    }
+    E_INVALID, E_SHAPE = 1, 2
+    assert codes["null layout"] == E_INVALID
+    assert codes["dim range"] == E_INVALID
+    assert codes["bad dtype"] == E_INVALID
+    assert codes["wrong dim"] == E_SHAPE
+    assert codes["decouple shape"] == E_SHAPE
+    assert codes["gemm z shape"] == E_SHAPE
+    assert codes["host pointers"] == E_INVALID
