@@ -1,0 +1,30 @@
+"""ncu target: one BERT FC GEMM (M 8192, K 768, N 3072) with a separate fp32
+bias (alt_matmul, B [N, K]) and the same GEMM reading the bias attached by
+store_at (alt_matmul_store_at, Z [N, K + 64]).  Two warm-up launches of each
+first, then one of each (profile with --launch-skip 4 --launch-count 2 -k regex:k_tc)."""
+import sys
+
+import torch
+
+sys.path.insert(0, __file__.rsplit("/", 2)[0])
+import paper_conf_eurosys_xuxpwwwdxcwc23_b200 as alt  # noqa: E402
+from paper_conf_eurosys_xuxpwwwdxcwc23_b200 import synth  # noqa: E402
+
+dt, M, K, N = torch.bfloat16, 8192, 768, 3072
+A = synth.activations("sab_A", (M, K)).to(dt).cuda()
+B = synth.weights("sab_B", (K, N)).to(dt)
+bias = synth.bn_bias("sab_b", N)
+La, Lc, Lb = alt.Layout((M, K), []), alt.Layout((M, N), []), alt.Layout((K, N), [])
+Lbt = alt.Layout((K, N), [("reorder", [1, 0])])
+bt = B.t().contiguous().cuda()
+Lz = alt.Layout((K + 1, N), [("reorder", [1, 0]), ("pad", 1, 0, 63)])
+z = torch.empty(Lz.phys_shape, dtype=dt, device="cuda")
+alt.store_at(Lb, B.cuda(), bias.to(dt).cuda(), 0, Lz, z)
+bf = bias.to(dt).float().cuda()
+c0, c1 = torch.empty((M, N), dtype=dt, device="cuda"), torch.empty((M, N), dtype=dt, device="cuda")
+for _ in range(3):
+    alt.matmul(M, N, K, La, A, Lbt, bt, Lc, c0, bias=bf)
+    alt.matmul_store_at(M, N, K, La, A, Lz, z, Lc, c1)
+torch.cuda.synchronize()
+assert torch.equal(c0, c1)
+print("ok")
