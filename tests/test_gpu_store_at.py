@@ -140,3 +140,56 @@ def test_matmul_store_at_rejects_separate_bias():
     assert rc != 0
     with pytest.raises(alt.AltError):  # Z must be [K + 1, N]
         alt.matmul_store_at(M, N, K + 1, La, a, Lz, z, Lc, c)
+
+
+def test_store_at_unfold_layout_writes_every_copy():
+    """Z stored with an overlapping unfold (several physical copies per element,
+    overhang zeros): every copy holds the value, bit-exact to the oracle."""
+    dtype = torch.bfloat16
+    ashape, dim = (6, 21), 0
+    zp = [("unfold", 1, 8, 5)]          # 22 -> tiles of 8 with step 5 (overlap 3)
+    A = synth.activations("sau_A", ashape)
+    b = synth.activations("sau_b", (21,))
+    _, _, ad = make_operand("sau_A", [], A, dtype)
+    bw = words(b.to(dtype))
+    zshape = (7, 21)
+    OZ = oracle.Layout(zshape, zp)
+    want = OZ.materialize(o_store_at(words(A.to(dtype)), bw, dim))
+    Lz = alt.Layout(zshape, zp)
+    z = torch.full(Lz.phys_shape, 7, dtype=dtype, device="cuda")
+    alt.store_at(alt.Layout(ashape, []), ad, from_words(bw, dtype), dim, Lz, z)
+    torch.cuda.synchronize()
+    assert np.array_equal(words(z).reshape(OZ.phys_shape), want.reshape(OZ.phys_shape))
+
+
+def test_store_at_is_a_bit_copy():
+    """NaN payloads, -0 and infinities survive store_at / decouple_at (fp32)."""
+    special = np.array([0x7FC00001, 0x80000000, 0x7F800000, 0xFF800000, 0x00000001, 0x3F800000],
+                       dtype=np.uint32)
+    aw = np.resize(special, (5, 6)).astype(np.uint32)
+    bw = special.copy()
+    ad, bd = from_words(aw, torch.float32), from_words(bw, torch.float32)
+    La, Lz = alt.Layout((5, 6), []), alt.Layout((6, 6), [("reorder", [1, 0])])
+    z = torch.empty(Lz.phys_shape, dtype=torch.float32, device="cuda")
+    alt.store_at(La, ad, bd, 0, Lz, z)
+    a2 = torch.empty_like(ad)
+    b2 = torch.empty_like(bd)
+    alt.decouple_at(Lz, z, 0, La, a2, b2)
+    torch.cuda.synchronize()
+    assert np.array_equal(words(a2).reshape(5, 6), aw)
+    assert np.array_equal(words(b2), bw)
+    OZ = oracle.Layout((6, 6), [("reorder", [1, 0])])
+    assert np.array_equal(words(z).reshape(OZ.phys_shape), OZ.materialize(o_store_at(aw, bw, 0)).reshape(6, 6))
+
+
+def test_matmul_store_at_empty_batch_is_noop():
+    """M = 0: nothing launched, nothing written (as alt_matmul)."""
+    N, K = 64, 64
+    La, Lz, Lc = alt.Layout((4, K), []), alt.Layout((K + 1, N), []), alt.Layout((4, N), [])
+    c = torch.full((4, N), 5.0, dtype=torch.bfloat16, device="cuda")
+    n0 = alt.launch_count()
+    alt.matmul_store_at(0, N, K, La, torch.zeros(4, K, dtype=torch.bfloat16, device="cuda"), Lz,
+                        torch.zeros(K + 1, N, dtype=torch.bfloat16, device="cuda"), Lc, c)
+    torch.cuda.synchronize()
+    assert alt.launch_count() == n0
+    assert bool((c == 5.0).all())
