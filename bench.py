@@ -281,6 +281,9 @@ def main():
     ap.add_argument("--batch", type=int, default=32, help="images per GPU")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--eager", action="store_true", help="time eager launches instead of a CUDA graph")
+    ap.add_argument("--bert-bias", default="none", choices=["none", "separate", "attached"],
+                    help="bert workload: no bias (default line), a separate fp32 bias, or the bias "
+                         "attached to the weight by store_at (P:786-792)")
     ap.add_argument("--workload", default="r50", choices=["r50", "r18", "mv2", "bert", "relayout", "fig12"],
                     help="r50 = BASELINE config 2 (the driver's default); r18 = config 5 "
                          "(batch-sharded chain, global batch 256); mv2 = config 4; bert = config 3; "

@@ -129,7 +129,13 @@ def run(args):
             Lc = alt.Layout((M, N), LY.gemm_c_tiled(M, N, 128, 64))
             a, b, c = La.empty(torch.bfloat16, dev).normal_(), Lb.empty(torch.bfloat16, dev).normal_(), \
                 Lc.empty(torch.bfloat16, dev)
-            items.append((name, M, N, K, La, a, Lb, b, Lc, c))
+            bias = torch.randn(N, device=dev).to(torch.bfloat16)
+            if args.bert_bias == "attached":   # store_at: the bias rides in the weight
+                Lz = alt.Layout((K + 1, N), LY.gemm_z_tiled_nk(K, N, tuned.get("b_nt", 256), 64))
+                z = Lz.empty(torch.bfloat16, dev)
+                alt.store_at(Lb, b, bias, 0, Lz, z)
+                Lb, b = Lz, z
+            items.append((name, M, N, K, La, a, Lb, b, Lc, c, bias.float()))
 
         cfgs = {}
         for it in items:
@@ -137,22 +143,31 @@ def run(args):
             c.pop("b_nt", None)  # a layout parameter, not a kernel one
             cfgs[(it[1], it[2], it[3])] = c
 
+        def gemm(it):
+            _, M_, N_, K_, La, a, Lb, b, Lc, c, bias = it
+            if args.bert_bias == "attached":
+                alt.matmul_store_at(M_, N_, K_, La, a, Lb, b, Lc, c, cfg=cfgs[(M_, N_, K_)])
+            else:
+                alt.matmul(M_, N_, K_, La, a, Lb, b, Lc, c, bias=bias if args.bert_bias == "separate" else None,
+                           cfg=cfgs[(M_, N_, K_)])
+
         def step():
-            for (_, M_, N_, K_, La, a, Lb, b, Lc, c) in items:
-                alt.matmul(M_, N_, K_, La, a, Lb, b, Lc, c, cfg=cfgs[(M_, N_, K_)])
+            for it in items:
+                gemm(it)
 
         ms = _time(step, args.steps, args.warmup, ws)
         flops = sum(2.0 * M_ * N_ * K_ for (_, M_, N_, K_, *_r) in items) * ws
         per = []
         for it in items:
-            t = _time(lambda it=it: alt.matmul(it[1], it[2], it[3], it[4], it[5], it[6], it[7], it[8],
-                                               it[9], cfg=cfgs[(it[1], it[2], it[3])]),
-                      max(3, args.steps), 2, ws)
+            t = _time(lambda it=it: gemm(it), max(3, args.steps), 2, ws)
             per.append({"gemm": it[0], "M": it[1], "us": round(t * 1e3, 2), "cfg": cfgs[(it[1], it[2], it[3])],
                         "tflops": round(2.0 * it[1] * it[2] * it[3] / (t * 1e-3) / 1e12, 1)})
         out = _line(args, ws, flops / (ms * 1e-3) / 1e12, "TFLOP/s", ms,
                     {"workload": "BERT-base GEMMs at seq 512 x 16 sequences (M=8192): 768x768, "
-                                 "768x3072, 3072x768, tiled A M/128 K/64, B N/nt K/64 (nt tuned), C M/128 N/64",
+                                 "768x3072, 3072x768, tiled A M/128 K/64, B N/nt K/64 (nt tuned), C M/128 N/64"
+                                 + {"none": "", "separate": ", fp32 bias vector in the epilogue",
+                                    "attached": ", bias attached to the weight columns by store_at "
+                                                "(Z N/nt (K+64)/64 nt 64), read in place"}[args.bert_bias],
                      "global_batch": 16 * ws, "seq_len": 512, "parallelism": f"dp{ws}"},
                     {"scaling": "weak", "per_gemm": per, "gpu_launches": 3 * args.steps})
     elif args.workload == "relayout":

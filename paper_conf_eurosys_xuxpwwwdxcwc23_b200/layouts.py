@@ -71,6 +71,14 @@ def gemm_b_tiled_nk(K: int, N: int, nt: int, kt: int):
     return [("split", 0, [K // kt, kt]), ("split", 2, [N // nt, nt]), ("reorder", [2, 0, 3, 1])]
 
 
+def gemm_z_tiled_nk(K: int, N: int, nt: int, kt: int):
+    """Z = store_at(B, bias, 0), logical [K + 1, N], stored like
+    gemm_b_tiled_nk with one more K tile: N/nt (K+kt)/kt nt kt, K a multiple
+    of kt; the bias row k = K opens the last K tile (pad zeros after it)."""
+    return [("pad", 0, 0, kt - 1), ("split", 0, [(K + kt) // kt, kt]), ("split", 2, [N // nt, nt]),
+            ("reorder", [2, 0, 3, 1])]
+
+
 def gemm_b_tiled_kn(K: int, N: int, kt: int, nt: int):
     """B: K/kt N/nt kt nt (the paper's template; N innermost)."""
     return [("split", 0, [K // kt, kt]), ("split", 2, [N // nt, nt]), ("reorder", [0, 2, 1, 3])]

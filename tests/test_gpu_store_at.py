@@ -193,3 +193,31 @@ def test_matmul_store_at_empty_batch_is_noop():
     torch.cuda.synchronize()
     assert alt.launch_count() == n0
     assert bool((c == 5.0).all())
+
+
+@pytest.mark.parametrize("nt", [128, 256])
+def test_matmul_store_at_tiled_z_bench_layout(nt):
+    """the bench's attached-bias layout (layouts.gemm_z_tiled_nk: N/nt (K+64)/64
+    nt 64, bias row opening the last K tile) on the tensor-core path, tiled A / C."""
+    from paper_conf_eurosys_xuxpwwwdxcwc23_b200 import layouts as LY
+    dtype = torch.bfloat16
+    M, N, K = 512, 512, 256
+    A = synth.activations("mzt_A", (M, K))
+    B = synth.weights("mzt_B", (K, N))
+    bias = synth.bn_bias("mzt_b", N)
+    ap, cp = LY.gemm_a_tiled(M, K, 128, 64), LY.gemm_c_tiled(M, N, 128, 64)
+    _, _, ad = make_operand("mzt_A", ap, A, dtype)
+    _, _, bd = make_operand("mzt_B", LY.gemm_b_tiled_nk(K, N, nt, 64), B, dtype)
+    Lb = alt.Layout((K, N), LY.gemm_b_tiled_nk(K, N, nt, 64))
+    Lz = alt.Layout((K + 1, N), LY.gemm_z_tiled_nk(K, N, nt, 64))
+    z = Lz.empty(dtype)
+    alt.store_at(Lb, bd, bias.to(dtype).cuda(), 0, Lz, z)
+    La, Lc = alt.Layout((M, K), ap), alt.Layout((M, N), cp)
+    c = Lc.empty(dtype)
+    alt.matmul_store_at(M, N, K, La, ad, Lz, z, Lc, c, act="relu", cfg={"path": alt.PATH_TC, "block_n": nt})
+    torch.cuda.synchronize()
+    assert alt.last_plan()["path"] == alt.PATH_TC
+    f64 = lambda t: t.to(dtype).double().numpy()  # noqa: E731
+    want = gemm_store_at_f64(f64(A), o_store_at(f64(B), f64(bias), 0), act="relu")
+    got = read_output(oracle.Layout((M, N), cp), c, dtype)
+    assert_parity(got, want, dtype)
