@@ -272,6 +272,48 @@ def oracle_sample(seconds_budget=15.0, image=0):
 
 
 # ------------------------------------------------------------------- main -
+def spawn(args) -> int:
+    """`--gpus N` (N > 1) outside torchrun: launch N ranks of this script
+    (one process per GPU over NCCL, rendezvous on 127.0.0.1)."""
+    import socket
+    import torch
+    have = torch.cuda.device_count()
+    if have < args.gpus:
+        print(f"bench.py: --gpus {args.gpus} but only {have} CUDA device(s) visible", file=sys.stderr)
+        return 2
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
+
+
+def roofline_by_class(S, times_ms, bf16_peak, hbm_peak):
+    """Per-class roofline over the layer set: layers whose FLOPs / tensor peak
+    exceed their algorithmic bytes / HBM peak are tensor-bound and judged in
+    TFLOP/s against the tensor peak; the others are HBM-bound and judged in
+    GB/s against HBM bandwidth."""
+    cls = {"tensor": [0.0, 0.0, 0], "hbm": [0.0, 0.0, 0]}
+    for l, t in zip(S.layers, times_ms):
+        f, b = l["L"].flops(S.N), l["L"].min_bytes(S.N)
+        k = "tensor" if f / (bf16_peak * 1e12) >= b / (hbm_peak * 1e9) else "hbm"
+        cls[k][0] += f if k == "tensor" else b
+        cls[k][1] += t * 1e-3
+        cls[k][2] += 1
+    out = {}
+    if cls["tensor"][2]:
+        a = cls["tensor"][0] / cls["tensor"][1] / 1e12
+        out["tensor"] = {"layers": cls["tensor"][2], "achieved": round(a, 2), "peak": bf16_peak,
+                         "unit": "TFLOP/s", "frac": round(a / bf16_peak, 4)}
+    if cls["hbm"][2]:
+        a = cls["hbm"][0] / cls["hbm"][1] / 1e9
+        out["hbm"] = {"layers": cls["hbm"][2], "achieved": round(a, 1), "peak": hbm_peak, "unit": "GB/s",
+                      "frac": round(a / hbm_peak, 4)}
+    return out
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -280,6 +322,8 @@ def main():
     ap.add_argument("--impl", default="alt", choices=["alt", "reference"])
     ap.add_argument("--batch", type=int, default=32, help="images per GPU")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-aux", action="store_true",
+                    help="skip the other BASELINE configs (chains, BERT, relayout, fixed layouts) in the line")
     ap.add_argument("--eager", action="store_true", help="time eager launches instead of a CUDA graph")
     ap.add_argument("--bert-bias", default="none", choices=["none", "separate", "attached"],
                     help="bert workload: no bias (default line), a separate fp32 bias, or the bias "
@@ -289,10 +333,13 @@ def main():
                          "(batch-sharded chain, global batch 256); mv2 = config 4; bert = config 3; "
                          "relayout = the D6 bandwidth set; fig12 = the paper's propagation study")
     args = ap.parse_args()
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ and args.impl != "reference":
+        sys.exit(spawn(args))
     if args.workload != "r50":
         import bench_workloads
         return bench_workloads.run(args)
-    ws, rank, local = dist_init()
+    ws, rank, local = (max(1, args.gpus), int(os.environ.get("RANK", "0")), 0) if args.impl == "reference" \
+        else dist_init()
     config = {"workload": "ResNet-50 conv2d layer set (23 unique torchvision-v1.5 convs), "
                           f"batch {args.batch} per GPU, bf16, tuned ALT layouts, fused BN+ReLU",
               "global_batch": args.batch * ws, "per_gpu_batch": args.batch,
@@ -390,8 +437,10 @@ def main():
     per_layer = []
     bf16_peak, hbm_peak, peak_src = peaks()
     t_roof_sum = t_meas_sum = 0.0
+    layer_ms = []
     for i, l in enumerate(S.layers):
         t = statistics.median(ev[k][i][0].elapsed_time(ev[k][i][1]) for k in range(args.steps))
+        layer_ms.append(t)
         # per-layer roofline time: max(FLOPs / tensor peak, algorithmic bytes / HBM peak)
         t_tc = l["L"].flops(S.N) / (bf16_peak * 1e12)
         t_hbm = l["L"].min_bytes(S.N) / (hbm_peak * 1e9)
@@ -401,46 +450,51 @@ def main():
                           "bound": "tensor" if t_tc >= t_hbm else "hbm",
                           "roofline_frac": round(max(t_tc, t_hbm) / (t * 1e-3), 3),
                           "tflops": round(l["L"].flops(S.N) / (t * 1e-3) / 1e12, 1),
+                          "gbs": round(l["L"].min_bytes(S.N) / (t * 1e-3) / 1e9, 1),
                           "path": plans[i]["path"], "tile": [plans[i]["tile_n"], plans[i]["tile_h"],
                                                              plans[i]["tile_w"]],
                           "block_n": plans[i]["block_n"]})
     value = S.flops * ws / (ms * 1e-3) / 1e12
+    by_class = roofline_by_class(S, layer_ms, bf16_peak, hbm_peak)
 
     # e2e through the public API with host buffers (copies overlapped with
-    # the conversions and convs on their own streams)
+    # the conversions and convs on their own streams), every timed step
     for _ in range(2):
         S.step_e2e_overlap()
     torch.cuda.synchronize()
     barrier(ws)
     e0 = torch.cuda.Event(enable_timing=True)
     e1 = torch.cuda.Event(enable_timing=True)
-    e_steps = max(1, min(args.steps, 5))
     e0.record(stream)
-    for k in range(e_steps):
+    for k in range(args.steps):
         S.step_e2e_overlap(start_ev=e0 if k == 0 else None)
     e1.record(stream)
     torch.cuda.synchronize()
-    e_ms = max_over_ranks(e0.elapsed_time(e1) / e_steps, ws)
+    e_ms = max_over_ranks(e0.elapsed_time(e1) / args.steps, ws)
     h2d, d2h = S.io_bytes()
 
-    achieved = S.flops / (conv_ms * 1e-3) / 1e12
+    tb = by_class.get("tensor", {})
     line = {"metric": METRIC, "value": round(value, 2), "unit": "TFLOP/s", "n_gpus": ws,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 4),
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "bf16",
             "data": "synthetic", "config": config,
-            "roofline": {"kernel": "k_tc_conv (tcgen05 implicit-GEMM conv, all 23 launches)",
-                         "bound": "tensor", "achieved": round(achieved, 2), "peak": bf16_peak,
+            "roofline": {"kernel": "k_tc_conv (tcgen05 implicit-GEMM conv) on the tensor-bound layers",
+                         "bound": "tensor", "achieved": tb.get("achieved"), "peak": bf16_peak,
                          "peak_source": f"{peak_src} bf16 dense (burst)", "unit": "TFLOP/s",
-                         "frac": round(achieved / bf16_peak, 4),
-                         "traffic": None, "algorithmic_bytes_per_step": S.alg_bytes,
+                         "frac": tb.get("frac"), "traffic": None,
+                         "by_class": by_class,
+                         "all_layers_tflops": round(S.flops / (conv_ms * 1e-3) / 1e12, 2),
+                         "graph_step_frac": round(value / ws / bf16_peak, 4),
+                         "algorithmic_bytes_per_step": S.alg_bytes,
                          "set_roofline_time_frac": round(t_roof_sum / t_meas_sum, 4),
-                         "note": "achieved = sum of layer FLOPs / sum of per-launch CUDA-event times; "
-                                 "13 of 23 layers are HBM-bound at batch 32 (SURVEY §8d); "
+                         "note": "achieved / frac = tensor-bound layers' FLOPs / their summed per-launch "
+                                 "CUDA-event times (event nodes in the graph); by_class.hbm = HBM-bound "
+                                 "layers' algorithmic bytes / their times vs measured HBM; "
                                  "set_roofline_time_frac = sum over layers of max(FLOPs/tensor peak, "
                                  "bytes/HBM peak) / sum of measured layer times"},
             "e2e": {"value": round(S.flops * ws / (e_ms * 1e-3) / 1e12, 3), "unit": "TFLOP/s",
                     "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
-                    "ms_per_step": round(e_ms, 3),
+                    "ms_per_step": round(e_ms, 3), "steps": args.steps,
                     "note": "per layer: pinned H2D of the NCHW input, conversion to the tuned layout, "
                             "conv, D2H of the output; copies on their own streams overlap compute"},
             "gpu_launches": launches, "clocks": getattr(clk, "summary", None),
@@ -449,9 +503,31 @@ def main():
     if os.path.exists(traffic_file):
         try:
             with open(traffic_file) as f:
-                line["roofline"]["traffic"] = json.load(f).get("dram_bytes_per_step")
+                tr = json.load(f)
+            line["roofline"]["traffic"] = tr.get("dram_bytes_per_step")
+            line["roofline"]["traffic_source"] = tr.get("source")
         except Exception:
             pass
+    del S
+    torch.cuda.empty_cache()
+    import bench_workloads as BW
+    # BASELINE config 5 at this N: the batch-sharded R18 chain (strong scaling,
+    # NCCL all-gather timed), every rank takes part
+    line["chain_scaling"] = BW.r18_strong(args.steps, args.warmup, ws, rank, dev)
+    torch.cuda.empty_cache()
+    if ws == 1 and not args.no_aux:
+        aux = {}
+        aux["mv2_b16"] = BW.mv2_chain(args.steps, args.warmup, ws, dev)
+        aux["bert_m8192"] = BW.bert_set(args.steps, args.warmup, ws, dev)
+        torch.cuda.empty_cache()
+        aux["relayout_d6"] = BW.relayout_run(args.steps, ws, dev)
+        torch.cuda.empty_cache()
+        try:
+            import bench_layouts as BL
+            aux["fixed_layouts"] = BL.run_all(dev, steps=max(5, min(args.steps, 10)))
+        except ImportError:
+            pass
+        line["aux"] = aux
     if rank == 0 and ws == 1 and not args.no_cpu_baseline:
         tf, threads, sample = oracle_sample(seconds_budget=15.0)
         line["cpu_baseline"] = {"value": tf, "unit": "TFLOP/s", "cores": threads, "kind": "oracle",

@@ -74,121 +74,160 @@ def _line(args, ws, metric_value, unit, ms, config, extra):
     return line
 
 
-def run(args):
-    ws, rank, local = bench.dist_init()
+def r18_strong(steps, warmup, ws, rank, dev, graph=True):
+    """BASELINE config 5: the ResNet-18 chain at GLOBAL batch 256, sharded by
+    batch over the ws ranks (strong scaling, row a10).  Each rank runs the
+    whole chain on its contiguous shard; the final 512x7x7 feature maps are
+    all-gathered over NCCL inside the timed region (the path's only
+    collective).  Returns a dict (time = max over ranks of chain + gather)."""
     import paper_conf_eurosys_xuxpwwwdxcwc23_b200 as alt
     from paper_conf_eurosys_xuxpwwwdxcwc23_b200 import chain as CH
+    global_batch = 256
+    lo, hi = D.shard_range(global_batch, rank, ws)
+    ch = CH.resnet18(hi - lo, dev)
+    gathered = {}
+
+    def step():
+        y = ch.run()
+        gathered["y"] = D.gather_outputs(y, ws)   # identity at ws = 1
+    n0 = alt.launch_count()
+    step()
+    torch.cuda.synchronize()
+    per_step = alt.launch_count() - n0
+    ms = _time(step, steps, warmup, ws, graph=graph)
+    flops = ch.flops * (global_batch / ch.N)
+    recorded, launched = ch.plan()
+    out_bytes = gathered["y"].numel() * gathered["y"].element_size()
+    return {"workload": "ResNet-18 conv chain (conv1 7x7 + 16 3x3 + 3 1x1 ds, maxpool, BN+ReLU, residual "
+                        "adds), global batch 256 sharded by batch, NCCL all-gather of the 512x7x7 output",
+            "global_batch": global_batch, "per_gpu_batch": ch.N, "n_gpus": ws, "ms_per_step": round(ms, 4),
+            "tflops": round(flops / (ms * 1e-3) / 1e12, 2), "scaling": "strong",
+            "gathered_bytes": out_bytes, "gpu_launches_per_step": per_step,
+            "cfgs": "chain_tune.json" if ch.cfgs_loaded else "heuristic",
+            "propagation": {"alg1_recorded_conversions": recorded, "standalone_conversion_kernels": launched}}
+
+
+def mv2_chain(steps, warmup, ws, dev, N=16):
+    """BASELINE config 4: MobileNet-V2 (52 convs, 17 depthwise) at batch N
+    per GPU with layout propagation (Alg. 1)."""
+    import paper_conf_eurosys_xuxpwwwdxcwc23_b200 as alt
+    from paper_conf_eurosys_xuxpwwwdxcwc23_b200 import chain as CH
+    ch = CH.mobilenet_v2(N, dev)
+    n0 = alt.launch_count()
+    ch.run()
+    torch.cuda.synchronize()
+    per_step = alt.launch_count() - n0
+    ms = _time(ch.run, steps, warmup, ws)
+    recorded, launched = ch.plan()
+    return {"workload": f"MobileNet-V2 chain (52 convs, 17 depthwise, BN+ReLU6, residual adds), batch {N}",
+            "per_gpu_batch": N, "ms_per_step": round(ms, 4), "tflops": round(ch.flops / (ms * 1e-3) / 1e12, 2),
+            "hbm_bytes_min": ch.min_bytes(), "hbm_gbs_min": round(ch.min_bytes() / (ms * 1e-3) / 1e9, 1),
+            "gpu_launches_per_step": per_step,
+            "propagation": {"alg1_recorded_conversions": recorded, "standalone_conversion_kernels": launched}}
+
+
+def bert_set(steps, warmup, ws, dev, bias="none"):
+    """BASELINE config 3: BERT-base GEMMs at M = 8192 on tiled layouts."""
+    import paper_conf_eurosys_xuxpwwwdxcwc23_b200 as alt
+    from paper_conf_eurosys_xuxpwwwdxcwc23_b200 import layouts as LY
+    from paper_conf_eurosys_xuxpwwwdxcwc23_b200 import nets
+    from paper_conf_eurosys_xuxpwwwdxcwc23_b200 import tunecache
+    M = 8192
+    items = []
+    for name, K, N in nets.BERT_GEMMS:
+        tuned = tunecache.lookup_gemm(M, N, K) or {}
+        La = alt.Layout((M, K), LY.gemm_a_tiled(M, K, 128, 64))
+        Lb = alt.Layout((K, N), LY.gemm_b_tiled_nk(K, N, tuned.get("b_nt", 256), 64))
+        Lc = alt.Layout((M, N), LY.gemm_c_tiled(M, N, 128, 64))
+        a, b, c = La.empty(torch.bfloat16, dev).normal_(), Lb.empty(torch.bfloat16, dev).normal_(), \
+            Lc.empty(torch.bfloat16, dev)
+        bvec = torch.randn(N, device=dev).to(torch.bfloat16)
+        if bias == "attached":   # store_at (P:786-792): the bias rides in the weight
+            Lz = alt.Layout((K + 1, N), LY.gemm_z_tiled_nk(K, N, tuned.get("b_nt", 256), 64))
+            z = Lz.empty(torch.bfloat16, dev)
+            alt.store_at(Lb, b, bvec, 0, Lz, z)
+            Lb, b = Lz, z
+        cfg = dict(tuned or {"path": 1, "block_n": 256})
+        cfg.pop("b_nt", None)  # a layout parameter, not a kernel one
+        items.append((name, M, N, K, La, a, Lb, b, Lc, c, bvec.float(), cfg))
+
+    def gemm(it):
+        _, M_, N_, K_, La, a, Lb, b, Lc, c, bv, cfg = it
+        if bias == "attached":
+            alt.matmul_store_at(M_, N_, K_, La, a, Lb, b, Lc, c, cfg=cfg)
+        else:
+            alt.matmul(M_, N_, K_, La, a, Lb, b, Lc, c, bias=bv if bias == "separate" else None, cfg=cfg)
+
+    def step():
+        for it in items:
+            gemm(it)
+    ms = _time(step, steps, warmup, ws)
+    flops = sum(2.0 * it[1] * it[2] * it[3] for it in items)
+    per = []
+    for it in items:
+        t = _time(lambda it=it: gemm(it), max(3, steps), 2, ws)
+        per.append({"gemm": it[0], "M": it[1], "N": it[2], "K": it[3], "us": round(t * 1e3, 2), "cfg": it[11],
+                    "tflops": round(2.0 * it[1] * it[2] * it[3] / (t * 1e-3) / 1e12, 1)})
+    return {"workload": "BERT-base GEMMs at seq 512 x 16 sequences (M=8192): 768x768, 768x3072, 3072x768, "
+                        "tiled A M/128 K/64, B N/nt K/64 (nt tuned), C M/128 N/64"
+                        + {"none": "", "separate": ", fp32 bias vector in the epilogue",
+                           "attached": ", bias attached to the weight columns by store_at "
+                                       "(Z N/nt (K+64)/64 nt 64), read in place"}[bias],
+            "ms_per_step": round(ms, 4), "tflops": round(flops / (ms * 1e-3) / 1e12, 2), "per_gemm": per}
+
+
+def relayout_run(steps, ws, dev):
+    """The D6 relayout set: algorithmic HBM GB/s per case and in aggregate."""
+    import paper_conf_eurosys_xuxpwwwdxcwc23_b200 as alt
+    from paper_conf_eurosys_xuxpwwwdxcwc23_b200 import relayout_set
+    peak = bench.peaks()[1]
+    cases, tot_bytes, tot_ms = [], 0.0, 0.0
+    for name, shape, sp, dp in relayout_set.cases():
+        for dt in (torch.bfloat16, torch.float32):
+            S, Dl = alt.Layout(shape, sp), alt.Layout(shape, dp)
+            src = S.empty(dt, dev).normal_()
+            dst = Dl.empty(dt, dev)
+            t = _time(lambda: alt.relayout(S, src, Dl, dst), max(5, steps), 2, ws)
+            nbytes = relayout_set.alg_bytes(S, Dl, src.element_size())
+            gbs = nbytes / (t * 1e-3) / 1e9
+            cases.append({"case": name, "dtype": str(dt)[6:], "MB": round(nbytes / 1e6, 1),
+                          "us": round(t * 1e3, 1), "GB/s": round(gbs), "frac": round(gbs / peak, 3)})
+            tot_bytes += nbytes
+            tot_ms += t
+            del src, dst
+    return {"workload": "D6 relayout set (ResNet tensors at batch 256, BERT A, KCRS weights)",
+            "gbs": round(tot_bytes / (tot_ms * 1e-3) / 1e9, 1), "hbm_peak_gbs": peak,
+            "frac": round(tot_bytes / (tot_ms * 1e-3) / 1e9 / peak, 3), "ms": round(tot_ms, 4), "cases": cases}
+
+
+def run(args):
+    ws, rank, local = bench.dist_init()
     dev = torch.device("cuda", local)
     torch.cuda.set_device(dev)
     out = None
-    if args.workload in ("r18", "mv2"):
-        if args.workload == "r18":
-            global_batch = 256
-            lo, hi = D.shard_range(global_batch, rank, ws)
-            ch = CH.resnet18(hi - lo, dev)
-        else:
-            global_batch = 16 * ws
-            ch = CH.mobilenet_v2(16, dev)
-        gathered = {}
-
-        def step():
-            y = ch.run()
-            if args.workload == "r18" and ws > 1:
-                gathered["y"] = D.gather_outputs(y, ws)   # the only cross-GPU step
-
-        n0 = alt.launch_count()
-        step()
-        torch.cuda.synchronize()
-        per_step_launches = alt.launch_count() - n0
-        ms = _time(step, args.steps, args.warmup, ws, graph=(ws == 1 or args.workload != "r18"))
-        flops = ch.flops * (global_batch / ch.N if args.workload == "r18" else ws)
-        recorded, launched = ch.plan()
-        cfg = {"workload": ("ResNet-18 conv chain (conv1 7x7 + 16 3x3 + 3 1x1 ds, maxpool, BN+ReLU, "
-                            "residual adds), global batch 256 sharded by batch, NCCL all-gather of the "
-                            "512x7x7 output" if args.workload == "r18" else
-                            "MobileNet-V2 chain (52 convs, 17 depthwise, BN+ReLU6, residual adds), "
-                            "batch 16 per GPU"),
-               "global_batch": global_batch, "per_gpu_batch": ch.N, "parallelism": f"dp{ws}"}
-        out = _line(args, ws, flops / (ms * 1e-3) / 1e12, "TFLOP/s", ms, cfg,
-                    {"scaling": "strong" if args.workload == "r18" else "weak",
-                     "gpu_launches": per_step_launches * args.steps,
-                     "propagation": {"alg1_recorded_conversions": recorded,
-                                     "standalone_conversion_kernels": launched,
-                                     "launches_per_step": per_step_launches,
-                                     "ops_per_step": len(ch.ops) + 1}})
+    if args.workload == "r18":
+        r = r18_strong(args.steps, args.warmup, ws, rank, dev)
+        out = _line(args, ws, r["tflops"], "TFLOP/s", r["ms_per_step"],
+                    {"workload": r["workload"], "global_batch": 256, "per_gpu_batch": r["per_gpu_batch"],
+                     "parallelism": f"dp{ws}"},
+                    {"scaling": "strong", "gpu_launches": r["gpu_launches_per_step"] * args.steps,
+                     "propagation": r["propagation"], "gathered_bytes": r["gathered_bytes"]})
+    elif args.workload == "mv2":
+        r = mv2_chain(args.steps, args.warmup, ws, dev)
+        out = _line(args, ws, r["tflops"] * ws, "TFLOP/s", r["ms_per_step"],
+                    {"workload": r["workload"], "global_batch": 16 * ws, "per_gpu_batch": 16,
+                     "parallelism": f"dp{ws}"},
+                    {"scaling": "weak", "gpu_launches": r["gpu_launches_per_step"] * args.steps,
+                     "propagation": r["propagation"], "hbm_gbs_min": r["hbm_gbs_min"]})
     elif args.workload == "bert":
-        from paper_conf_eurosys_xuxpwwwdxcwc23_b200 import layouts as LY
-        from paper_conf_eurosys_xuxpwwwdxcwc23_b200 import nets
-        from paper_conf_eurosys_xuxpwwwdxcwc23_b200 import tunecache
-        M = 8192
-        items = []
-        for name, K, N in nets.BERT_GEMMS:
-            tuned = tunecache.lookup_gemm(M, N, K) or {}
-            La = alt.Layout((M, K), LY.gemm_a_tiled(M, K, 128, 64))
-            Lb = alt.Layout((K, N), LY.gemm_b_tiled_nk(K, N, tuned.get("b_nt", 256), 64))
-            Lc = alt.Layout((M, N), LY.gemm_c_tiled(M, N, 128, 64))
-            a, b, c = La.empty(torch.bfloat16, dev).normal_(), Lb.empty(torch.bfloat16, dev).normal_(), \
-                Lc.empty(torch.bfloat16, dev)
-            bias = torch.randn(N, device=dev).to(torch.bfloat16)
-            if args.bert_bias == "attached":   # store_at: the bias rides in the weight
-                Lz = alt.Layout((K + 1, N), LY.gemm_z_tiled_nk(K, N, tuned.get("b_nt", 256), 64))
-                z = Lz.empty(torch.bfloat16, dev)
-                alt.store_at(Lb, b, bias, 0, Lz, z)
-                Lb, b = Lz, z
-            items.append((name, M, N, K, La, a, Lb, b, Lc, c, bias.float()))
-
-        cfgs = {}
-        for it in items:
-            c = dict(tunecache.lookup_gemm(it[1], it[2], it[3]) or {"path": 1, "block_n": 256})
-            c.pop("b_nt", None)  # a layout parameter, not a kernel one
-            cfgs[(it[1], it[2], it[3])] = c
-
-        def gemm(it):
-            _, M_, N_, K_, La, a, Lb, b, Lc, c, bias = it
-            if args.bert_bias == "attached":
-                alt.matmul_store_at(M_, N_, K_, La, a, Lb, b, Lc, c, cfg=cfgs[(M_, N_, K_)])
-            else:
-                alt.matmul(M_, N_, K_, La, a, Lb, b, Lc, c, bias=bias if args.bert_bias == "separate" else None,
-                           cfg=cfgs[(M_, N_, K_)])
-
-        def step():
-            for it in items:
-                gemm(it)
-
-        ms = _time(step, args.steps, args.warmup, ws)
-        flops = sum(2.0 * M_ * N_ * K_ for (_, M_, N_, K_, *_r) in items) * ws
-        per = []
-        for it in items:
-            t = _time(lambda it=it: gemm(it), max(3, args.steps), 2, ws)
-            per.append({"gemm": it[0], "M": it[1], "us": round(t * 1e3, 2), "cfg": cfgs[(it[1], it[2], it[3])],
-                        "tflops": round(2.0 * it[1] * it[2] * it[3] / (t * 1e-3) / 1e12, 1)})
-        out = _line(args, ws, flops / (ms * 1e-3) / 1e12, "TFLOP/s", ms,
-                    {"workload": "BERT-base GEMMs at seq 512 x 16 sequences (M=8192): 768x768, "
-                                 "768x3072, 3072x768, tiled A M/128 K/64, B N/nt K/64 (nt tuned), C M/128 N/64"
-                                 + {"none": "", "separate": ", fp32 bias vector in the epilogue",
-                                    "attached": ", bias attached to the weight columns by store_at "
-                                                "(Z N/nt (K+64)/64 nt 64), read in place"}[args.bert_bias],
-                     "global_batch": 16 * ws, "seq_len": 512, "parallelism": f"dp{ws}"},
-                    {"scaling": "weak", "per_gemm": per, "gpu_launches": 3 * args.steps})
+        r = bert_set(args.steps, args.warmup, ws, dev, args.bert_bias)
+        out = _line(args, ws, r["tflops"] * ws, "TFLOP/s", r["ms_per_step"],
+                    {"workload": r["workload"], "global_batch": 16 * ws, "seq_len": 512, "parallelism": f"dp{ws}"},
+                    {"scaling": "weak", "per_gemm": r["per_gemm"], "gpu_launches": 3 * args.steps})
     elif args.workload == "relayout":
-        from paper_conf_eurosys_xuxpwwwdxcwc23_b200 import relayout_set
-        peak = bench.peaks()[1]
-        cases, tot_bytes, tot_ms = [], 0.0, 0.0
-        for name, shape, sp, dp in relayout_set.cases():
-            for dt in (torch.bfloat16, torch.float32):
-                S, Dl = alt.Layout(shape, sp), alt.Layout(shape, dp)
-                src = S.empty(dt, dev).normal_()
-                dst = Dl.empty(dt, dev)
-                t = _time(lambda: alt.relayout(S, src, Dl, dst), max(5, args.steps), 2, ws)
-                nbytes = relayout_set.alg_bytes(S, Dl, src.element_size())
-                gbs = nbytes / (t * 1e-3) / 1e9
-                cases.append({"case": name, "dtype": str(dt)[6:], "MB": round(nbytes / 1e6, 1),
-                              "us": round(t * 1e3, 1), "GB/s": round(gbs), "frac": round(gbs / peak, 3)})
-                tot_bytes += nbytes
-                tot_ms += t
-        out = _line(args, ws, tot_bytes / (tot_ms * 1e-3) / 1e9, "GB/s", tot_ms, {
-            "workload": "D6 relayout set (ResNet tensors at batch 256, BERT A, KCRS weights)",
-            "parallelism": f"dp{ws}"}, {"scaling": "weak", "hbm_peak_gbs": peak, "cases": cases})
+        r = relayout_run(args.steps, ws, dev)
+        out = _line(args, ws, r["gbs"], "GB/s", r["ms"], {"workload": r["workload"], "parallelism": f"dp{ws}"},
+                    {"scaling": "weak", "hbm_peak_gbs": r["hbm_peak_gbs"], "cases": r["cases"]})
     elif args.workload == "fig12":
         out = fig12(args, ws)
     if rank == 0 and out is not None:

@@ -254,10 +254,13 @@ alt_status alt_matmul(int64_t M, int64_t N, int64_t K, alt_layout a_l,
  * [K + 1, N] = store_at(B, bias, 0), i.e. column n is (B[:, n], bias[n]):
  *   C[m,n] = act(scale[n] * sum_{k<K} A[m,k] Z[k,n] + Z[K,n] + residual).
  * The contraction reads rows k < K of Z through z_l (the same kernels as
- * alt_matmul); the attached row Z[K, :] is the bias, widened to fp32 by one
- * N-element gather launch on `stream` into stream-ordered scratch.  epi may
- * carry scale / residual / act; epi->bias must be NULL (ALT_E_INVALID).
- * Other errors as alt_matmul. */
+ * alt_matmul); the attached row Z[K, :] is the bias.  Separable z_l: the
+ * epilogue reads bias[n] in place at Z's owner offset rd0[K] + rd1[n] (no
+ * extra launch).  Non-separable z_l: the row is first gathered to fp32 by
+ * one N-element launch on `stream` into stream-ordered scratch.  z_l must
+ * be lossless (every element stored; else ALT_E_LOSSY).  epi may carry
+ * scale / residual / act; epi->bias must be NULL (ALT_E_INVALID).  Other
+ * errors as alt_matmul. */
 alt_status alt_matmul_store_at(int64_t M, int64_t N, int64_t K, alt_layout a_l,
                                const void *a, alt_layout z_l, const void *z,
                                alt_layout c_l, void *c, alt_dtype dtype,

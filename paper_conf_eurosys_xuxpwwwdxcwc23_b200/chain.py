@@ -25,6 +25,13 @@ from . import nets, synth
 _TUNE_PATH = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "chain_tune.json")
 
 
+def _numel(shape) -> int:
+    n = 1
+    for v in shape:
+        n *= v
+    return n
+
+
 def chan_tile(C: int) -> int:
     """largest power of two <= 64 dividing C (>= 8 for the tensor-core path)"""
     x = 64
@@ -63,8 +70,13 @@ def wgt_prims(L: nets.ConvShape):
 class Chain:
     """Device state + launch sequence of one network chain at batch N."""
 
-    def __init__(self, ops, N: int, dev, dtype=torch.bfloat16, name="chain", img_hw=224):
+    def __init__(self, ops, N: int, dev, dtype=torch.bfloat16, name="chain", img_hw=224, policy="propagated"):
+        """policy: "propagated" (every tensor in its consumer's tuned layout,
+        Alg. 1 + Fig. 5b) or a fixed activation layout for the whole chain,
+        "nhwc" / "nchw" (the fixed-layout baseline of P:426-465; weights keep
+        their offline layouts)."""
         self.ops, self.N, self.dev, self.dtype = ops, N, dev, dtype
+        self.policy = policy
         # logical shapes of every tensor
         shapes = {"img": (N, 3, img_hw, img_hw)}
         for op in ops:
@@ -79,11 +91,15 @@ class Chain:
         self.shapes = shapes
         # layout of each tensor: the input layout of its first consumer (the
         # same NCHW[x]c family for every consumer here, see act_prims)
-        self.layouts = {t: A.Layout(shp, act_prims(shp[1])) for t, shp in shapes.items()}
+        fixed = {"nhwc": LY.nhwc(), "nchw": LY.nchw()}.get(policy)
+        if policy != "propagated" and fixed is None:
+            raise ValueError(f"unknown layout policy {policy!r}")
+        self.layouts = {t: A.Layout(shp, act_prims(shp[1]) if fixed is None else fixed)
+                        for t, shp in shapes.items()}
         # a few-channel first conv (C = 3) reads the image window-folded
         # (reading A23): the input pad op writes that layout directly
         L0 = ops[0][1]
-        if ops[0][0] == "conv" and ops[0][2] == "img" and L0.C % 8 and L0.groups == 1:
+        if fixed is None and ops[0][0] == "conv" and ops[0][2] == "img" and L0.C % 8 and L0.groups == 1:
             self.layouts["img"] = A.Layout(shapes["img"], LY.conv_input_wfold(L0.C, L0.S, L0.stride, L0.pad))
         self.img_plain = A.Layout(shapes["img"], [])
         self.buf = {t: torch.zeros(self.layouts[t].phys_shape, dtype=dtype, device=dev) for t in shapes}
@@ -119,6 +135,19 @@ class Chain:
         torch.cuda.synchronize(dev) if dev.type == "cuda" else None
         self.flops = sum(op[1].flops(N) for op in ops if op[0] == "conv")
 
+    def min_bytes(self, esize: int = 2) -> float:
+        """algorithmic HBM bytes of one pass: every op reads its inputs once
+        (a residual too) and writes its output once"""
+        tot = 0.0
+        for op in self.ops:
+            if op[0] == "conv":
+                tot += op[1].min_bytes(self.N, esize)
+                if op[3] is not None:
+                    tot += esize * _numel(self.shapes[op[3]])
+            else:
+                tot += esize * (_numel(self.shapes[op[4]]) + _numel(self.shapes[op[5]]))
+        return tot
+
     # ------------------------------------------------------------ planning
     def plan(self):
         """Alg. 1 over the chain's DAG via alt_plan_chain.  Returns
@@ -149,7 +178,7 @@ class Chain:
 
     # -------------------------------------------------------------- tuning
     def tune_key(self):
-        return f"{self.name}|N{self.N}"
+        return f"{self.name}|N{self.N}" + ("" if self.policy == "propagated" else f"|{self.policy}")
 
     def tune(self, reps=10, warmup=3, store=True, log=None):
         """Per conv op, time candidate kernel configurations (BLOCK_N, CTA
@@ -263,11 +292,11 @@ class Chain:
         return self.ops[-1][5]
 
 
-def resnet18(N, dev, dtype=torch.bfloat16, img_hw=224):
-    return Chain(nets.resnet18_chain(img_hw), N, dev, dtype, "r18", img_hw)
+def resnet18(N, dev, dtype=torch.bfloat16, img_hw=224, policy="propagated"):
+    return Chain(nets.resnet18_chain(img_hw), N, dev, dtype, "r18", img_hw, policy)
 
 
-def mobilenet_v2(N, dev, dtype=torch.bfloat16, img_hw=224):
-    c = Chain(nets.mobilenet_v2_chain(img_hw), N, dev, dtype, "mv2", img_hw)
+def mobilenet_v2(N, dev, dtype=torch.bfloat16, img_hw=224, policy="propagated"):
+    c = Chain(nets.mobilenet_v2_chain(img_hw), N, dev, dtype, "mv2", img_hw, policy)
     c._relu6 = True
     return c

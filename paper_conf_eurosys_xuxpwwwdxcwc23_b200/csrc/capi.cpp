@@ -358,6 +358,9 @@ alt_status alt_matmul_store_at(int64_t M, int64_t N, int64_t K, alt_layout a_l, 
     set_error("alt_matmul_store_at: layout logical shapes do not match A[M,K] / Z[K+1,N] / C[M,N]");
     return ALT_E_SHAPE;
   }
+  // every element of Z (B and the attached bias row) must have a stored copy:
+  // a lossy Z (e.g. unfold with B < S) has owner offsets of -1 (reading A4)
+  if (!(z_l->impl.flags & ALT_LOSSLESS)) { set_error("alt_matmul_store_at: z's layout is lossy"); return ALT_E_LOSSY; }
   if (M == 0) return ALT_OK;
   if (!is_device_ptr(a) || !is_device_ptr(z) || !is_device_ptr(c)) { set_error("alt_matmul_store_at: A/Z/C must be device pointers"); return ALT_E_INVALID; }
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);

@@ -38,11 +38,23 @@ def init_from_env(backend: str | None = None):
     return world, rank, local
 
 
-def gather_outputs(local: torch.Tensor, world: int) -> torch.Tensor:
-    """All-gather equal-sized per-rank outputs along dim 0 (the batch dim of
-    the physical layout) into one tensor on every rank."""
+def gather_outputs(local: torch.Tensor, world: int, N: int | None = None) -> torch.Tensor:
+    """All-gather per-rank outputs along dim 0 (the batch dim of the physical
+    layout) into one tensor on every rank.  With N given, shards may be
+    uneven (shard_range): each rank pads its shard to ceil(N / world) rows,
+    and the padding rows are dropped after the gather."""
     if world == 1:
         return local
+    if N is not None and N % world:
+        per = -(-N // world)
+        if local.shape[0] < per:
+            pad = torch.zeros((per - local.shape[0],) + tuple(local.shape[1:]), dtype=local.dtype,
+                              device=local.device)
+            local = torch.cat([local, pad])
+        full = gather_outputs(local, world)
+        parts = [full[r * per: r * per + (shard_range(N, r, world)[1] - shard_range(N, r, world)[0])]
+                 for r in range(world)]
+        return torch.cat(parts)
     out = torch.empty((world * local.shape[0],) + tuple(local.shape[1:]), dtype=local.dtype,
                       device=local.device)
     if local.device.type == "cuda":
@@ -61,3 +73,14 @@ def max_over_ranks(x: float, world: int, device=None) -> float:
     t = torch.tensor([x], dtype=torch.float64, device=device)
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return float(t.item())
+
+
+def sharded_forward(N: int, world: int, rank: int, run_shard) -> torch.Tensor:
+    """Row a10: rank `rank` runs the whole chain on its contiguous image range
+    (run_shard(lo, hi) -> that shard's output, N outermost in its physical
+    layout, so the shard is a contiguous slice) and one all-gather assembles
+    the full batch on every rank.  Images are independent (O8), so the result
+    equals the unsharded chain's."""
+    lo, hi = shard_range(N, rank, world)
+    local = run_shard(lo, hi)
+    return gather_outputs(local, world, N)

@@ -69,3 +69,27 @@ def read_output(OL: oracle.Layout, y: torch.Tensor, dtype) -> np.ndarray:
     bad = OL.check_consistent(w)
     assert bad == 0, f"{bad} inconsistent physical positions (pad != 0 or copies differ)"
     return OL.read_f64(w)
+
+
+# Per-element bar next to the normwise one (bf16 path): the GPU's error on
+# every output is bounded by its bf16 output rounding (unit roundoff 2^-8 of
+# |y|) plus the fp32 accumulation error (<= n 2^-24 sum |x w| |scale|, n <=
+# 4608 reduction terms < 2^-11).  2^-7 (|ref| + absref) is a safe envelope
+# of both; a corrupted or misplaced element (a wrong row, a stale tile)
+# exceeds it.  absref = |scale| conv(|x|, |w|) + |bias| + |residual| in fp64.
+ELEM_REL = 2.0 ** -7
+
+
+def assert_elementwise(got: np.ndarray, ref: np.ndarray, absref: np.ndarray, what=""):
+    bad = np.abs(got - ref) > ELEM_REL * (np.abs(ref) + absref)
+    n = int(bad.sum())
+    if n:
+        idx = np.argwhere(bad)[0]
+        raise AssertionError(f"{what}: {n} element(s) outside 2^-7 (|ref| + sum|x w|), first at {tuple(idx)}: "
+                             f"got {got[tuple(idx)]!r} ref {ref[tuple(idx)]!r} absref {absref[tuple(idx)]!r}")
+
+
+def abs_conv_ref(p: dict, xl: np.ndarray, wl: np.ndarray, scale=None, bias=None, res=None) -> np.ndarray:
+    """|scale| conv(|x|, |w|) + |bias| + |res| (fp64 oracle, logical operands)"""
+    return oracle.conv2d_f64(p, np.abs(xl), np.abs(wl), None if scale is None else np.abs(scale),
+                             None if bias is None else np.abs(bias), None if res is None else np.abs(res), 0)

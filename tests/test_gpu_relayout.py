@@ -100,6 +100,19 @@ def test_relayout_full_size_r1_sampled():
     assert np.array_equal(dw[js], xw[src_idx])
 
 
+from paper_conf_eurosys_xuxpwwwdxcwc23_b200 import relayout_set  # noqa: E402
+
+
+@pytest.mark.parametrize("dtype", [torch.bfloat16, torch.float32])
+@pytest.mark.parametrize("case", relayout_set.cases(), ids=[c[0] for c in relayout_set.cases()])
+def test_relayout_d6_full_size_bit_exact(case, dtype):
+    """every D6 case at the size and in the launch configuration the bench
+    times (ResNet tensors at batch 256, BERT A 8192x3072, 512x512x3x3
+    weights): the whole destination, bit-exact against the oracle (O2)"""
+    name, shape, sp, dp = case
+    _gpu_relayout(shape, sp, dp, dtype, "full" + name)
+
+
 def test_relayout_shape_mismatch_and_lossy():
     a = alt.Layout((4, 8), [])
     b = alt.Layout((8, 4), [])

@@ -215,6 +215,13 @@ def test_G_and_F_bruteforce_vs_numpy(seed):
     want = np.where(ref >= 0, x.reshape(-1)[np.maximum(ref, 0)], 0).astype(np.uint32)
     assert np.array_equal(L.materialize(x), want)
     assert L.check_consistent(want) == 0
+    # unmaterialise (O2, F side) == numpy scatter of the owner copies: every
+    # held element reads back from the numpy image, a lossy layout is refused
+    if len(held) == n:
+        assert np.array_equal(L.unmaterialize(want), x)
+    else:
+        with pytest.raises(oracle.OracleError):
+            L.unmaterialize(want)
 
 
 def test_pad_matches_numpy_pad():
