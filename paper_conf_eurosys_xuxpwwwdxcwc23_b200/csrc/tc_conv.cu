@@ -53,6 +53,11 @@ struct OperandMap {
   int32_t slab_bytes;
   int32_t oob0;  // dim-0 coordinate that makes a box all zeros
   int32_t sw;    // slab width (channels)
+  // MN-major operand (mnw > 0): the stride-1 physical dim is the M (or N)
+  // dim, not the reduction; smem holds ng groups of mnw M-elements x 64
+  // K rows (gbytes each, K rows mnw * 2 bytes apart), one TMA box per
+  // (group, channel slab).  mnw = 0: K-major (channel run innermost).
+  int32_t mnw, ng, gbytes;
 };
 
 struct TcArgs {
@@ -365,7 +370,21 @@ __global__ void __launch_bounds__(kThreads, 1)
     const CUtensorMap *tmap = isA ? &tmA : &tmB;
     unsigned char *sbase = isA ? sA : sB;
     const int sbytes = isA ? kStageBytesA : L::kB;
-    const bool active = j < a.spi;
+    // issues per stage: (group, channel slab) pairs; a K-major operand has
+    // one group, an MN-major one ng groups of mnw rows (planner: <= 16)
+    const bool active = j < om.ng * a.spi;
+    const int gi = om.mnw ? j % om.ng : 0, si = om.mnw ? j / om.ng : j;
+    // this lane's group: rows [gi * mnw, (gi + 1) * mnw) of the tile
+    int g_dn = 0, g_dh = 0, g_dw = 0;
+    if (om.mnw && isA) {
+      const int r = gi * om.mnw;
+      g_dn = r / (a.tile_h * a.tile_w);
+      g_dh = (r / a.tile_w) % a.tile_h;
+      g_dw = r % a.tile_w;
+    } else if (om.mnw) {
+      g_dw = gi * om.mnw;
+    }
+    const uint32_t goff = (uint32_t)(gi * om.gbytes);
     int it = 0, ti = 0;
     for (int tile = unit0; tile < a.num_tiles; tile += unit_step, ti++) {
       const UnitInfo ui = unit_info(a, tile);
@@ -373,8 +392,8 @@ __global__ void __launch_bounds__(kThreads, 1)
       const int k_begin = ui.kb, k_end = ui.ke;
       int32_t v[NVAR];
       // B rows of this CTA: its 1/CG share of the unit's BN output channels
-      const int pp = isA ? tc.p0 : 0, qq = isA ? tc.q0 : tc.k0 + rank * (BN / CG) + a.b_koff;
-      v[V_N0] = isA ? tc.n0 : 0;
+      const int pp = isA ? tc.p0 + g_dh : 0, qq = (isA ? tc.q0 : tc.k0 + rank * (BN / CG) + a.b_koff) + g_dw;
+      v[V_N0] = isA ? tc.n0 + g_dn : 0;
       v[V_PT] = (int)om.fp.div((uint32_t)pp); v[V_PR] = pp - v[V_PT] * om.divp;
       v[V_QT] = (int)om.fq.div((uint32_t)qq); v[V_QR] = qq - v[V_QT] * om.divq;
       v[V_ONE] = 1;
@@ -388,7 +407,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           vt[V_R] = 0; vt[V_S] = 0; vt[V_GT] = 0; vt[V_GR] = 0;
           coords(om, vt, base);
         }
-        const uint32_t trow = smem_u32(tab) + (uint32_t)((isA ? 0 : 8) * 4 + j * 64);
+        const uint32_t trow = smem_u32(tab) + (uint32_t)((isA ? 0 : 8) * 4 + si * 64);
         int stage = it % STAGES;
         uint32_t ph = (uint32_t)((it / STAGES) & 1);
         for (int kit = k_begin; kit < k_end; kit++, it++) {
@@ -400,7 +419,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             int32_t o0, o1, o2, o3, o4;
             asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];" : "=r"(o0), "=r"(o1), "=r"(o2), "=r"(o3) : "r"(ta));
             asm volatile("ld.shared.b32 %0, [%1];" : "=r"(o4) : "r"(ta + 16));
-            unsigned char *dst = sbase + stage * sbytes + j * om.slab_bytes;
+            unsigned char *dst = sbase + stage * sbytes + goff + si * om.slab_bytes;
             if constexpr (CG == 2)
               tma_load_5d_2cta(dst, tmap, &full[stage], base[0] + o0, base[1] + o1, base[2] + o2, base[3] + o3,
                                base[4] + o4);
@@ -421,7 +440,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         if (lane == 0 && rank == 0) mbar_expect_tx(&full[stage], CG * (kStageBytesA + L::kB));
         __syncwarp();
         if (active) {
-          const int slab = kit * a.spi + j;
+          const int slab = kit * a.spi + si;
           const bool valid = slab < a.total_slabs;
           const int sl = valid ? slab : 0;
           const int tap = (int)a.f_Gc.div((uint32_t)sl), g = sl - tap * a.Gc;
@@ -432,10 +451,10 @@ __global__ void __launch_bounds__(kThreads, 1)
           coords(om, v, c);
           if (!valid) c[0] = om.oob0;
           if constexpr (CG == 2)
-            tma_load_5d_2cta(sbase + stage * sbytes + j * om.slab_bytes, tmap, &full[stage], c[0], c[1], c[2], c[3],
-                             c[4]);
+            tma_load_5d_2cta(sbase + stage * sbytes + goff + si * om.slab_bytes, tmap, &full[stage], c[0], c[1], c[2],
+                             c[3], c[4]);
           else
-            tma_load_5d(sbase + stage * sbytes + j * om.slab_bytes, tmap, &full[stage], c[0], c[1], c[2], c[3],
+            tma_load_5d(sbase + stage * sbytes + goff + si * om.slab_bytes, tmap, &full[stage], c[0], c[1], c[2], c[3],
                         c[4]);
         }
       }
@@ -445,22 +464,35 @@ __global__ void __launch_bounds__(kThreads, 1)
     if (lane == 0 && rank == 0) {
       // ------------------------------------------------------ MMA issuer
       // (the leader CTA issues for the pair: M = 128 * CG)
-      constexpr uint32_t idesc = idesc_f32acc(1 /*bf16*/, 128 * CG, BN);
+      // a_major / b_major (bits 15 / 16): MN-major operands
+      const uint32_t idesc = idesc_f32acc(1 /*bf16*/, 128 * CG, BN) | (a.A.mnw ? 1u << 15 : 0u) |
+                             (a.B.mnw ? 1u << 16 : 0u);
       const int sw = a.sw;
-      const uint32_t layout = sw == 8 ? 0u : (sw == 16 ? 6u : (sw == 32 ? 4u : 2u));
-      const uint32_t sbo = sw == 8 ? 128u : (uint32_t)(8 * sw * 2);
-      const uint32_t aS = (uint32_t)a.A.slab_bytes, bS = (uint32_t)a.B.slab_bytes;
-      const uint32_t lboA = sw == 8 ? aS : 16u, lboB = sw == 8 ? bS : 16u;
       // descriptors of stage 0's four K=16 steps; stage s adds s * stage bytes
       // to the start-address field (addr >> 4 in bits 0-13, no carry out)
+      auto desc = [&](const OperandMap &om, uint32_t base, int kk) -> uint64_t {
+        const int kc = kk * 16;
+        if (om.mnw == 0) {
+          // K-major: slab = sw channels x rows, each row one sw-channel run
+          const uint32_t layout = sw == 8 ? 0u : (sw == 16 ? 6u : (sw == 32 ? 4u : 2u));
+          const uint32_t sbo = sw == 8 ? 128u : (uint32_t)(8 * sw * 2);
+          const uint32_t lbo = sw == 8 ? (uint32_t)om.slab_bytes : 16u;
+          return smem_desc(base + (uint32_t)((kc / sw) * om.slab_bytes + (kc % sw) * 2), lbo, sbo, layout);
+        }
+        // MN-major: K row k of a group at k * mnw * 2 bytes; groups of mnw
+        // rows gbytes apart.  Swizzled: LBO = group stride, SBO = 8 K rows;
+        // interleaved (mnw = 8): SBO = group stride, LBO = 8 K rows (128 B)
+        const uint32_t rowb = (uint32_t)om.mnw * 2;
+        const uint32_t addr = base + (uint32_t)kc * rowb;
+        if (om.mnw == 8) return smem_desc(addr, 128u, (uint32_t)om.gbytes, 0u);
+        const uint32_t layout = om.mnw == 16 ? 6u : (om.mnw == 32 ? 4u : 2u);
+        return smem_desc(addr, (uint32_t)om.gbytes, 8u * rowb, layout);
+      };
       uint64_t dA[4], dB[4];
 #pragma unroll
       for (int kk = 0; kk < 4; kk++) {
-        const int kc = kk * 16;
-        const int slab = kc / sw;
-        const uint32_t off = (uint32_t)((kc % sw) * 2);
-        dA[kk] = smem_desc(smem_u32(sA) + slab * aS + off, lboA, sbo, layout);
-        dB[kk] = smem_desc(smem_u32(sB) + slab * bS + off, lboB, sbo, layout);
+        dA[kk] = desc(a.A, smem_u32(sA), kk);
+        dB[kk] = desc(a.B, smem_u32(sB), kk);
       }
       int it = 0, i = 0;
       for (int tile = unit0; tile < a.num_tiles; tile += unit_step, i++) {
@@ -1085,7 +1117,11 @@ static bool fold_window(const LView &x, const LView &w, int64_t S, int Vw, int p
 // Cut a TMA view out of a compiled layout: per logical dim a role (rows n/h/w,
 // channel c, filter taps r/s).  Requires the layout's affine map (split /
 // reorder / pad / unfold sequences); see DESIGN.md §5.
-static bool build_view(const LView &L, const RoleInfo *roles, int sw, View *out, char *why) {
+// mnw > 0 builds an MN-major view: the R_W role's in-tile dim must be the
+// stride-1 dim (box = mnw, the caller sets that role's tile to mnw and the
+// other row roles' tiles to 1: one box per group of mnw rows), the channel
+// dim is an ordinary box dim of sw channels.
+static bool build_view(const LView &L, const RoleInfo *roles, int sw, View *out, char *why, int mnw = 0) {
   auto fail = [&](const char *m) { snprintf(why, 160, "%s", m); return false; };
   if (!L.ok) return fail("layout not separable-affine");
   View v;
@@ -1118,13 +1154,13 @@ static bool build_view(const LView &L, const RoleInfo *roles, int sw, View *out,
           const int p = plist[d][i];
           if (L.coef[p] == 1) plo = p; else phi = p;
         }
-        if (plo < 0 || L.pstride[plo] != 1) return fail("channel tile is not the innermost (stride-1) dim");
+        if (plo < 0 || (!mnw && L.pstride[plo] != 1)) return fail("channel tile is not the innermost (stride-1) dim");
         const int64_t xlo = L.pshape[plo];
         if (xlo % sw) return fail("slab width does not divide channel tile");
         if (phi >= 0 && L.coef[phi] != xlo) return fail("channel digits not a plain split");
         v.xlo = xlo;
         v.divg = (int)(xlo / sw);
-        VDim &lo = add(plo, sw, 1, 0);
+        VDim &lo = add(plo, sw, 1, mnw ? 5 : 0);
         lo.coef[V_GR] = sw;
         if (phi >= 0) {
           VDim &hi = add(phi, 1, 1, 100);
@@ -1151,7 +1187,14 @@ static bool build_view(const LView &L, const RoleInfo *roles, int sw, View *out,
       case R_W: {
         const bool isH = ri.role == R_H;
         const int VT = isH ? V_PT : V_QT, VR = isH ? V_PR : V_QR, VTAP = isH ? V_R : V_S;
-        const int base_order = isH ? 20 : 10;
+        // MN-major: the W role's in-tile dim is the innermost box dim
+        const int base_order = isH ? 20 : (mnw ? 0 : 10);
+        if (mnw && !isH && ri.V != 1) return fail("MN-major operand with a strided M dim");
+        // a box's start along the stride-1 dim must stay 16-byte aligned (a
+        // filter tap / padding shift of the MN run traps in TMA): MN-major
+        // activations take 1x1 unpadded convs (and GEMM rows) only
+        if (mnw && !isH && (ri.win != 1 || ri.pad != 0 || off != 0))
+          return fail("MN-major operand with filter taps / padding along its stride-1 dim");
         int &div = isH ? v.divp : v.divq;
         if (nphys[d] == 0) {
           if (ri.tile != 1 || ri.win != 1) return fail("tile > 1 on a size-1 spatial dim");
@@ -1180,6 +1223,7 @@ static bool build_view(const LView &L, const RoleInfo *roles, int sw, View *out,
         if (ch == Elo) {
           // plain split (GEMM-like): no window, no stride, no padding
           if (ri.V != 1 || ri.win != 1 || ri.pad != 0 || off != 0) return fail("split spatial dim with window/stride");
+          if (mnw && !isH && ri.tile > Elo) return fail("MN-major group wider than the inner M tile");
           div = (int)Elo;
           if (ri.tile <= Elo) {
             if (Elo % ri.tile) return fail("tile does not divide spatial split");
@@ -1220,6 +1264,12 @@ static bool build_view(const LView &L, const RoleInfo *roles, int sw, View *out,
     }
   }
   if (v.xlo == 0) return fail("no channel dim");
+  if (mnw) {  // the group's mnw rows must be the stride-1 dim
+    bool ok = false;
+    for (int i = 0; i < v.rank; i++)
+      if (v.d[i].order == 0 && v.d[i].stride == 1 && v.d[i].box == mnw && v.d[i].estride == 1) ok = true;
+    if (!ok) return fail("MN-major: the M tile's run is not the stride-1 dim");
+  }
   // order: dim 0 = channel run, then box>1 dims inner->outer, then box-1
   std::stable_sort(v.d, v.d + v.rank, [](const VDim &x, const VDim &y) { return x.order < y.order; });
   // merge box-1 dims adjacent in memory until rank <= 5
@@ -1256,8 +1306,10 @@ static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
   return fn;
 }
 
+// sw: channels per slab; the swizzle follows the innermost box dim (sw for a
+// K-major view, the group width mnw for an MN-major one)
 static bool encode_view(const View &v, const void *base, int esize, int sw, CUtensorMap *tm, OperandMap *om,
-                        char *why) {
+                        char *why, int mnw = 0) {
   cuuint64_t dims[5], strides[4];
   cuuint32_t box[5], es[5];
   int64_t prev = 1;
@@ -1279,7 +1331,7 @@ static bool encode_view(const View &v, const void *base, int esize, int sw, CUte
   for (int i = 0; i < 4; i++)
     if (strides[i] % 16) { snprintf(why, 160, "TMA stride %llu not a multiple of 16 B", (unsigned long long)strides[i]); return false; }
   if ((reinterpret_cast<uintptr_t>(base) & 15)) { snprintf(why, 160, "base not 16-B aligned"); return false; }
-  const int row_bytes = sw * esize;
+  const int row_bytes = (mnw ? mnw : sw) * esize;
   CUtensorMapSwizzle swz = row_bytes == 16 ? CU_TENSOR_MAP_SWIZZLE_NONE
                            : row_bytes == 32 ? CU_TENSOR_MAP_SWIZZLE_32B
                            : row_bytes == 64 ? CU_TENSOR_MAP_SWIZZLE_64B
@@ -1304,6 +1356,9 @@ static bool encode_view(const View &v, const void *base, int esize, int sw, CUte
   om->slab_bytes = (int32_t)(rows * row_bytes);
   om->oob0 = (int32_t)v.d[0].extent;
   om->sw = sw;
+  om->mnw = mnw;
+  om->ng = 1;
+  om->gbytes = 0;
   return true;
 }
 
@@ -1594,17 +1649,44 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
     }
     for (int sw = 64; sw >= 8; sw /= 2) {
       View va, vb;
-      if (!build_view(P.va, ra, sw, &va, why)) continue;
-      if (!build_view(P.vb, rb, sw, &vb, why)) continue;
+      // K-major first (the channel run innermost); otherwise an MN-major
+      // view whose stride-1 dim is the M (A) / N (B) run: groups of mnw rows
+      // (mnw = the widest of 64 / 32 / 16 / 8 that tiles the run), one TMA box
+      // of mnw x sw per (group, slab)
+      auto view_of = [&](const LView &L, const RoleInfo *roles, int rows, int run, View *v, int *mnw) -> bool {
+        *mnw = 0;
+        if (build_view(L, roles, sw, v, why)) return true;
+        char why2[160];
+        for (int w = 64; w >= 8; w /= 2) {
+          if (run % w || rows % w || (rows / w) * (64 / sw) > 16) continue;
+          RoleInfo rm[kMaxL];
+          memcpy(rm, roles, sizeof(rm));
+          for (int d = 0; d < kMaxL; d++) {
+            if (rm[d].role == R_W) rm[d].tile = w;
+            if (rm[d].role == R_H || rm[d].role == R_N) rm[d].tile = 1;
+          }
+          if (build_view(L, rm, sw, v, why2, w)) { *mnw = w; return true; }
+        }
+        return false;
+      };
+      int mnA = 0, mnB = 0;
+      if (!view_of(P.va, ra, 128, c.tw, &va, &mnA)) continue;
+      if (!view_of(P.vb, rb, BN / cg, BN / cg, &vb, &mnB)) continue;
       int64_t rowsA = 1, rowsB = 1;
       for (int i = 1; i < va.rank; i++) rowsA *= (va.d[i].box + va.d[i].estride - 1) / va.d[i].estride;
       for (int i = 1; i < vb.rank; i++) rowsB *= (vb.d[i].box + vb.d[i].estride - 1) / vb.d[i].estride;
-      if (rowsA != 128 || rowsB != BN / cg) { snprintf(why, 160, "rows A %lld B %lld", (long long)rowsA, (long long)rowsB); continue; }
+      // K-major: a box holds the tile's rows; MN-major: sw K rows of one group
+      if (rowsA != (mnA ? sw : 128) || rowsB != (mnB ? sw : BN / cg)) {
+        snprintf(why, 160, "rows A %lld B %lld", (long long)rowsA, (long long)rowsB);
+        continue;
+      }
       TcPlan pl;
       TcArgs &a = pl.a;
       memset(&a, 0, sizeof(a));
-      if (!encode_view(va, P.a, esize, sw, &pl.ta, &a.A, why)) continue;
-      if (!encode_view(vb, P.b, esize, sw, &pl.tb, &a.B, why)) continue;
+      if (!encode_view(va, P.a, esize, sw, &pl.ta, &a.A, why, mnA)) continue;
+      if (!encode_view(vb, P.b, esize, sw, &pl.tb, &a.B, why, mnB)) continue;
+      if (mnA) { a.A.ng = 128 / mnA; a.A.gbytes = 64 * mnA * esize; }
+      if (mnB) { a.B.ng = BN / cg / mnB; a.B.gbytes = 64 * mnB * esize; }
       // output: TMA-store view when y holds one copy per element (no pads /
       // unfold duplicates) and a >= 8-channel contiguous run, else the writer
       a.out_mode = 0;
