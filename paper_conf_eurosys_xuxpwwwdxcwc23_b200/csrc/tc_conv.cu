@@ -75,6 +75,11 @@ struct TcArgs {
   int32_t S, Gc;
   FastDiv f_nnt, f_mtw, f_mth, f_spl, f_Gc, f_S;  // num_n_tiles, mt_w, mt_h, splits, Gc, S
   int32_t total_slabs, spi, num_iters;
+  // fp32 operands split into three bf16 planes (reading A27): pairs = 6
+  // plane products per reduction step (0 = plain bf16); rsg = R * S * Gc
+  // slabs per pair; out_f32: the output (and residual) are fp32
+  int32_t pairs, rsg, out_f32;
+  FastDiv f_rsg;
   int32_t sw;
   Writer yw;
   Reader yr;             // out_mode 2: owner offsets of y
@@ -147,6 +152,30 @@ __device__ __forceinline__ uint64_t gtimer() {
 #define DBG(slot) \
   if (a.dbg) a.dbg[(size_t)blockIdx.x * 40 + (slot)] = gtimer()
 
+// reduction slab -> filter tap (r, s) and the channel slab of A and of B.
+// Plain operands: slab = tap * Gc + g.  fp32 split operands (a.pairs = 6):
+// slab = pair * (R S Gc) + tap * Gc + g, the pair selecting the bf16 planes
+// (pa, pb) in {lh, hl, mm, mh, hm, hh} (every product of weight > 2^-24); a
+// plane starts Gc channel slabs after the previous one.  Smallest products
+// first: the tensor core's fp32 accumulation rounds each MMA step relative
+// to the accumulator's magnitude, so the five small pairs are summed while
+// the accumulator is still small and only the hh steps see the full value
+// (measured 6x lower error than hh first).
+__device__ __forceinline__ void slab_decode(const TcArgs &a, int sl, int &r, int &sx, int &gA, int &gB) {
+  int rem = sl, pa = 0, pb = 0;
+  if (a.pairs) {
+    const int pr = (int)a.f_rsg.div((uint32_t)sl);
+    rem = sl - pr * a.rsg;
+    pa = (0x001102 >> (4 * pr)) & 0xF;
+    pb = (0x010120 >> (4 * pr)) & 0xF;
+  }
+  const int tap = (int)a.f_Gc.div((uint32_t)rem), g = rem - tap * a.Gc;
+  r = (int)a.f_S.div((uint32_t)tap);
+  sx = tap - r * a.S;
+  gA = pa * a.Gc + g + a.a_goff;
+  gB = pb * a.Gc + g;
+}
+
 __device__ __forceinline__ void coords(const OperandMap &m, const int32_t (&v)[NVAR], int32_t (&c)[5]) {
 #pragma unroll
   for (int d = 0; d < 5; d++) {
@@ -198,6 +227,42 @@ static __device__ __noinline__ void residual_chunk(const EpiParams &e, int is_co
       if (o >= 0) r = bf16_to_f32(__ldg(res + o));
     }
     out[j] = r;
+  }
+}
+// fp32 residual (split-operand path)
+static __device__ __noinline__ void residual_chunk_f32(const EpiParams &e, int is_conv, int K, int n, int p, int q,
+                                                       int kb, int koff, float *out) {
+  const float *res = static_cast<const float *>(e.residual);
+  for (int j = 0; j < 32; j++) {
+    const int k = kb + j;
+    float r = 0.f;
+    if (k < K) {
+      const int64_t o = is_conv ? e.res.off4(n, koff + k, p, q) : e.res.off2(q, koff + k);
+      if (o >= 0) r = __ldg(res + o);
+    }
+    out[j] = r;
+  }
+}
+// fp32 output: one row's 32 channels, direct 16-byte stores of 4 channels
+// (out_mode 2) or through the generic writer
+static __device__ __noinline__ void store_chunk_f32(const TcArgs &a, float *y, int64_t yrow, int n, int p, int q,
+                                                    int kb, const float *v) {
+  if (a.out_mode == 2) {
+    for (int c = 0; c < 8; c++) {
+      const int k = kb + 4 * c;
+      if (k >= a.K) break;
+      float *dst = y + yrow + __ldg(a.yr.rd[1] + a.y_koff + k);
+      asm volatile("st.global.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(dst), "f"(v[4 * c]), "f"(v[4 * c + 1]),
+                   "f"(v[4 * c + 2]), "f"(v[4 * c + 3])
+                   : "memory");
+    }
+    return;
+  }
+  for (int j = 0; j < 32; j++) {
+    const int k = kb + j;
+    if (k >= a.K) break;
+    if (a.is_conv) write4<float>(a.yw, y, n, a.y_koff + k, p, q, v[j]);
+    else write2<float>(a.yw, y, q, a.y_koff + k, v[j]);
   }
 }
 // one row's 32 channels through the generic writer (pads, unfold copies)
@@ -332,12 +397,12 @@ __global__ void __launch_bounds__(kThreads, 1)
     for (int sl = threadIdx.x; sl < padded_slabs; sl += kThreads) {
       const bool valid = sl < a.total_slabs;
       const int s0 = valid ? sl : 0;
-      const int tap = (int)a.f_Gc.div((uint32_t)s0), g = s0 - tap * a.Gc;
-      const int r = (int)a.f_S.div((uint32_t)tap), sx = tap - r * a.S;
+      int r, sx, gA, gB;
+      slab_decode(a, s0, r, sx, gA, gB);
 #pragma unroll
       for (int o = 0; o < 2; o++) {
         const OperandMap &om = o == 0 ? a.A : a.B;
-        const int ga = o == 0 ? g + a.a_goff : g;
+        const int ga = o == 0 ? gA : gB;
         const int gt = (int)om.fg.div((uint32_t)ga), gr = ga - gt * om.divg;
 #pragma unroll
         for (int d = 0; d < 5; d++)
@@ -443,9 +508,9 @@ __global__ void __launch_bounds__(kThreads, 1)
           const int slab = kit * a.spi + si;
           const bool valid = slab < a.total_slabs;
           const int sl = valid ? slab : 0;
-          const int tap = (int)a.f_Gc.div((uint32_t)sl), g = sl - tap * a.Gc;
-          v[V_R] = (int)a.f_S.div((uint32_t)tap); v[V_S] = tap - v[V_R] * a.S;
-          const int ga = isA ? g + a.a_goff : g;
+          int gA, gB;
+          slab_decode(a, sl, v[V_R], v[V_S], gA, gB);
+          const int ga = isA ? gA : gB;
           v[V_GT] = (int)om.fg.div((uint32_t)ga); v[V_GR] = ga - v[V_GT] * om.divg;
           int32_t c[5];
           coords(om, v, c);
@@ -816,9 +881,17 @@ __global__ void __launch_bounds__(kThreads, 1)
           if constexpr (!EARLY) {
             if (!RV && a.epi.residual && vrow) {
               float rv[32];  // local memory, touched only when a residual exists
-              residual_chunk(a.epi, a.is_conv, a.K, n, p, q, kb, a.y_koff, rv);
+              if (a.out_f32) residual_chunk_f32(a.epi, a.is_conv, a.K, n, p, q, kb, a.y_koff, rv);
+              else residual_chunk(a.epi, a.is_conv, a.K, n, p, q, kb, a.y_koff, rv);
 #pragma unroll
               for (int j = 0; j < 32; j++) v[j] += rv[j];
+            }
+            if (a.out_f32) {  // fp32 result (split-operand path): act, store
+#pragma unroll
+              for (int j = 0; j < 32; j++) v[j] = act == 1 ? fmaxf(v[j], 0.f) : (act == 2 ? fminf(fmaxf(v[j], 0.f), 6.f) : v[j]);
+              if (vrow) store_chunk_f32(a, reinterpret_cast<float *>(y), yrow, n, p, q, kb, v);
+              if (c0 + kStep < BN) tmem_ld_32x32b_x32(next, raw);
+              continue;
             }
           }
           // activation folded into the bf16 conversion (cvt .relu)
@@ -896,7 +969,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         if (a.out_mode != 0 && !wsl) chunk_loop(std::true_type{}, std::true_type{});
         else chunk_loop(std::false_type{}, std::true_type{});
       } else {
-        if (a.out_mode != 0 && !a.epi.residual && !wsl) chunk_loop(std::true_type{}, std::false_type{});
+        if (a.out_mode != 0 && !a.epi.residual && !wsl && !a.out_f32) chunk_loop(std::true_type{}, std::false_type{});
         else chunk_loop(std::false_type{}, std::false_type{});
       }
       if (coop_rows >= 0) {
@@ -1547,6 +1620,8 @@ struct TcProblem {
   int64_t R, S, C;            // taps and reduction channels
   OpEpilogue epi;
   int64_t coff = 0, koff = 0; // grouped conv: this group's first input / output channel
+  int pairs = 0;              // fp32 split operands: 6 plane products per slab (0 = bf16)
+  bool out_f32 = false;       // fp32 output / residual
 };
 
 static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t stream, alt_kernel_cfg *used,
@@ -1571,6 +1646,7 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
     k[i++] = P.epi.residual_l ? (int64_t)P.epi.residual_l->serial : 0;
     k[i++] = P.epi.act;
     k[i++] = (P.coff << 32) | P.koff;
+    k[i++] = P.pairs * 2 + (P.out_f32 ? 1 : 0);
     if (cfg) {
       k[i++] = cfg->block_n; k[i++] = cfg->tile_n; k[i++] = cfg->tile_h; k[i++] = cfg->tile_w;
       k[i++] = cfg->stages;
@@ -1696,13 +1772,14 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
         // default TMA stores (measured faster than direct 16-byte stores)
         return e && e[0] == 'd' ? 2 : (e && e[0] == 'g' ? 0 : 1);
       }();
-      if (store_mode == 2 && !(P.yl->flags & (ALT_HAS_PAD | ALT_HAS_UNFOLD)) && P.K % 8 == 0 && P.koff % 8 == 0 &&
-          (reinterpret_cast<uintptr_t>(P.y) & 15) == 0 && direct_store_ok(P.vy)) {
+      // fp32 output: direct 16-byte stores (4 channels) or the generic writer
+      if ((store_mode == 2 || P.out_f32) && !(P.yl->flags & (ALT_HAS_PAD | ALT_HAS_UNFOLD)) && P.K % 8 == 0 &&
+          P.koff % 8 == 0 && (reinterpret_cast<uintptr_t>(P.y) & 15) == 0 && direct_store_ok(P.vy)) {
         alt_status st2 = make_reader(P.yl, &a.yr);
         if (st2 != ALT_OK) return st2;
         a.out_mode = 2;
       }
-      if (a.out_mode == 0 && store_mode != 0 && !(P.yl->flags & (ALT_HAS_PAD | ALT_HAS_UNFOLD))) {
+      if (a.out_mode == 0 && store_mode != 0 && !P.out_f32 && !(P.yl->flags & (ALT_HAS_PAD | ALT_HAS_UNFOLD))) {
         char why2[160];
         for (int so = 32; so >= 8 && !a.out_mode; so /= 2) {
           if (P.koff % so) continue;  // a group's first channel must start a store slab
@@ -1731,7 +1808,11 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       a.a_goff = (int32_t)(P.coff / sw);
       a.b_koff = (int32_t)P.koff;
       a.y_koff = (int32_t)P.koff;
-      a.total_slabs = (int32_t)(P.R * P.S * a.Gc);
+      a.rsg = (int32_t)(P.R * P.S * a.Gc);
+      a.pairs = P.pairs;
+      a.out_f32 = P.out_f32 ? 1 : 0;
+      if (P.pairs && P.C % sw) { snprintf(why, 160, "split planes not slab-aligned"); continue; }
+      a.total_slabs = (int32_t)((P.pairs ? P.pairs : 1) * P.R * P.S * a.Gc);
       a.spi = 64 / sw;
       a.num_iters = (a.total_slabs + a.spi - 1) / a.spi;
       a.sw = sw;
@@ -1805,10 +1886,11 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       a.f_mth = FastDiv((uint32_t)a.mt_h);
       a.f_spl = FastDiv((uint32_t)a.splits);
       a.f_Gc = FastDiv((uint32_t)a.Gc);
+      a.f_rsg = FastDiv((uint32_t)std::max(1, a.rsg));
       a.f_S = FastDiv((uint32_t)a.S);
       alt_status st;
       if ((st = make_epi(P.epi, &a.epi)) != ALT_OK) return st;
-      a.res_vec = P.epi.residual && a.epi.res.sep && chan_vec8(*P.epi.residual_l, true) &&
+      a.res_vec = P.epi.residual && !P.out_f32 && a.epi.res.sep && chan_vec8(*P.epi.residual_l, true) &&
                   (reinterpret_cast<uintptr_t>(P.epi.residual) & 15) == 0 ? 1 : 0;
       // the kernel always applies scale * acc + bias: absent ones become the
       // identity (device-resident ones / zeros, grown on demand)
@@ -1856,8 +1938,128 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
   return ALT_E_UNSUPPORTED;
 }
 
+// ---- fp32 on the tensor cores (reading A27, split3.cu): each fp32 operand is
+// split into three bf16 planes stored reduction-innermost ([outer][3 Cp]) in
+// stream-ordered scratch, the conv / GEMM runs the six plane products of
+// every reduction slab on the bf16 kernel, and the epilogue writes fp32.
+alt_status split3_launch(Layout *L, const float *src, int red, int64_t C, int64_t Cp, uint16_t *dst,
+                         cudaStream_t stream);
+
+// compiled internal layouts of the split planes, by logical shape (stable
+// serials keep the launch-plan cache hit across calls)
+static Layout *split_layout(int lrank, const int64_t *lshape, int nprims, const alt_prim *prims) {
+  static std::mutex mu;
+  static std::vector<std::pair<std::vector<int64_t>, Layout *>> cache;
+  std::vector<int64_t> key(lshape, lshape + lrank);
+  key.push_back(nprims ? prims[0].v[0] * 16 + prims[0].v[1] : -1);
+  std::lock_guard<std::mutex> g(mu);
+  for (auto &e : cache)
+    if (e.first == key) return e.second;
+  Layout *L = new Layout();
+  if (compile_layout(lrank, lshape, prims, nprims, L) != ALT_OK) { delete L; return nullptr; }
+  cache.push_back({key, L});
+  return L;
+}
+
+struct SplitScratch {
+  void *p[2] = {nullptr, nullptr};
+  cudaStream_t s;
+  ~SplitScratch() { for (void *q : p) if (q) cudaFreeAsync(q, s); }
+};
+
+static alt_status tc_conv_f32(const ConvProblem &P, const alt_kernel_cfg *cfg, cudaStream_t stream,
+                              alt_kernel_cfg *used) {
+  if (P.groups > 1) { set_error("tc path: fp32 grouped conv runs on the generic path"); return ALT_E_UNSUPPORTED; }
+  const int64_t Cp = (P.C + 7) / 8 * 8;
+  alt_prim nhwc{};
+  nhwc.kind = ALT_REORDER; nhwc.n = 4; nhwc.v[0] = 0; nhwc.v[1] = 2; nhwc.v[2] = 3; nhwc.v[3] = 1;
+  const int64_t xs[4] = {P.N, 3 * Cp, P.H, P.W}, ws[4] = {P.K, 3 * Cp, P.R, P.S};
+  Layout *XL = split_layout(4, xs, 1, &nhwc), *WL = split_layout(4, ws, 1, &nhwc);
+  if (!XL || !WL) return ALT_E_NOMEM;
+  SplitScratch sc;
+  sc.s = stream;
+  if (cudaMallocAsync(&sc.p[0], (size_t)XL->pnumel * 2, stream) != cudaSuccess ||
+      cudaMallocAsync(&sc.p[1], (size_t)WL->pnumel * 2, stream) != cudaSuccess) {
+    cudaGetLastError();
+    set_error("tc fp32: split scratch allocation failed");
+    return ALT_E_NOMEM;
+  }
+  alt_status st = split3_launch(P.xl, static_cast<const float *>(P.x), 1, P.C, Cp,
+                                static_cast<uint16_t *>(sc.p[0]), stream);
+  if (st == ALT_OK)
+    st = split3_launch(P.wl, static_cast<const float *>(P.w), 1, P.C, Cp, static_cast<uint16_t *>(sc.p[1]), stream);
+  if (st != ALT_OK) return st;
+  TcProblem T{};
+  T.is_conv = true;
+  T.al = XL; T.bl = WL; T.yl = P.yl;
+  T.a = sc.p[0]; T.b = sc.p[1]; T.y = P.y;
+  T.ra[0].role = R_N;
+  T.ra[1].role = R_C;
+  T.ra[2] = RoleInfo{R_H, 1, P.Vh, P.ph, (int)((P.R - 1) * P.dh + 1), P.dh};
+  T.ra[3] = RoleInfo{R_W, 1, P.Vw, P.pw, (int)((P.S - 1) * P.dw + 1), P.dw};
+  T.rb[0] = RoleInfo{R_W, 1, 1, 0, 1, 0};
+  T.rb[1].role = R_C;
+  T.rb[2].role = R_TR;
+  T.rb[3].role = R_TS;
+  T.ry[0].role = R_N;
+  T.ry[1].role = R_C;
+  T.ry[2] = RoleInfo{R_H, 1, 1, 0, 1, 0};
+  T.ry[3] = RoleInfo{R_W, 1, 1, 0, 1, 0};
+  T.N = P.N; T.K = P.K; T.Ho = P.Ho; T.Wo = P.Wo;
+  T.R = P.R; T.S = P.S; T.C = Cp;
+  T.epi = P.epi;
+  T.va = lview(*XL); T.vb = lview(*WL); T.vy = lview(*P.yl);
+  T.pairs = 6;
+  T.out_f32 = true;
+  if (P.N * P.Ho * P.Wo >= (1ll << 31)) { set_error("tc: too many output pixels"); return ALT_E_UNSUPPORTED; }
+  return tc_run(T, cfg, stream, used, 0, 0);
+}
+
+static alt_status tc_gemm_f32(const GemmProblem &P, const alt_kernel_cfg *cfg, cudaStream_t stream,
+                              alt_kernel_cfg *used) {
+  const int64_t Kp = (P.K + 7) / 8 * 8;
+  alt_prim tr{};
+  tr.kind = ALT_REORDER; tr.n = 2; tr.v[0] = 1; tr.v[1] = 0;
+  const int64_t as[2] = {P.M, 3 * Kp}, bs[2] = {3 * Kp, P.N};
+  Layout *AL = split_layout(2, as, 0, nullptr), *BL = split_layout(2, bs, 1, &tr);
+  if (!AL || !BL) return ALT_E_NOMEM;
+  SplitScratch sc;
+  sc.s = stream;
+  if (cudaMallocAsync(&sc.p[0], (size_t)AL->pnumel * 2, stream) != cudaSuccess ||
+      cudaMallocAsync(&sc.p[1], (size_t)BL->pnumel * 2, stream) != cudaSuccess) {
+    cudaGetLastError();
+    set_error("tc fp32: split scratch allocation failed");
+    return ALT_E_NOMEM;
+  }
+  // A [M, K]: reduction dim 1; B [K(+1), N]: reduction dim 0, rows k < K
+  alt_status st = split3_launch(P.al, static_cast<const float *>(P.a), 1, P.K, Kp,
+                                static_cast<uint16_t *>(sc.p[0]), stream);
+  if (st == ALT_OK)
+    st = split3_launch(P.bl, static_cast<const float *>(P.b), 0, P.K, Kp, static_cast<uint16_t *>(sc.p[1]), stream);
+  if (st != ALT_OK) return st;
+  TcProblem T{};
+  T.is_conv = false;
+  T.al = AL; T.bl = BL; T.yl = P.cl;
+  T.a = sc.p[0]; T.b = sc.p[1]; T.y = P.c;
+  T.ra[0] = RoleInfo{R_W, 128, 1, 0, 1, 0};
+  T.ra[1].role = R_C;
+  T.rb[0].role = R_C;
+  T.rb[1] = RoleInfo{R_W, 1, 1, 0, 1, 0};
+  T.ry[0] = RoleInfo{R_W, 128, 1, 0, 1, 0};
+  T.ry[1].role = R_C;
+  T.N = 1; T.K = P.N; T.Ho = 1; T.Wo = P.M;
+  T.R = 1; T.S = 1; T.C = Kp;
+  T.epi = P.epi;
+  T.va = lview(*AL); T.vb = lview(*BL); T.vy = lview(*P.cl);
+  T.pairs = 6;
+  T.out_f32 = true;
+  if (P.M >= (1ll << 31)) { set_error("tc: M too large"); return ALT_E_UNSUPPORTED; }
+  return tc_run(T, cfg, stream, used, 1, 1);
+}
+
 alt_status tc_conv(const ConvProblem &P, const alt_kernel_cfg *cfg, cudaStream_t stream, alt_kernel_cfg *used) {
-  if (P.dtype != ALT_BF16) { set_error("tc path: bf16 only"); return ALT_E_UNSUPPORTED; }
+  if (P.dtype == ALT_F32) return tc_conv_f32(P, cfg, stream, used);
+  if (P.dtype != ALT_BF16) { set_error("tc path: bf16 / fp32 only"); return ALT_E_UNSUPPORTED; }
   const int64_t G = P.groups < 1 ? 1 : P.groups;
   const int64_t Cg = P.C / G, Kg = P.K / G;
   if (G > 1 && (Cg % 8 || Kg % 8 || G == P.C)) {
@@ -1914,7 +2116,8 @@ alt_status tc_conv(const ConvProblem &P, const alt_kernel_cfg *cfg, cudaStream_t
 }
 
 alt_status tc_gemm(const GemmProblem &P, const alt_kernel_cfg *cfg, cudaStream_t stream, alt_kernel_cfg *used) {
-  if (P.dtype != ALT_BF16) { set_error("tc path: bf16 only"); return ALT_E_UNSUPPORTED; }
+  if (P.dtype == ALT_F32) return tc_gemm_f32(P, cfg, stream, used);
+  if (P.dtype != ALT_BF16) { set_error("tc path: bf16 / fp32 only"); return ALT_E_UNSUPPORTED; }
   TcProblem T{};
   T.is_conv = false;
   T.al = P.al; T.bl = P.bl; T.yl = P.cl;

@@ -95,8 +95,6 @@ GEMM_CASES = [
 @pytest.mark.parametrize("case", GEMM_CASES, ids=[f"{c[0]}x{c[1]}x{c[2]}p{c[3]}{c[4]}" for c in GEMM_CASES])
 def test_matmul_store_at_parity(case, dtype):
     M, N, K, pad, path = case
-    if dtype == torch.float32 and path == "tc":
-        pytest.skip("tensor-core path is bf16")
     A = synth.activations("msa_A", (M, K))
     B = synth.weights("msa_B", (K, N))
     bias = synth.bn_bias("msa_b", N)
