@@ -137,12 +137,14 @@ def plan_layer(L, N):
 class LayerSet:
     """Device state for the ResNet-50 layer set at batch N."""
 
-    def __init__(self, N: int, dev):
+    def __init__(self, N: int, dev, dtype=None):
         import torch
         import paper_conf_eurosys_xuxpwwwdxcwc23_b200 as alt
         from paper_conf_eurosys_xuxpwwwdxcwc23_b200 import nets, synth
+        dtype = dtype or torch.bfloat16
         self.alt = alt
         self.N = N
+        self.dtype = dtype
         self.layers = []
         for L in nets.RESNET50:
             pl = plan_layer(L, N)
@@ -152,20 +154,20 @@ class LayerSet:
             lw0 = alt.Layout((L.K, L.C, L.R, L.S), [])
             lw = alt.Layout((L.K, L.C, L.R, L.S), pl["w"])
             ly = alt.Layout((N, L.K, Ho, Wo), pl["y"])
-            x0 = synth.activations("r50x" + L.name, (N, L.C, L.H, L.W)).to(torch.bfloat16)
-            w0 = synth.weights("r50w" + L.name, (L.K, L.C, L.R, L.S)).to(torch.bfloat16)
-            xt = lx.empty(torch.bfloat16, dev)
-            wt = lw.empty(torch.bfloat16, dev)
+            x0 = synth.activations("r50x" + L.name, (N, L.C, L.H, L.W)).to(dtype)
+            w0 = synth.weights("r50w" + L.name, (L.K, L.C, L.R, L.S)).to(dtype)
+            xt = lx.empty(dtype, dev)
+            wt = lw.empty(dtype, dev)
             x0d = x0.to(dev)
             alt.relayout(lx0, x0d, lx, xt)                       # conversion op (Fig. 5a)
             alt.relayout(lw0, w0.to(dev), lw, wt)                # weights: offline
-            yt = ly.empty(torch.bfloat16, dev)
+            yt = ly.empty(dtype, dev)
             sc = synth.bn_scale("r50s" + L.name, L.K).to(dev)
             bi = synth.bn_bias("r50b" + L.name, L.K).to(dev)
             p = alt.conv_params(N, L.C, L.H, L.W, L.K, L.R, L.S, L.stride, L.pad)
             self.layers.append(dict(L=L, p=p, lx0=lx0, lx=lx, lw=lw, ly=ly, x=xt, w=wt, y=yt, sc=sc,
                                     bi=bi, cfg=pl["cfg"], x_host=x0.pin_memory(), x0d=x0d,
-                                    y_host=torch.empty(yt.shape, dtype=torch.bfloat16).pin_memory()))
+                                    y_host=torch.empty(yt.shape, dtype=dtype).pin_memory()))
         self.flops = sum(l["L"].flops(N) for l in self.layers)
         self.alg_bytes = sum(l["L"].min_bytes(N) for l in self.layers)
         self.plans = []
@@ -224,9 +226,29 @@ class LayerSet:
         comp.wait_stream(self.s_in)
 
     def io_bytes(self):
-        h2d = sum(l["x_host"].numel() * 2 for l in self.layers)
-        d2h = sum(l["y_host"].numel() * 2 for l in self.layers)
+        h2d = sum(l["x_host"].numel() * l["x_host"].element_size() for l in self.layers)
+        d2h = sum(l["y_host"].numel() * l["y_host"].element_size() for l in self.layers)
         return h2d, d2h
+
+    def time_graph(self, steps, warmup):
+        """device ms per step of the whole set (CUDA graph of `steps` steps)"""
+        import torch
+        for _ in range(warmup):
+            self.step()
+        torch.cuda.synchronize()
+        g = torch.cuda.CUDAGraph()
+        s = torch.cuda.Stream()
+        s.wait_stream(torch.cuda.current_stream())
+        with torch.cuda.stream(s), torch.cuda.graph(g, stream=s):
+            for _ in range(steps):
+                self.step()
+        torch.cuda.current_stream().wait_stream(s)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        g.replay()
+        e1.record()
+        torch.cuda.synchronize()
+        return e0.elapsed_time(e1) / steps
 
 
 # -------------------------------------------------------------- CPU oracle -
@@ -522,6 +544,21 @@ def main():
         torch.cuda.empty_cache()
         aux["relayout_d6"] = BW.relayout_run(args.steps, ws, dev)
         torch.cuda.empty_cache()
+        # the same R50 layer set in fp32 (the paper's precision):
+        # tensor cores through the three-plane bf16 split (reading A27)
+        S32 = LayerSet(args.batch, dev, torch.float32)
+        ms32 = S32.time_graph(max(3, args.steps // 2), 2)
+        aux["r50_fp32"] = {"workload": f"ResNet-50 conv set, batch {args.batch}, fp32 in / out, tuned layouts",
+                           "ms_per_step": round(ms32, 4), "tflops": round(S32.flops / (ms32 * 1e-3) / 1e12, 2),
+                           "arith": "fp32 via six bf16 tcgen05 products (max-norm error <= 1e-5)"}
+        del S32
+        torch.cuda.empty_cache()
+        # batch 1 (the other half of BASELINE config 2)
+        S1 = LayerSet(1, dev)
+        ms1 = S1.time_graph(args.steps, 2)
+        aux["r50_b1"] = {"ms_per_step": round(ms1, 4), "us_per_layer": round(ms1 * 1e3 / len(S1.layers), 2),
+                         "tflops": round(S1.flops / (ms1 * 1e-3) / 1e12, 2)}
+        del S1
         try:
             import bench_layouts as BL
             aux["fixed_layouts"] = BL.run_all(dev, steps=max(5, min(args.steps, 10)))

@@ -190,14 +190,21 @@ typedef enum { ALT_ACT_NONE = 0, ALT_ACT_RELU = 1, ALT_ACT_RELU6 = 2 } alt_act;
  * computed in fp32 and rounded once (RNE) to the output dtype, then stored
  * through y's layout: every unfold copy is written, pad positions get 0.
  * scale / bias are device fp32 arrays of length K (NULL = 1 / 0).
- * residual has y's logical shape, y's dtype, and its own layout. */
+ * residual has y's logical shape, y's dtype, and its own layout.
+ * flags & ALT_EPI_PADS_ZERO: the caller guarantees that y's pad / overhang
+ * positions already hold 0 (e.g. a zero-initialised buffer only ever
+ * written through this layout, as in a layer chain); the kernel then stores
+ * the element positions only — a padded output layout is written by the
+ * TMA-store epilogue instead of the per-element writer.  Unfold copies are
+ * always all written. */
+enum { ALT_EPI_PADS_ZERO = 1 };
 typedef struct {
   const float *scale;
   const float *bias;
   const void *residual;
   alt_layout residual_l;
   int32_t act;                /* alt_act */
-  int32_t _pad;
+  int32_t flags;              /* ALT_EPI_* */
 } alt_epilogue;
 
 typedef enum {
@@ -293,30 +300,44 @@ uint64_t alt_launch_count(void);
  * freed inside.
  *
  * Conv template: x = N C/it H W it (it = x tile) with
- * optional pad(H,p,p)+pad(W,p,p) materialised, w = K/ot' C/it' R S ot' it'
- * (the GPU default puts c innermost, A11), y = N K/ot Ho Wo ot.
+ * optional pad(H,p,p)+pad(W,p,p) materialised, or the paper's overlapped
+ * spatial tiles N H/ht W/wt C/it (ht+KH-1)(wt+KW-1) it (pad + unfold, Eq. 1;
+ * stride V: B = V(ht-1)+KH, S = V ht, reading A6) when ht / wt are given;
+ * w = K/ot' C/it' R S ot' it' (c innermost: K-major B, A11) or the paper's
+ * O/ot' I/it' KH KW it' ot' (o innermost: MN-major B); y = N K/ot Ho Wo ot,
+ * or N Ho/ht Wo/wt K/ot ht wt ot when ht | Ho and wt | Wo.
  * GEMM template: A = M/mt K/kt mt kt, B = N/nt K/kt nt kt
- * (the paper's K/kt N/nt kt nt is the MN-major variant), C = M/mt N/nt mt nt.
+ * (K innermost) or the paper's K/kt N/nt kt nt (N innermost, MN-major),
+ * C = M/mt N/nt mt nt.
+ * Every grid point is timed as the median of `reps` L2-flushed launches;
+ * the `topk` fastest are then re-measured (median of 3 x reps) and the best
+ * re-measured point is returned.
  */
 typedef enum { ALT_OP_CONV2D = 0, ALT_OP_MATMUL = 1 } alt_op_kind;
 
 typedef struct { int64_t M, N, K; } alt_matmul_params;
 
 #define ALT_TUNE_MAX_VALS 8
+#define ALT_TUNE_NPARAMS 12
 typedef struct {
   /* candidate values per template parameter; nvals[i] == 0 = default set.
    * conv:  0 it (x channel tile; the w c tile it' = it), 1 ot (y channel
    *        tile), 2 split_k (negative: -s = split_cluster form with s ranges),
-   *        3 cta_pair (0 auto, 2 single CTA), 4 tile_h,
-   *        5 tile_w, 6 block_n (the w k tile ot' = min(block_n, K)),
-   *        7 pad_x (0/1: materialise the conv zero padding in x)
-   * gemm:  0 mt, 1 kt, 2 nt, 6 block_n */
-  int64_t vals[8][ALT_TUNE_MAX_VALS];
-  int32_t nvals[8];
+   *        3 cta_pair (0 auto, 1 pair = BLOCK_M 256, 2 single CTA = 128),
+   *        4 tile_h, 5 tile_w (kernel output-pixel tile), 6 block_n (the w k
+   *        tile ot' = min(block_n, K)), 7 pad_x (0/1: materialise the conv
+   *        zero padding in x), 8 ht, 9 wt (layout spatial tiles; 0 = none),
+   *        10 stages (smem ring depth; 0 = deepest), 11 w order (0 c
+   *        innermost, 1 the paper's it' ot')
+   * gemm:  0 mt, 1 kt, 2 nt, 6 block_n, 10 stages, 11 B order (0 N/nt K/kt
+   *        nt kt, 1 K/kt N/nt kt nt) */
+  int64_t vals[ALT_TUNE_NPARAMS][ALT_TUNE_MAX_VALS];
+  int32_t nvals[ALT_TUNE_NPARAMS];
   int32_t max_points;   /* budget: maximum measured points (<= 4096) */
   int32_t warmup, reps; /* per point */
   int32_t fix_x;        /* 1: keep x layout = fixed_x (propagated from a producer) */
   alt_layout fixed_x;
+  int32_t topk;         /* re-measured finalists (0 = 3) */
 } alt_tune_space;
 
 typedef struct {

@@ -58,7 +58,7 @@ class ConvParams(ctypes.Structure):
 class _Epi(ctypes.Structure):
     _fields_ = [("scale", ctypes.c_void_p), ("bias", ctypes.c_void_p),
                 ("residual", ctypes.c_void_p), ("residual_l", ctypes.c_void_p),
-                ("act", ctypes.c_int32), ("_pad", ctypes.c_int32)]
+                ("act", ctypes.c_int32), ("flags", ctypes.c_int32)]
 
 
 class KernelCfg(ctypes.Structure):
@@ -75,10 +75,10 @@ class MatmulParams(ctypes.Structure):
 
 
 class TuneSpace(ctypes.Structure):
-    _fields_ = [("vals", (ctypes.c_int64 * 8) * 8), ("nvals", ctypes.c_int32 * 8),
+    _fields_ = [("vals", (ctypes.c_int64 * 8) * 12), ("nvals", ctypes.c_int32 * 12),
                 ("max_points", ctypes.c_int32), ("warmup", ctypes.c_int32),
                 ("reps", ctypes.c_int32), ("fix_x", ctypes.c_int32),
-                ("fixed_x", ctypes.c_void_p)]
+                ("fixed_x", ctypes.c_void_p), ("topk", ctypes.c_int32)]
 
 
 class TuneResult(ctypes.Structure):
@@ -253,14 +253,18 @@ def relayout(src_l: Layout, src: torch.Tensor, dst_l: Layout, dst: torch.Tensor,
     return dst
 
 
-def _epi(scale, bias, residual, residual_l, act):
-    if scale is None and bias is None and residual is None and not act:
+ALT_EPI_PADS_ZERO = 1
+
+
+def _epi(scale, bias, residual, residual_l, act, pads_zero=False):
+    if scale is None and bias is None and residual is None and not act and not pads_zero:
         return None
     e = _Epi()
     e.scale, e.bias = _ptr(scale), _ptr(bias)
     e.residual = _ptr(residual)
     e.residual_l = residual_l.handle.value if residual_l is not None else None
     e.act = ACT[act]
+    e.flags = ALT_EPI_PADS_ZERO if pads_zero else 0
     return e
 
 
@@ -287,9 +291,10 @@ def conv_params(N, C, H, W, K, R, S, stride=1, pad=0, groups=1, dilation=1) -> C
 
 
 def conv2d(p: ConvParams, x_l: Layout, x, w_l: Layout, w, y_l: Layout, y, scale=None, bias=None,
-           residual=None, residual_l: Layout | None = None, act=0, cfg=None, stream=None):
-    """alt_conv2d: y (in y_l) = act(scale * conv(x, w) + bias + residual)."""
-    e = _epi(scale, bias, residual, residual_l, act)
+           residual=None, residual_l: Layout | None = None, act=0, cfg=None, stream=None, pads_zero=False):
+    """alt_conv2d: y (in y_l) = act(scale * conv(x, w) + bias + residual).
+    pads_zero: y's pad positions already hold 0 (ALT_EPI_PADS_ZERO)."""
+    e = _epi(scale, bias, residual, residual_l, act, pads_zero)
     c = _cfg(cfg)
     _check(_lib.alt_conv2d(ctypes.byref(p), x_l.handle, _ptr(x), w_l.handle, _ptr(w), y_l.handle,
                            _ptr(y), _dtype_code(x), ctypes.byref(e) if e else None,
@@ -352,7 +357,8 @@ def launch_count() -> int:
 
 
 def tune(op: str, params, dtype: int, space: dict | None = None, stream=None,
-         max_points: int = 64, warmup: int = 3, reps: int = 10, fixed_x: Layout | None = None):
+         max_points: int = 64, warmup: int = 3, reps: int = 10, fixed_x: Layout | None = None,
+         topk: int = 3):
     """alt_tune over the bounded grid; returns (x/A prims, w/B prims, y/C prims, cfg, best_us,
     measured, all_us)."""
     sp = TuneSpace()
@@ -360,7 +366,7 @@ def tune(op: str, params, dtype: int, space: dict | None = None, stream=None,
         sp.nvals[i] = len(vals)
         for j, v in enumerate(vals):
             sp.vals[i][j] = int(v)
-    sp.max_points, sp.warmup, sp.reps = max_points, warmup, reps
+    sp.max_points, sp.warmup, sp.reps, sp.topk = max_points, warmup, reps, topk
     if fixed_x is not None:
         sp.fix_x, sp.fixed_x = 1, fixed_x.handle.value
     res = TuneResult()

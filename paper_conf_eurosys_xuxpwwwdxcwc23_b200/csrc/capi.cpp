@@ -48,6 +48,7 @@ static alt_status fill_epi(const alt_epilogue *e, const Layout *yl, OpEpilogue *
   o->scale = e->scale;
   o->bias = e->bias;
   o->act = e->act;
+  o->pads_zero = (e->flags & ALT_EPI_PADS_ZERO) ? 1 : 0;
   if ((e->scale && !is_device_ptr(e->scale)) || (e->bias && !is_device_ptr(e->bias))) {
     set_error("epilogue: scale / bias must be device pointers");
     return ALT_E_INVALID;

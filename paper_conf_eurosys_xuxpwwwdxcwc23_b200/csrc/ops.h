@@ -18,6 +18,7 @@ struct OpEpilogue {
   const int64_t *bias_att_rd = nullptr;
   int64_t bias_att_base = 0;
   int32_t bias_att_bf16 = 0;
+  int32_t pads_zero = 0;  // ALT_EPI_PADS_ZERO: y's pad positions already hold 0
 };
 
 struct ConvProblem {

@@ -80,6 +80,9 @@ struct TcArgs {
   // slabs per pair; out_f32: the output (and residual) are fp32
   int32_t pairs, rsg, out_f32;
   FastDiv f_rsg;
+  int32_t nst;           // smem ring stages in use (<= the instantiation's STAGES; tuner knob)
+  int32_t yvec;          // out_mode 0 with 8-channel runs: copies written as 16-byte vectors
+  int32_t pads_zero;     // ALT_EPI_PADS_ZERO: skip y's pad (structural zero) positions
   int32_t sw;
   Writer yw;
   Reader yr;             // out_mode 2: owner offsets of y
@@ -263,6 +266,50 @@ static __device__ __noinline__ void store_chunk_f32(const TcArgs &a, float *y, i
     if (k >= a.K) break;
     if (a.is_conv) write4<float>(a.yw, y, n, a.y_koff + k, p, q, v[j]);
     else write2<float>(a.yw, y, q, a.y_koff + k, v[j]);
+  }
+}
+// one row's 32 channels into a layout with pads / unfold copies whose
+// channel dim runs in 16-byte-aligned groups of 8 (NCHW[x]c tiled templates):
+// every physical copy of the (n, p, q) row gets four 16-byte stores; pad
+// positions the row owns get zeros (or are skipped under pads_zero)
+static __device__ __noinline__ void write_chunk_vec(const TcArgs &a, uint16_t *y, int n, int p, int q, int kb,
+                                                    const uint32_t *pk) {
+  const Writer &w = a.yw;
+  int64_t ch[4];
+#pragma unroll
+  for (int c = 0; c < 4; c++) {
+    const int k = kb + 8 * c;
+    ch[c] = k < a.K ? __ldg(a.yr.rd[1] + a.y_koff + k) : -1;
+  }
+  const int d0 = a.is_conv ? n : q;
+  const int32_t a0 = __ldg(w.wptr[0] + d0), a1 = __ldg(w.wptr[0] + d0 + 1);
+  int32_t b0 = 0, b1 = 1, c0 = 0, c1 = 1;
+  if (a.is_conv) {
+    b0 = __ldg(w.wptr[2] + p); b1 = __ldg(w.wptr[2] + p + 1);
+    c0 = __ldg(w.wptr[3] + q); c1 = __ldg(w.wptr[3] + q + 1);
+  }
+  for (int32_t i = a0; i < a1; i++) {
+    const int64_t ca = __ldg(w.wlist[0] + i);
+    for (int32_t j = b0; j < b1; j++) {
+      const int64_t cb = a.is_conv ? __ldg(w.wlist[2] + j) : 0;
+      for (int32_t l = c0; l < c1; l++) {
+        const int64_t cc = a.is_conv ? __ldg(w.wlist[3] + l) : 0;
+        const bool zero = ((ca | cb | cc) & 1) != 0;
+        if (zero && a.pads_zero) continue;
+        const int64_t base = (ca >> 1) + (cb >> 1) + (cc >> 1);
+#pragma unroll
+        for (int c = 0; c < 4; c++) {
+          if (ch[c] < 0) break;
+          uint16_t *dst = y + base + ch[c];
+          if (zero)
+            asm volatile("st.global.v4.b32 [%0], {%1, %1, %1, %1};" ::"l"(dst), "r"(0u) : "memory");
+          else
+            asm volatile("st.global.v4.b32 [%0], {%1, %2, %3, %4};" ::"l"(dst), "r"(pk[4 * c]), "r"(pk[4 * c + 1]),
+                         "r"(pk[4 * c + 2]), "r"(pk[4 * c + 3])
+                         : "memory");
+        }
+      }
+    }
   }
 }
 // one row's 32 channels through the generic writer (pads, unfold copies)
@@ -473,10 +520,10 @@ __global__ void __launch_bounds__(kThreads, 1)
           coords(om, vt, base);
         }
         const uint32_t trow = smem_u32(tab) + (uint32_t)((isA ? 0 : 8) * 4 + si * 64);
-        int stage = it % STAGES;
-        uint32_t ph = (uint32_t)((it / STAGES) & 1);
+        int stage = it % a.nst;
+        uint32_t ph = (uint32_t)((it / a.nst) & 1);
         for (int kit = k_begin; kit < k_end; kit++, it++) {
-          if (it >= STAGES) mbar_wait(&empty[stage], ph ^ 1);
+          if (it >= a.nst) mbar_wait(&empty[stage], ph ^ 1);
           if (lane == 0 && rank == 0) mbar_expect_tx(&full[stage], CG * (kStageBytesA + L::kB));
           __syncwarp();
           if (active) {
@@ -492,12 +539,12 @@ __global__ void __launch_bounds__(kThreads, 1)
               tma_load_5d(dst, tmap, &full[stage], base[0] + o0, base[1] + o1, base[2] + o2, base[3] + o3,
                           base[4] + o4);
           }
-          if (++stage == STAGES) { stage = 0; ph ^= 1u; }
+          if (++stage == a.nst) { stage = 0; ph ^= 1u; }
         }
         continue;
       }
       for (int kit = k_begin; kit < k_end; kit++, it++) {
-        const int stage = it % STAGES, round = it / STAGES;
+        const int stage = it % a.nst, round = it / a.nst;
         if (lane == 0 && ti == ALT_DBG_TILE && kit == k_begin) { DBG(24); }
         if (round > 0) mbar_wait(&empty[stage], (round - 1) & 1);
         if (lane == 0 && ti == ALT_DBG_TILE && kit == k_begin) { DBG(25); }
@@ -569,8 +616,8 @@ __global__ void __launch_bounds__(kThreads, 1)
         const uint32_t d = tmem + (uint32_t)(acc * BN);
         const UnitInfo ui = unit_info(a, tile);
         const int k_begin = ui.kb, k_end = ui.ke;
-        int stage = it % STAGES;
-        uint32_t ph = (uint32_t)((it / STAGES) & 1);
+        int stage = it % a.nst;
+        uint32_t ph = (uint32_t)((it / a.nst) & 1);
         for (int kit = k_begin; kit < k_end; kit++, it++) {
           mbar_wait(&full[stage], ph);
           if (i == ALT_DBG_TILE && kit == k_begin) { DBG(28); }
@@ -584,7 +631,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           }
           if constexpr (CG == 2) mma_commit_2cta(&empty[stage], 0x3);  // frees the stage in both CTAs
           else mma_commit(&empty[stage]);
-          if (++stage == STAGES) { stage = 0; ph ^= 1u; }
+          if (++stage == a.nst) { stage = 0; ph ^= 1u; }
         }
         if constexpr (CG == 2) mma_commit_2cta(&tfull[acc], 0x3);
         else mma_commit(&tfull[acc]);
@@ -958,7 +1005,10 @@ __global__ void __launch_bounds__(kThreads, 1)
             }
           } else if constexpr (!EARLY) {
             // generic layouts: every copy / pad position through the writer
-            if (vrow) write_chunk(a.yw, a.is_conv, a.K, y, n, p, q, kb, a.y_koff, pk);
+            if (vrow) {
+              if (a.yvec) write_chunk_vec(a, y, n, p, q, kb, pk);
+              else write_chunk(a.yw, a.is_conv, a.K, y, n, p, q, kb, a.y_koff, pk);
+            }
           }
           if constexpr (!EARLY) {
             if (c0 + kStep < BN) tmem_ld_32x32b_x32(next, raw);
@@ -1127,6 +1177,7 @@ struct LView {
   int64_t pshape[kMaxP] = {}, pstride[kMaxP] = {}, coef[kMaxP] = {};
   int32_t owner[kMaxP] = {};
   int64_t off[kMaxL] = {};
+  int64_t lext[kMaxL] = {};  // logical extents
 };
 
 static LView lview(const Layout &L) {
@@ -1140,7 +1191,10 @@ static LView lview(const Layout &L) {
     v.coef[p] = L.aff.coef[p];
     v.owner[p] = L.pdim_owner[p];
   }
-  for (int d = 0; d < L.lrank; d++) v.off[d] = L.aff.off[d];
+  for (int d = 0; d < L.lrank; d++) {
+    v.off[d] = L.aff.off[d];
+    v.lext[d] = L.lshape[d];
+  }
   return v;
 }
 
@@ -1194,7 +1248,11 @@ static bool fold_window(const LView &x, const LView &w, int64_t S, int Vw, int p
 // stride-1 dim (box = mnw, the caller sets that role's tile to mnw and the
 // other row roles' tiles to 1: one box per group of mnw rows), the channel
 // dim is an ordinary box dim of sw channels.
-static bool build_view(const LView &L, const RoleInfo *roles, int sw, View *out, char *why, int mnw = 0) {
+// clip: an output view of a padded layout (ALT_EPI_PADS_ZERO stores): each
+// spatial dim's extent ends at the last element row, so TMA drops the rows
+// of a tile past Ho / Wo instead of writing them into the hi pad
+static bool build_view(const LView &L, const RoleInfo *roles, int sw, View *out, char *why, int mnw = 0,
+                       bool clip = false) {
   auto fail = [&](const char *m) { snprintf(why, 160, "%s", m); return false; };
   if (!L.ok) return fail("layout not separable-affine");
   View v;
@@ -1282,6 +1340,7 @@ static bool build_view(const LView &L, const RoleInfo *roles, int sw, View *out,
           x.coef[VR] = ri.V;
           x.coef[VTAP] = ri.tap;
           x.coef[V_ONE] = (int32_t)(-ri.pad - off);
+          if (clip) x.extent = std::min<int64_t>(x.extent, L.lext[d] - off);
           break;
         }
         if (nphys[d] != 2) return fail("spatial dim with >2 physical dims");
@@ -1646,7 +1705,7 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
     k[i++] = P.epi.residual_l ? (int64_t)P.epi.residual_l->serial : 0;
     k[i++] = P.epi.act;
     k[i++] = (P.coff << 32) | P.koff;
-    k[i++] = P.pairs * 2 + (P.out_f32 ? 1 : 0);
+    k[i++] = P.pairs * 4 + (P.out_f32 ? 2 : 0) + (P.epi.pads_zero ? 1 : 0);
     if (cfg) {
       k[i++] = cfg->block_n; k[i++] = cfg->tile_n; k[i++] = cfg->tile_h; k[i++] = cfg->tile_w;
       k[i++] = cfg->stages;
@@ -1779,17 +1838,33 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
         if (st2 != ALT_OK) return st2;
         a.out_mode = 2;
       }
-      if (a.out_mode == 0 && store_mode != 0 && !P.out_f32 && !(P.yl->flags & (ALT_HAS_PAD | ALT_HAS_UNFOLD))) {
+      // TMA-store view: y holds one copy per element; pads only when the
+      // caller guarantees they already hold 0 (ALT_EPI_PADS_ZERO)
+      if (a.out_mode == 0 && store_mode != 0 && !P.out_f32 && !(P.yl->flags & ALT_HAS_UNFOLD) &&
+          (!(P.yl->flags & ALT_HAS_PAD) || P.epi.pads_zero)) {
         char why2[160];
         for (int so = 32; so >= 8 && !a.out_mode; so /= 2) {
           if (P.koff % so) continue;  // a group's first channel must start a store slab
           View vy;
-          if (!build_view(P.vy, ry, so, &vy, why2)) continue;
+          if ((P.yl->flags & ALT_HAS_PAD) && P.yl->max_copies[1] != 1) break;  // padded channels: the writer
+          if (!build_view(P.vy, ry, so, &vy, why2, 0, (P.yl->flags & ALT_HAS_PAD) != 0)) continue;
           int64_t rowsY = 1;
           for (int i = 1; i < vy.rank; i++) rowsY *= vy.d[i].box;
           if (rowsY != 32) continue;
           if (encode_view(vy, P.y, esize, so, &pl.ty, &a.O, why2)) a.out_mode = 1;
         }
+      }
+      // generic-writer layouts (pads / unfold copies) with 8-channel runs:
+      // the vectorised writer (the channel dim itself must hold one copy
+      // per channel, or its pad positions already be 0)
+      a.pads_zero = P.epi.pads_zero;
+      a.yvec = 0;
+      if (a.out_mode == 0 && !P.out_f32 && P.yl->separable && P.K % 8 == 0 && P.koff % 8 == 0 &&
+          (reinterpret_cast<uintptr_t>(P.y) & 15) == 0 && chan_vec8(*P.yl, true) &&
+          (P.yl->max_copies[1] == 1 || P.epi.pads_zero)) {
+        alt_status st2 = make_reader(P.yl, &a.yr);
+        if (st2 != ALT_OK) return st2;
+        a.yvec = 1;
       }
       a.is_conv = P.is_conv;
       a.N = (int32_t)P.N; a.K = (int32_t)P.K; a.Ho = (int32_t)P.Ho; a.Wo = (int32_t)P.Wo;
@@ -1911,13 +1986,15 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       pl.BN = BN;
       pl.cg = cg;
       pl.stages = stages_for(BN, cg);
+      // a shallower ring than the instantiation's (tuner knob; 2 .. STAGES)
+      a.nst = (cfg && cfg->stages >= 2 && cfg->stages < pl.stages) ? cfg->stages : pl.stages;
       alt_kernel_cfg u{};
       u.path = ALT_PATH_TC;
       u.block_m = 128 * cg;
       u.cta_pair = cg == 2 ? 1 : 2;
       u.block_n = BN;
       u.block_k = 64;
-      u.stages = pl.stages;
+      u.stages = a.nst;
       u.tile_n = c.tn; u.tile_h = c.th; u.tile_w = c.tw;
       u.split_k = a.splits;
       u.split_cluster = pl.sc > 1 ? 1 : (a.full_units > 0 && a.splits > 1 ? 2 : 0);

@@ -90,14 +90,60 @@ def test_pool_parity(kind):
         assert norm_rel(got, ref) <= 4e-3
 
 
+def _check_tuned_conv(p, N, C, H, K, R, pad, res, stride=1):
+    """the tuner's winner: a valid layout pair whose conv is oracle-exact"""
+    x = synth.activations("tunex", (N, C, H, H))
+    w = synth.weights("tunew", (K, C, R, R))
+    Ho = (H + 2 * pad - R) // stride + 1
+    Ox, xph, xd = make_operand("tunex", res["x"], x, torch.bfloat16)
+    Ow, wph, wd = make_operand("tunew", res["w"], w, torch.bfloat16)
+    Ly = alt.Layout((N, K, Ho, Ho), res["y"])
+    y = torch.zeros(Ly.phys_shape, dtype=torch.bfloat16, device="cuda")
+    alt.conv2d(p, alt.Layout(x.shape, res["x"]), xd, alt.Layout(w.shape, res["w"]), wd, Ly, y, cfg=res["cfg"])
+    torch.cuda.synchronize()
+    ref = oracle.conv2d(dict(N=N, C=C, H=H, W=H, K=K, R=R, S=R, pad_h=pad, pad_w=pad, stride_h=stride,
+                             stride_w=stride), Ox, xph, Ow, wph)
+    got = read_output(oracle.Layout((N, K, Ho, Ho), res["y"]), y, torch.bfloat16)
+    assert norm_rel(got, ref) <= BF16_TOL
+
+
+@pytest.mark.parametrize("space", [
+    {8: [7], 9: [7]},                         # overlapped input tiles + tiled output (ht = wt = 7)
+    {8: [14], 9: [2]},
+    {11: [1]},                                # the paper's weight order it' ot' (MN-major B)
+    {10: [3], 3: [1]},                        # 3-stage ring, BLOCK_M 256
+    {8: [7, 0], 9: [7, 0], 11: [0, 1], 10: [0, 4], 3: [0, 2]},   # mixed grid
+], ids=["ht7wt7", "ht14wt2", "paper-w", "stages3-bm256", "mixed"])
+def test_tune_conv_template_knobs(space):
+    """the widened grid: spatial layout tiles, the
+    paper's weight order, BLOCK_M and ring stages; every returned winner is
+    a valid layout pair whose conv is oracle-exact"""
+    p = alt.conv_params(4, 64, 14, 14, 128, 3, 3, 1, 1)
+    sp = {0: [64], 1: [64], 6: [128]}
+    sp.update(space)
+    res = alt.tune("conv2d", p, alt.ALT_BF16, sp, max_points=32, warmup=1, reps=3)
+    assert res["measured"] >= 1 and res["best_us"] > 0
+    if 8 in space and space[8][0]:
+        assert any(q[0] == "unfold" for q in res["x"]) or len(space[8]) > 1
+    _check_tuned_conv(p, 4, 64, 14, 128, 3, 1, res)
+
+
+def test_tune_conv_strided_spatial_template():
+    p = alt.conv_params(2, 64, 28, 28, 128, 3, 3, 2, 1)
+    res = alt.tune("conv2d", p, alt.ALT_BF16, {0: [64], 1: [64], 6: [128], 8: [7], 9: [7]}, max_points=4,
+                   warmup=1, reps=3)
+    _check_tuned_conv(p, 2, 64, 28, 128, 3, 1, res, stride=2)
+
+
 def test_tune_conv_small():
     """alt_tune (bounded grid, parity unpinned A19): the winner is a valid
-    layout pair whose conv is oracle-exact."""
+    layout pair whose conv is oracle-exact; the returned time is the
+    re-measured median of a finalist."""
     p = alt.conv_params(4, 64, 14, 14, 128, 3, 3, 1, 1)
     res = alt.tune("conv2d", p, alt.ALT_BF16, {0: [64, 32], 1: [64], 6: [128, 256]}, max_points=8,
                    warmup=1, reps=3)
     assert res["measured"] >= 2 and res["best_us"] > 0
-    assert all(t >= res["best_us"] for t in res["all_us"])
+    assert res["best_us"] <= 2.0 * min(res["all_us"])
     x = synth.activations("tunex", (4, 64, 14, 14))
     w = synth.weights("tunew", (128, 64, 3, 3))
     Ox, xph, xd = make_operand("tunex", res["x"], x, torch.bfloat16)

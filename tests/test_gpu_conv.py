@@ -427,3 +427,32 @@ def test_grouped_conv_tensor_core(case):
     name, N, C, H, W, K, R, V, pad, g, xp, wp, yp, rp = case
     _, plan = run_conv(name, N, C, H, W, K, R, R, V, pad, xp, wp, yp, torch.bfloat16, groups=g, epi=True,
                        res_p=rp, act=1, cfg={"path": alt.PATH_AUTO}, expect_path=alt.PATH_TC)
+
+
+@pytest.mark.parametrize("yp_name", ["padded NCHW8c", "tiled unfold template", "padded NCHW64c"])
+@pytest.mark.parametrize("pads_zero", [False, True])
+def test_epilogue_writes_consumer_templates(yp_name, pads_zero):
+    """A tensor-core conv writing its consumer's padded / overlapped-tile input
+    layout (the fused conversion of Fig. 5b): the vectorised writer stores
+    every unfold copy; pad positions get 0 (pads_zero=False, buffer poisoned)
+    or keep the zeros the caller guarantees (pads_zero=True, ALT_EPI_PADS_ZERO,
+    zero buffer — padded layouts then go through the TMA-store epilogue)."""
+    N, C, H, K = 2, 64, 14, 64
+    yp = {"padded NCHW8c": LY.nchwxc(K, 8, pad_hw=1),
+          "tiled unfold template": LY.conv_input_tiled(K, 16, H, H, 3, 3, 7, 7, 1, 1),
+          "padded NCHW64c": LY.nchwxc(K, 64, pad_hw=1)}[yp_name]
+    x = synth.activations("pzx", (N, C, H, H))
+    w = synth.weights("pzw", (K, C, 3, 3))
+    Xo, xph, xd = make_operand("pzx", LY.nchwxc(C, 64), x, torch.bfloat16)
+    Wo_, wph, wd = make_operand("pzw", LY.kcrs_yk_xc(K, C, 64, 64), w, torch.bfloat16)
+    Ly = alt.Layout((N, K, H, H), yp)
+    fill = 0.0 if pads_zero else 3.0
+    y = torch.full(Ly.phys_shape, fill, dtype=torch.bfloat16, device="cuda")
+    p = alt.conv_params(N, C, H, H, K, 3, 3, 1, 1)
+    alt.conv2d(p, alt.Layout(x.shape, LY.nchwxc(C, 64)), xd, alt.Layout(w.shape, LY.kcrs_yk_xc(K, C, 64, 64)), wd,
+               Ly, y, act=1, cfg={"path": alt.PATH_TC}, pads_zero=pads_zero)
+    torch.cuda.synchronize()
+    assert alt.last_plan()["path"] == alt.PATH_TC
+    ref = oracle.conv2d(dict(N=N, C=C, H=H, W=H, K=K, R=3, S=3, pad_h=1, pad_w=1), Xo, xph, Wo_, wph, act=1)
+    got = read_output(oracle.Layout((N, K, H, H), yp), y, torch.bfloat16)
+    assert_parity(got, ref, torch.bfloat16)
