@@ -82,6 +82,8 @@ struct TcArgs {
   FastDiv f_rsg;
   int32_t nst;           // smem ring stages in use (<= the instantiation's STAGES; tuner knob)
   int32_t yvec;          // out_mode 0 with 8-channel runs: copies written as 16-byte vectors
+  int32_t out_round;     // out_mode 1, round stores: the 8 epilogue warps stage a whole 128-row x
+                         // 64-channel round in smem, one thread TMA-stores it (a.O views 128 rows)
   int32_t pads_zero;     // ALT_EPI_PADS_ZERO: skip y's pad (structural zero) positions
   int32_t sw;
   Writer yw;
@@ -682,7 +684,20 @@ __global__ void __launch_bounds__(kThreads, 1)
     uint32_t so[4];
 #pragma unroll
     for (int c = 0; c < 4; c++) so[c] = soff(c);
-    const int lg_sw = sw_o == 32 ? 5 : (sw_o == 16 ? 4 : 3);  // sw_o is 8, 16 or 32
+    // round stores: this thread's four 16-byte pieces in a 16 KB round buffer
+    // [64 / sw_o slabs][128 rows][sw_o channels], rows swizzled as the store box
+    if (a.out_round) {
+#pragma unroll
+      for (int c = 0; c < 4; c++) {
+        const int ch = half * 32 + c * 8;
+        uint32_t off = (uint32_t)(row * pitch + (ch & (sw_o - 1)) * 2);
+        off ^= ((off >> 7) & ((1u << swz) - 1u)) << 4;
+        so[c] = (uint32_t)((ch / sw_o) * 128 * pitch) + off;
+      }
+    }
+    const uint32_t rbase = smem_u32(sOut);
+    uint32_t round_ctr = 0;  // round-store buffer parity (across tiles)
+    const int lg_sw = sw_o == 64 ? 6 : (sw_o == 32 ? 5 : (sw_o == 16 ? 4 : 3));  // sw_o is 8 .. 64
     const int nslab = 32 >> lg_sw;
     int32_t ocg[5], ocr[5];  // store coordinates per channel slab (tile, in-tile)
     uint32_t sbuf_ctr = 0;   // TMA-store staging buffer parity (per warp, across tiles)
@@ -708,7 +723,9 @@ __global__ void __launch_bounds__(kThreads, 1)
       // computed while the MMA may still be running
       int32_t cbase[5] = {0, 0, 0, 0, 0};
       if (a.out_mode == 1 && lane == 0) {
-        const int sn = tc.n0 + sn0, sp = tc.p0 + sp0, sq = tc.q0 + sq0;
+        // round stores: the box is the whole tile (origin n0, p0, q0)
+        const int sn = tc.n0 + (a.out_round ? 0 : sn0), sp = tc.p0 + (a.out_round ? 0 : sp0),
+                  sq = tc.q0 + (a.out_round ? 0 : sq0);
         int32_t vo[NVAR];
         vo[V_N0] = sn;
         vo[V_PT] = (int)a.O.fp.div((uint32_t)sp); vo[V_PR] = sp - vo[V_PT] * a.O.divp;
@@ -969,6 +986,39 @@ __global__ void __launch_bounds__(kThreads, 1)
                                : "memory");
                 }
               }
+            }
+          } else if (a.out_mode == 1 && a.out_round) {
+            // Round store: every epilogue warp writes its 32 x 32 piece of the
+            // round's 128 x 64 block into one of two 16 KB buffers; thread 0
+            // then stores the block with one TMA store per channel slab.
+            // Buffer reuse: thread 0 waits (before the "free" barrier) until
+            // the store issued two rounds ago has read its buffer.
+            const uint32_t rbuf = rbase + (uint32_t)(round_ctr++ & 1u) * 16384u;
+            if (et == 0) bulk_wait_read1();
+            named_bar(3, kEpiThreads);
+#pragma unroll
+            for (int c = 0; c < 4; c++)
+              asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(rbuf + so[c]), "r"(pk[4 * c]),
+                           "r"(pk[4 * c + 1]), "r"(pk[4 * c + 2]), "r"(pk[4 * c + 3])
+                           : "memory");
+            fence_async_smem();
+            named_bar(4, kEpiThreads);
+            if (et == 0) {
+              const int kr = tc.k0 + c0;  // the round's first channel
+              for (int j = 0; j < (64 >> lg_sw); j++) {
+                if (kr + (j << lg_sw) >= a.K) break;
+                const int g = ((kr + a.y_koff) >> lg_sw) + j;
+                const int gt = (int)a.O.fg.div((uint32_t)g), gr = g - gt * a.O.divg;
+                int32_t co[5];
+#pragma unroll
+                for (int d = 0; d < 5; d++) co[d] = cbase[d] + ocg[d] * gt + ocr[d] * gr;
+                asm volatile(
+                    "cp.async.bulk.tensor.5d.global.shared::cta.tile.bulk_group [%0, {%2, %3, %4, %5, %6}], [%1];" ::"l"(
+                        reinterpret_cast<uint64_t>(&tmY)),
+                    "r"(rbuf + (uint32_t)(j * 128 * pitch)), "r"(co[0]), "r"(co[1]), "r"(co[2]), "r"(co[3]), "r"(co[4])
+                    : "memory");
+              }
+              bulk_commit();
             }
           } else if (a.out_mode == 1) {
             // Each warp stores its own 32-row x 32-channel sub-tile: private
@@ -1843,6 +1893,27 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       if (a.out_mode == 0 && store_mode != 0 && !P.out_f32 && !(P.yl->flags & ALT_HAS_UNFOLD) &&
           (!(P.yl->flags & ALT_HAS_PAD) || P.epi.pads_zero)) {
         char why2[160];
+        // round stores (one 128-row box per channel slab and round) unless a
+        // split-K / cluster form is requested (their epilogues skip rounds)
+        static const bool rounds_on = [] { const char *e = getenv("ALT_TC_ROUND"); return !(e && e[0] == '0'); }();
+        const bool want_round = rounds_on && !(cfg && (cfg->split_k > 1 || cfg->split_cluster)) && kEpiWarps == 8;
+        for (int so = 64; so >= 8 && want_round && !a.out_mode; so /= 2) {
+          if (P.koff % so) continue;
+          if ((P.yl->flags & ALT_HAS_PAD) && P.yl->max_copies[1] != 1) break;
+          RoleInfo rr[kMaxL];
+          memcpy(rr, ry, sizeof(rr));
+          for (int d = 0; d < kMaxL; d++) {
+            if (rr[d].role == R_N) rr[d].tile = c.tn;
+            if (rr[d].role == R_H) rr[d].tile = c.th;
+            if (rr[d].role == R_W) rr[d].tile = c.tw;
+          }
+          View vy;
+          if (!build_view(P.vy, rr, so, &vy, why2, 0, (P.yl->flags & ALT_HAS_PAD) != 0)) continue;
+          int64_t rowsY = 1;
+          for (int i = 1; i < vy.rank; i++) rowsY *= vy.d[i].box;
+          if (rowsY != 128) continue;
+          if (encode_view(vy, P.y, esize, so, &pl.ty, &a.O, why2)) { a.out_mode = 1; a.out_round = 1; }
+        }
         for (int so = 32; so >= 8 && !a.out_mode; so /= 2) {
           if (P.koff % so) continue;  // a group's first channel must start a store slab
           View vy;

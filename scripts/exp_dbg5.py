@@ -35,6 +35,9 @@ for name in sys.argv[1].split(","):
     buf = np.zeros(ncta * 40, np.uint64)
     lib.alt__debug_tc(buf.ctypes.data, ncta * 40)
     t = buf.reshape(ncta, 40).astype(np.int64)
+    # only the CTAs of the last launch (slots of unused CTAs hold older stamps)
+    last = t[:, 0].max()
+    t = t[t[:, 0] > last - 200_000]
     t0 = t[:, 0][t[:, 0] > 0].min()
     rel = np.where(t > 0, (t - t0) / 1000.0, np.nan)
     print(name, alt.last_plan())

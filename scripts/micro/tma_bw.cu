@@ -54,7 +54,30 @@ __global__ void __launch_bounds__(64, 1) k_tma(const __grid_constant__ CUtensorM
   }
   __syncthreads();
   unsigned long long t0 = clock64();
-  if (MODE == 6) {
+  if (MODE == 7 || MODE == 8) {
+    // one box per lane: lanes 0 .. loads-1 of warp 0 issue the boxes of a
+    // stage concurrently (the conv kernel's producer pattern)
+    if (warp == 0) {
+      int stage = 0; uint32_t ph = 0;
+      for (int it = 0; it < iters; it++) {
+        if (it >= STAGES) mbar_wait(&empty[stage], ph ^ 1);
+        if (lane == 0) mbar_expect_tx(&full[stage], sbytes);
+        __syncwarp();
+        const int32_t cc = ((blockIdx.x * 37 + it * p.loads + lane) & 63);
+        if (lane < p.loads)
+          tma_load_5d(smem + stage * sbytes + lane * p.box_bytes, &tm, &full[stage], 0,
+                      MODE == 7 ? cc * p.step[1] : 0, MODE == 8 ? cc * p.step[2] : 0, 0, 0);
+        if (++stage == STAGES) { stage = 0; ph ^= 1; }
+      }
+    } else if (warp == 1 && lane == 0) {
+      int stage = 0; uint32_t ph = 0;
+      for (int it = 0; it < iters; it++) {
+        mbar_wait(&full[stage], ph);
+        mbar_arrive(&empty[stage]);
+        if (++stage == STAGES) { stage = 0; ph ^= 1; }
+      }
+    }
+  } else if (MODE == 6) {
     if (warp == 0 && lane == 0) {
       int stage = 0; uint32_t ph = 0;
       for (int it = 0; it < iters; it++) {
@@ -150,13 +173,13 @@ int main() {
   cudaMemset(buf, 0, big);
   unsigned long long *cyc;
   cudaMalloc(&cyc, 4 * nsm * sizeof(unsigned long long));
-  for (auto f : {k_tma<0>, k_tma<1>, k_tma<2>, k_tma<3>, k_tma<4>, k_tma<5>, k_tma<6>}) if (cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, 210 * 1024) != cudaSuccess) printf("attr failed\n");
+  for (auto f : {k_tma<0>, k_tma<1>, k_tma<2>, k_tma<3>, k_tma<4>, k_tma<5>, k_tma<6>, k_tma<7>, k_tma<8>}) if (cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, 210 * 1024) != cudaSuccess) printf("attr failed\n");
   cudaEvent_t e0, e1;
   cudaEventCreate(&e0);
   cudaEventCreate(&e1);
   auto run = [&](const char *name, std::vector<uint64_t> dims, std::vector<uint32_t> box, Pat p, int ctas_per_sm, int mode = 0) {
     CUtensorMap tm = make_map(buf, dims, box, 128, {}, (mode == 1 || mode == 3) ? 2 : 5);
-    auto kern = mode == 0 ? k_tma<0> : mode == 1 ? k_tma<1> : mode == 2 ? k_tma<2> : mode == 3 ? k_tma<3> : mode == 4 ? k_tma<4> : mode == 5 ? k_tma<5> : k_tma<6>;
+    auto kern = mode == 0 ? k_tma<0> : mode == 1 ? k_tma<1> : mode == 2 ? k_tma<2> : mode == 3 ? k_tma<3> : mode == 4 ? k_tma<4> : mode == 5 ? k_tma<5> : mode == 6 ? k_tma<6> : mode == 7 ? k_tma<7> : k_tma<8>;
     const int iters = 2048;
     const int smem = p.stages * p.box_bytes * p.loads + 1024;
     const int grid = nsm * ctas_per_sm;
@@ -173,7 +196,30 @@ int main() {
     printf("mode %d %-44s box %5d B x%d, %2d st, %d CTA/SM: %8.1f GB/s %6.1f B/clk/SM@1.965\n", mode, name, p.box_bytes, p.loads,
            p.stages, ctas_per_sm, bytes / ms / 1e6, bytes / ms / 1e6 / nsm / 1.965);
   };
-  for (int mode : {2, 6}) {
+  {
+    uint64_t R = (uint64_t)1 << 22;
+    // concurrent lanes: (rows per box, boxes per stage, stages)
+    int cfgs[][3] = {{128, 1, 6}, {128, 2, 4}, {64, 2, 6}, {32, 4, 6}, {16, 8, 6}, {128, 3, 3}, {64, 4, 4},
+                     {32, 8, 4}, {128, 4, 3}, {256, 1, 4}, {256, 2, 3}};
+    for (auto &c : cfgs) {
+      Pat p = {2, c[0] * 128, {1, (int32_t)(R / c[0])}, {0, c[0]}, c[1], c[2]};
+      run("2D [R][64] concurrent lanes", {64, R}, {64, (uint32_t)c[0]}, p, 1, 7);
+    }
+  }
+  {
+    // conv-like scattered A boxes: [R][14 pixels][64 ch]; box {64, w, g}: g
+    // segments of w pixels (w*128 B contiguous) 1792 B apart
+    uint64_t R = (uint64_t)1 << 18;
+    int cfgs[][4] = {{4, 32, 1, 5}, {4, 16, 2, 5}, {4, 8, 4, 5}, {8, 16, 1, 5}, {8, 8, 2, 5}, {14, 8, 1, 5},
+                     {14, 4, 2, 5}, {4, 32, 2, 3}};
+    for (auto &c : cfgs) {
+      Pat p = {3, c[0] * c[1] * 128, {1, 1, 64}, {0, 0, c[1]}, c[2], c[3]};
+      char nm[64];
+      snprintf(nm, 64, "3D scattered seg %d px x %d", c[0], c[1]);
+      run(nm, {64, 14, R}, {64, (uint32_t)c[0], (uint32_t)c[1]}, p, 1, 8);
+    }
+  }
+  for (int mode : {6}) {
     uint64_t R = (uint64_t)1 << 22;
     for (int rows : {64, 128, 256}) for (int st : {2, 4, 8}) {
       if (st * rows * 128 > 200 * 1024) continue;
