@@ -165,8 +165,13 @@ class LayerSet:
             sc = synth.bn_scale("r50s" + L.name, L.K).to(dev)
             bi = synth.bn_bias("r50b" + L.name, L.K).to(dev)
             p = alt.conv_params(N, L.C, L.H, L.W, L.K, L.R, L.S, L.stride, L.pad)
+            cfg = pl["cfg"]
+            if dtype == torch.float32:
+                # fp32 (split-plane) path: fp32 epilogue stores, so no cluster /
+                # tail split-K forms (bf16 TMA-store epilogues); tiles / BLOCK_N kept
+                cfg = {k: v for k, v in cfg.items() if k not in ("split_k", "split_cluster")}
             self.layers.append(dict(L=L, p=p, lx0=lx0, lx=lx, lw=lw, ly=ly, x=xt, w=wt, y=yt, sc=sc,
-                                    bi=bi, cfg=pl["cfg"], x_host=x0.pin_memory(), x0d=x0d,
+                                    bi=bi, cfg=cfg, x_host=x0.pin_memory(), x0d=x0d,
                                     y_host=torch.empty(yt.shape, dtype=dtype).pin_memory()))
         self.flops = sum(l["L"].flops(N) for l in self.layers)
         self.alg_bytes = sum(l["L"].min_bytes(N) for l in self.layers)

@@ -318,7 +318,7 @@ typedef enum { ALT_OP_CONV2D = 0, ALT_OP_MATMUL = 1 } alt_op_kind;
 typedef struct { int64_t M, N, K; } alt_matmul_params;
 
 #define ALT_TUNE_MAX_VALS 8
-#define ALT_TUNE_NPARAMS 12
+#define ALT_TUNE_NPARAMS 15
 typedef struct {
   /* candidate values per template parameter; nvals[i] == 0 = default set.
    * conv:  0 it (x channel tile; the w c tile it' = it), 1 ot (y channel
@@ -328,7 +328,9 @@ typedef struct {
    *        tile ot' = min(block_n, K)), 7 pad_x (0/1: materialise the conv
    *        zero padding in x), 8 ht, 9 wt (layout spatial tiles; 0 = none),
    *        10 stages (smem ring depth; 0 = deepest), 11 w order (0 c
-   *        innermost, 1 the paper's it' ot')
+   *        innermost, 1 the paper's it' ot'), 12 h't, 13 w't, 14 o't: the
+   *        two-level output template N H/(h't ht) W/(w't wt) K/(o't ot)
+   *        h't w't o't ht wt ot (0 or 1 = one level)
    * gemm:  0 mt, 1 kt, 2 nt, 6 block_n, 10 stages, 11 B order (0 N/nt K/kt
    *        nt kt, 1 K/kt N/nt kt nt) */
   int64_t vals[ALT_TUNE_NPARAMS][ALT_TUNE_MAX_VALS];

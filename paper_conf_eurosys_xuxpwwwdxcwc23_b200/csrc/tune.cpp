@@ -148,6 +148,18 @@ Seq out_layout_tiled(int64_t K, int64_t ot, int64_t Ho, int64_t Wo, int64_t ht, 
   s.p.push_back(r);
   return s;
 }
+// Two-level output template: N H/(h2 ht) W/(w2 wt) K/(o2 ot)
+// h2 w2 o2 ht wt ot; h2 (w2) | Ho / ht (Wo / wt), o2 | K / ot
+Seq out_layout_two_level(int64_t K, int64_t ot, int64_t o2, int64_t Ho, int64_t Wo, int64_t ht, int64_t wt,
+                         int64_t h2, int64_t w2) {
+  Seq s;
+  s.p.push_back(P_split(2, {Ho / (h2 * ht), h2, ht}));                // N K Hoo h2 ht W
+  s.p.push_back(P_split(5, {Wo / (w2 * wt), w2, wt}));                // N K Hoo h2 ht Woo w2 wt
+  s.p.push_back(P_split(1, {K / (o2 * ot), o2, ot}));                 // N Koo o2 ot Hoo h2 ht Woo w2 wt
+  // -> N Hoo Woo Koo h2 w2 o2 ht wt ot
+  s.p.push_back(P_reorder({0, 4, 7, 1, 5, 8, 2, 6, 9, 3}));
+  return s;
+}
 // the paper's weight order O/ot I/it KH KW it ot (o innermost)
 Seq wgt_layout_paper(int64_t K, int64_t C, int64_t Cp, int64_t y, int64_t x) {
   Seq s;
@@ -289,6 +301,9 @@ extern "C" alt_status alt_tune(alt_op_kind op, const void *op_params, alt_dtype 
     std::vector<int64_t> lwts = vals_or(space, 9, {0});
     std::vector<int64_t> stgs = vals_or(space, 10, {0});
     std::vector<int64_t> words = vals_or(space, 11, {0});
+    std::vector<int64_t> h2s = vals_or(space, 12, {0});   // two-level output factors (0 / 1 = one level)
+    std::vector<int64_t> w2s = vals_or(space, 13, {0});
+    std::vector<int64_t> o2s = vals_or(space, 14, {0});
     for (int64_t it : its) {
       if (it > Cp || Cp % it || it % 8) continue;
       if (space && space->fix_x) { if (it != its[0]) continue; }
@@ -302,6 +317,9 @@ extern "C" alt_status alt_tune(alt_op_kind op, const void *op_params, alt_dtype 
           for (int64_t lht : lhts)
           for (int64_t lwt : lwts)
           for (int64_t wo : words)
+          for (int64_t h2 : h2s)
+          for (int64_t w2 : w2s)
+          for (int64_t o2 : o2s)
           for (int64_t th : ths)
           for (int64_t tw : tws)
           for (int64_t pr : pairs)
@@ -316,7 +334,11 @@ extern "C" alt_status alt_tune(alt_op_kind op, const void *op_params, alt_dtype 
                                      : act_layout(p.C, Cp, it, pad ? p.pad_h : 0);
             pt.seq[1] = wo ? wgt_layout_paper(p.K, p.C, Cp, y_w, it) : wgt_layout(p.K, p.C, Cp, y_w, it);
             const bool ytiled = (lht || lwt) && (!lht || Ho % lht == 0) && (!lwt || Wo % lwt == 0);
-            pt.seq[2] = ytiled ? out_layout_tiled(p.K, ot, Ho, Wo, lht, lwt) : act_layout(p.K, p.K, ot, 0);
+            const int64_t H2 = h2 > 1 ? h2 : 1, W2 = w2 > 1 ? w2 : 1, O2 = o2 > 1 ? o2 : 1;
+            const bool two = (H2 > 1 || W2 > 1 || O2 > 1);
+            if (two && !(lht && lwt && Ho % (H2 * lht) == 0 && Wo % (W2 * lwt) == 0 && p.K % (O2 * ot) == 0)) continue;
+            pt.seq[2] = two ? out_layout_two_level(p.K, ot, O2, Ho, Wo, lht, lwt, H2, W2)
+                            : ytiled ? out_layout_tiled(p.K, ot, Ho, Wo, lht, lwt) : act_layout(p.K, p.K, ot, 0);
             pt.fixed_x = space && space->fix_x && space->fixed_x;
             alt_kernel_cfg &cfg = pt.cfg;
             cfg.path = ALT_PATH_AUTO;

@@ -128,6 +128,19 @@ def test_tune_conv_template_knobs(space):
     _check_tuned_conv(p, 4, 64, 14, 128, 3, 1, res)
 
 
+def test_tune_conv_two_level_output_template():
+    """the two-level output template N H/(h't ht) W/(w't wt) K/(o't ot)
+    h't w't o't ht wt ot is a measured grid point; the winner
+    restricted to it is oracle-exact"""
+    p = alt.conv_params(2, 64, 28, 28, 64, 3, 3, 1, 1)
+    res = alt.tune("conv2d", p, alt.ALT_BF16, {0: [64], 1: [8], 6: [64], 8: [7], 9: [7], 12: [2], 13: [2], 14: [2]},
+                   max_points=4, warmup=1, reps=3)
+    assert res["measured"] >= 1
+    split_y = [q for q in res["y"] if q[0] == "split"]
+    assert len(split_y) == 3 and all(len(q[2]) == 3 for q in split_y)
+    _check_tuned_conv(p, 2, 64, 28, 64, 3, 1, res)
+
+
 def test_tune_conv_strided_spatial_template():
     p = alt.conv_params(2, 64, 28, 28, 128, 3, 3, 2, 1)
     res = alt.tune("conv2d", p, alt.ALT_BF16, {0: [64], 1: [64], 6: [128], 8: [7], 9: [7]}, max_points=4,

@@ -120,7 +120,13 @@ def test_matmul_store_at_parity(case, dtype):
     Z = o_store_at(f64(B), f64(bias), 0)
     want = gemm_store_at_f64(f64(A), Z, scale=scale.double().numpy(), residual=f64(res), act="relu")
     got = read_output(oracle.Layout((M, N), []), c, dtype)
-    assert_parity(got, want, dtype)
+    try:
+        assert_parity(got, want, dtype)
+    except AssertionError as e:  # locate the wrong outputs (diagnostics for an intermittent failure)
+        d = np.abs(got - want) > 0.05 * np.abs(want).max()
+        rows, cols = np.where(d.any(1))[0], np.where(d.any(0))[0]
+        raise AssertionError(f"{e}; plan {alt.last_plan()}; wrong rows {rows[:8]}..{rows[-8:]} ({len(rows)}), "
+                             f"cols {cols[:8]}..{cols[-8:]} ({len(cols)})") from None
 
 
 def test_matmul_store_at_rejects_separate_bias():
