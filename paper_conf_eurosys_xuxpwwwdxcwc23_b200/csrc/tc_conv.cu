@@ -90,7 +90,8 @@ struct TcArgs {
   Reader yr;             // out_mode 2: owner offsets of y
   EpiParams epi;
   uint64_t *dbg;         // optional per-CTA timestamps (ALT_TC_DEBUG)
-  int32_t epi_dbg;       // developer knob (ALT_TC_EPI_DBG): 1 skip output stores, 2 skip the whole drain
+  int32_t epi_dbg;       // developer knob (ALT_TC_EPI_DBG): 1 skip output stores, 2 skip the whole drain,
+                         // 3 also skip the MMAs (the TMA pipeline alone)
   // split-K: work unit = (output tile, reduction range); partial fp32 tiles
   // in ws[cta_tile][split][BN/32][128][32], arrivals counted in cnt[cta_tile]
   int32_t splits;
@@ -625,11 +626,13 @@ __global__ void __launch_bounds__(kThreads, 1)
           if (i == ALT_DBG_TILE && kit == k_begin) { DBG(28); }
           tc_fence_after();
           const uint64_t oA = (uint64_t)((stage * kStageBytesA) >> 4), oB = (uint64_t)((stage * L::kB) >> 4);
+          if (a.epi_dbg != 3) {  // developer knob 3: the TMA pipeline alone (no MMA, no drain)
 #pragma unroll
-          for (int kk = 0; kk < 4; kk++) {
-            const uint32_t accum = (kit != k_begin || kk != 0) ? 1u : 0u;
-            if constexpr (CG == 2) mma_bf16_2cta(d, dA[kk] + oA, dB[kk] + oB, idesc, accum);
-            else mma_bf16(d, dA[kk] + oA, dB[kk] + oB, idesc, accum);
+            for (int kk = 0; kk < 4; kk++) {
+              const uint32_t accum = (kit != k_begin || kk != 0) ? 1u : 0u;
+              if constexpr (CG == 2) mma_bf16_2cta(d, dA[kk] + oA, dB[kk] + oB, idesc, accum);
+              else mma_bf16(d, dA[kk] + oA, dB[kk] + oB, idesc, accum);
+            }
           }
           if constexpr (CG == 2) mma_commit_2cta(&empty[stage], 0x3);  // frees the stage in both CTAs
           else mma_commit(&empty[stage]);
@@ -860,7 +863,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       // function calls while a load is in flight (a call would save / restore
       // the registers the asynchronous load is writing); the other variant
       // issues the next load at the end of the chunk.
-      if (a.epi_dbg == 2) {
+      if (a.epi_dbg == 2 || a.epi_dbg == 3) {
         tc_fence_before();
         __syncwarp();
         if (lane == 0) {
@@ -1520,9 +1523,16 @@ static bool encode_view(const View &v, const void *base, int esize, int sw, CUte
                                              : CU_TENSOR_MAP_SWIZZLE_128B;
   auto enc = get_encode();
   if (!enc) { snprintf(why, 160, "cuTensorMapEncodeTiled unavailable"); return false; }
+  static const CUtensorMapL2promotion promo = [] {
+    const char *e = getenv("ALT_TMA_L2PROMO");  // developer A/B knob: 0 none, 64, 128, 256 (default)
+    const int v = e ? atoi(e) : 256;
+    return v == 0 ? CU_TENSOR_MAP_L2_PROMOTION_NONE
+                  : v == 64 ? CU_TENSOR_MAP_L2_PROMOTION_L2_64B
+                            : v == 128 ? CU_TENSOR_MAP_L2_PROMOTION_L2_128B : CU_TENSOR_MAP_L2_PROMOTION_L2_256B;
+  }();
   CUresult r = enc(tm, esize == 2 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 5,
-                   const_cast<void *>(base), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, swz,
-                   CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+                   const_cast<void *>(base), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, swz, promo,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) { snprintf(why, 160, "cuTensorMapEncodeTiled failed (%d)", (int)r); return false; }
   memset(om, 0, sizeof(*om));
   for (int i = 0; i < 5; i++)

@@ -1,3 +1,2 @@
-python scripts/epi_probe.py > gpurun_out/epi_round.txt 2>&1
-ALT_TC_ROUND=0 python scripts/epi_probe.py > gpurun_out/epi_warp.txt 2>&1
-python -m pytest tests/test_gpu_conv.py tests/test_gpu_mnmajor.py tests/test_gpu_fp32tc.py tests/test_gpu_chain.py -q -x --timeout 900 -p no:cacheprovider > gpurun_out/conv.txt 2>&1; echo "rc=$?" >> gpurun_out/conv.txt
+ALT_TC_EPI_DBG=3 python scripts/stage_probe.py l1.3x3,l3.3x3,l2.1x1a,l3.1x1a,l1.1x1a > gpurun_out/stages3.txt 2>&1
+python scripts/stage_probe.py l1.3x3,l3.3x3,l2.1x1a,l3.1x1a,l1.1x1a > gpurun_out/stages0.txt 2>&1
