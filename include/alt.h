@@ -221,7 +221,10 @@ typedef struct {
   int32_t path;        /* alt_path */
   int32_t block_m;     /* 128 (or 256 with cta_pair) */
   int32_t block_n;     /* 32..256, multiple of 16 */
-  int32_t block_k;     /* 64 */
+  int32_t block_k;     /* 64 (reduction slab per stage); tensor-core stride-1 3x3:
+                          1 = request the halo mode (one A load per filter row,
+                          the 3 taps along W read it shifted), 2 = refuse it;
+                          reported back as 1 when the plan uses it */
   int32_t stages;      /* smem pipeline depth */
   int32_t cta_pair;    /* 0 auto, 1 = tcgen05 cta_group::2 CTA pair, 2 = one CTA */
   int32_t tile_n, tile_h, tile_w;
@@ -318,7 +321,7 @@ typedef enum { ALT_OP_CONV2D = 0, ALT_OP_MATMUL = 1 } alt_op_kind;
 typedef struct { int64_t M, N, K; } alt_matmul_params;
 
 #define ALT_TUNE_MAX_VALS 8
-#define ALT_TUNE_NPARAMS 15
+#define ALT_TUNE_NPARAMS 16
 typedef struct {
   /* candidate values per template parameter; nvals[i] == 0 = default set.
    * conv:  0 it (x channel tile; the w c tile it' = it), 1 ot (y channel
@@ -330,7 +333,9 @@ typedef struct {
    *        10 stages (smem ring depth; 0 = deepest), 11 w order (0 c
    *        innermost, 1 the paper's it' ot'), 12 h't, 13 w't, 14 o't: the
    *        two-level output template N H/(h't ht) W/(w't wt) K/(o't ot)
-   *        h't w't o't ht wt ot (0 or 1 = one level)
+   *        h't w't o't ht wt ot (0 or 1 = one level),
+   *        15 halo (1: stride-1 3x3 taps along W from one row-shifted A
+   *        load, cfg.block_k = 1; needs a pixel tile with tile_w >= Wo + 2)
    * gemm:  0 mt, 1 kt, 2 nt, 6 block_n, 10 stages, 11 B order (0 N/nt K/kt
    *        nt kt, 1 K/kt N/nt kt nt) */
   int64_t vals[ALT_TUNE_NPARAMS][ALT_TUNE_MAX_VALS];

@@ -75,7 +75,7 @@ class MatmulParams(ctypes.Structure):
 
 
 class TuneSpace(ctypes.Structure):
-    _fields_ = [("vals", (ctypes.c_int64 * 8) * 15), ("nvals", ctypes.c_int32 * 15),
+    _fields_ = [("vals", (ctypes.c_int64 * 8) * 16), ("nvals", ctypes.c_int32 * 16),
                 ("max_points", ctypes.c_int32), ("warmup", ctypes.c_int32),
                 ("reps", ctypes.c_int32), ("fix_x", ctypes.c_int32),
                 ("fixed_x", ctypes.c_void_p), ("topk", ctypes.c_int32)]

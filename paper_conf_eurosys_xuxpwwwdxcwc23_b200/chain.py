@@ -432,8 +432,17 @@ class Chain:
             Ho, Wo = L.out_hw()
             tiles = [None] + [(128 // (th * tw), th, tw) for th in (1, 2, 4) for tw in (4, 8, 16, 32)
                               if tw <= 2 * Wo and th <= 2 * Ho and 128 // (th * tw) <= max(self.N, 1)]
+            # halo tiles (stride-1 3x3: a W run of 16 / 32 / 64 >= Wo + 2)
+            halo_tiles = [] if (L.R != 3 or L.stride != 1) else \
+                [(128 // (th * tw), th, tw) for tw in (16, 32, 64) for th in (1, 2, 4, 8)
+                 if tw >= Wo + 2 and 128 % (th * tw) == 0 and 1 <= 128 // (th * tw) <= max(self.N, 1)]
             cands = []
             M = self.N * Ho * Wo
+            for bn, pair, t in itertools.product((64, 128, 256), (0, 2), halo_tiles):
+                if bn > 64 and bn >= 2 * L.K:
+                    continue
+                cands.append({"path": A.PATH_TC, "block_n": bn, "cta_pair": pair, "split_k": 1, "split_cluster": 0,
+                              "tile_n": t[0], "tile_h": t[1], "tile_w": t[2], "block_k": 1})
             for bn, pair, sk, t in itertools.product((64, 128, 256), (0, 2), (1, 2, 4, -2, -4), tiles):
                 if bn > 64 and bn >= 2 * L.K:
                     continue

@@ -81,6 +81,7 @@ struct TcArgs {
   int32_t pairs, rsg, out_f32;
   FastDiv f_rsg;
   int32_t nst;           // smem ring stages in use (<= the instantiation's STAGES; tuner knob)
+  int32_t hboff;         // halo mode: set the descriptor base-offset field for row-shifted A starts
   int32_t yvec;          // out_mode 0 with 8-channel runs: copies written as 16-byte vectors
   int32_t out_round;     // out_mode 1, round stores: the 8 epilogue warps stage a whole 128-row x
                          // 64-channel round in smem, one thread TMA-stores it (a.O views 128 rows)
@@ -136,10 +137,15 @@ constexpr int tmem_cols(int c) { return c <= 32 ? 32 : (c <= 64 ? 64 : (c <= 128
 constexpr int kTabSlabs = kEpiWarps == 8 ? 288 : 240;
 constexpr int kTabBytes = kTabSlabs * 64;
 
-template <int BN, int STAGES, int CG = 1>
+// HS > 0: halo mode for stride-1 filters of width HS (3x3): an A stage is
+// loaded once per (filter row, channel slab) with 8 spare rows after the
+// 128, and the HS taps along W read it at row offsets 0 .. HS-1; B holds the
+// HS tap slabs of the stage
+template <int BN, int STAGES, int CG = 1, int HS = 0>
 struct TcSmem {
-  static constexpr int kB = (BN / CG) * 64 * 2;  // this CTA's share of the B tile
-  static constexpr int kRing = STAGES * (kStageBytesA + kB);
+  static constexpr int kAst = kStageBytesA + (HS ? 1024 : 0);  // A stage stride
+  static constexpr int kB = (BN / CG) * 64 * 2 * (HS ? HS : 1);  // this CTA's share of the B tile(s)
+  static constexpr int kRing = STAGES * (kAst + kB);
   static constexpr int kOut = kRing;                       // 2 staging buffers for TMA stores
   static constexpr int kSB = kOut + kEpiWarps * 4096;      // scale / bias of the tile (2 x BN floats)
   static constexpr int kBar = kSB + 2 * BN * 4;             // barriers
@@ -397,19 +403,19 @@ __device__ __forceinline__ TileCoord tile_coord(const TcArgs &a, int tile, int B
 // cluster barrier CTA r reduces rows [r * 128 / SC, (r + 1) * 128 / SC) of all
 // SC partials through distributed shared memory in split order, applies the
 // epilogue and stores them — the reduction and the epilogue are split SC ways.
-template <int BN, int STAGES, int CG, bool RV, int SC>
+template <int BN, int STAGES, int CG, bool RV, int SC, int HS = 0>
 __global__ void __launch_bounds__(kThreads, 1)
     k_tc_conv(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
               const __grid_constant__ CUtensorMap tmY, const __grid_constant__ TcArgs a, uint16_t *__restrict__ y) {
   using namespace sm100;
-  using L = TcSmem<BN, STAGES, CG>;
+  using L = TcSmem<BN, STAGES, CG, HS>;
   const int rank = CG == 2 ? (int)cluster_ctarank() : 0;
   const int unit0 = blockIdx.x / CG, unit_step = gridDim.x / CG;
   extern __shared__ __align__(1024) unsigned char smem_raw[];
   unsigned char *smem = reinterpret_cast<unsigned char *>(
       (reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   unsigned char *sA = smem;
-  unsigned char *sB = smem + STAGES * kStageBytesA;
+  unsigned char *sB = smem + STAGES * L::kAst;
   unsigned char *sOut = smem + L::kOut;
   const uint32_t sSB = sm100::smem_u32(smem + L::kSB);  // scale [BN] then bias [BN] (fp32)
   uint64_t *full = reinterpret_cast<uint64_t *>(smem + L::kBar);
@@ -484,11 +490,18 @@ __global__ void __launch_bounds__(kThreads, 1)
     const OperandMap &om = isA ? a.A : a.B;
     const CUtensorMap *tmap = isA ? &tmA : &tmB;
     unsigned char *sbase = isA ? sA : sB;
-    const int sbytes = isA ? kStageBytesA : L::kB;
+    const int sbytes = isA ? L::kAst : L::kB;
     // issues per stage: (group, channel slab) pairs; a K-major operand has
-    // one group, an MN-major one ng groups of mnw rows (planner: <= 16)
-    const bool active = j < om.ng * a.spi;
-    const int gi = om.mnw ? j % om.ng : 0, si = om.mnw ? j / om.ng : j;
+    // one group, an MN-major one ng groups of mnw rows (planner: <= 16);
+    // halo mode: B issues one box per (tap s, slab), lane j -> s = j / spi
+    const int hsb = (HS && !isA) ? HS : 1;
+    const bool active = j < om.ng * a.spi * hsb;
+    const int hs_s = (HS && !isA) ? j / a.spi : 0;
+    const int jj = (HS && !isA) ? j - hs_s * a.spi : j;
+    const int gi = om.mnw ? jj % om.ng : 0, si = om.mnw ? jj / om.ng : jj;
+    const int32_t hs_c[5] = {om.coef[0][V_S] * hs_s, om.coef[1][V_S] * hs_s, om.coef[2][V_S] * hs_s,
+                             om.coef[3][V_S] * hs_s, om.coef[4][V_S] * hs_s};
+    const uint32_t hs_off = (uint32_t)(hs_s * (BN / CG) * 128);
     // this lane's group: rows [gi * mnw, (gi + 1) * mnw) of the tile
     int g_dn = 0, g_dh = 0, g_dw = 0;
     if (om.mnw && isA) {
@@ -534,13 +547,13 @@ __global__ void __launch_bounds__(kThreads, 1)
             int32_t o0, o1, o2, o3, o4;
             asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];" : "=r"(o0), "=r"(o1), "=r"(o2), "=r"(o3) : "r"(ta));
             asm volatile("ld.shared.b32 %0, [%1];" : "=r"(o4) : "r"(ta + 16));
-            unsigned char *dst = sbase + stage * sbytes + goff + si * om.slab_bytes;
+            unsigned char *dst = sbase + stage * sbytes + goff + hs_off + si * om.slab_bytes;
             if constexpr (CG == 2)
-              tma_load_5d_2cta(dst, tmap, &full[stage], base[0] + o0, base[1] + o1, base[2] + o2, base[3] + o3,
-                               base[4] + o4);
+              tma_load_5d_2cta(dst, tmap, &full[stage], base[0] + o0 + hs_c[0], base[1] + o1 + hs_c[1],
+                               base[2] + o2 + hs_c[2], base[3] + o3 + hs_c[3], base[4] + o4 + hs_c[4]);
             else
-              tma_load_5d(dst, tmap, &full[stage], base[0] + o0, base[1] + o1, base[2] + o2, base[3] + o3,
-                          base[4] + o4);
+              tma_load_5d(dst, tmap, &full[stage], base[0] + o0 + hs_c[0], base[1] + o1 + hs_c[1],
+                          base[2] + o2 + hs_c[2], base[3] + o3 + hs_c[3], base[4] + o4 + hs_c[4]);
           }
           if (++stage == a.nst) { stage = 0; ph ^= 1u; }
         }
@@ -563,14 +576,15 @@ __global__ void __launch_bounds__(kThreads, 1)
           const int ga = isA ? gA : gB;
           v[V_GT] = (int)om.fg.div((uint32_t)ga); v[V_GR] = ga - v[V_GT] * om.divg;
           int32_t c[5];
+          v[V_S] += hs_s;  // halo mode: this lane's tap s (B); 0 otherwise
           coords(om, v, c);
           if (!valid) c[0] = om.oob0;
           if constexpr (CG == 2)
-            tma_load_5d_2cta(sbase + stage * sbytes + goff + si * om.slab_bytes, tmap, &full[stage], c[0], c[1], c[2],
-                             c[3], c[4]);
+            tma_load_5d_2cta(sbase + stage * sbytes + goff + hs_off + si * om.slab_bytes, tmap, &full[stage], c[0], c[1],
+                             c[2], c[3], c[4]);
           else
-            tma_load_5d(sbase + stage * sbytes + goff + si * om.slab_bytes, tmap, &full[stage], c[0], c[1], c[2], c[3],
-                        c[4]);
+            tma_load_5d(sbase + stage * sbytes + goff + hs_off + si * om.slab_bytes, tmap, &full[stage], c[0], c[1], c[2],
+                        c[3], c[4]);
         }
       }
     }
@@ -625,13 +639,20 @@ __global__ void __launch_bounds__(kThreads, 1)
           mbar_wait(&full[stage], ph);
           if (i == ALT_DBG_TILE && kit == k_begin) { DBG(28); }
           tc_fence_after();
-          const uint64_t oA = (uint64_t)((stage * kStageBytesA) >> 4), oB = (uint64_t)((stage * L::kB) >> 4);
+          const uint64_t oA = (uint64_t)((stage * L::kAst) >> 4), oB = (uint64_t)((stage * L::kB) >> 4);
           if (a.epi_dbg != 3) {  // developer knob 3: the TMA pipeline alone (no MMA, no drain)
 #pragma unroll
-            for (int kk = 0; kk < 4; kk++) {
-              const uint32_t accum = (kit != k_begin || kk != 0) ? 1u : 0u;
-              if constexpr (CG == 2) mma_bf16_2cta(d, dA[kk] + oA, dB[kk] + oB, idesc, accum);
-              else mma_bf16(d, dA[kk] + oA, dB[kk] + oB, idesc, accum);
+            for (int hs = 0; hs < (HS ? HS : 1); hs++) {
+              // halo: tap s reads A rows shifted by s (128-byte rows: + s * 8
+              // in 16-byte units; base-offset field = s when requested)
+              const uint64_t sA_off = HS ? (uint64_t)(hs * 8) | (a.hboff ? ((uint64_t)hs << 49) : 0ull) : 0ull;
+              const uint64_t sB_off = HS ? (uint64_t)((hs * (BN / CG) * 128) >> 4) : 0ull;
+#pragma unroll
+              for (int kk = 0; kk < 4; kk++) {
+                const uint32_t accum = (kit != k_begin || kk != 0 || hs != 0) ? 1u : 0u;
+                if constexpr (CG == 2) mma_bf16_2cta(d, dA[kk] + oA + sA_off, dB[kk] + oB + sB_off, idesc, accum);
+                else mma_bf16(d, dA[kk] + oA + sA_off, dB[kk] + oB + sB_off, idesc, accum);
+              }
             }
           }
           if constexpr (CG == 2) mma_commit_2cta(&empty[stage], 0x3);  // frees the stage in both CTAs
@@ -1632,13 +1653,13 @@ static int num_sms() {
   return n;
 }
 
-template <int BN, int STAGES, int CG_, bool RV, int SC = 1>
+template <int BN, int STAGES, int CG_, bool RV, int SC = 1, int HS = 0>
 static cudaError_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUtensorMap &ty, const TcArgs &a,
                              uint16_t *y, int grid, cudaStream_t s) {
   constexpr int CG = CG_;
-  auto kern = k_tc_conv<BN, STAGES, CG, RV, SC>;
-  const int smem = TcSmem<BN, STAGES, CG>::kBytes;
-  static_assert(TcSmem<BN, STAGES, CG>::kBytes <= 232448, "smem budget");
+  auto kern = k_tc_conv<BN, STAGES, CG, RV, SC, HS>;
+  const int smem = TcSmem<BN, STAGES, CG, HS>::kBytes;
+  static_assert(TcSmem<BN, STAGES, CG, HS>::kBytes <= 232448, "smem budget");
   static bool attr_set = false;  // once per instantiation (not capture-safe to repeat)
   if (!attr_set) {
     cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
@@ -1693,6 +1714,7 @@ struct TcPlan {
   int grid;
   int BN, stages, cg;
   int sc;  // cluster split-K factor (1 = off)
+  int hs;  // halo mode: filter width S folded into row-shifted A reads (0 = off)
   alt_kernel_cfg used;
 };
 static std::mutex g_tc_mu;
@@ -1704,8 +1726,18 @@ constexpr int stages_for(int BN, int CG) {
   return kEpiWarps == 8 ? (CG == 2 ? (BN == 128 ? 7 : 5) : (BN == 64 ? 7 : (BN == 128 ? 5 : 3)))  // BN 192: pair, 5
                         : (CG == 2 ? (BN == 128 ? 5 : 4) : (BN == 64 ? 5 : (BN == 128 ? 4 : 3)));
 }
+// halo-mode ring depth (A stage + 8 spare rows, three B tap slabs per stage)
+constexpr int stages_halo(int BN, int CG) { return BN / CG == 64 ? 4 : 2; }
 template <bool RV>
 static cudaError_t launch_plan_rv(const TcPlan &pl, uint16_t *yy, cudaStream_t stream) {
+  if (pl.hs == 3) {
+    if (pl.cg == 2) {
+      if (pl.BN == 128) return launch_tc<128, stages_halo(128, 2), 2, RV, 1, 3>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+      return launch_tc<256, stages_halo(256, 2), 2, RV, 1, 3>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+    }
+    if (pl.BN == 64) return launch_tc<64, stages_halo(64, 1), 1, RV, 1, 3>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+    return launch_tc<128, stages_halo(128, 1), 1, RV, 1, 3>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+  }
   if (pl.cg == 2) {
     if (pl.BN == 128) return launch_tc<128, stages_for(128, 2), 2, RV>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
     if (pl.BN == 192) return launch_tc<192, stages_for(192, 2), 2, RV>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
@@ -1842,7 +1874,21 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       if (ry[d].role == R_W) ry[d].tile = sw_w;
       if (rb[d].role == R_W) rb[d].tile = BN / cg;
     }
+    // halo mode (stride-1 3x3, 64-channel slabs, K-major A): the tile's W run
+    // tw in {16, 32, 64} must leave S - 1 spare columns past Wo, so the row
+    // shifts of the valid outputs stay inside their own W run
+    static const int halo_env = [] { const char *e = getenv("ALT_TC_HALO"); return e ? atoi(e) : -1; }();
+    const int halo_cfg = cfg && cfg->block_k == 1 ? 1 : (cfg && cfg->block_k == 2 ? 0 : -1);
+    const int halo_want = halo_env >= 0 ? halo_env : (halo_cfg >= 0 ? halo_cfg : 0);
+    const bool halo_ok = halo_want && P.is_conv && P.S == 3 && !P.pairs && P.ra[3].role == R_W && P.ra[3].V == 1 &&
+                         P.ra[3].tap == 1 && (c.tw == 16 || c.tw == 32 || c.tw == 64) && P.Wo + P.S - 2 < c.tw &&
+                         !(cfg && (cfg->split_k > 1 || cfg->split_cluster)) && BN / cg <= 128;
+    for (int hmode = halo_ok ? 1 : 0; hmode >= 0; hmode--)
     for (int sw = 64; sw >= 8; sw /= 2) {
+      if (hmode && sw != 64) continue;
+      RoleInfo rah[kMaxL];
+      memcpy(rah, ra, sizeof(rah));
+      if (hmode) rah[3].tap = 0;  // the A box does not move with the tap s
       View va, vb;
       // K-major first (the channel run innermost); otherwise an MN-major
       // view whose stride-1 dim is the M (A) / N (B) run: groups of mnw rows
@@ -1865,7 +1911,8 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
         return false;
       };
       int mnA = 0, mnB = 0;
-      if (!view_of(P.va, ra, 128, c.tw, &va, &mnA)) continue;
+      if (!view_of(P.va, rah, 128, c.tw, &va, &mnA)) continue;
+      if (hmode && mnA) continue;
       if (!view_of(P.vb, rb, BN / cg, BN / cg, &vb, &mnB)) continue;
       int64_t rowsA = 1, rowsB = 1;
       for (int i = 1; i < va.rank; i++) rowsA *= (va.d[i].box + va.d[i].estride - 1) / va.d[i].estride;
@@ -1958,17 +2005,22 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       if (mtiles * ntiles > 0x7fffffff) { set_error("tc: too many tiles"); return ALT_E_UNSUPPORTED; }
       a.num_n_tiles = (int32_t)ntiles;
       a.num_tiles = (int32_t)(((mtiles + cg - 1) / cg) * ntiles);  // work units
-      a.S = (int32_t)P.S;
+      a.S = (int32_t)(hmode ? 1 : P.S);  // halo: the slabs enumerate (r, g); the S taps ride in each stage
       a.Gc = (int32_t)((P.C + sw - 1) / sw);
       if (P.coff % sw) { snprintf(why, 160, "group channel offset %% slab"); continue; }
       a.a_goff = (int32_t)(P.coff / sw);
       a.b_koff = (int32_t)P.koff;
       a.y_koff = (int32_t)P.koff;
-      a.rsg = (int32_t)(P.R * P.S * a.Gc);
+      a.rsg = (int32_t)(P.R * a.S * a.Gc);
       a.pairs = P.pairs;
       a.out_f32 = P.out_f32 ? 1 : 0;
       if (P.pairs && P.C % sw) { snprintf(why, 160, "split planes not slab-aligned"); continue; }
-      a.total_slabs = (int32_t)((P.pairs ? P.pairs : 1) * P.R * P.S * a.Gc);
+      a.total_slabs = (int32_t)((P.pairs ? P.pairs : 1) * P.R * a.S * a.Gc);
+      pl.hs = hmode ? (int)P.S : 0;
+      {
+        static const int hboff = [] { const char *e = getenv("ALT_HALO_BOFF"); return e ? atoi(e) : 0; }();
+        a.hboff = hboff;
+      }
       a.spi = 64 / sw;
       a.num_iters = (a.total_slabs + a.spi - 1) / a.spi;
       a.sw = sw;
@@ -2066,7 +2118,7 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
                           : (int)std::min<int64_t>((int64_t)a.num_tiles * cg, num_sms() / cg * cg);
       pl.BN = BN;
       pl.cg = cg;
-      pl.stages = stages_for(BN, cg);
+      pl.stages = pl.hs ? stages_halo(BN, cg) : stages_for(BN, cg);
       // a shallower ring than the instantiation's (tuner knob; 2 .. STAGES)
       a.nst = (cfg && cfg->stages >= 2 && cfg->stages < pl.stages) ? cfg->stages : pl.stages;
       alt_kernel_cfg u{};
@@ -2079,6 +2131,7 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       u.tile_n = c.tn; u.tile_h = c.th; u.tile_w = c.tw;
       u.split_k = a.splits;
       u.split_cluster = pl.sc > 1 ? 1 : (a.full_units > 0 && a.splits > 1 ? 2 : 0);
+      u.block_k = pl.hs ? 1 : 64;  // 1 = halo mode (cfg->block_k: 1 request, 2 refuse)
       pl.used = u;
       cudaError_t e = launch_plan(pl, P.y, stream);
       count_launch();

@@ -304,6 +304,7 @@ extern "C" alt_status alt_tune(alt_op_kind op, const void *op_params, alt_dtype 
     std::vector<int64_t> h2s = vals_or(space, 12, {0});   // two-level output factors (0 / 1 = one level)
     std::vector<int64_t> w2s = vals_or(space, 13, {0});
     std::vector<int64_t> o2s = vals_or(space, 14, {0});
+    std::vector<int64_t> halos = vals_or(space, 15, {0});  // 1: halo mode (stride-1 3x3)
     for (int64_t it : its) {
       if (it > Cp || Cp % it || it % 8) continue;
       if (space && space->fix_x) { if (it != its[0]) continue; }
@@ -320,6 +321,7 @@ extern "C" alt_status alt_tune(alt_op_kind op, const void *op_params, alt_dtype 
           for (int64_t h2 : h2s)
           for (int64_t w2 : w2s)
           for (int64_t o2 : o2s)
+          for (int64_t hl : halos)
           for (int64_t th : ths)
           for (int64_t tw : tws)
           for (int64_t pr : pairs)
@@ -347,6 +349,7 @@ extern "C" alt_status alt_tune(alt_op_kind op, const void *op_params, alt_dtype 
             cfg.split_k = (int32_t)(sk < 0 ? -sk : sk);  // negative: the cluster (DSMEM) form
             cfg.split_cluster = sk < 0 ? 1 : 0;
             cfg.stages = (int32_t)sg;
+            cfg.block_k = hl ? 1 : 0;
             if (th && tw) {
               cfg.tile_h = (int32_t)th;
               cfg.tile_w = (int32_t)tw;

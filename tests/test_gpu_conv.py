@@ -456,3 +456,27 @@ def test_epilogue_writes_consumer_templates(yp_name, pads_zero):
     ref = oracle.conv2d(dict(N=N, C=C, H=H, W=H, K=K, R=3, S=3, pad_h=1, pad_w=1), Xo, xph, Wo_, wph, act=1)
     got = read_output(oracle.Layout((N, K, H, H), yp), y, torch.bfloat16)
     assert_parity(got, ref, torch.bfloat16)
+
+
+HALO_CASES = [
+    # name, (N, C, H, W, K), cfg (tile with a W run of 16 / 32 / 64)
+    ("14x14 tw16 bn64", (4, 64, 14, 14, 64), {"block_n": 64, "tile_n": 1, "tile_h": 8, "tile_w": 16}),
+    ("28x28 tw32 bn128", (2, 128, 28, 28, 128), {"block_n": 128, "cta_pair": 2, "tile_n": 1, "tile_h": 4, "tile_w": 32}),
+    ("56x56 tw64 pair", (2, 64, 56, 56, 128), {"block_n": 128, "tile_n": 1, "tile_h": 2, "tile_w": 64}),
+    ("56x56 tw64 bn256 pair", (2, 64, 56, 56, 256), {"block_n": 256, "tile_n": 2, "tile_h": 1, "tile_w": 64}),
+    ("ragged 13x13 tw16 residual", (3, 64, 13, 13, 64), {"block_n": 64, "tile_n": 2, "tile_h": 4, "tile_w": 16}),
+]
+
+
+@pytest.mark.parametrize("pad_x", [0, 1], ids=["oob-pad", "materialised-pad"])
+@pytest.mark.parametrize("case", HALO_CASES, ids=[c[0] for c in HALO_CASES])
+def test_tc_conv_halo(case, pad_x):
+    """halo mode for stride-1 3x3 (block_k = 1 requests it): each input row
+    segment is loaded once per filter row and the three taps along W read it
+    at row offsets 0 / 1 / 2 (descriptor shift); vs the oracle"""
+    name, (N, C, H, W, K), cfg = case
+    res = LY.nchwxc(K, 64) if "residual" in name else None
+    _, plan = run_conv("halo" + name, N, C, H, W, K, 3, 3, 1, 1, LY.nchwxc(C, 64, pad_hw=pad_x),
+                       LY.kcrs_yk_xc(K, C, min(K, cfg["block_n"]), 64), LY.nchwxc(K, 64), torch.bfloat16, epi=True,
+                       res_p=res, act=1, cfg={"path": alt.PATH_TC, "block_k": 1, **cfg}, expect_path=alt.PATH_TC)
+    assert plan["block_k"] == 1, plan   # the halo plan ran
