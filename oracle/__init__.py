@@ -81,6 +81,7 @@ def lib():
         L.orc_read_logical.argtypes = [c_p, c_p, c_i, c_p]
         L.orc_read_logical.restype = c_i
         L.orc_conv2d_f64.argtypes = [c_p, c_p, c_p, c_p, c_p, c_p, c_i, c_ll, c_ll, c_p]
+        L.orc_conv3d_f64.argtypes = [c_p, c_p, c_p, c_p, c_p, c_p, c_i, c_p]
         L.orc_conv2d_points.argtypes = [c_p, c_p, c_p, c_p, c_p, c_i, c_p, c_p, c_p, c_p,
                                         c_i, c_ll, c_p, c_p]
         L.orc_conv2d_points.restype = c_i
@@ -253,6 +254,38 @@ def conv2d(p: dict, x_l: Layout, x: np.ndarray, w_l: Layout, w: np.ndarray,
     wl = w_l.read_f64(w)
     rl = res_l.read_f64(residual) if residual is not None else None
     return conv2d_f64(p, xl, wl, scale, bias, rl, act, images)
+
+
+def conv3d_out(p: dict):
+    """(Do, Ho, Wo) of a 3-D conv (the standard definition, as O3)."""
+    g = lambda k, d=1: p.get(k, d)  # noqa: E731
+    D, H, W, T, R, S = (p[k] for k in "DHWTRS")
+    return ((D + 2 * g("pad_d", 0) - g("dil_d") * (T - 1) - 1) // g("stride_d") + 1,
+            (H + 2 * g("pad_h", 0) - g("dil_h") * (R - 1) - 1) // g("stride_h") + 1,
+            (W + 2 * g("pad_w", 0) - g("dil_w") * (S - 1) - 1) // g("stride_w") + 1)
+
+
+def conv3d_f64(p: dict, x: np.ndarray, w: np.ndarray, scale=None, bias=None,
+               residual=None, act: int = 0) -> np.ndarray:
+    """O3b (C3D) + O6 on fp64 logical arrays x[N,C,D,H,W],
+    w[K,C/g,T,R,S] -> y[N,K,Do,Ho,Wo]."""
+    N, C, D, H, W, K, T, R, S = (p[k] for k in ("N", "C", "D", "H", "W", "K", "T", "R", "S"))
+    g = lambda k, d=1: p.get(k, d)  # noqa: E731
+    pr = np.array([N, C, D, H, W, K, T, R, S, g("stride_d"), g("stride_h"), g("stride_w"), g("pad_d", 0),
+                   g("pad_h", 0), g("pad_w", 0), g("dil_d"), g("dil_h"), g("dil_w"), g("groups")], np.int64)
+    x, w = _f64(x), _f64(w)
+    assert x.shape == (N, C, D, H, W) and w.shape == (K, C // g("groups"), T, R, S)
+    y = np.zeros((N, K) + conv3d_out(p), np.float64)
+    lib().orc_conv3d_f64(_ptr(pr), _ptr(x), _ptr(w), _ptr(_f64(scale)), _ptr(_f64(bias)), _ptr(_f64(residual)),
+                         int(act), _ptr(y))
+    return y
+
+
+def conv3d(p: dict, x_l: Layout, x: np.ndarray, w_l: Layout, w: np.ndarray, scale=None, bias=None,
+           res_l: Layout | None = None, residual=None, act: int = 0) -> np.ndarray:
+    """O3b + O6 with operands as physical word buffers in declared layouts."""
+    return conv3d_f64(p, x_l.read_f64(x), w_l.read_f64(w), scale, bias,
+                      res_l.read_f64(residual) if residual is not None else None, act)
 
 
 def conv2d_points(p: dict, x_l: Layout, x: np.ndarray, w_l: Layout, w: np.ndarray,

@@ -467,6 +467,48 @@ void orc_conv2d_f64(const long long *p, const double *x, const double *w,
     }
 }
 
+/* ----------------------------------------------------------------- O3b --- */
+/* Direct (textbook) 3-D convolution, the paper's C3D operator (
+ * "for other convolutions (e.g., 3-D case), the template is similar",
+ * P:1146-1150): on fp64 row-major logical arrays x[N,C,D,H,W],
+ * w[K,C/G,T,R,S], y[N,K,Do,Ho,Wo],
+ *   y[n,k,od,oh,ow] = sum_{c<C/G, t<T, r<R, s<S}
+ *       x[n, g(k) C/G + c, od Vd - pd + dd t, oh Vh - ph + dh r, ow Vw - pw + dw s]
+ *       * w[k, c, t, r, s]      (x = 0 outside the tensor),
+ * summed in (c, t, r, s) ascending order, then the O6 epilogue.
+ * p[] = {N,C,D,H,W,K,T,R,S, Vd,Vh,Vw, pd,ph,pw, dd,dh,dw, G}. */
+void orc_conv3d_f64(const long long *p, const double *x, const double *w,
+                    const double *scale, const double *bias, const double *res,
+                    int act, double *y) {
+  long long N = p[0], C = p[1], D = p[2], H = p[3], W = p[4], K = p[5], T = p[6], R = p[7], S = p[8];
+  long long Vd = p[9], Vh = p[10], Vw = p[11], pd = p[12], ph = p[13], pw = p[14];
+  long long dd = p[15], dh = p[16], dw = p[17], G = p[18];
+  long long Do = (D + 2 * pd - dd * (T - 1) - 1) / Vd + 1;
+  long long Ho = (H + 2 * ph - dh * (R - 1) - 1) / Vh + 1, Wo = (W + 2 * pw - dw * (S - 1) - 1) / Vw + 1;
+  long long Cg = C / G;
+#pragma omp parallel for collapse(2) schedule(dynamic)
+  for (long long n = 0; n < N; n++)
+    for (long long k = 0; k < K; k++) {
+      long long g = k * G / K;
+      for (long long od = 0; od < Do; od++)
+        for (long long oh = 0; oh < Ho; oh++)
+          for (long long ow = 0; ow < Wo; ow++) {
+            double acc = 0.0;
+            for (long long c = 0; c < Cg; c++)
+              for (long long t = 0; t < T; t++)
+                for (long long r = 0; r < R; r++)
+                  for (long long s = 0; s < S; s++) {
+                    long long id = od * Vd - pd + dd * t, ih = oh * Vh - ph + dh * r, iw = ow * Vw - pw + dw * s;
+                    if (id < 0 || id >= D || ih < 0 || ih >= H || iw < 0 || iw >= W) continue;
+                    acc += x[(((n * C + g * Cg + c) * D + id) * H + ih) * W + iw] *
+                           w[(((k * Cg + c) * T + t) * R + r) * S + s];
+                  }
+            long long idx = (((n * K + k) * Do + od) * Ho + oh) * Wo + ow;
+            y[idx] = epilogue(acc, scale, bias, res, k, idx, act);
+          }
+    }
+}
+
 /* Same definition evaluated one output at a time, reading x and w through
  * their layouts' F maps directly (for sampled checks at full size).
  * pts: npts x 4 (n,k,p,q). */
