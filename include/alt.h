@@ -251,6 +251,30 @@ alt_status alt_conv2d(const alt_conv2d_params *p, alt_layout x_l, const void *x,
                       const alt_kernel_cfg *cfg /*nullable*/,
                       alt_stream_t stream);
 
+/* 3-D convolution, the paper's C3D operator (its layout
+ * template is "similar" to C2D's):
+ *   y[n,k,od,oh,ow] = act(scale[k] * sum_{c<C/G, t<T, r<R, s<S}
+ *       x[n, g(k) C/G + c, od Vd - pd + dd t, oh Vh - ph + dh r, ow Vw - pw + dw s]
+ *       * w[k,c,t,r,s] + bias[k] + residual[n,k,od,oh,ow])
+ * with x = 0 outside the tensor; Do = (D + 2 pd - dd (T - 1) - 1) / Vd + 1
+ * (Ho, Wo alike).  Logical shapes: x [N,C,D,H,W], w [K,C/groups,T,R,S],
+ * y / residual [N,K,Do,Ho,Wo], each in its own declared layout (errors,
+ * ownership, asynchrony as alt_conv2d).  Tensor-core path: groups = 1, bf16 /
+ * fp32 operands whose layouts admit a TMA view (channel tile innermost, the
+ * depth dim plain or padded), output stored by TMA (no unfold copies; pads
+ * only under ALT_EPI_PADS_ZERO), no residual; one output depth slice per
+ * M tile (tile_n = 1).  Everything else: the generic CUDA-core path. */
+typedef struct {
+  int64_t N, C, D, H, W, K, T, R, S;
+  int32_t stride_d, stride_h, stride_w, pad_d, pad_h, pad_w;
+  int32_t dil_d, dil_h, dil_w, groups;
+} alt_conv3d_params;
+alt_status alt_conv3d(const alt_conv3d_params *p, alt_layout x_l, const void *x,
+                      alt_layout w_l, const void *w, alt_layout y_l, void *y,
+                      alt_dtype dtype, const alt_epilogue *epi /*nullable*/,
+                      const alt_kernel_cfg *cfg /*nullable*/,
+                      alt_stream_t stream);
+
 /* GEMM: C[m,n] = sum_k A[m,k] B[k,n] with logical
  * A [M,K], B [K,N], C [M,N] in arbitrary declared layouts; epilogue as above
  * (per-column scale / bias, i.e. indexed by n). */

@@ -15,7 +15,8 @@ CPU fallback.
 import importlib
 
 __all__ = ["ACT", "ALT_BF16", "ALT_F32", "AltError", "ConvParams", "KernelCfg", "Layout",
-           "PATH_AUTO", "PATH_DW", "PATH_SIMT", "PATH_TC", "conv2d", "conv_params", "last_plan",
+           "PATH_AUTO", "PATH_DW", "PATH_SIMT", "PATH_TC", "conv2d", "conv_params", "conv3d", "conv3d_params",
+           "last_plan",
            "launch_count", "lib_path", "matmul", "matmul_store_at", "store_at", "decouple_at", "plan_chain",
            "pool2d", "relayout", "tune"]
 

@@ -55,6 +55,12 @@ class ConvParams(ctypes.Structure):
                                               "dil_h", "dil_w", "groups", "_pad")]
 
 
+class Conv3dParams(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_int64) for n in ("N", "C", "D", "H", "W", "K", "T", "R", "S")] + \
+               [(n, ctypes.c_int32) for n in ("stride_d", "stride_h", "stride_w", "pad_d", "pad_h", "pad_w",
+                                              "dil_d", "dil_h", "dil_w", "groups")]
+
+
 class _Epi(ctypes.Structure):
     _fields_ = [("scale", ctypes.c_void_p), ("bias", ctypes.c_void_p),
                 ("residual", ctypes.c_void_p), ("residual_l", ctypes.c_void_p),
@@ -98,6 +104,7 @@ _lib.alt_layout_phys_to_logical.argtypes = [_p, _i64, _p, _p]
 _lib.alt_layout_logical_to_phys.argtypes = [_p, _p, _p]
 _lib.alt_relayout.argtypes = [_p, _p, _p, _p, ctypes.c_int, _p]
 _lib.alt_conv2d.argtypes = [_p, _p, _p, _p, _p, _p, _p, ctypes.c_int, _p, _p, _p]
+_lib.alt_conv3d.argtypes = [_p, _p, _p, _p, _p, _p, _p, ctypes.c_int, _p, _p, _p]
 _lib.alt_matmul.argtypes = [_i64, _i64, _i64, _p, _p, _p, _p, _p, _p, ctypes.c_int, _p, _p, _p]
 _lib.alt_last_plan.argtypes = [_p]
 _lib.alt_launch_count.restype = ctypes.c_uint64
@@ -302,6 +309,25 @@ def conv2d(p: ConvParams, x_l: Layout, x, w_l: Layout, w, y_l: Layout, y, scale=
     return y
 
 
+def conv3d_params(N, C, D, H, W, K, T, R, S, stride=1, pad=0, dilation=1, groups=1) -> Conv3dParams:
+    """alt_conv3d_params; stride / pad / dilation: an int or a (d, h, w) triple"""
+    tri = lambda v: tuple(v) if isinstance(v, (tuple, list)) else (v, v, v)  # noqa: E731
+    st, pd, dl = tri(stride), tri(pad), tri(dilation)
+    return Conv3dParams(N, C, D, H, W, K, T, R, S, st[0], st[1], st[2], pd[0], pd[1], pd[2], dl[0], dl[1], dl[2],
+                        groups)
+
+
+def conv3d(p: Conv3dParams, x_l: Layout, x, w_l: Layout, w, y_l: Layout, y, scale=None, bias=None,
+           residual=None, residual_l: Layout | None = None, act=0, cfg=None, stream=None, pads_zero=False):
+    """alt_conv3d (C3D, P:1546-1549): y (in y_l) = act(scale * conv3d(x, w) + bias + residual)."""
+    e = _epi(scale, bias, residual, residual_l, act, pads_zero)
+    c = _cfg(cfg)
+    _check(_lib.alt_conv3d(ctypes.byref(p), x_l.handle, _ptr(x), w_l.handle, _ptr(w), y_l.handle,
+                           _ptr(y), _dtype_code(x), ctypes.byref(e) if e else None,
+                           ctypes.byref(c) if c else None, _stream_ptr(stream)), "alt_conv3d")
+    return y
+
+
 def matmul(M, N, K, a_l: Layout, a, b_l: Layout, b, c_l: Layout, c, scale=None, bias=None,
            residual=None, residual_l=None, act=0, cfg=None, stream=None):
     """alt_matmul: C (in c_l) = act(scale * A B + bias + residual)."""
@@ -400,4 +426,4 @@ EXPORTED = ["alt_status_str", "alt_last_error", "alt_layout_create", "alt_layout
             "alt_layout_query", "alt_layout_logical", "alt_layout_phys_to_logical",
             "alt_layout_logical_to_phys", "alt_relayout", "alt_conv2d", "alt_matmul",
             "alt_last_plan", "alt_launch_count", "alt_tune", "alt_plan_chain", "alt_pool2d",
-            "alt_store_at", "alt_decouple_at", "alt_matmul_store_at"]
+            "alt_store_at", "alt_decouple_at", "alt_matmul_store_at", "alt_conv3d"]

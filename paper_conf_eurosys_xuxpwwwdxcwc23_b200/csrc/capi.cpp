@@ -221,6 +221,66 @@ alt_status alt_conv2d(const alt_conv2d_params *p, alt_layout x_l, const void *x,
   return st;
 }
 
+alt_status alt_conv3d(const alt_conv3d_params *p, alt_layout x_l, const void *x, alt_layout w_l,
+                      const void *w, alt_layout y_l, void *y, alt_dtype dtype,
+                      const alt_epilogue *epi, const alt_kernel_cfg *cfg, alt_stream_t stream) {
+  if (!p || !x_l || !w_l || !y_l) { set_error("alt_conv3d: NULL argument"); return ALT_E_INVALID; }
+  if (dtype != ALT_F32 && dtype != ALT_BF16) { set_error("alt_conv3d: bad dtype"); return ALT_E_INVALID; }
+  if (p->N < 0 || p->C < 1 || p->D < 1 || p->H < 1 || p->W < 1 || p->K < 1 || p->T < 1 || p->R < 1 || p->S < 1 ||
+      p->stride_d < 1 || p->stride_h < 1 || p->stride_w < 1 || p->pad_d < 0 || p->pad_h < 0 || p->pad_w < 0) {
+    set_error("alt_conv3d: bad geometry");
+    return ALT_E_INVALID;
+  }
+  const int32_t dd = p->dil_d < 1 ? 1 : p->dil_d, dh = p->dil_h < 1 ? 1 : p->dil_h, dw = p->dil_w < 1 ? 1 : p->dil_w;
+  const int32_t G = p->groups < 1 ? 1 : p->groups;
+  if (p->C % G || p->K % G) { set_error("alt_conv3d: groups must divide C and K"); return ALT_E_INVALID; }
+  const int64_t Do = (p->D + 2 * p->pad_d - (int64_t)dd * (p->T - 1) - 1) / p->stride_d + 1;
+  const int64_t Ho = (p->H + 2 * p->pad_h - (int64_t)dh * (p->R - 1) - 1) / p->stride_h + 1;
+  const int64_t Wo = (p->W + 2 * p->pad_w - (int64_t)dw * (p->S - 1) - 1) / p->stride_w + 1;
+  if (p->D + 2 * p->pad_d < (int64_t)dd * (p->T - 1) + 1 || p->H + 2 * p->pad_h < (int64_t)dh * (p->R - 1) + 1 ||
+      p->W + 2 * p->pad_w < (int64_t)dw * (p->S - 1) + 1 || Do < 1 || Ho < 1 || Wo < 1) {
+    set_error("alt_conv3d: empty output");
+    return ALT_E_INVALID;
+  }
+  const int64_t xs[5] = {p->N, p->C, p->D, p->H, p->W}, wsh[5] = {p->K, p->C / G, p->T, p->R, p->S},
+                ys[5] = {p->N, p->K, Do, Ho, Wo};
+  if (p->N > 0 && (!shape_is(&x_l->impl, 5, xs) || !shape_is(&w_l->impl, 5, wsh) || !shape_is(&y_l->impl, 5, ys))) {
+    set_error("alt_conv3d: layout logical shapes do not match x[N,C,D,H,W] / w[K,C/g,T,R,S] / y[N,K,Do,Ho,Wo]");
+    return ALT_E_SHAPE;
+  }
+  if (p->N == 0) return ALT_OK;
+  if (!is_device_ptr(x) || !is_device_ptr(w) || !is_device_ptr(y)) { set_error("alt_conv3d: x/w/y must be device pointers"); return ALT_E_INVALID; }
+  ConvProblem P{};
+  P.N = p->N; P.C = p->C; P.H = p->H; P.W = p->W; P.K = p->K; P.R = p->R; P.S = p->S;
+  P.Ho = Ho; P.Wo = Wo;
+  P.Vh = p->stride_h; P.Vw = p->stride_w; P.ph = p->pad_h; P.pw = p->pad_w; P.groups = G;
+  P.dh = dh; P.dw = dw;
+  P.D = p->D; P.T = p->T; P.Do = Do; P.Vd = p->stride_d; P.pd = p->pad_d; P.dd = dd; P.c3d = true;
+  P.xl = &x_l->impl; P.wl = &w_l->impl; P.yl = &y_l->impl;
+  P.x = x; P.w = w; P.y = y; P.dtype = dtype;
+  alt_status st = fill_epi(epi, P.yl, &P.epi);
+  if (st != ALT_OK) return st;
+  if (P.epi.bias_att) { set_error("alt_conv3d: attached bias unsupported"); return ALT_E_INVALID; }
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  const int32_t path = cfg ? cfg->path : ALT_PATH_AUTO;
+  alt_kernel_cfg used{};
+  if (path == ALT_PATH_TC || (path == ALT_PATH_AUTO && G == 1)) {
+    st = tc_conv(P, cfg, s, &used);
+    if (st != ALT_E_UNSUPPORTED || path == ALT_PATH_TC) {
+      if (st == ALT_OK) set_last_plan(used);
+      return st;
+    }
+  }
+  if (path == ALT_PATH_DW) { set_error("alt_conv3d: no depthwise kernel"); return ALT_E_UNSUPPORTED; }
+  st = simt_conv3d(P, s);
+  if (st == ALT_OK) {
+    used = alt_kernel_cfg{};
+    used.path = ALT_PATH_SIMT;
+    set_last_plan(used);
+  }
+  return st;
+}
+
 static alt_status gemm_dispatch(GemmProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s);
 
 alt_status alt_matmul(int64_t M, int64_t N, int64_t K, alt_layout a_l, const void *a,

@@ -37,6 +37,28 @@ struct Reader {
   }
 };
 
+// Rank-5 reader / writer (C3D operands): owner offsets of a separable layout,
+// or the primitive interpreter; every position an element owns.
+struct Reader5 {
+  int32_t sep;
+  const int64_t *rd[5];
+  const LayoutDesc *desc;
+  __device__ __forceinline__ int64_t off5(int64_t i0, int64_t i1, int64_t i2, int64_t i3, int64_t i4) const {
+    if (sep) {
+      const int64_t a = __ldg(rd[0] + i0), b = __ldg(rd[1] + i1), c = __ldg(rd[2] + i2), d = __ldg(rd[3] + i3),
+                    e = __ldg(rd[4] + i4);
+      if ((a | b | c | d | e) < 0) return -1;
+      return a + b + c + d + e;
+    }
+    int64_t l[5] = {i0, i1, i2, i3, i4};
+    return dev_F_offset(*desc, l);
+  }
+};
+struct Writer5 {
+  const int32_t *wptr[5];
+  const int64_t *wlist[5];
+};
+
 // Every physical position owned by a logical element (separable layouts).
 struct Writer {
   int32_t lrank;

@@ -25,6 +25,11 @@ struct ConvProblem {
   int64_t N, C, H, W, K, R, S, Ho, Wo;
   int32_t Vh, Vw, ph, pw, groups;
   int32_t dh = 1, dw = 1;  // dilation (SIMT path)
+  // 3-D convolution (C3D): depth extent / taps / output depth and its
+  // stride, padding, dilation; D = T = Do = 1 for conv2d (logical rank 4)
+  int64_t D = 1, T = 1, Do = 1;
+  int32_t Vd = 1, pd = 0, dd = 1;
+  bool c3d = false;
   Layout *xl, *wl, *yl;
   const void *x, *w;
   void *y;
@@ -44,6 +49,7 @@ struct GemmProblem {
 alt_status relayout_launch(Layout *S, const void *src, Layout *D, void *dst, int wb,
                            cudaStream_t stream);
 alt_status simt_conv(const ConvProblem &P, cudaStream_t stream);
+alt_status simt_conv3d(const ConvProblem &P, cudaStream_t stream);
 alt_status simt_gemm(const GemmProblem &P, cudaStream_t stream);
 // tensor-core path; returns ALT_E_UNSUPPORTED (without launching) when the
 // layouts / shapes cannot be served, filling *why

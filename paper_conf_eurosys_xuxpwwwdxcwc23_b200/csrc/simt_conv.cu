@@ -292,3 +292,133 @@ alt_status simt_gemm(const GemmProblem &P, cudaStream_t stream) {
 }
 
 }  // namespace alt
+
+// ------------------------------------------------------------ C3D (SIMT) --
+// The generic CUDA-core path of alt_conv3d: one thread per
+// output element y[n,k,od,oh,ow], the (c, t, r, s) sum in fp32 with x / w
+// gathered through any compiled rank-5 layout, the epilogue of O6, and the
+// result written to every position y's layout holds it at (pad zeros
+// included).  Correctness fallback; the tensor-core path (tc_conv.cu) serves
+// the layouts a TMA box can be cut from.
+namespace alt {
+
+struct Simt3Args {
+  int64_t N, C, D, H, W, K, T, R, S, Do, Ho, Wo;
+  int32_t Vd, Vh, Vw, pd, ph, pw, dd, dh, dw, G;
+  Reader5 xr, wr, rr;
+  Writer5 yw;
+  const float *scale, *bias;
+  const void *residual;
+  int32_t act;
+};
+
+template <typename T>
+__global__ void __launch_bounds__(256) k_simt_conv3d(const Simt3Args a, const T *__restrict__ x,
+                                                     const T *__restrict__ w, T *__restrict__ y) {
+  const int64_t total = a.N * a.K * a.Do * a.Ho * a.Wo;
+  const int64_t Cg = a.C / a.G;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    int64_t r_ = i;
+    const int64_t ow = r_ % a.Wo; r_ /= a.Wo;
+    const int64_t oh = r_ % a.Ho; r_ /= a.Ho;
+    const int64_t od = r_ % a.Do; r_ /= a.Do;
+    const int64_t k = r_ % a.K;
+    const int64_t n = r_ / a.K;
+    const int64_t g = k * a.G / a.K;
+    float acc = 0.f;
+    for (int64_t c = 0; c < Cg; c++)
+      for (int64_t t = 0; t < a.T; t++) {
+        const int64_t id = od * a.Vd - a.pd + a.dd * t;
+        if (id < 0 || id >= a.D) continue;
+        for (int64_t r = 0; r < a.R; r++) {
+          const int64_t ih = oh * a.Vh - a.ph + a.dh * r;
+          if (ih < 0 || ih >= a.H) continue;
+          for (int64_t s = 0; s < a.S; s++) {
+            const int64_t iw = ow * a.Vw - a.pw + a.dw * s;
+            if (iw < 0 || iw >= a.W) continue;
+            const int64_t xo = a.xr.off5(n, g * Cg + c, id, ih, iw), wo = a.wr.off5(k, c, t, r, s);
+            if (xo < 0 || wo < 0) continue;
+            acc = fmaf(load_as_f32<T>(x, xo), load_as_f32<T>(w, wo), acc);
+          }
+        }
+      }
+    float v = (a.scale ? __ldg(a.scale + k) : 1.f) * acc + (a.bias ? __ldg(a.bias + k) : 0.f);
+    if (a.residual) {
+      const int64_t ro = a.rr.off5(n, k, od, oh, ow);
+      if (ro >= 0) v += load_as_f32<T>(static_cast<const T *>(a.residual), ro);
+    }
+    v = apply_act(v, a.act);
+    const T out = from_f32<T>(v);
+    // every position y's layout holds (n, k, od, oh, ow) at; owned pads get 0
+    const int64_t idx[5] = {n, k, od, oh, ow};
+    int32_t lo[5], hi[5];
+#pragma unroll
+    for (int d = 0; d < 5; d++) {
+      lo[d] = __ldg(a.yw.wptr[d] + idx[d]);
+      hi[d] = __ldg(a.yw.wptr[d] + idx[d] + 1);
+    }
+    for (int32_t i0 = lo[0]; i0 < hi[0]; i0++) {
+      const int64_t c0 = __ldg(a.yw.wlist[0] + i0);
+      for (int32_t i1 = lo[1]; i1 < hi[1]; i1++) {
+        const int64_t c1 = __ldg(a.yw.wlist[1] + i1);
+        for (int32_t i2 = lo[2]; i2 < hi[2]; i2++) {
+          const int64_t c2 = __ldg(a.yw.wlist[2] + i2);
+          for (int32_t i3 = lo[3]; i3 < hi[3]; i3++) {
+            const int64_t c3 = __ldg(a.yw.wlist[3] + i3);
+            for (int32_t i4 = lo[4]; i4 < hi[4]; i4++) {
+              const int64_t c4 = __ldg(a.yw.wlist[4] + i4);
+              const int64_t o = (c0 >> 1) + (c1 >> 1) + (c2 >> 1) + (c3 >> 1) + (c4 >> 1);
+              y[o] = ((c0 | c1 | c2 | c3 | c4) & 1) ? T(0) : out;
+            }
+          }
+        }
+      }
+    }
+  }
+}
+
+static alt_status make_reader5(Layout *L, Reader5 *r) {
+  SepDev sd{};
+  const LayoutDesc *desc = nullptr;
+  alt_status st = device_tables(L, &sd, &desc);
+  if (st != ALT_OK) return st;
+  r->sep = L->separable ? 1 : 0;
+  for (int d = 0; d < 5; d++) r->rd[d] = sd.rd[d];
+  r->desc = desc;
+  return ALT_OK;
+}
+
+alt_status simt_conv3d(const ConvProblem &P, cudaStream_t stream) {
+  if (!P.yl->separable) {
+    set_error("output layouts must be separable (no fuse across logical dims); relayout instead");
+    return ALT_E_UNSUPPORTED;
+  }
+  Simt3Args a{};
+  a.N = P.N; a.C = P.C; a.D = P.D; a.H = P.H; a.W = P.W; a.K = P.K; a.T = P.T; a.R = P.R; a.S = P.S;
+  a.Do = P.Do; a.Ho = P.Ho; a.Wo = P.Wo;
+  a.Vd = P.Vd; a.Vh = P.Vh; a.Vw = P.Vw; a.pd = P.pd; a.ph = P.ph; a.pw = P.pw;
+  a.dd = P.dd; a.dh = P.dh; a.dw = P.dw; a.G = P.groups;
+  alt_status st;
+  if ((st = make_reader5(P.xl, &a.xr)) != ALT_OK) return st;
+  if ((st = make_reader5(P.wl, &a.wr)) != ALT_OK) return st;
+  if (P.epi.residual && (st = make_reader5(P.epi.residual_l, &a.rr)) != ALT_OK) return st;
+  SepDev sy{};
+  if ((st = device_tables(P.yl, &sy, nullptr)) != ALT_OK) return st;
+  for (int d = 0; d < 5; d++) { a.yw.wptr[d] = sy.wptr[d]; a.yw.wlist[d] = sy.wlist[d]; }
+  a.scale = P.epi.scale;
+  a.bias = P.epi.bias;
+  a.residual = P.epi.residual;
+  a.act = P.epi.act;
+  const int64_t total = P.N * P.K * P.Do * P.Ho * P.Wo;
+  if (total == 0) return ALT_OK;
+  const int grid = (int)std::min<int64_t>((total + 255) / 256, 148 * 32);
+  if (P.dtype == ALT_BF16)
+    k_simt_conv3d<uint16_t><<<grid, 256, 0, stream>>>(a, (const uint16_t *)P.x, (const uint16_t *)P.w, (uint16_t *)P.y);
+  else
+    k_simt_conv3d<float><<<grid, 256, 0, stream>>>(a, (const float *)P.x, (const float *)P.w, (float *)P.y);
+  count_launch();
+  if (cudaGetLastError() != cudaSuccess) { set_error("simt conv3d launch failed"); return ALT_E_CUDA; }
+  return ALT_OK;
+}
+
+}  // namespace alt

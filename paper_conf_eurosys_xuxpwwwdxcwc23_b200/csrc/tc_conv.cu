@@ -43,7 +43,8 @@
 
 namespace alt {
 
-enum Var { V_N0 = 0, V_PT, V_PR, V_QT, V_QR, V_GT, V_GR, V_R, V_S, V_ONE, NVAR };
+// V_DO / V_T: output depth and depth tap of a 3-D conv (C3D), 0 for conv2d
+enum Var { V_N0 = 0, V_PT, V_PR, V_QT, V_QR, V_GT, V_GR, V_R, V_S, V_ONE, V_DO, V_T, NVAR };
 
 // box-coordinate rule for one tensor map: coord[d] = sum_k coef[d][k] * var[k]
 struct OperandMap {
@@ -82,6 +83,9 @@ struct TcArgs {
   FastDiv f_rsg;
   int32_t nst;           // smem ring stages in use (<= the instantiation's STAGES; tuner knob)
   int32_t hboff;         // halo mode: set the descriptor base-offset field for row-shifted A starts
+  // C3D: tile batch index b = n Do + od (tile_n = 1); taps (t, r, s), RS = R S
+  int32_t Do3, RS3;
+  FastDiv f_Do3, f_RS3;
   int32_t yvec;          // out_mode 0 with 8-channel runs: copies written as 16-byte vectors
   int32_t out_round;     // out_mode 1, round stores: the 8 epilogue warps stage a whole 128-row x
                          // 64-channel round in smem, one thread TMA-stores it (a.O views 128 rows)
@@ -173,7 +177,7 @@ __device__ __forceinline__ uint64_t gtimer() {
 // to the accumulator's magnitude, so the five small pairs are summed while
 // the accumulator is still small and only the hh steps see the full value
 // (measured 6x lower error than hh first).
-__device__ __forceinline__ void slab_decode(const TcArgs &a, int sl, int &r, int &sx, int &gA, int &gB) {
+__device__ __forceinline__ void slab_decode(const TcArgs &a, int sl, int &r, int &sx, int &t, int &gA, int &gB) {
   int rem = sl, pa = 0, pb = 0;
   if (a.pairs) {
     const int pr = (int)a.f_rsg.div((uint32_t)sl);
@@ -181,7 +185,13 @@ __device__ __forceinline__ void slab_decode(const TcArgs &a, int sl, int &r, int
     pa = (0x001102 >> (4 * pr)) & 0xF;
     pb = (0x010120 >> (4 * pr)) & 0xF;
   }
-  const int tap = (int)a.f_Gc.div((uint32_t)rem), g = rem - tap * a.Gc;
+  int tap = (int)a.f_Gc.div((uint32_t)rem);
+  const int g = rem - tap * a.Gc;
+  t = 0;
+  if (a.Do3) {  // C3D: tap = (t, r, s)
+    t = (int)a.f_RS3.div((uint32_t)tap);
+    tap -= t * a.RS3;
+  }
   r = (int)a.f_S.div((uint32_t)tap);
   sx = tap - r * a.S;
   gA = pa * a.Gc + g + a.a_goff;
@@ -382,7 +392,7 @@ __device__ __forceinline__ UnitInfo unit_info(const TcArgs &a, int tile) {
   return u;
 }
 
-struct TileCoord { int n0, p0, q0, k0; };
+struct TileCoord { int n0, p0, q0, k0, d0; };
 // work unit `tile` -> this CTA's 128-row M tile and the unit's N tile; with a
 // CTA pair (CG = 2) a unit is two consecutive M tiles, one per CTA rank
 __device__ __forceinline__ TileCoord tile_coord(const TcArgs &a, int tile, int BN, int CG, int rank) {
@@ -392,7 +402,11 @@ __device__ __forceinline__ TileCoord tile_coord(const TcArgs &a, int tile, int B
   const int tw_i = mt - mw * a.mt_w;
   const int tn_i = (int)a.f_mth.div((uint32_t)mw);
   const int th_i = mw - tn_i * a.mt_h;
-  return {tn_i * a.tile_n, th_i * a.tile_h, tw_i * a.tile_w, nt * BN};
+  if (a.Do3) {  // C3D: the batch index of a tile is (n, od), one output depth slice per tile
+    const int n = (int)a.f_Do3.div((uint32_t)tn_i);
+    return {n, th_i * a.tile_h, tw_i * a.tile_w, nt * BN, tn_i - n * a.Do3};
+  }
+  return {tn_i * a.tile_n, th_i * a.tile_h, tw_i * a.tile_w, nt * BN, 0};
 }
 
 // RV: epilogue reads the residual as 16-byte vectors (a separate
@@ -453,8 +467,8 @@ __global__ void __launch_bounds__(kThreads, 1)
     for (int sl = threadIdx.x; sl < padded_slabs; sl += kThreads) {
       const bool valid = sl < a.total_slabs;
       const int s0 = valid ? sl : 0;
-      int r, sx, gA, gB;
-      slab_decode(a, s0, r, sx, gA, gB);
+      int r, sx, tt, gA, gB;
+      slab_decode(a, s0, r, sx, tt, gA, gB);
 #pragma unroll
       for (int o = 0; o < 2; o++) {
         const OperandMap &om = o == 0 ? a.A : a.B;
@@ -462,8 +476,8 @@ __global__ void __launch_bounds__(kThreads, 1)
         const int gt = (int)om.fg.div((uint32_t)ga), gr = ga - gt * om.divg;
 #pragma unroll
         for (int d = 0; d < 5; d++)
-          tab[sl * 16 + o * 8 + d] = om.coef[d][V_R] * r + om.coef[d][V_S] * sx + om.coef[d][V_GT] * gt +
-                                     om.coef[d][V_GR] * gr;
+          tab[sl * 16 + o * 8 + d] = om.coef[d][V_R] * r + om.coef[d][V_S] * sx + om.coef[d][V_T] * tt +
+                                     om.coef[d][V_GT] * gt + om.coef[d][V_GR] * gr;
         if (!valid) tab[sl * 16 + o * 8] = om.oob0;  // all-zero box (dim 0 has no tile term)
       }
     }
@@ -522,6 +536,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       // B rows of this CTA: its 1/CG share of the unit's BN output channels
       const int pp = isA ? tc.p0 + g_dh : 0, qq = (isA ? tc.q0 : tc.k0 + rank * (BN / CG) + a.b_koff) + g_dw;
       v[V_N0] = isA ? tc.n0 + g_dn : 0;
+      v[V_DO] = isA ? tc.d0 : 0;
       v[V_PT] = (int)om.fp.div((uint32_t)pp); v[V_PR] = pp - v[V_PT] * om.divp;
       v[V_QT] = (int)om.fq.div((uint32_t)qq); v[V_QR] = qq - v[V_QT] * om.divq;
       v[V_ONE] = 1;
@@ -532,7 +547,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           int32_t vt[NVAR];
 #pragma unroll
           for (int k = 0; k < NVAR; k++) vt[k] = v[k];
-          vt[V_R] = 0; vt[V_S] = 0; vt[V_GT] = 0; vt[V_GR] = 0;
+          vt[V_R] = 0; vt[V_S] = 0; vt[V_T] = 0; vt[V_GT] = 0; vt[V_GR] = 0;
           coords(om, vt, base);
         }
         const uint32_t trow = smem_u32(tab) + (uint32_t)((isA ? 0 : 8) * 4 + si * 64);
@@ -572,7 +587,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           const bool valid = slab < a.total_slabs;
           const int sl = valid ? slab : 0;
           int gA, gB;
-          slab_decode(a, sl, v[V_R], v[V_S], gA, gB);
+          slab_decode(a, sl, v[V_R], v[V_S], v[V_T], gA, gB);
           const int ga = isA ? gA : gB;
           v[V_GT] = (int)om.fg.div((uint32_t)ga); v[V_GR] = ga - v[V_GT] * om.divg;
           int32_t c[5];
@@ -728,17 +743,24 @@ __global__ void __launch_bounds__(kThreads, 1)
 #pragma unroll
     for (int d = 0; d < 5; d++) { ocg[d] = a.O.coef[d][V_GT]; ocr[d] = a.O.coef[d][V_GR]; }
     int i = 0;
+    int sb_k0 = -1;  // output-channel block whose scale / bias sSB holds
     for (int tile = unit0; tile < a.num_tiles; tile += unit_step, i++) {
       const int acc = i % NACC, use = i / NACC;
       const UnitInfo ui = unit_info(a, tile);
       const int mn = ui.mn, ksp = ui.sp;
       const TileCoord tc = tile_coord(a, mn, BN, CG, rank);
-      named_bar(2, kEpiThreads);  // every epilogue warp is done with the previous tile's values
-      if (et < BN) {  // explicit shared-space stores (the aligned base is a generic pointer)
-        asm volatile("st.shared.f32 [%0], %1;" ::"r"(sSB + 4u * et), "f"(pf_s) : "memory");
-        asm volatile("st.shared.f32 [%0], %1;" ::"r"(sSB + 4u * (BN + et)), "f"(pf_b) : "memory");
+      // restage scale / bias only when the tile's channel block changes (the
+      // same for every epilogue warp: all walk the same tile sequence); with
+      // one N tile (K_out <= BLOCK_N) the two CTA-wide barriers go away
+      if (tc.k0 != sb_k0) {
+        named_bar(2, kEpiThreads);  // every epilogue warp is done with the previous tile's values
+        if (et < BN) {  // explicit shared-space stores (the aligned base is a generic pointer)
+          asm volatile("st.shared.f32 [%0], %1;" ::"r"(sSB + 4u * et), "f"(pf_s) : "memory");
+          asm volatile("st.shared.f32 [%0], %1;" ::"r"(sSB + 4u * (BN + et)), "f"(pf_b) : "memory");
+        }
+        named_bar(2, kEpiThreads);
+        sb_k0 = tc.k0;
       }
-      named_bar(2, kEpiThreads);
       if (et == 0 && i == ALT_DBG_TILE) { DBG(30); }
       fetch_sb(tile + unit_step, pf_s, pf_b);
       const int n = tc.n0 + rn, p = tc.p0 + rp, q = tc.q0 + rq;
@@ -754,7 +776,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         vo[V_N0] = sn;
         vo[V_PT] = (int)a.O.fp.div((uint32_t)sp); vo[V_PR] = sp - vo[V_PT] * a.O.divp;
         vo[V_QT] = (int)a.O.fq.div((uint32_t)sq); vo[V_QR] = sq - vo[V_QT] * a.O.divq;
-        vo[V_GT] = 0; vo[V_GR] = 0; vo[V_R] = 0; vo[V_S] = 0; vo[V_ONE] = 1;
+        vo[V_GT] = 0; vo[V_GR] = 0; vo[V_R] = 0; vo[V_S] = 0; vo[V_ONE] = 1; vo[V_DO] = tc.d0; vo[V_T] = 0;
         coords(a.O, vo, cbase);
       }
       int64_t yrow = 0;  // out_mode 2: offset of this thread's output row
@@ -1188,7 +1210,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           vo[V_N0] = sn;
           vo[V_PT] = (int)a.O.fp.div((uint32_t)spp); vo[V_PR] = spp - vo[V_PT] * a.O.divp;
           vo[V_QT] = (int)a.O.fq.div((uint32_t)sq); vo[V_QR] = sq - vo[V_QT] * a.O.divq;
-          vo[V_GT] = 0; vo[V_GR] = 0; vo[V_R] = 0; vo[V_S] = 0; vo[V_ONE] = 1;
+          vo[V_GT] = 0; vo[V_GR] = 0; vo[V_R] = 0; vo[V_S] = 0; vo[V_ONE] = 1; vo[V_DO] = tc.d0; vo[V_T] = 0;
           coords(a.O, vo, cbq);
           for (int j = 0; j < nslab; j++) {
             if (kb + (j << lg_sw) >= a.K) break;
@@ -1216,7 +1238,7 @@ __global__ void __launch_bounds__(kThreads, 1)
 }
 
 // =========================================================== host planner ==
-enum Role { R_NONE = 0, R_N, R_H, R_W, R_C, R_TR, R_TS };
+enum Role { R_NONE = 0, R_N, R_H, R_W, R_C, R_TR, R_TS, R_D, R_TT };  // R_D / R_TT: C3D depth / depth tap
 
 struct RoleInfo {
   int role = R_NONE;
@@ -1381,11 +1403,23 @@ static bool build_view(const LView &L, const RoleInfo *roles, int sw, View *out,
         break;
       }
       case R_TR:
-      case R_TS: {
+      case R_TS:
+      case R_TT: {
         if (nphys[d] == 0) break;
         if (nphys[d] != 1 || L.coef[plist[d][0]] != 1 || off != 0) return fail("filter tap dim must be plain");
         VDim &x = add(plist[d][0], 1, 1, 100);
-        x.coef[ri.role == R_TR ? V_R : V_S] = 1;
+        x.coef[ri.role == R_TR ? V_R : (ri.role == R_TS ? V_S : V_T)] = 1;
+        break;
+      }
+      case R_D: {
+        // C3D depth (box 1): input coordinate od Vd - pd + dd t (+ the
+        // layout's own pad offset), output coordinate od; plain dim only
+        if (nphys[d] == 0) { if (ri.V != 1 || ri.win != 1) return fail("depth window on a size-1 dim"); break; }
+        if (nphys[d] != 1 || L.coef[plist[d][0]] != 1) return fail("depth dim must be plain (no split / unfold)");
+        VDim &x = add(plist[d][0], 1, 1, 100);
+        x.coef[V_DO] = ri.V;
+        x.coef[V_T] = ri.tap;
+        x.coef[V_ONE] = (int32_t)(-ri.pad - off);
         break;
       }
       case R_H:
@@ -1771,6 +1805,7 @@ struct TcProblem {
   int64_t R, S, C;            // taps and reduction channels
   OpEpilogue epi;
   int64_t coff = 0, koff = 0; // grouped conv: this group's first input / output channel
+  int64_t T = 1, Do = 0;      // C3D: depth taps, output depth (Do = 0: conv2d / GEMM)
   int pairs = 0;              // fp32 split operands: 6 plane products per slab (0 = bf16)
   bool out_f32 = false;       // fp32 output / residual
 };
@@ -1787,10 +1822,11 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
     k[i++] = (int64_t)P.al->serial; k[i++] = (int64_t)P.bl->serial; k[i++] = (int64_t)P.yl->serial;
     k[i++] = (int64_t)(uintptr_t)P.a; k[i++] = (int64_t)(uintptr_t)P.b; k[i++] = (int64_t)(uintptr_t)P.y;
     k[i++] = P.N; k[i++] = P.K; k[i++] = P.Ho; k[i++] = P.Wo; k[i++] = P.R; k[i++] = P.S; k[i++] = P.C;
-    for (int d = 0; d < 4; d++) {
+    for (int d = 0; d < 5; d++) {
       k[i++] = ((int64_t)P.ra[d].role << 48) | ((int64_t)P.ra[d].V << 32) | ((int64_t)P.ra[d].pad << 16) |
                P.ra[d].win;
     }
+    k[i++] = (P.T << 32) | P.Do;
     k[i++] = (int64_t)(uintptr_t)P.epi.scale; k[i++] = (int64_t)(uintptr_t)P.epi.bias;
     k[i++] = (int64_t)(uintptr_t)P.epi.bias_att;
     k[i++] = (int64_t)(uintptr_t)P.epi.residual;
@@ -1804,6 +1840,7 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       k[i++] = cfg->cta_pair;
       k[i++] = cfg->split_k;
       k[i++] = cfg->split_cluster;
+      k[i++] = cfg->block_k;  // halo request / refusal
     }
     int dev = 0;
     cudaGetDevice(&dev);
@@ -1825,6 +1862,7 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
   struct Cand { int tn, th, tw; };
   std::vector<Cand> cands;
   if (cfg && cfg->tile_n * cfg->tile_h * cfg->tile_w == 128) {
+    if (P.Do && cfg->tile_n != 1) { set_error("tc: C3D tiles hold one output depth slice (tile_n = 1)"); return ALT_E_UNSUPPORTED; }
     cands.push_back({cfg->tile_n, cfg->tile_h, cfg->tile_w});
   } else if (!P.is_conv) {
     cands.push_back({1, 1, 128});
@@ -1994,12 +2032,13 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
         if (st2 != ALT_OK) return st2;
         a.yvec = 1;
       }
+      if (P.Do && a.out_mode != 1) { snprintf(why, 160, "C3D needs a TMA-store output layout"); continue; }
       a.is_conv = P.is_conv;
       a.N = (int32_t)P.N; a.K = (int32_t)P.K; a.Ho = (int32_t)P.Ho; a.Wo = (int32_t)P.Wo;
       a.tile_n = c.tn; a.tile_h = c.th; a.tile_w = c.tw;
       a.mt_h = (int32_t)((P.Ho + c.th - 1) / c.th);
       a.mt_w = (int32_t)((P.Wo + c.tw - 1) / c.tw);
-      const int64_t mt_n = (P.N + c.tn - 1) / c.tn;
+      const int64_t mt_n = (P.N * (P.Do ? P.Do : 1) + c.tn - 1) / c.tn;  // C3D: tiles over (n, od)
       const int64_t mtiles = mt_n * a.mt_h * a.mt_w;
       const int64_t ntiles = (P.K + BN - 1) / BN;
       if (mtiles * ntiles > 0x7fffffff) { set_error("tc: too many tiles"); return ALT_E_UNSUPPORTED; }
@@ -2015,7 +2054,11 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       a.pairs = P.pairs;
       a.out_f32 = P.out_f32 ? 1 : 0;
       if (P.pairs && P.C % sw) { snprintf(why, 160, "split planes not slab-aligned"); continue; }
-      a.total_slabs = (int32_t)((P.pairs ? P.pairs : 1) * P.R * a.S * a.Gc);
+      a.total_slabs = (int32_t)((P.pairs ? P.pairs : 1) * P.T * P.R * a.S * a.Gc);
+      a.Do3 = (int32_t)P.Do;
+      a.RS3 = (int32_t)(P.R * a.S);
+      a.f_Do3 = FastDiv((uint32_t)std::max<int64_t>(1, P.Do));
+      a.f_RS3 = FastDiv((uint32_t)std::max(1, a.RS3));
       pl.hs = hmode ? (int)P.S : 0;
       {
         static const int hboff = [] { const char *e = getenv("ALT_HALO_BOFF"); return e ? atoi(e) : 0; }();
@@ -2268,7 +2311,46 @@ static alt_status tc_gemm_f32(const GemmProblem &P, const alt_kernel_cfg *cfg, c
   return tc_run(T, cfg, stream, used, 1, 1);
 }
 
+// C3D on the tensor cores: the conv2d kernel with a depth role — each M tile
+// is one output depth slice od of one image n (tile_n = 1, tiles over
+// (n, od)), the reduction runs over (t, r, s, channel slab) and the depth tap
+// t moves the A box along D (od Vd - pd + dd t; out of range = TMA zero fill)
+static alt_status tc_conv3d(const ConvProblem &P, const alt_kernel_cfg *cfg, cudaStream_t stream,
+                            alt_kernel_cfg *used) {
+  if (P.dtype != ALT_BF16) { set_error("tc path: C3D is bf16 (fp32 runs on the generic path)"); return ALT_E_UNSUPPORTED; }
+  if (P.groups > 1) { set_error("tc path: grouped C3D runs on the generic path"); return ALT_E_UNSUPPORTED; }
+  if (P.epi.residual) { set_error("tc path: C3D with a residual runs on the generic path"); return ALT_E_UNSUPPORTED; }
+  TcProblem T{};
+  T.is_conv = true;
+  T.al = P.xl; T.bl = P.wl; T.yl = P.yl;
+  T.a = P.x; T.b = P.w; T.y = P.y;
+  // x (n, c, d, h, w); w (k, c, t, r, s); y (n, k, od, oh, ow)
+  T.ra[0].role = R_N;
+  T.ra[1].role = R_C;
+  T.ra[2] = RoleInfo{R_D, 1, P.Vd, P.pd, (int)((P.T - 1) * P.dd + 1), P.dd};
+  T.ra[3] = RoleInfo{R_H, 1, P.Vh, P.ph, (int)((P.R - 1) * P.dh + 1), P.dh};
+  T.ra[4] = RoleInfo{R_W, 1, P.Vw, P.pw, (int)((P.S - 1) * P.dw + 1), P.dw};
+  T.rb[0] = RoleInfo{R_W, 1, 1, 0, 1, 0};
+  T.rb[1].role = R_C;
+  T.rb[2].role = R_TT;
+  T.rb[3].role = R_TR;
+  T.rb[4].role = R_TS;
+  T.ry[0].role = R_N;
+  T.ry[1].role = R_C;
+  T.ry[2] = RoleInfo{R_D, 1, 1, 0, 1, 0};
+  T.ry[3] = RoleInfo{R_H, 1, 1, 0, 1, 0};
+  T.ry[4] = RoleInfo{R_W, 1, 1, 0, 1, 0};
+  T.N = P.N; T.K = P.K; T.Ho = P.Ho; T.Wo = P.Wo;
+  T.R = P.R; T.S = P.S; T.C = P.C;
+  T.T = P.T; T.Do = P.Do;
+  T.epi = P.epi;
+  T.va = lview(*P.xl); T.vb = lview(*P.wl); T.vy = lview(*P.yl);
+  if (P.N * P.Do * P.Ho * P.Wo >= (1ll << 31)) { set_error("tc: too many output pixels"); return ALT_E_UNSUPPORTED; }
+  return tc_run(T, cfg, stream, used, 1, 0);
+}
+
 alt_status tc_conv(const ConvProblem &P, const alt_kernel_cfg *cfg, cudaStream_t stream, alt_kernel_cfg *used) {
+  if (P.c3d) return tc_conv3d(P, cfg, stream, used);
   if (P.dtype == ALT_F32) return tc_conv_f32(P, cfg, stream, used);
   if (P.dtype != ALT_BF16) { set_error("tc path: bf16 / fp32 only"); return ALT_E_UNSUPPORTED; }
   const int64_t G = P.groups < 1 ? 1 : P.groups;

@@ -16,12 +16,17 @@ h = rows[0]
 ki, mi, vi, ui = h.index("Kernel Name"), h.index("Metric Name"), h.index("Metric Value"), h.index("Metric Unit")
 idi = h.index("ID")
 per = {}
-scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "usecond": 1, "nsecond": 1e-3, "msecond": 1e3}
+scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "usecond": 1, "nsecond": 1e-3, "msecond": 1e3,
+         "ns": 1e-3, "us": 1, "ms": 1e3, "B": 1, "KB": 1e3, "MB": 1e6, "GB": 1e9}
 for r in rows[1:]:
-    per.setdefault(int(r[idi]), {})[r[mi]] = float(r[vi].replace(",", "")) * scale.get(r[ui], 1)
+    try:
+        val = float(r[vi].replace(",", ""))
+    except ValueError:
+        continue
+    per.setdefault(int(r[idi]), {})[r[mi]] = val * scale.get(r[ui], 1)
 launches = [per[k] for k in sorted(per)][-23:]  # the last step: one launch per layer
 out = {"source": f"ncu launch list, commit {sys.argv[2]}, L2 flushed before each kernel (cold reads); "
-                 "writes = L2 write bytes from the SMs (dram__bytes_write misses lines still dirty in L2)",
+                 "writes = bytes the kernel stores (TMA stores / L2 write sectors; dram__bytes_write misses lines still dirty in L2)",
        "layers": []}
 tot_r = tot_w = tot_alg = 0.0
 for L, m in zip(nets.RESNET50, launches):
@@ -29,8 +34,12 @@ for L, m in zip(nets.RESNET50, launches):
     alg_r = 2.0 * (32 * L.C * L.H * L.W + L.K * L.C * L.R * L.S)
     alg_w = 2.0 * 32 * L.K * Ho * Wo
     rd = m.get("dram__bytes_read.sum", 0.0)
-    wr = m.get("lts__t_bytes_srcunit_tex_op_write.sum", m.get("dram__bytes_write.sum", 0.0))
-    out["layers"].append({"layer": L.name, "us": m.get("gpu__time_duration.sum"), "dram_read": rd, "l2_write": wr,
+    # bytes the kernel stores: TMA stores (the epilogue's main path), else L2 write sectors
+    wr = max(m.get("l1tex__m_l1tex2xbar_write_bytes_mem_global_op_tma_st.sum", 0.0),
+             32.0 * m.get("lts__t_sectors_op_write.sum", 0.0))
+    us = m.get("gpu__time_duration.sum", 0.0)
+    us = us / 1e3 if us > 1e4 else us  # ncu reports ns or us
+    out["layers"].append({"layer": L.name, "us": us, "dram_read": rd, "bytes_written": wr,
                           "alg_read": alg_r, "alg_write": alg_w})
     tot_r += rd
     tot_w += wr

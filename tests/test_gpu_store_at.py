@@ -109,7 +109,7 @@ def test_matmul_store_at_parity(case, dtype):
     z = torch.empty(Lz.phys_shape, dtype=dtype, device="cuda")
     alt.store_at(Lb, bd, bb, 0, Lz, z)
     La, Lc = alt.Layout((M, K), []), alt.Layout((M, N), [])
-    c = torch.empty((M, N), dtype=dtype, device="cuda")
+    c = torch.full((M, N), float("nan"), dtype=dtype, device="cuda")  # poison: every element must be written
     cfg = {"path": {"tc": alt.PATH_TC, "simt": alt.PATH_SIMT, "auto": alt.PATH_AUTO}[path]}
     alt.matmul_store_at(M, N, K, La, ad, Lz, z, Lc, c, scale=scale.cuda(), residual=rd, residual_l=Lc,
                         act="relu", cfg=cfg)
@@ -125,8 +125,10 @@ def test_matmul_store_at_parity(case, dtype):
     except AssertionError as e:  # locate the wrong outputs (diagnostics for an intermittent failure)
         d = np.abs(got - want) > 0.05 * np.abs(want).max()
         rows, cols = np.where(d.any(1))[0], np.where(d.any(0))[0]
+        unwritten = int(np.isnan(got).sum())
         raise AssertionError(f"{e}; plan {alt.last_plan()}; wrong rows {rows[:8]}..{rows[-8:]} ({len(rows)}), "
-                             f"cols {cols[:8]}..{cols[-8:]} ({len(cols)})") from None
+                             f"cols {cols[:8]}..{cols[-8:]} ({len(cols)}); {unwritten} outputs never written; "
+                             f"sample got {got[rows[0], cols[:3]]} want {want[rows[0], cols[:3]]}") from None
 
 
 def test_matmul_store_at_rejects_separate_bias():
