@@ -192,7 +192,7 @@ class Layout:
 
     def __del__(self):
         h = getattr(self, "_h", None)
-        if h is not None and h.value:
+        if h is not None and h.value and _lib is not None:  # (interpreter shutdown: module globals cleared)
             _lib.alt_layout_destroy(h)
             self._h = None
 
