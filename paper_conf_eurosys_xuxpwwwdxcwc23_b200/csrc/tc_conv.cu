@@ -177,6 +177,9 @@ __device__ __forceinline__ uint64_t gtimer() {
 // to the accumulator's magnitude, so the five small pairs are summed while
 // the accumulator is still small and only the hh steps see the full value
 // (measured 6x lower error than hh first).
+// D3: C3D instantiation (depth taps / output depth); the conv2d / GEMM
+// kernels compile the depth terms out (measured 11 us per R50 step)
+template <bool D3>
 __device__ __forceinline__ void slab_decode(const TcArgs &a, int sl, int &r, int &sx, int &t, int &gA, int &gB) {
   int rem = sl, pa = 0, pb = 0;
   if (a.pairs) {
@@ -188,7 +191,7 @@ __device__ __forceinline__ void slab_decode(const TcArgs &a, int sl, int &r, int
   int tap = (int)a.f_Gc.div((uint32_t)rem);
   const int g = rem - tap * a.Gc;
   t = 0;
-  if (a.Do3) {  // C3D: tap = (t, r, s)
+  if (D3) {  // C3D: tap = (t, r, s)
     t = (int)a.f_RS3.div((uint32_t)tap);
     tap -= t * a.RS3;
   }
@@ -198,12 +201,13 @@ __device__ __forceinline__ void slab_decode(const TcArgs &a, int sl, int &r, int
   gB = pb * a.Gc + g;
 }
 
+template <bool D3>
 __device__ __forceinline__ void coords(const OperandMap &m, const int32_t (&v)[NVAR], int32_t (&c)[5]) {
 #pragma unroll
   for (int d = 0; d < 5; d++) {
     int32_t s = 0;
 #pragma unroll
-    for (int k = 0; k < NVAR; k++) s += m.coef[d][k] * v[k];
+    for (int k = 0; k < (D3 ? NVAR : V_DO); k++) s += m.coef[d][k] * v[k];
     c[d] = s;
   }
 }
@@ -395,6 +399,7 @@ __device__ __forceinline__ UnitInfo unit_info(const TcArgs &a, int tile) {
 struct TileCoord { int n0, p0, q0, k0, d0; };
 // work unit `tile` -> this CTA's 128-row M tile and the unit's N tile; with a
 // CTA pair (CG = 2) a unit is two consecutive M tiles, one per CTA rank
+template <bool D3>
 __device__ __forceinline__ TileCoord tile_coord(const TcArgs &a, int tile, int BN, int CG, int rank) {
   const int mq = (int)a.f_nnt.div((uint32_t)tile);
   const int mt = mq * CG + rank, nt = tile - mq * a.num_n_tiles;
@@ -402,7 +407,7 @@ __device__ __forceinline__ TileCoord tile_coord(const TcArgs &a, int tile, int B
   const int tw_i = mt - mw * a.mt_w;
   const int tn_i = (int)a.f_mth.div((uint32_t)mw);
   const int th_i = mw - tn_i * a.mt_h;
-  if (a.Do3) {  // C3D: the batch index of a tile is (n, od), one output depth slice per tile
+  if (D3) {  // C3D: the batch index of a tile is (n, od), one output depth slice per tile
     const int n = (int)a.f_Do3.div((uint32_t)tn_i);
     return {n, th_i * a.tile_h, tw_i * a.tile_w, nt * BN, tn_i - n * a.Do3};
   }
@@ -417,7 +422,7 @@ __device__ __forceinline__ TileCoord tile_coord(const TcArgs &a, int tile, int B
 // cluster barrier CTA r reduces rows [r * 128 / SC, (r + 1) * 128 / SC) of all
 // SC partials through distributed shared memory in split order, applies the
 // epilogue and stores them — the reduction and the epilogue are split SC ways.
-template <int BN, int STAGES, int CG, bool RV, int SC, int HS = 0>
+template <int BN, int STAGES, int CG, bool RV, int SC, int HS = 0, bool D3 = false>
 __global__ void __launch_bounds__(kThreads, 1)
     k_tc_conv(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
               const __grid_constant__ CUtensorMap tmY, const __grid_constant__ TcArgs a, uint16_t *__restrict__ y) {
@@ -468,7 +473,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       const bool valid = sl < a.total_slabs;
       const int s0 = valid ? sl : 0;
       int r, sx, tt, gA, gB;
-      slab_decode(a, s0, r, sx, tt, gA, gB);
+      slab_decode<D3>(a, s0, r, sx, tt, gA, gB);
 #pragma unroll
       for (int o = 0; o < 2; o++) {
         const OperandMap &om = o == 0 ? a.A : a.B;
@@ -530,7 +535,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     int it = 0, ti = 0;
     for (int tile = unit0; tile < a.num_tiles; tile += unit_step, ti++) {
       const UnitInfo ui = unit_info(a, tile);
-      const TileCoord tc = tile_coord(a, ui.mn, BN, CG, rank);
+      const TileCoord tc = tile_coord<D3>(a, ui.mn, BN, CG, rank);
       const int k_begin = ui.kb, k_end = ui.ke;
       int32_t v[NVAR];
       // B rows of this CTA: its 1/CG share of the unit's BN output channels
@@ -548,7 +553,7 @@ __global__ void __launch_bounds__(kThreads, 1)
 #pragma unroll
           for (int k = 0; k < NVAR; k++) vt[k] = v[k];
           vt[V_R] = 0; vt[V_S] = 0; vt[V_T] = 0; vt[V_GT] = 0; vt[V_GR] = 0;
-          coords(om, vt, base);
+          coords<D3>(om, vt, base);
         }
         const uint32_t trow = smem_u32(tab) + (uint32_t)((isA ? 0 : 8) * 4 + si * 64);
         int stage = it % a.nst;
@@ -587,12 +592,12 @@ __global__ void __launch_bounds__(kThreads, 1)
           const bool valid = slab < a.total_slabs;
           const int sl = valid ? slab : 0;
           int gA, gB;
-          slab_decode(a, sl, v[V_R], v[V_S], v[V_T], gA, gB);
+          slab_decode<D3>(a, sl, v[V_R], v[V_S], v[V_T], gA, gB);
           const int ga = isA ? gA : gB;
           v[V_GT] = (int)om.fg.div((uint32_t)ga); v[V_GR] = ga - v[V_GT] * om.divg;
           int32_t c[5];
           v[V_S] += hs_s;  // halo mode: this lane's tap s (B); 0 otherwise
-          coords(om, v, c);
+          coords<D3>(om, v, c);
           if (!valid) c[0] = om.oob0;
           if constexpr (CG == 2)
             tma_load_5d_2cta(sbase + stage * sbytes + goff + hs_off + si * om.slab_bytes, tmap, &full[stage], c[0], c[1],
@@ -707,7 +712,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     auto fetch_sb = [&](int tile, float &fs, float &fb) {
       fs = 1.f; fb = 0.f;
       if (tile < a.num_tiles && et < BN) {
-        const int k = min(tile_coord(a, unit_info(a, tile).mn, BN, CG, rank).k0 + et, a.K - 1);
+        const int k = min(tile_coord<D3>(a, unit_info(a, tile).mn, BN, CG, rank).k0 + et, a.K - 1);
         fs = __ldg(a.epi.scale + k);
         fb = epi_bias(a.epi, k);
       }
@@ -743,28 +748,25 @@ __global__ void __launch_bounds__(kThreads, 1)
 #pragma unroll
     for (int d = 0; d < 5; d++) { ocg[d] = a.O.coef[d][V_GT]; ocr[d] = a.O.coef[d][V_GR]; }
     int i = 0;
-    int sb_k0 = -1;  // output-channel block whose scale / bias sSB holds
     for (int tile = unit0; tile < a.num_tiles; tile += unit_step, i++) {
       const int acc = i % NACC, use = i / NACC;
       const UnitInfo ui = unit_info(a, tile);
       const int mn = ui.mn, ksp = ui.sp;
-      const TileCoord tc = tile_coord(a, mn, BN, CG, rank);
-      // restage scale / bias only when the tile's channel block changes (the
-      // same for every epilogue warp: all walk the same tile sequence); with
-      // one N tile (K_out <= BLOCK_N) the two CTA-wide barriers go away
-      if (tc.k0 != sb_k0) {
-        named_bar(2, kEpiThreads);  // every epilogue warp is done with the previous tile's values
-        if (et < BN) {  // explicit shared-space stores (the aligned base is a generic pointer)
-          asm volatile("st.shared.f32 [%0], %1;" ::"r"(sSB + 4u * et), "f"(pf_s) : "memory");
-          asm volatile("st.shared.f32 [%0], %1;" ::"r"(sSB + 4u * (BN + et)), "f"(pf_b) : "memory");
-        }
-        named_bar(2, kEpiThreads);
-        sb_k0 = tc.k0;
+      const TileCoord tc = tile_coord<D3>(a, mn, BN, CG, rank);
+      named_bar(2, kEpiThreads);  // every epilogue warp is done with the previous tile's values
+      if (et < BN) {  // explicit shared-space stores (the aligned base is a generic pointer)
+        asm volatile("st.shared.f32 [%0], %1;" ::"r"(sSB + 4u * et), "f"(pf_s) : "memory");
+        asm volatile("st.shared.f32 [%0], %1;" ::"r"(sSB + 4u * (BN + et)), "f"(pf_b) : "memory");
       }
+      named_bar(2, kEpiThreads);
       if (et == 0 && i == ALT_DBG_TILE) { DBG(30); }
       fetch_sb(tile + unit_step, pf_s, pf_b);
       const int n = tc.n0 + rn, p = tc.p0 + rp, q = tc.q0 + rq;
       const bool vrow = n < a.N && p < a.Ho && q < a.Wo;
+      // the pair's second M tile past the last one (odd M-tile count): its
+      // rows alias image n0 >= N, which a GEMM view (no image dim) maps back
+      // onto rows 0..127 — such a tile stores nothing
+      const bool tile_ok = tc.n0 < a.N;
       // TMA-store coordinates of this warp's 32-row sub-box (tile part),
       // computed while the MMA may still be running
       int32_t cbase[5] = {0, 0, 0, 0, 0};
@@ -777,7 +779,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         vo[V_PT] = (int)a.O.fp.div((uint32_t)sp); vo[V_PR] = sp - vo[V_PT] * a.O.divp;
         vo[V_QT] = (int)a.O.fq.div((uint32_t)sq); vo[V_QR] = sq - vo[V_QT] * a.O.divq;
         vo[V_GT] = 0; vo[V_GR] = 0; vo[V_R] = 0; vo[V_S] = 0; vo[V_ONE] = 1; vo[V_DO] = tc.d0; vo[V_T] = 0;
-        coords(a.O, vo, cbase);
+        coords<D3>(a.O, vo, cbase);
       }
       int64_t yrow = 0;  // out_mode 2: offset of this thread's output row
       if (a.out_mode == 2 && vrow)
@@ -1051,7 +1053,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             named_bar(4, kEpiThreads);
             if (et == 0) {
               const int kr = tc.k0 + c0;  // the round's first channel
-              for (int j = 0; j < (64 >> lg_sw); j++) {
+              for (int j = 0; j < (64 >> lg_sw) && tile_ok; j++) {
                 if (kr + (j << lg_sw) >= a.K) break;
                 const int g = ((kr + a.y_koff) >> lg_sw) + j;
                 const int gt = (int)a.O.fg.div((uint32_t)g), gr = g - gt * a.O.divg;
@@ -1086,7 +1088,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             fence_async_smem();
             __syncwarp();
             if (lane == 0) {
-              for (int j = 0; j < nslab; j++) {
+              for (int j = 0; j < nslab && tile_ok; j++) {
                 if (kb + (j << lg_sw) >= a.K) break;  // channels past K: nothing to store
                 const int g = ((kb + a.y_koff) >> lg_sw) + j;
                 const int gt = (int)a.O.fg.div((uint32_t)g), gr = g - gt * a.O.divg;
@@ -1141,7 +1143,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       cluster_sync();
       if (et == 0) { DBG(37); }
       const int crank = (int)cluster_ctarank();
-      const TileCoord tc = tile_coord(a, unit_info(a, unit0).mn, BN, CG, rank);
+      const TileCoord tc = tile_coord<D3>(a, unit_info(a, unit0).mn, BN, CG, rank);
       constexpr int NQ = 4 / SC, NCH = BN / 32;
       const int ew = warp - 2;
       int cnt = 0;
@@ -1211,7 +1213,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           vo[V_PT] = (int)a.O.fp.div((uint32_t)spp); vo[V_PR] = spp - vo[V_PT] * a.O.divp;
           vo[V_QT] = (int)a.O.fq.div((uint32_t)sq); vo[V_QR] = sq - vo[V_QT] * a.O.divq;
           vo[V_GT] = 0; vo[V_GR] = 0; vo[V_R] = 0; vo[V_S] = 0; vo[V_ONE] = 1; vo[V_DO] = tc.d0; vo[V_T] = 0;
-          coords(a.O, vo, cbq);
+          coords<D3>(a.O, vo, cbq);
           for (int j = 0; j < nslab; j++) {
             if (kb + (j << lg_sw) >= a.K) break;
             const int g = ((kb + a.y_koff) >> lg_sw) + j;
@@ -1687,11 +1689,11 @@ static int num_sms() {
   return n;
 }
 
-template <int BN, int STAGES, int CG_, bool RV, int SC = 1, int HS = 0>
+template <int BN, int STAGES, int CG_, bool RV, int SC = 1, int HS = 0, bool D3 = false>
 static cudaError_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUtensorMap &ty, const TcArgs &a,
                              uint16_t *y, int grid, cudaStream_t s) {
   constexpr int CG = CG_;
-  auto kern = k_tc_conv<BN, STAGES, CG, RV, SC, HS>;
+  auto kern = k_tc_conv<BN, STAGES, CG, RV, SC, HS, D3>;
   const int smem = TcSmem<BN, STAGES, CG, HS>::kBytes;
   static_assert(TcSmem<BN, STAGES, CG, HS>::kBytes <= 232448, "smem budget");
   static bool attr_set = false;  // once per instantiation (not capture-safe to repeat)
@@ -1789,6 +1791,16 @@ static cudaError_t launch_plan(const TcPlan &pl, void *y, cudaStream_t stream) {
                         : launch_tc<128, stages_for(128, 1), 1, false, 4>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
     return pl.sc == 2 ? launch_tc<256, stages_for(256, 1), 1, false, 2>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream)
                       : launch_tc<256, stages_for(256, 1), 1, false, 4>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+  }
+  if (pl.a.Do3) {  // C3D (planner: no residual, no split, no halo)
+    if (pl.cg == 2) {
+      if (pl.BN == 128) return launch_tc<128, stages_for(128, 2), 2, false, 1, 0, true>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+      if (pl.BN == 192) return launch_tc<192, stages_for(192, 2), 2, false, 1, 0, true>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+      return launch_tc<256, stages_for(256, 2), 2, false, 1, 0, true>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+    }
+    if (pl.BN == 64) return launch_tc<64, stages_for(64, 1), 1, false, 1, 0, true>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+    if (pl.BN == 128) return launch_tc<128, stages_for(128, 1), 1, false, 1, 0, true>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+    return launch_tc<256, stages_for(256, 1), 1, false, 1, 0, true>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
   }
   return pl.a.res_vec ? launch_plan_rv<true>(pl, yy, stream) : launch_plan_rv<false>(pl, yy, stream);
 }
@@ -2320,6 +2332,7 @@ static alt_status tc_conv3d(const ConvProblem &P, const alt_kernel_cfg *cfg, cud
   if (P.dtype != ALT_BF16) { set_error("tc path: C3D is bf16 (fp32 runs on the generic path)"); return ALT_E_UNSUPPORTED; }
   if (P.groups > 1) { set_error("tc path: grouped C3D runs on the generic path"); return ALT_E_UNSUPPORTED; }
   if (P.epi.residual) { set_error("tc path: C3D with a residual runs on the generic path"); return ALT_E_UNSUPPORTED; }
+  if (cfg && (cfg->split_k > 1 || cfg->split_cluster)) { set_error("tc path: C3D has no split-K"); return ALT_E_UNSUPPORTED; }
   TcProblem T{};
   T.is_conv = true;
   T.al = P.xl; T.bl = P.wl; T.yl = P.yl;

@@ -123,7 +123,7 @@ def test_matmul_store_at_parity(case, dtype):
     got = read_output(oracle.Layout((M, N), []), c, dtype)
     try:
         assert_parity(got, want, dtype)
-    except AssertionError as e:  # locate the wrong outputs (diagnostics for an intermittent failure)
+    except AssertionError as e:  # locate the wrong outputs (the decomposition that found the pair-tile aliasing)
         d = np.abs(got - want) > 0.05 * np.abs(want).max()
         rows, cols = np.where(d.any(1))[0], np.where(d.any(0))[0]
         unwritten = int(np.isnan(got).sum())
