@@ -37,6 +37,34 @@ struct SepPair {
   const int64_t *rd[kMaxL];    // src owner offsets
 };
 
+template <typename T>
+__device__ __forceinline__ uint4 ld16(const T *p) { return __ldg(reinterpret_cast<const uint4 *>(p)); }
+
+// Warp-cooperative store of per-lane contiguous runs.  Lane l holds NVO
+// 16-byte vectors forming one contiguous dst run that starts at element
+// offset off (-1: the lane stores nothing).  Written straight from registers,
+// store instruction k would touch 32 runs 16 bytes each (32 partial lines per
+// instruction); staged through this warp's shared buffer st[32 * NVO], store
+// instruction k moves the warp's vectors [32k, 32k + 32) in lane order — one
+// 512-byte span when the lanes' runs are adjacent, which they are except
+// where a warp straddles a batch boundary.  Slots are XOR-swizzled so both
+// the staging writes and the reads hit distinct banks per 8-lane phase.
+template <typename T, int NVO>
+__device__ __forceinline__ void warp_store_runs(uint4 *st, const uint4 (&w)[NVO], int64_t off, T *dst, int lane) {
+  constexpr int VE = 16 / sizeof(T);
+  auto key = [](int s) { return ((s * NVO) >> 3) & (NVO - 1); };
+#pragma unroll
+  for (int k = 0; k < NVO; k++) st[lane * NVO + (k ^ key(lane))] = w[k];
+  __syncwarp();
+#pragma unroll
+  for (int k = 0; k < NVO; k++) {
+    const int j = k * 32 + lane, s = j / NVO, r = j % NVO;
+    const long long so = __shfl_sync(0xffffffffu, (long long)off, s);
+    if (so >= 0) *reinterpret_cast<uint4 *>(dst + so + (int64_t)r * VE) = st[s * NVO + (r ^ key(s))];
+  }
+  __syncwarp();
+}
+
 // ------------------------------------------------------------------ K_SEP --
 template <typename T, int V>
 __global__ void __launch_bounds__(256) k_relayout_sep(SepPair P, const T *__restrict__ src,
@@ -540,18 +568,29 @@ __global__ void __launch_bounds__(256) k_relayout_row(RowPlan R, const T *__rest
 
 
 // K_ROW, identity suffix (dst positions = the b indices in order, e.g. the
-// padded-channel image layout N C/8 H W 8c) with 16-byte X-runs: no staging —
+// padded-channel image layout N C/8 H W 8c) with 16- or 32-byte X-runs: no
+// shared-memory transpose —
 // a thread loads one 16-byte b-vector of each of the X rows (pad rows are
 // zeros), transposes it in registers and stores the V runs, which are
 // adjacent in dst.  Neighbouring threads take neighbouring b-vectors.
-template <typename T>
+// X = V (16-byte runs) or, for fp32, 2 V (32-byte runs: 8 channels); a
+// thread's V runs (V X elements) are one contiguous dst span, written through
+// warp_store_runs.
+template <typename T, int X>
 __global__ void __launch_bounds__(256) k_relayout_row_ident(RowPlan R, const T *__restrict__ src,
                                                             T *__restrict__ dst, uint32_t nthr) {
   pdl_wait();
   constexpr int V = 16 / sizeof(T);
-  constexpr int X = V;  // 16-byte runs
+  constexpr int NVO = X;  // 16-byte output vectors per thread: V runs of X elements
+  __shared__ uint4 stage[8][32 * NVO];
+  const int lane = threadIdx.x & 31;
+  uint4 *st = stage[threadIdx.x >> 5];
   const uint32_t nv = (uint32_t)(R.Lb / V);
-  for (uint32_t t = blockIdx.x * blockDim.x + threadIdx.x; t < nthr; t += gridDim.x * blockDim.x) {
+  for (uint32_t t0 = blockIdx.x * blockDim.x + (threadIdx.x & ~31u); t0 < nthr; t0 += gridDim.x * blockDim.x) {
+    const uint32_t t = t0 + lane;
+    uint4 w[NVO];
+    int64_t off = -1;
+    if (t < nthr) {
     const uint32_t o = t / nv, bv = t - o * nv;
     uint32_t rem = o;
     int32_t combo[kMaxL];
@@ -578,23 +617,396 @@ __global__ void __launch_bounds__(256) k_relayout_row_ident(RowPlan R, const T *
       u[j] = ai < 0 ? make_uint4(0u, 0u, 0u, 0u)
                     : __ldg(reinterpret_cast<const uint4 *>(src + base + __ldg(R.rd[R.a] + ai) + (int64_t)bv * V));
     }
-    T *d = dst + (int64_t)o * (R.npos * X) + (int64_t)bv * V * X;
+    // run k = element k of rows 0 .. X-1 (X / V vectors)
 #pragma unroll
     for (int k = 0; k < V; k++) {
-      uint32_t w[4];
-      if constexpr (sizeof(T) == 2) {
-        const uint32_t sel = (k & 1) ? 0x7632u : 0x5410u;
 #pragma unroll
-        for (int jp = 0; jp < 4; jp++)
-          w[jp] = __byte_perm(reinterpret_cast<const uint32_t *>(&u[2 * jp])[k >> 1],
-                              reinterpret_cast<const uint32_t *>(&u[2 * jp + 1])[k >> 1], sel);
-      } else {
+      for (int h = 0; h < X / V; h++) {
+        uint32_t ww[4];
+        if constexpr (sizeof(T) == 2) {
+          const uint32_t sel = (k & 1) ? 0x7632u : 0x5410u;
 #pragma unroll
-        for (int j = 0; j < 4; j++) w[j] = reinterpret_cast<const uint32_t *>(&u[j])[k];
+          for (int jp = 0; jp < 4; jp++)
+            ww[jp] = __byte_perm(reinterpret_cast<const uint32_t *>(&u[h * V + 2 * jp])[k >> 1],
+                                 reinterpret_cast<const uint32_t *>(&u[h * V + 2 * jp + 1])[k >> 1], sel);
+        } else {
+#pragma unroll
+          for (int j = 0; j < 4; j++) ww[j] = reinterpret_cast<const uint32_t *>(&u[h * V + j])[k];
+        }
+        w[k * (X / V) + h] = make_uint4(ww[0], ww[1], ww[2], ww[3]);
       }
-      *reinterpret_cast<uint4 *>(d + k * X) = make_uint4(w[0], w[1], w[2], w[3]);
+    }
+    off = (int64_t)o * (R.npos * X) + (int64_t)bv * V * X;
+    }
+    warp_store_runs<T, NVO>(st, w, off, dst, lane);
+  }
+}
+
+// ------------------------------------------------------------------ K_WIN --
+// Group form of K_ROW for the conv input templates (pad + unfold of H and W
+// + NCHW[x]c, Fig. 5 / §5.1; window-folded images).  dst's
+// innermost physical dims G = [pg, p0] (p0: the X-run of logical dim a) are
+// one contiguous dst block per outer index.  The rows the block reads are
+// the combinations of G's dims not owned by the src-contiguous dim b (x the
+// X run); each is staged once per block over the b window the block touches
+// (whole rows when G holds every b dim), 16-byte coalesced loads, pad rows
+// as zeros.  The write phase then emits every X-run of the block as 16-byte
+// vectors with one b-table lookup per run.  K_ROW stages a separate window
+// per innermost outer index (for the 8 x 8 unfold template: 10 x overlapping
+// windows and per-element lookups; ncu: instruction-bound at 62 % SM busy).
+constexpr int kWinG = 6;
+struct WinPlan {
+  int32_t a, b;
+  int32_t X, Lb, LbS, span;    // run length, b extent, staged row pitch, window (elements)
+  int32_t nvs;                 // 16-byte vectors per staged row
+  int32_t ng;                  // G dims above p0 (dst order, innermost last)
+  FastDiv gdiv[kWinG];
+  int32_t gowner[kWinG], grad[kWinG];
+  int32_t nrq;                 // row groups (product of G's non-b dims above p0)
+  int32_t nrun;                // X-runs per block
+  int32_t nbg;                 // combinations of G's b coordinates
+  int32_t nout;
+  FastDiv odiv[kMaxP];
+  int32_t oowner[kMaxP], orad[kMaxP];
+  uint32_t nouter;
+  int32_t lrank;
+  const int32_t *rev[kMaxL];
+  const int64_t *rd[kMaxL];
+  const int32_t *blo;          // window start per outer b combo
+  FastDiv f_x, f_nvs;
+  // per-block offset tables: for every logical dim d != b owning G dims (a
+  // always: p0 is its innermost), T_d[local] = rd_d[rev_d(outer_d + G part)]
+  // over d's G coordinates (mixed radix, innermost first); a staged row's src
+  // offset is base + sum_d T_d[local_d] — a few dozen lookups per block
+  // instead of a dependent rev -> rd chain per dim for each of its rows
+  int32_t nt;                  // tables
+  int32_t tdim[kMaxL];         // logical dim of table t
+  int32_t toff[kMaxL + 1];     // entry offsets (prefix sums)
+  int32_t tn[kMaxL];           // coordinates of table t
+  FastDiv text[kMaxL][kWinG + 1];
+  int32_t trad[kMaxL][kWinG + 1];
+  int32_t gti[kWinG];          // table of G dim k's owner (-1: b)
+  int32_t gmul[kWinG];         // place value of G dim k in its table's local index
+  int32_t ati;                 // table of a (local index = a's G part * X + j)
+  uint32_t notab;              // bit d: logical dim d (!= b) has no G dims (block base only)
+};
+
+// outer index o -> per-logical-dim combos of the outer dims
+__device__ __forceinline__ void win_outer(const WinPlan &P, uint32_t o, int32_t (&combo)[kMaxL]) {
+#pragma unroll
+  for (int d = 0; d < kMaxL; d++) combo[d] = 0;
+  for (int k = P.nout - 1; k >= 0; k--) {
+    uint32_t q, r;
+    P.odiv[k].divmod(o, q, r);
+    combo[P.oowner[k]] += (int32_t)r * P.orad[k];
+    o = q;
+  }
+}
+
+template <typename T, int X>
+__global__ void __launch_bounds__(256) k_relayout_win(WinPlan P, const T *__restrict__ src, T *__restrict__ dst) {
+  extern __shared__ __align__(16) unsigned char win_smem[];
+  const int ntab = P.toff[P.nt];
+  int64_t *s_tab = reinterpret_cast<int64_t *>(win_smem);                     // [ntab]
+  int32_t *s_bsl = reinterpret_cast<int32_t *>(win_smem + (size_t)ntab * 8);  // [nbg] run slot of G's b coords
+  // runs staged transposed: [rq][window slot][X], the slots of a row
+  // XOR-swizzled within each V-run group (conflict-free staging stores)
+  uint4 *runs = reinterpret_cast<uint4 *>(win_smem + (((size_t)ntab * 8 + (size_t)P.nbg * 4 + 15) & ~size_t(15)));
+  __shared__ int64_t s_base;
+  constexpr int V = 16 / sizeof(T);
+  constexpr int NV = X / V;                         // 16-byte vectors per run (1 or 2)
+  auto slot = [](int bl) { return bl ^ ((bl / V) & (V - 1)); };
+  pdl_wait();
+  const int64_t blk = (int64_t)P.nrun * X;
+  for (uint32_t o = blockIdx.x; o < P.nouter; o += gridDim.x) {
+    int32_t oc[kMaxL];
+    win_outer(P, o, oc);
+    const int lo = __ldg(P.blo + oc[P.b]);
+    __syncthreads();  // the previous block's runs are consumed
+    if (threadIdx.x == 0) {
+      int64_t base = 0;
+      for (int d = 0; d < P.lrank; d++) {
+        if (!((P.notab >> d) & 1u)) continue;
+        const int32_t i = __ldg(P.rev[d] + oc[d]);
+        if (i < 0) { base = -1; break; }
+        base += __ldg(P.rd[d] + i);
+      }
+      s_base = base;
+    }
+    for (int e = threadIdx.x; e < ntab; e += blockDim.x) {
+      int t = 0;
+      while (e >= P.toff[t + 1]) t++;
+      uint32_t rem = (uint32_t)(e - P.toff[t]);
+      int32_t sub = 0;
+      for (int k = 0; k < P.tn[t]; k++) {
+        uint32_t q, r;
+        P.text[t][k].divmod(rem, q, r);
+        sub += (int32_t)r * P.trad[t][k];
+        rem = q;
+      }
+      const int d = P.tdim[t];
+      const int32_t i = __ldg(P.rev[d] + oc[d] + sub);
+      s_tab[e] = i < 0 ? -1 : __ldg(P.rd[d] + i);
+    }
+    for (int g = threadIdx.x; g < P.nbg; g += blockDim.x) {
+      uint32_t rem = (uint32_t)g;
+      int32_t cb = oc[P.b];
+      for (int k = P.ng - 1; k >= 0; k--) {
+        if (P.gowner[k] != P.b) continue;
+        uint32_t q, rr;
+        P.gdiv[k].divmod(rem, q, rr);
+        cb += (int32_t)rr * P.grad[k];
+        rem = q;
+      }
+      const int32_t bi = __ldg(P.rev[P.b] + cb);
+      s_bsl[g] = bi < 0 ? -1 : slot(bi - lo);
+    }
+    __syncthreads();
+    const int64_t base = s_base;
+    // stage: item (rq, b-vector v) loads the X rows' 16-byte vectors at
+    // b0 = lo + v V and transposes them into V runs of X elements
+    for (int e = threadIdx.x; e < P.nrq * P.nvs; e += blockDim.x) {
+      const int rq = (int)P.f_nvs.div((uint32_t)e), v = e - rq * P.nvs;
+      const int b0 = lo + v * V;
+      int loc[kMaxL];
+#pragma unroll
+      for (int t = 0; t < kMaxL; t++) loc[t] = 0;
+      uint32_t rem = (uint32_t)rq;
+      for (int k = P.ng - 1; k >= 0; k--) {
+        if (P.gti[k] < 0) continue;
+        uint32_t q, rr;
+        P.gdiv[k].divmod(rem, q, rr);
+        loc[P.gti[k]] += (int)rr * P.gmul[k];
+        rem = q;
+      }
+      int64_t off = base;
+      for (int t = 0; t < P.nt && off >= 0; t++) {
+        if (t == P.ati) continue;
+        const int64_t x = s_tab[P.toff[t] + loc[t]];
+        off = x < 0 ? -1 : off + x;
+      }
+      const int64_t *ta = s_tab + P.toff[P.ati] + loc[P.ati] * X;
+      uint4 u[X];
+#pragma unroll
+      for (int j = 0; j < X; j++) {
+        const int64_t xa = ta[j];
+        u[j] = (off < 0 || xa < 0 || b0 >= P.Lb) ? make_uint4(0u, 0u, 0u, 0u) : ld16(src + off + xa + b0);
+      }
+      uint4 *rrow = runs + (size_t)rq * P.LbS * NV;
+#pragma unroll
+      for (int k = 0; k < V; k++) {
+        const int sl = slot(v * V + k);
+#pragma unroll
+        for (int h = 0; h < NV; h++) {
+          uint32_t ww[4];
+          if constexpr (sizeof(T) == 2) {
+            const uint32_t sel = (k & 1) ? 0x7632u : 0x5410u;
+#pragma unroll
+            for (int jp = 0; jp < 4; jp++)
+              ww[jp] = __byte_perm(reinterpret_cast<const uint32_t *>(&u[h * V + 2 * jp])[k >> 1],
+                                   reinterpret_cast<const uint32_t *>(&u[h * V + 2 * jp + 1])[k >> 1], sel);
+          } else {
+#pragma unroll
+            for (int jj = 0; jj < 4; jj++) ww[jj] = reinterpret_cast<const uint32_t *>(&u[h * V + jj])[k];
+          }
+          rrow[sl * NV + h] = make_uint4(ww[0], ww[1], ww[2], ww[3]);
+        }
+      }
+    }
+    __syncthreads();
+    T *db = dst + (int64_t)o * blk;
+    for (int q = threadIdx.x; q < P.nrun; q += blockDim.x) {
+      uint32_t rem = (uint32_t)q;
+      int rq = 0, rmul = 1, gb = 0, gmul = 1;
+      for (int k = P.ng - 1; k >= 0; k--) {
+        uint32_t qq, rr;
+        P.gdiv[k].divmod(rem, qq, rr);
+        if (P.gowner[k] == P.b) { gb += (int)rr * gmul; gmul *= (int)P.gdiv[k].d; }
+        else { rq += (int)rr * rmul; rmul *= (int)P.gdiv[k].d; }
+        rem = qq;
+      }
+      const int sl = s_bsl[gb];
+      const uint4 *rr = runs + ((size_t)rq * P.LbS + (sl < 0 ? 0 : sl)) * NV;
+#pragma unroll
+      for (int h = 0; h < NV; h++)
+        *reinterpret_cast<uint4 *>(db + (int64_t)q * X + h * V) = sl < 0 ? make_uint4(0u, 0u, 0u, 0u) : rr[h];
     }
   }
+}
+
+// host side of K_WIN: false (nothing launched) when the layouts do not fit
+static bool win_launch(Layout *S, const void *src, Layout *D, void *dst, int wb, const SepDev &ss,
+                       const SepDev &ds, cudaStream_t stream, int nsm, alt_status *st) {
+  const int V = 16 / wb;
+  if (D->prank < 3 || D->pnumel >= (1ll << 31)) return false;
+  if ((reinterpret_cast<uintptr_t>(dst) | reinterpret_cast<uintptr_t>(src)) & 15) return false;
+  const int p0 = D->prank - 1;
+  const int a = D->pdim_owner[p0];
+  const int b = S->pdim_owner[S->prank - 1];
+  if (D->pdim_rad[p0] != 1 || a == b || D->pdim_owner[p0 - 1] != b) return false;
+  const int64_t X = D->pshape[p0];
+  if (!(X * wb == 16 || X * wb == 32)) return false;
+  // measured (R3, 256 x 64 x 56 x 56): bf16 149 us vs K_ROW 170 us; fp32
+  // 250 vs 198 (its whole-row group does not fit the budget), so fp32 stays
+  // on K_ROW unless forced (ALT_WIN_FP32=1)
+  static const bool win_f32 = getenv("ALT_WIN_FP32") != nullptr;
+  if (wb == 4 && !win_f32) return false;
+  const int64_t Lb = S->lshape[b];
+  if (Lb % V || Lb >= (1 << 20)) return false;
+  for (int64_t i = 0; i < Lb; i++) if (S->rd[b][i] != i) return false;  // b contiguous in src
+  for (int d = 0; d < S->lrank; d++) {
+    if (d == b) continue;
+    for (int64_t o : S->rd[d]) if (o >= 0 && o % V) return false;   // rows start on 16 bytes
+  }
+  // the largest group G = [pg, p0] whose staged rows fit the budget
+  // budget: staged bytes per CTA (a larger group removes the window overlap
+  // between neighbouring blocks but lowers residency); developer knob
+  static const size_t budget = getenv("ALT_WIN_BUDGET") ? (size_t)atol(getenv("ALT_WIN_BUDGET")) : 110 * 1000;
+  int best_pg = -1;
+  int64_t best_span = 0, best_nrq = 0, best_ngb = 0;
+  std::vector<int32_t> best_blo;
+  for (int pg = p0 - 1; pg >= 1 && p0 - pg <= kWinG; pg--) {
+    int64_t nrq = 1;
+    for (int p = pg; p < p0; p++) if (D->pdim_owner[p] != b) nrq *= D->pshape[p];
+    // window per outer b combo: the b indices the block's G coordinates reach
+    std::vector<int> bo, bg;
+    for (int p = 0; p < pg; p++) if (D->pdim_owner[p] == b) bo.push_back(p);
+    for (int p = pg; p < p0; p++) if (D->pdim_owner[p] == b) bg.push_back(p);
+    int64_t nob = 1, ngb = 1;
+    for (int p : bo) nob *= D->pshape[p];
+    for (int p : bg) ngb *= D->pshape[p];
+    if (nob * ngb > (1 << 22)) continue;
+    std::vector<int32_t> blo((size_t)D->rev[b].size(), 0);
+    int64_t span = 0;
+    for (int64_t k = 0; k < nob; k++) {
+      int64_t rem = k, ob = 0;
+      for (int t = (int)bo.size() - 1; t >= 0; t--) {
+        ob += (rem % D->pshape[bo[(size_t)t]]) * D->pdim_rad[bo[(size_t)t]];
+        rem /= D->pshape[bo[(size_t)t]];
+      }
+      int64_t lo = INT64_MAX, hi = -1;
+      for (int64_t g = 0; g < ngb; g++) {
+        int64_t rg = g, cbv = ob;
+        for (int t = (int)bg.size() - 1; t >= 0; t--) {
+          cbv += (rg % D->pshape[bg[(size_t)t]]) * D->pdim_rad[bg[(size_t)t]];
+          rg /= D->pshape[bg[(size_t)t]];
+        }
+        const int32_t bi = D->rev[b][(size_t)cbv];
+        if (bi >= 0) { lo = std::min<int64_t>(lo, bi); hi = std::max<int64_t>(hi, bi); }
+      }
+      if (hi < 0) lo = hi = 0;
+      lo = lo / V * V;
+      blo[(size_t)ob] = (int32_t)lo;
+      span = std::max<int64_t>(span, hi - lo + 1);
+    }
+    span = (span + V - 1) / V * V;
+    const size_t smem = (((size_t)nrq * X * 8 + (size_t)ngb * 4 + 15) & ~size_t(15)) + (size_t)nrq * X * span * wb;
+    if (smem > budget || nrq * X > 8192) break;
+    best_pg = pg; best_span = span; best_nrq = nrq; best_ngb = ngb; best_blo.swap(blo);
+  }
+  if (best_pg < 0 || best_nrq == 1) return false;  // one row group: K_ROW's forms serve it
+  const int pg = best_pg;
+  WinPlan P{};
+  int tabn = 0;
+  P.a = a; P.b = b;
+  P.X = (int32_t)X; P.Lb = (int32_t)Lb; P.span = (int32_t)best_span;
+  const int64_t LbS = best_span;  // run slots per staged row group
+  P.LbS = (int32_t)LbS;
+  P.nvs = (int32_t)(best_span / V);
+  P.ng = p0 - pg;
+  int64_t nrun = 1;
+  for (int p = pg; p < p0; p++) {
+    const int k = p - pg;
+    P.gdiv[k] = FastDiv((uint32_t)D->pshape[p]);
+    P.gowner[k] = D->pdim_owner[p];
+    P.grad[k] = D->pdim_rad[p];
+    nrun *= D->pshape[p];
+  }
+  P.nrq = (int32_t)best_nrq;
+  P.nrun = (int32_t)nrun;
+  int k = 0;
+  int64_t nouter = 1;
+  for (int p = 0; p < pg; p++) {
+    P.odiv[k] = FastDiv((uint32_t)D->pshape[p]);
+    P.oowner[k] = D->pdim_owner[p];
+    P.orad[k] = D->pdim_rad[p];
+    nouter *= D->pshape[p];
+    k++;
+  }
+  P.nout = k;
+  P.nouter = (uint32_t)nouter;
+  P.lrank = D->lrank;
+  for (int d = 0; d < D->lrank; d++) { P.rev[d] = ds.rev[d]; P.rd[d] = ss.rd[d]; }
+  P.f_x = FastDiv((uint32_t)X);
+  P.f_nvs = FastDiv((uint32_t)P.nvs);
+  P.nbg = (int32_t)best_ngb;
+  {
+    // per-logical-dim offset tables over the G coordinates (see WinPlan)
+    int nt = 0, tot = 0;
+    P.notab = 0;
+    for (int d = 0; d < D->lrank; d++) {
+      if (d == b) continue;
+      std::vector<int> gd;  // G dims of d above p0, innermost first
+      for (int p = p0 - 1; p >= pg; p--) if (D->pdim_owner[p] == d) gd.push_back(p);
+      if (d != a && gd.empty()) { P.notab |= 1u << d; continue; }
+      if (nt >= kMaxL || (int)gd.size() + 1 > kWinG + 1) return false;
+      P.tdim[nt] = d;
+      P.toff[nt] = tot;
+      int k = 0, sz = 1;
+      if (d == a) { P.text[nt][k] = FastDiv((uint32_t)X); P.trad[nt][k] = 1; k++; sz *= (int)X; P.ati = nt; }
+      for (int p : gd) {
+        P.text[nt][k] = FastDiv((uint32_t)D->pshape[p]);
+        P.trad[nt][k] = D->pdim_rad[p];
+        P.gti[p - pg] = nt;
+        P.gmul[p - pg] = sz / (d == a ? (int)X : 1);
+        sz *= (int)D->pshape[p];
+        k++;
+      }
+      P.tn[nt] = k;
+      tot += sz;
+      nt++;
+    }
+    for (int p = pg; p < p0; p++) if (D->pdim_owner[p] == b) P.gti[p - pg] = -1;
+    P.nt = nt;
+    P.toff[nt] = tot;
+    if (tot > 4096) return false;
+    tabn = tot;
+  }
+  const size_t smem = (((size_t)tabn * 8 + (size_t)best_ngb * 4 + 15) & ~size_t(15)) + (size_t)best_nrq * X * LbS * wb;
+  // device copy of the window-start table, cached per (layout pair, device)
+  static std::mutex mu;
+  struct Ent { uint64_t s, d; int dev; int32_t *ptr; };
+  static std::vector<Ent> cache;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  int32_t *dt = nullptr;
+  {
+    std::lock_guard<std::mutex> g(mu);
+    for (auto &e : cache) if (e.s == S->serial && e.d == D->serial && e.dev == dev) dt = e.ptr;
+    if (!dt) {
+      if (cudaMalloc(&dt, best_blo.size() * 4) != cudaSuccess) { cudaGetLastError(); return false; }
+      if (cudaMemcpy(dt, best_blo.data(), best_blo.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess) { cudaGetLastError(); return false; }
+      cache.push_back({S->serial, D->serial, dev, dt});
+    }
+  }
+  P.blo = dt;
+  const int per_sm = std::max(1, (int)std::min<size_t>(8, (size_t)(200 * 1024) / smem));
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(nouter, (int64_t)nsm * per_sm));
+#define WIN_LAUNCH(T, XX)                                                                                 \
+  do {                                                                                                   \
+    cudaFuncSetAttribute(k_relayout_win<T, XX>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem); \
+    launch_pdl(k_relayout_win<T, XX>, grid, 256, smem, stream, P, (const T *)src, (T *)dst);             \
+  } while (0)
+  if (wb == 2) {
+    if (X == 8) WIN_LAUNCH(uint16_t, 8); else WIN_LAUNCH(uint16_t, 16);
+  } else {
+    if (X == 4) WIN_LAUNCH(uint32_t, 4); else WIN_LAUNCH(uint32_t, 8);
+  }
+#undef WIN_LAUNCH
+  count_launch();
+  *st = cudaGetLastError() == cudaSuccess ? ALT_OK : ALT_E_CUDA;
+  if (*st != ALT_OK) set_error("relayout (window group) launch failed");
+  return true;
 }
 
 // position q of the suffix holds b index q (no pad / unfold of b)
@@ -728,17 +1140,19 @@ static bool row_launch(Layout *S, const void *src, Layout *D, void *dst, int wb,
     for (int64_t o : S->rd[d]) if (o >= 0 && o % V) { vl = false; break; }
   }
   R.vec_load = vl ? 1 : 0;
-  // identity suffix with 16-byte runs: the staging-free register-transpose form
+  // identity suffix with 16- or 32-byte runs: the register-transpose form
   {
-    bool ident = R.bstatic && npos == Lb && X * wb == 16 && vl0;
+    bool ident = R.bstatic && npos == Lb && (X * wb == 16 || (X * wb == 32 && wb == 4)) && vl0;
     for (int64_t q = 0; q < npos && ident; q++) ident = bmap_static_is(D, b, sbc, q);
     static const bool no_id = getenv("ALT_RELAYOUT_NOID") != nullptr;  // developer A/B knob
     if (ident && !no_id) {
       const int64_t nthr = nouter * (Lb / V);
       if (nthr < (1ll << 31)) {
         const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((nthr + 255) / 256, (int64_t)nsm * 16));
-        if (wb == 2) launch_pdl(k_relayout_row_ident<uint16_t>, grid, 256, 0, stream, R, (const uint16_t *)src, (uint16_t *)dst, (uint32_t)nthr);
-        else launch_pdl(k_relayout_row_ident<uint32_t>, grid, 256, 0, stream, R, (const uint32_t *)src, (uint32_t *)dst, (uint32_t)nthr);
+        const bool x2 = X * wb == 32;
+        if (wb == 2 && !x2) launch_pdl(k_relayout_row_ident<uint16_t, 8>, grid, 256, 0, stream, R, (const uint16_t *)src, (uint16_t *)dst, (uint32_t)nthr);
+        else if (!x2) launch_pdl(k_relayout_row_ident<uint32_t, 4>, grid, 256, 0, stream, R, (const uint32_t *)src, (uint32_t *)dst, (uint32_t)nthr);
+        else launch_pdl(k_relayout_row_ident<uint32_t, 8>, grid, 256, 0, stream, R, (const uint32_t *)src, (uint32_t *)dst, (uint32_t)nthr);
         count_launch();
         *st = cudaGetLastError() == cudaSuccess ? ALT_OK : ALT_E_CUDA;
         if (*st != ALT_OK) set_error("relayout (row, identity) launch failed");
@@ -844,8 +1258,6 @@ static bool refine_perm(const Layout &S, const Layout &D, std::vector<RDim> &out
   return true;
 }
 
-template <typename T>
-__device__ __forceinline__ uint4 ld16(const T *p) { return __ldg(reinterpret_cast<const uint4 *>(p)); }
 
 // vector copy: each thread moves VPT vectors of 16 bytes along X (contiguous
 // in both layouts); batch dims decoded per vector
@@ -1042,6 +1454,208 @@ __global__ void __launch_bounds__(256) k_perm_rt(PermDims P, const T *__restrict
   }
 }
 
+// k_perm_rt, flat mapping with ex == V and dy == V (e.g. NCHW -> NCHW[V]c):
+// a thread's V x V block is one contiguous dst run of V vectors, stored
+// through warp_store_runs (512-byte spans per store instruction instead of
+// 32 lanes x 16 bytes at a 128-byte stride: measured 0.68 -> see DESIGN §5).
+template <typename T>
+__global__ void __launch_bounds__(256) k_perm_rt_ws(PermDims P, const T *__restrict__ src, T *__restrict__ dst,
+                                                  uint32_t nblk) {
+  pdl_wait();
+  constexpr int V = 16 / sizeof(T);
+  __shared__ uint4 stage[8][32 * V];
+  const int lane = threadIdx.x & 31;
+  uint4 *st = stage[threadIdx.x >> 5];
+  const uint32_t byn = (uint32_t)(P.ey / V);
+  for (uint32_t t0 = blockIdx.x * blockDim.x + (threadIdx.x & ~31u); t0 < nblk; t0 += gridDim.x * blockDim.x) {
+    const uint32_t t = t0 + lane;
+    uint4 w[V];
+    int64_t off = -1;
+    if (t < nblk) {
+      uint32_t rem = t / byn;
+      const uint32_t by = t - rem * byn;
+      int64_t sb = 0, db = 0;
+      for (int k = P.nd - 1; k >= 0; k--) {
+        uint32_t q, r;
+        P.ext[k].divmod(rem, q, r);
+        sb += (int64_t)r * P.sstr[k];
+        db += (int64_t)r * P.dstr[k];
+        rem = q;
+      }
+      const int64_t y0 = (int64_t)by * V;
+      uint4 u[V];
+#pragma unroll
+      for (int j = 0; j < V; j++) u[j] = ld16(src + sb + j * P.sx + y0);
+#pragma unroll
+      for (int k = 0; k < V; k++) {
+        uint32_t ww[4];
+        if constexpr (sizeof(T) == 2) {
+          const uint32_t sel = (k & 1) ? 0x7632u : 0x5410u;
+#pragma unroll
+          for (int jp = 0; jp < 4; jp++)
+            ww[jp] = __byte_perm(reinterpret_cast<const uint32_t *>(&u[2 * jp])[k >> 1],
+                                 reinterpret_cast<const uint32_t *>(&u[2 * jp + 1])[k >> 1], sel);
+        } else {
+#pragma unroll
+          for (int j = 0; j < 4; j++) ww[j] = reinterpret_cast<const uint32_t *>(&u[j])[k];
+        }
+        w[k] = make_uint4(ww[0], ww[1], ww[2], ww[3]);
+      }
+      off = db + y0 * V;
+    }
+    warp_store_runs<T, V>(st, w, off, dst, lane);
+  }
+}
+
+// K_PBLOCK: the X x Y transpose tile would be mostly empty (X and Y both
+// short, e.g. weights KCRS -> KCRS16k16c: X = 16 c, Y = R S = 9), so the tile
+// grows by the batch dims nearest to dst-contiguity until it holds up to
+// 4096 elements; a CTA iteration moves one such block: scalar loads in src
+// order (coalesced along the src runs) into shared memory at the block's
+// compact dst position, then 16-byte stores of the block (contiguous in dst
+// when the block dims nest, which the selection favours) or scalar stores.
+constexpr int kPbMax = 6;
+struct PermBlock {
+  int32_t nb;                     // block dims
+  int32_t bsize;                  // elements per block
+  FastDiv sext[kPbMax];           // block dims in src order (innermost first)
+  int64_t ssrc[kPbMax];           //   their src strides
+  int32_t sloc[kPbMax];           //   their compact dst-order (local) strides
+  FastDiv dext[kPbMax];           // block dims in dst order (innermost first)
+  int64_t ddst[kPbMax];           //   their dst strides
+  int32_t dcontig;                // block is one contiguous dst range
+  int32_t nd;                     // batch dims
+  FastDiv ext[kMaxP];
+  int64_t sstr[kMaxP], dstr[kMaxP];
+  uint32_t nbatch;
+};
+
+template <typename T>
+__global__ void __launch_bounds__(256) k_perm_block(PermBlock B, const T *__restrict__ src, T *__restrict__ dst) {
+  pdl_wait();
+  extern __shared__ __align__(16) unsigned char pb_smem[];
+  T *tile = reinterpret_cast<T *>(pb_smem);
+  constexpr int V = 16 / sizeof(T);
+  for (uint32_t bi = blockIdx.x; bi < B.nbatch; bi += gridDim.x) {
+    uint32_t rem = bi;
+    int64_t sb = 0, db = 0;
+    for (int k = B.nd - 1; k >= 0; k--) {
+      uint32_t q, r;
+      B.ext[k].divmod(rem, q, r);
+      sb += (int64_t)r * B.sstr[k];
+      db += (int64_t)r * B.dstr[k];
+      rem = q;
+    }
+    __syncthreads();
+    // eight loads in flight per thread before the shared stores
+    for (int e0 = threadIdx.x; e0 < B.bsize; e0 += blockDim.x * 8) {
+      T val[8];
+      int loc[8];
+#pragma unroll
+      for (int u = 0; u < 8; u++) {
+        const int e = e0 + u * (int)blockDim.x;
+        loc[u] = -1;
+        if (e >= B.bsize) continue;
+        uint32_t re = (uint32_t)e;
+        int lc = 0;
+        int64_t so = 0;
+        for (int i = 0; i < B.nb; i++) {
+          uint32_t q, ii;
+          B.sext[i].divmod(re, q, ii);
+          re = q;
+          so += (int64_t)ii * B.ssrc[i];
+          lc += (int)ii * B.sloc[i];
+        }
+        loc[u] = lc;
+        val[u] = src[sb + so];
+      }
+#pragma unroll
+      for (int u = 0; u < 8; u++)
+        if (loc[u] >= 0) tile[loc[u]] = val[u];
+    }
+    __syncthreads();
+    if (B.dcontig && ((db % V) == 0)) {
+      for (int v = threadIdx.x; v < B.bsize / V; v += blockDim.x)
+        *reinterpret_cast<uint4 *>(dst + db + (int64_t)v * V) = *reinterpret_cast<const uint4 *>(tile + v * V);
+    } else {
+      for (int l = threadIdx.x; l < B.bsize; l += blockDim.x) {
+        uint32_t rl = (uint32_t)l;
+        int64_t dof = 0;
+        for (int i = 0; i < B.nb; i++) {
+          uint32_t q, ii;
+          B.dext[i].divmod(rl, q, ii);
+          rl = q;
+          dof += (int64_t)ii * B.ddst[i];
+        }
+        dst[db + dof] = tile[l];
+      }
+    }
+  }
+}
+
+// host side of K_PBLOCK over the refined dims r (X = ix, Y = iy); false when
+// the block would not beat the transpose tiles
+static bool pblock_launch(const std::vector<RDim> &r, int ix, int iy, const void *src, void *dst, int wb,
+                          cudaStream_t stream, int nsm) {
+  const int V = 16 / wb;
+  std::vector<int> in = {ix, iy};
+  int64_t bsize = r[ix].ext * r[iy].ext;
+  for (;;) {
+    int best = -1;
+    for (int i = 0; i < (int)r.size(); i++) {
+      if (std::find(in.begin(), in.end(), i) != in.end()) continue;
+      if (best < 0 || r[i].dstr < r[best].dstr) best = i;
+    }
+    if (best < 0 || bsize * r[best].ext > 4096 || (int)in.size() >= kPbMax) break;
+    in.push_back(best);
+    bsize *= r[best].ext;
+  }
+  if (bsize < 256 || bsize % V) return false;
+  PermBlock B{};
+  B.nb = (int)in.size();
+  B.bsize = (int32_t)bsize;
+  std::vector<int> so(in), dor(in);
+  std::sort(so.begin(), so.end(), [&](int a, int b) { return r[a].sstr < r[b].sstr; });
+  std::sort(dor.begin(), dor.end(), [&](int a, int b) { return r[a].dstr < r[b].dstr; });
+  std::vector<int64_t> loc(r.size(), 0);
+  int64_t acc = 1;
+  bool contig = true;
+  for (int k = 0; k < B.nb; k++) {
+    const int i = dor[(size_t)k];
+    loc[(size_t)i] = acc;
+    if (r[i].dstr != acc) contig = false;
+    B.dext[k] = FastDiv((uint32_t)r[i].ext);
+    B.ddst[k] = r[i].dstr;
+    acc *= r[i].ext;
+  }
+  for (int k = 0; k < B.nb; k++) {
+    const int i = so[(size_t)k];
+    B.sext[k] = FastDiv((uint32_t)r[i].ext);
+    B.ssrc[k] = r[i].sstr;
+    B.sloc[k] = (int32_t)loc[(size_t)i];
+  }
+  B.dcontig = contig ? 1 : 0;
+  int nd = 0;
+  int64_t nbatch = 1;
+  for (int i = 0; i < (int)r.size(); i++) {
+    if (std::find(in.begin(), in.end(), i) != in.end()) continue;
+    if (nd >= kMaxP) return false;
+    B.ext[nd] = FastDiv((uint32_t)r[i].ext);
+    B.sstr[nd] = r[i].sstr;
+    B.dstr[nd] = r[i].dstr;
+    nbatch *= r[i].ext;
+    nd++;
+  }
+  if (nbatch >= (1ll << 31)) return false;
+  B.nd = nd;
+  B.nbatch = (uint32_t)nbatch;
+  const size_t smem = (size_t)bsize * wb;
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(nbatch, (int64_t)nsm * 8));
+  if (wb == 2) launch_pdl(k_perm_block<uint16_t>, grid, 256, smem, stream, B, (const uint16_t *)src, (uint16_t *)dst);
+  else launch_pdl(k_perm_block<uint32_t>, grid, 256, smem, stream, B, (const uint32_t *)src, (uint32_t *)dst);
+  return true;
+}
+
 static bool perm_launch(Layout *S, const void *src, Layout *D, void *dst, int wb, cudaStream_t stream, int nsm,
                         alt_status *st) {
   std::vector<RDim> r;
@@ -1107,7 +1721,11 @@ static bool perm_launch(Layout *S, const void *src, Layout *D, void *dst, int wb
     }
     if (rt && nblk < (1ll << 31)) {
       const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((nblk + 255) / 256, (int64_t)nsm * 16));
-      if (wb == 2) launch_pdl(k_perm_rt<uint16_t>, grid, 256, 0, stream, P, (const uint16_t *)src, (uint16_t *)dst, (uint32_t)nblk, lgLY);
+      static const bool no_ws = getenv("ALT_RELAYOUT_NOWS") != nullptr;  // developer A/B knob
+      if (lgLY < 0 && P.ex == V && P.dy == V && !no_ws) {
+        if (wb == 2) launch_pdl(k_perm_rt_ws<uint16_t>, grid, 256, 0, stream, P, (const uint16_t *)src, (uint16_t *)dst, (uint32_t)nblk);
+        else launch_pdl(k_perm_rt_ws<uint32_t>, grid, 256, 0, stream, P, (const uint32_t *)src, (uint32_t *)dst, (uint32_t)nblk);
+      } else if (wb == 2) launch_pdl(k_perm_rt<uint16_t>, grid, 256, 0, stream, P, (const uint16_t *)src, (uint16_t *)dst, (uint32_t)nblk, lgLY);
       else launch_pdl(k_perm_rt<uint32_t>, grid, 256, 0, stream, P, (const uint32_t *)src, (uint32_t *)dst, (uint32_t)nblk, lgLY);
       count_launch();
       *st = cudaGetLastError() == cudaSuccess ? ALT_OK : ALT_E_CUDA;
@@ -1125,6 +1743,13 @@ static bool perm_launch(Layout *S, const void *src, Layout *D, void *dst, int wb
       const double waste = (double)((P.ex + tx - 1) / tx * tx) * ((P.ey + ty - 1) / ty * ty) / ((double)P.ex * P.ey);
       const double score = waste * 1.0 + 1e-3 * std::abs(std::log2((double)tx / ty));
       if (score < best) { best = score; TX = tx; }
+    }
+    static const bool no_pb = getenv("ALT_RELAYOUT_NOPB") != nullptr;  // developer A/B knob
+    if (best > 2.0 && !no_pb && pblock_launch(r, ix, iy, src, dst, wb, stream, nsm)) {
+      count_launch();
+      *st = cudaGetLastError() == cudaSuccess ? ALT_OK : ALT_E_CUDA;
+      if (*st != ALT_OK) set_error("relayout (permutation block) launch failed");
+      return true;
     }
     const int64_t TY = area / TX;
     const int64_t tiles = ((P.ex + TX - 1) / TX) * ((P.ey + TY - 1) / TY) * (D->pnumel / (P.ex * P.ey));
@@ -1187,6 +1812,8 @@ alt_status relayout_launch(Layout *S, const void *src, Layout *D, void *dst, int
     {
       alt_status rst = ALT_OK;
       static const bool no_row = getenv("ALT_RELAYOUT_NOROW") != nullptr;  // developer A/B knob
+      static const bool no_win = getenv("ALT_RELAYOUT_NOWIN") != nullptr;  // developer A/B knob
+      if (!no_win && win_launch(S, src, D, dst, wb, ss, ds, stream, nsm, &rst)) return rst;
       if (!no_row && row_launch(S, src, D, dst, wb, ss, ds, stream, nsm, &rst)) return rst;
     }
     SepPair P{};

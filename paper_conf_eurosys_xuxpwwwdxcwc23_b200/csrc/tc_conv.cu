@@ -83,6 +83,10 @@ struct TcArgs {
   FastDiv f_rsg;
   int32_t nst;           // smem ring stages in use (<= the instantiation's STAGES; tuner knob)
   int32_t hboff;         // halo mode: set the descriptor base-offset field for row-shifted A starts
+  int32_t b_res;         // resident weights: every unit of this CTA has the same N tile and the
+                         // reduction fits the ring (num_iters <= nst), so the B slabs loaded with
+                         // the first tile stay in the ring's B slots (slot = k iteration) and later
+                         // tiles stream A only (one B read per CTA instead of one per tile)
   // C3D: tile batch index b = n Do + od (tile_n = 1); taps (t, r, s), RS = R S
   int32_t Do3, RS3;
   FastDiv f_Do3, f_RS3;
@@ -558,11 +562,12 @@ __global__ void __launch_bounds__(kThreads, 1)
         const uint32_t trow = smem_u32(tab) + (uint32_t)((isA ? 0 : 8) * 4 + si * 64);
         int stage = it % a.nst;
         uint32_t ph = (uint32_t)((it / a.nst) & 1);
+        const bool bload = !(a.b_res && ti > 0);  // resident B: loaded with the first tile only
         for (int kit = k_begin; kit < k_end; kit++, it++) {
           if (it >= a.nst) mbar_wait(&empty[stage], ph ^ 1);
-          if (lane == 0 && rank == 0) mbar_expect_tx(&full[stage], CG * (kStageBytesA + L::kB));
+          if (lane == 0 && rank == 0) mbar_expect_tx(&full[stage], CG * (kStageBytesA + (bload ? L::kB : 0)));
           __syncwarp();
-          if (active) {
+          if (active && (isA || bload)) {
             const uint32_t ta = trow + (uint32_t)(kit * a.spi * 64);
             int32_t o0, o1, o2, o3, o4;
             asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];" : "=r"(o0), "=r"(o1), "=r"(o2), "=r"(o3) : "r"(ta));
@@ -585,9 +590,10 @@ __global__ void __launch_bounds__(kThreads, 1)
         if (round > 0) mbar_wait(&empty[stage], (round - 1) & 1);
         if (lane == 0 && ti == ALT_DBG_TILE && kit == k_begin) { DBG(25); }
         // the leader's full barrier counts the bytes of both CTAs of a pair
-        if (lane == 0 && rank == 0) mbar_expect_tx(&full[stage], CG * (kStageBytesA + L::kB));
+        const bool bload = !(a.b_res && ti > 0);
+        if (lane == 0 && rank == 0) mbar_expect_tx(&full[stage], CG * (kStageBytesA + (bload ? L::kB : 0)));
         __syncwarp();
-        if (active) {
+        if (active && (isA || bload)) {
           const int slab = kit * a.spi + si;
           const bool valid = slab < a.total_slabs;
           const int sl = valid ? slab : 0;
@@ -659,7 +665,9 @@ __global__ void __launch_bounds__(kThreads, 1)
           mbar_wait(&full[stage], ph);
           if (i == ALT_DBG_TILE && kit == k_begin) { DBG(28); }
           tc_fence_after();
-          const uint64_t oA = (uint64_t)((stage * L::kAst) >> 4), oB = (uint64_t)((stage * L::kB) >> 4);
+          // resident B: this k iteration's slabs sit in B slot (kit - k_begin)
+          const uint64_t oA = (uint64_t)((stage * L::kAst) >> 4),
+                         oB = (uint64_t)(((a.b_res ? kit - k_begin : stage) * L::kB) >> 4);
           if (a.epi_dbg != 3) {  // developer knob 3: the TMA pipeline alone (no MMA, no drain)
 #pragma unroll
             for (int hs = 0; hs < (HS ? HS : 1); hs++) {
@@ -2176,6 +2184,14 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       pl.stages = pl.hs ? stages_halo(BN, cg) : stages_for(BN, cg);
       // a shallower ring than the instantiation's (tuner knob; 2 .. STAGES)
       a.nst = (cfg && cfg->stages >= 2 && cfg->stages < pl.stages) ? cfg->stages : pl.stages;
+      {
+        // resident weights (see TcArgs::b_res): a CTA's units keep one N tile
+        // when its unit stride is a multiple of the N-tile count (N fastest)
+        static const bool no_res = getenv("ALT_TC_NO_BRES") != nullptr;  // developer A/B knob
+        const int64_t ustep = pl.grid / cg;
+        a.b_res = (!no_res && pl.sc == 1 && a.splits == 1 && a.full_units == 0 && a.num_iters <= a.nst &&
+                   ustep % a.num_n_tiles == 0 && a.num_tiles > ustep) ? 1 : 0;
+      }
       alt_kernel_cfg u{};
       u.path = ALT_PATH_TC;
       u.block_m = 128 * cg;

@@ -66,6 +66,16 @@ D6 = [
     ("R8 images -> window-folded 7x7 s2", (3, 3, 50, 46), [], LY.conv_input_wfold(3, 7, 2, 3)),
     ("R8 images -> window-folded 3x3 s2", (2, 3, 33, 31), [], LY.conv_input_wfold(3, 3, 2, 1)),
     ("window-folded C16 s1 -> NHWC", (2, 16, 9, 13), LY.conv_input_wfold(16, 3, 1, 1), LY.nhwc()),
+    # window-group kernel (K_WIN): ragged tile overhang, 4-channel runs, strided tiles
+    ("unfold 8x8 ragged 30x30", (3, 16, 30, 30), [], LY.conv_input_tiled(16, 8, 30, 30, 3, 3, 8, 8, 1, 1)),
+    ("unfold 5x10 it=4", (2, 32, 20, 20), [], LY.conv_input_tiled(32, 4, 20, 20, 3, 3, 5, 10, 1, 1)),
+    ("unfold from NHWC", (2, 16, 28, 28), LY.nhwc(), LY.conv_input_tiled(16, 8, 28, 28, 3, 3, 7, 7, 1, 1)),
+    # permutation block kernel (K_PBLOCK): short X and Y, contiguous and scattered dst blocks
+    ("KCRS->KCRS8k8c", (64, 32, 3, 3), [], LY.kcrs_yk_xc(64, 32, 8, 8)),
+    ("KCRS->CRSK", (32, 24, 3, 3), [], [("reorder", [1, 2, 3, 0])]),
+    ("KCRS->paper i't o't", (32, 64, 5, 3), [], LY.kcrs_paper(32, 64, 16, 8)),
+    # warp-staged register transpose: batch boundary inside a warp (H W / 8 = 13)
+    ("NCHW->NCHW8c HW=104", (3, 16, 8, 13), [], LY.nchwxc(16, 8)),
 ]
 
 
