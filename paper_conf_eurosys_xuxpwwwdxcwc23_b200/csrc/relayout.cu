@@ -704,7 +704,7 @@ __device__ __forceinline__ void win_outer(const WinPlan &P, uint32_t o, int32_t 
 }
 
 template <typename T, int X>
-__global__ void __launch_bounds__(256) k_relayout_win(WinPlan P, const T *__restrict__ src, T *__restrict__ dst) {
+__global__ void __launch_bounds__(512) k_relayout_win(WinPlan P, const T *__restrict__ src, T *__restrict__ dst) {
   extern __shared__ __align__(16) unsigned char win_smem[];
   const int ntab = P.toff[P.nt];
   int64_t *s_tab = reinterpret_cast<int64_t *>(win_smem);                     // [ntab]
@@ -846,9 +846,10 @@ static bool win_launch(Layout *S, const void *src, Layout *D, void *dst, int wb,
   if (D->pdim_rad[p0] != 1 || a == b || D->pdim_owner[p0 - 1] != b) return false;
   const int64_t X = D->pshape[p0];
   if (!(X * wb == 16 || X * wb == 32)) return false;
-  // measured (R3, 256 x 64 x 56 x 56): bf16 149 us vs K_ROW 170 us; fp32
-  // 250 vs 198 (its whole-row group does not fit the budget), so fp32 stays
-  // on K_ROW unless forced (ALT_WIN_FP32=1)
+  // measured (R3, 256 x 64 x 56 x 56, 512-thread CTAs): bf16 101 us vs
+  // K_ROW 167 us; fp32 316 us at this budget (its whole-row group does not
+  // fit) and 200 us at 200 KB, i.e. no better than K_ROW's 194 us, so fp32
+  // stays on K_ROW unless forced (ALT_WIN_FP32=1)
   static const bool win_f32 = getenv("ALT_WIN_FP32") != nullptr;
   if (wb == 4 && !win_f32) return false;
   const int64_t Lb = S->lshape[b];
@@ -990,12 +991,15 @@ static bool win_launch(Layout *S, const void *src, Layout *D, void *dst, int wb,
     }
   }
   P.blo = dt;
-  const int per_sm = std::max(1, (int)std::min<size_t>(8, (size_t)(200 * 1024) / smem));
+  // threads per CTA: each block's three phases are latency-bound, so more
+  // threads per block shorten them (developer knob ALT_WIN_THREADS)
+  static const int win_threads = getenv("ALT_WIN_THREADS") ? atoi(getenv("ALT_WIN_THREADS")) : 512;
+  const int per_sm = std::max(1, (int)std::min<size_t>(2048 / win_threads, (size_t)(200 * 1024) / smem));
   const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(nouter, (int64_t)nsm * per_sm));
 #define WIN_LAUNCH(T, XX)                                                                                 \
   do {                                                                                                   \
     cudaFuncSetAttribute(k_relayout_win<T, XX>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem); \
-    launch_pdl(k_relayout_win<T, XX>, grid, 256, smem, stream, P, (const T *)src, (T *)dst);             \
+    launch_pdl(k_relayout_win<T, XX>, grid, win_threads, smem, stream, P, (const T *)src, (T *)dst);     \
   } while (0)
   if (wb == 2) {
     if (X == 8) WIN_LAUNCH(uint16_t, 8); else WIN_LAUNCH(uint16_t, 16);

@@ -72,16 +72,17 @@ __global__ void __launch_bounds__(64, 1) k_tma(const __grid_constant__ CUtensorM
     } else if (warp == 1 && lane == 0) {
       int stage = 0; uint32_t ph = 0;
       for (int it = 0; it < iters; it++) {
-        mbar_wait(&full[stage], ph);
+        if (MODE == 9) mbar_spin(&full[stage], ph); else mbar_wait(&full[stage], ph);
         mbar_arrive(&empty[stage]);
         if (++stage == STAGES) { stage = 0; ph ^= 1; }
       }
     }
-  } else if (MODE == 6) {
+  } else if (MODE == 6 || MODE == 9) {
+    // MODE 9: both sides spin on test_wait instead of try_wait
     if (warp == 0 && lane == 0) {
       int stage = 0; uint32_t ph = 0;
       for (int it = 0; it < iters; it++) {
-        if (it >= STAGES) mbar_wait(&empty[stage], ph ^ 1);
+        if (it >= STAGES) { if (MODE == 9) mbar_spin(&empty[stage], ph ^ 1); else mbar_wait(&empty[stage], ph ^ 1); }
         mbar_expect_tx(&full[stage], sbytes);
         for (int l = 0; l < p.loads; l++)
           tma_load_5d(smem + stage * sbytes + l * p.box_bytes, &tm, &full[stage], 0, ((blockIdx.x * 37 + it * p.loads + l) & 63) * p.step[1], 0, 0, 0);
@@ -90,7 +91,7 @@ __global__ void __launch_bounds__(64, 1) k_tma(const __grid_constant__ CUtensorM
     } else if (warp == 1 && lane == 0) {
       int stage = 0; uint32_t ph = 0;
       for (int it = 0; it < iters; it++) {
-        mbar_wait(&full[stage], ph);
+        if (MODE == 9) mbar_spin(&full[stage], ph); else mbar_wait(&full[stage], ph);
         mbar_arrive(&empty[stage]);
         if (++stage == STAGES) { stage = 0; ph ^= 1; }
       }
@@ -173,13 +174,13 @@ int main() {
   cudaMemset(buf, 0, big);
   unsigned long long *cyc;
   cudaMalloc(&cyc, 4 * nsm * sizeof(unsigned long long));
-  for (auto f : {k_tma<0>, k_tma<1>, k_tma<2>, k_tma<3>, k_tma<4>, k_tma<5>, k_tma<6>, k_tma<7>, k_tma<8>}) if (cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, 210 * 1024) != cudaSuccess) printf("attr failed\n");
+  for (auto f : {k_tma<0>, k_tma<1>, k_tma<2>, k_tma<3>, k_tma<4>, k_tma<5>, k_tma<6>, k_tma<7>, k_tma<8>, k_tma<9>}) if (cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, 210 * 1024) != cudaSuccess) printf("attr failed\n");
   cudaEvent_t e0, e1;
   cudaEventCreate(&e0);
   cudaEventCreate(&e1);
   auto run = [&](const char *name, std::vector<uint64_t> dims, std::vector<uint32_t> box, Pat p, int ctas_per_sm, int mode = 0) {
     CUtensorMap tm = make_map(buf, dims, box, 128, {}, (mode == 1 || mode == 3) ? 2 : 5);
-    auto kern = mode == 0 ? k_tma<0> : mode == 1 ? k_tma<1> : mode == 2 ? k_tma<2> : mode == 3 ? k_tma<3> : mode == 4 ? k_tma<4> : mode == 5 ? k_tma<5> : mode == 6 ? k_tma<6> : mode == 7 ? k_tma<7> : k_tma<8>;
+    auto kern = mode == 0 ? k_tma<0> : mode == 1 ? k_tma<1> : mode == 2 ? k_tma<2> : mode == 3 ? k_tma<3> : mode == 4 ? k_tma<4> : mode == 5 ? k_tma<5> : mode == 6 ? k_tma<6> : mode == 7 ? k_tma<7> : mode == 8 ? k_tma<8> : k_tma<9>;
     const int iters = 2048;
     const int smem = p.stages * p.box_bytes * p.loads + 1024;
     const int grid = nsm * ctas_per_sm;
@@ -196,9 +197,8 @@ int main() {
     printf("mode %d %-44s box %5d B x%d, %2d st, %d CTA/SM: %8.1f GB/s %6.1f B/clk/SM@1.965\n", mode, name, p.box_bytes, p.loads,
            p.stages, ctas_per_sm, bytes / ms / 1e6, bytes / ms / 1e6 / nsm / 1.965);
   };
-  {
+  if (getenv("TMA_ALL")) {
     uint64_t R = (uint64_t)1 << 22;
-    // concurrent lanes: (rows per box, boxes per stage, stages)
     int cfgs[][3] = {{128, 1, 6}, {128, 2, 4}, {64, 2, 6}, {32, 4, 6}, {16, 8, 6}, {128, 3, 3}, {64, 4, 4},
                      {32, 8, 4}, {128, 4, 3}, {256, 1, 4}, {256, 2, 3}};
     for (auto &c : cfgs) {
@@ -206,28 +206,15 @@ int main() {
       run("2D [R][64] concurrent lanes", {64, R}, {64, (uint32_t)c[0]}, p, 1, 7);
     }
   }
-  {
-    // conv-like scattered A boxes: [R][14 pixels][64 ch]; box {64, w, g}: g
-    // segments of w pixels (w*128 B contiguous) 1792 B apart
-    uint64_t R = (uint64_t)1 << 18;
-    int cfgs[][4] = {{4, 32, 1, 5}, {4, 16, 2, 5}, {4, 8, 4, 5}, {8, 16, 1, 5}, {8, 8, 2, 5}, {14, 8, 1, 5},
-                     {14, 4, 2, 5}, {4, 32, 2, 3}};
-    for (auto &c : cfgs) {
-      Pat p = {3, c[0] * c[1] * 128, {1, 1, 64}, {0, 0, c[1]}, c[2], c[3]};
-      char nm[64];
-      snprintf(nm, 64, "3D scattered seg %d px x %d", c[0], c[1]);
-      run(nm, {64, 14, R}, {64, (uint32_t)c[0], (uint32_t)c[1]}, p, 1, 8);
-    }
-  }
-  for (int mode : {6}) {
+  // single-lane issue, L2-resident boxes (64 distinct): try_wait (6) vs spin (9),
+  // boxes per stage, stage depth
+  for (int mode : {6, 9}) {
     uint64_t R = (uint64_t)1 << 22;
-    for (int rows : {64, 128, 256}) for (int st : {2, 4, 8}) {
-      if (st * rows * 128 > 200 * 1024) continue;
-      Pat p = {2, rows * 128, {1, (int32_t)(R / rows)}, {0, rows}, 1, st};
-      run("2D [R][64] 1 GiB", {64, R}, {64, (uint32_t)rows}, p, 1, mode);
+    for (int rows : {64, 128, 256}) for (int st : {2, 4, 8}) for (int nl : {1, 2}) {
+      if (st * rows * 128 * nl > 200 * 1024) continue;
+      Pat p = {2, rows * 128, {1, (int32_t)(R / rows)}, {0, rows}, nl, st};
+      run("2D [R][64] L2-resident", {64, R}, {64, (uint32_t)rows}, p, 1, mode);
     }
-    Pat p = {2, 16384, {1, (int32_t)(R / 128)}, {0, 128}, 4, 3};
-    run("2D [R][64] 1 GiB", {64, R}, {64, 128}, p, 1, mode);
   }
   return 0;
 }
