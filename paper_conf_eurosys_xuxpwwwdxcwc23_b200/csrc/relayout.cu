@@ -1604,6 +1604,7 @@ static bool pblock_launch(const std::vector<RDim> &r, int ix, int iy, const void
   const int V = 16 / wb;
   std::vector<int> in = {ix, iy};
   int64_t bsize = r[ix].ext * r[iy].ext;
+  if (bsize > 4096) return false;  // the X x Y tile alone exceeds a block: transpose tiles
   for (;;) {
     int best = -1;
     for (int i = 0; i < (int)r.size(); i++) {

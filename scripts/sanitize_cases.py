@@ -2,7 +2,7 @@
 (memcheck / racecheck / synccheck): tensor-core conv (bf16, fp32 split,
 MN-major, split-K, cluster split-K, tail split, round stores, padded-output
 epilogue), GEMM, depthwise, pool, relayout (permutation, K_ROW, K_CT,
-generic), store_at.  Each case is checked against the oracle so a race that
+generic, K_WIN, K_PBLOCK, warp-staged stores), resident weights, store_at.  Each case is checked against the oracle so a race that
 corrupts data also fails here.  usage: sanitize_cases.py"""
 import os
 import sys
@@ -46,6 +46,14 @@ cases = [
     ("relayout wfold (K_ROW)", lambda: _gpu_relayout((2, 3, 33, 31), [], LY.conv_input_wfold(3, 3, 2, 1), BF, "r3")),
     ("relayout generic", lambda: _gpu_relayout((2, 16, 14, 14), [("fuse", 1, 3), ("split", 1, [4, 4, 196]),
                                                                  ("reorder", [0, 1, 3, 2])], [], F32, "r4")),
+    ("relayout window group (K_WIN)", lambda: _gpu_relayout((3, 16, 30, 30), [],
+                                                           LY.conv_input_tiled(16, 8, 30, 30, 3, 3, 8, 8, 1, 1), BF, "r5")),
+    ("relayout perm block (K_PBLOCK)", lambda: _gpu_relayout((64, 32, 3, 3), [], LY.kcrs_yk_xc(64, 32, 8, 8), BF, "r6")),
+    ("relayout warp-staged rt", lambda: _gpu_relayout((3, 16, 8, 13), [], LY.nchwxc(16, 8), BF, "r7")),
+    ("relayout ident fp32 32-byte runs", lambda: _gpu_relayout((2, 3, 20, 24), [], LY.nchwxc(3, 8, pad_c=5), F32, "r8")),
+    ("tc conv resident weights", lambda: run_conv("s11", 8, 64, 28, 28, 64, 3, 3, 1, 1, LY.nchwxc(64, 64),
+                                                  LY.kcrs_yk_xc(64, 64, 64, 64), LY.nchwxc(64, 64), BF, epi=True,
+                                                  act=1, cfg={**TC, "block_n": 64})),
 ]
 only = sys.argv[1:]
 for name, fn in cases:

@@ -76,6 +76,8 @@ D6 = [
     ("KCRS->paper i't o't", (32, 64, 5, 3), [], LY.kcrs_paper(32, 64, 16, 8)),
     # warp-staged register transpose: batch boundary inside a warp (H W / 8 = 13)
     ("NCHW->NCHW8c HW=104", (3, 16, 8, 13), [], LY.nchwxc(16, 8)),
+    # short X, long Y: the X x Y tile exceeds a permutation block (transpose tiles)
+    ("images NCHW->NHWC C=3", (2, 3, 64, 64), [], LY.nhwc()),
 ]
 
 
