@@ -37,12 +37,6 @@ struct DwArgs {
   int32_t vec_out;
   int32_t res_vec;        // residual read as 8-channel vectors (epi.res tables)
   int32_t sb_vec;         // scale / bias 16-byte aligned (float4 loads)
-  // affine h / w offsets (rd[d][i] = rd[d][0] + i * stride over the logical
-  // range, true for every NCHW[x]c / NHWC / padded-interior layout): the fast
-  // form then computes x / y / weight offsets instead of ~25 table loads per
-  // output vector (the kernel was LSU-bound on the lookups)
-  int32_t aff;
-  int64_t xh0, xhs, xw0, xws, yh0, yhs, yw0, yws, wr0, wrs, ws0, wss;
   Writer yw;
   EpiParams epi;
 };
@@ -179,21 +173,18 @@ __global__ void __launch_bounds__(256, 2) k_dw3x3_fast(DwArgs a, const uint16_t 
     for (int r = 0; r < 3; r++) {
       const int ih = it.p * a.Vh - a.ph + r;
       vr[r] = ih >= 0 && ih < a.H;
-      ro[r] = a.aff ? a.xh0 + (int64_t)(vr[r] ? ih : 0) * a.xhs : __ldg(a.xrd[2] + (vr[r] ? ih : 0));
+      ro[r] = __ldg(a.xrd[2] + (vr[r] ? ih : 0));
     }
 #pragma unroll
     for (int s2 = 0; s2 < 3; s2++) {
       const int iw = it.q * a.Vw - a.pw + s2;
       vc[s2] = iw >= 0 && iw < a.W;
-      co[s2] = a.aff ? a.xw0 + (int64_t)(vc[s2] ? iw : 0) * a.xws : __ldg(a.xrd[3] + (vc[s2] ? iw : 0));
+      co[s2] = __ldg(a.xrd[3] + (vc[s2] ? iw : 0));
     }
     const int64_t wk = __ldg(a.wrd[0] + it.c0);
     int64_t wro[3], wco[3];
 #pragma unroll
-    for (int r = 0; r < 3; r++) {
-      wro[r] = a.aff ? a.wr0 + r * a.wrs : __ldg(a.wrd[2] + r);
-      wco[r] = a.aff ? a.ws0 + r * a.wss : __ldg(a.wrd[3] + r);
-    }
+    for (int r = 0; r < 3; r++) { wro[r] = __ldg(a.wrd[2] + r); wco[r] = __ldg(a.wrd[3] + r); }
     uint4 xv[9], wv[9];
 #pragma unroll
     for (int r = 0; r < 3; r++)
@@ -211,9 +202,8 @@ __global__ void __launch_bounds__(256, 2) k_dw3x3_fast(DwArgs a, const uint16_t 
     const float4 *scp = reinterpret_cast<const float4 *>(a.epi.scale + it.c0);
     const float4 *bip = reinterpret_cast<const float4 *>(a.epi.bias + it.c0);
     const float4 s0 = __ldg(scp), s1 = __ldg(scp + 1), b0 = __ldg(bip), b1 = __ldg(bip + 1);
-    const int64_t yo = __ldg(a.yrd[0] + it.n) + __ldg(a.yrd[1] + it.c0) +
-                       (a.aff ? a.yh0 + it.p * a.yhs + a.yw0 + it.q * a.yws
-                              : __ldg(a.yrd[2] + it.p) + __ldg(a.yrd[3] + it.q));
+    const int64_t yo = __ldg(a.yrd[0] + it.n) + __ldg(a.yrd[1] + it.c0) + __ldg(a.yrd[2] + it.p) +
+                       __ldg(a.yrd[3] + it.q);
     float acc[8];
 #pragma unroll
     for (int j = 0; j < 8; j++) acc[j] = 0.f;
@@ -349,20 +339,6 @@ alt_status dw_conv(const ConvProblem &P, cudaStream_t stream, alt_kernel_cfg *us
   const auto *w = static_cast<const uint16_t *>(P.w);
   auto *y = static_cast<uint16_t *>(P.y);
   const bool fast = r3 && a.w_vec && a.vec_out && a.sb_vec && (!P.epi.residual || a.res_vec);
-  if (fast) {
-    // affine h / w offset tables of x, y and the weights (see DwArgs::aff)
-    auto affine = [](const std::vector<int64_t> &rd, int64_t n, int64_t *o0, int64_t *st) {
-      if ((int64_t)rd.size() < n || n < 1) return false;
-      *o0 = rd[0];
-      *st = n > 1 ? rd[1] - rd[0] : 0;
-      for (int64_t i = 0; i < n; i++) if (rd[(size_t)i] != *o0 + i * *st) return false;
-      return true;
-    };
-    static const bool no_aff = getenv("ALT_DW_NO_AFF") != nullptr;  // developer A/B knob
-    a.aff = !no_aff && affine(P.xl->rd[2], P.H, &a.xh0, &a.xhs) && affine(P.xl->rd[3], P.W, &a.xw0, &a.xws) &&
-            affine(P.yl->rd[2], P.Ho, &a.yh0, &a.yhs) && affine(P.yl->rd[3], P.Wo, &a.yw0, &a.yws) &&
-            affine(P.wl->rd[2], 3, &a.wr0, &a.wrs) && affine(P.wl->rd[3], 3, &a.ws0, &a.wss) ? 1 : 0;
-  }
   if (fast) launch_pdl(k_dw3x3_fast, grid, 256, 0, stream, a, x, w, y);
   else if (r3) launch_pdl(k_dw_vec8<3, 3>, grid, 256, 0, stream, a, x, w, y);
   else if (r1) launch_pdl(k_dw_vec8<1, 1>, grid, 256, 0, stream, a, x, w, y);
