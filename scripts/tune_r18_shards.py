@@ -1,7 +1,7 @@
 """Loop-tune the R18 chain (chain.tune: BLOCK_N, CTA pair, split-K, pixel
 tiles, halo tiles) at the per-GPU batches of the 1/2/4/8-GPU shards of the
 global batch 256 (chain_tune.json) and time each shard chain before / after
-(CUDA graph).  usage: tune_r18_shards.py OUT_COPY"""
+(CUDA graph).  usage: tune_r18_shards.py OUT_COPY [N ...]"""
 import os
 import shutil
 import sys
@@ -11,7 +11,7 @@ import bench_workloads as BW  # noqa: E402
 from paper_conf_eurosys_xuxpwwwdxcwc23_b200 import chain as CH  # noqa: E402
 
 dev = torch.device("cuda", 0)
-for N in (256, 128, 64, 32):
+for N in ([int(v) for v in sys.argv[2:]] or (256, 128, 64, 32)):
     ch = CH.resnet18(N, dev)
     before = BW._time(lambda: ch.run(), 10, 3, 1)
     ch.tune(log=lambda m: print(f"r18 N{N}", m, flush=True))
