@@ -83,6 +83,8 @@ struct TcArgs {
   FastDiv f_rsg;
   int32_t nst;           // smem ring stages in use (<= the instantiation's STAGES; tuner knob)
   int32_t hboff;         // halo mode: set the descriptor base-offset field for row-shifted A starts
+  int32_t a_bytes;       // bytes of one A stage's box(es) (expect_tx): 128 rows x 128 B, or the
+                         // 2-D halo tile's (tile_h + R - 1) tile_w rows
   int32_t b_res;         // resident weights: every unit of this CTA has the same N tile and the
                          // reduction fits the ring (num_iters <= nst), so the B slabs loaded with
                          // the first tile stay in the ring's B slots (slot = k iteration) and later
@@ -149,11 +151,16 @@ constexpr int kTabBytes = kTabSlabs * 64;
 // loaded once per (filter row, channel slab) with 8 spare rows after the
 // 128, and the HS taps along W read it at row offsets 0 .. HS-1; B holds the
 // HS tap slabs of the stage
-template <int BN, int STAGES, int CG = 1, int HS = 0>
+// HR > 0 (with HS): two-dimensional halo for stride-1 R x S filters with one
+// 64-channel slab (C <= 64): an A stage holds the tile's (tile_h + R - 1)
+// input rows of tile_w pixels (<= 256 rows, one TMA box per tile) and the
+// R x S taps read it at row offsets r tile_w + s; the weights of all taps sit
+// in one resident B slot after the A ring (loaded with the CTA's first tile)
+template <int BN, int STAGES, int CG = 1, int HS = 0, int HR = 0>
 struct TcSmem {
-  static constexpr int kAst = kStageBytesA + (HS ? 1024 : 0);  // A stage stride
-  static constexpr int kB = (BN / CG) * 64 * 2 * (HS ? HS : 1);  // this CTA's share of the B tile(s)
-  static constexpr int kRing = STAGES * (kAst + kB);
+  static constexpr int kAst = HR ? 256 * 128 + 1024 : kStageBytesA + (HS ? 1024 : 0);  // A stage stride
+  static constexpr int kB = (BN / CG) * 64 * 2 * (HS ? HS : 1) * (HR ? HR : 1);  // this CTA's share of the B tile(s)
+  static constexpr int kRing = HR ? STAGES * kAst + kB : STAGES * (kAst + kB);
   static constexpr int kOut = kRing;                       // 2 staging buffers for TMA stores
   static constexpr int kSB = kOut + kEpiWarps * 4096;      // scale / bias of the tile (2 x BN floats)
   static constexpr int kBar = kSB + 2 * BN * 4;             // barriers
@@ -426,12 +433,12 @@ __device__ __forceinline__ TileCoord tile_coord(const TcArgs &a, int tile, int B
 // cluster barrier CTA r reduces rows [r * 128 / SC, (r + 1) * 128 / SC) of all
 // SC partials through distributed shared memory in split order, applies the
 // epilogue and stores them — the reduction and the epilogue are split SC ways.
-template <int BN, int STAGES, int CG, bool RV, int SC, int HS = 0, bool D3 = false>
+template <int BN, int STAGES, int CG, bool RV, int SC, int HS = 0, bool D3 = false, int HR = 0>
 __global__ void __launch_bounds__(kThreads, 1)
     k_tc_conv(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
               const __grid_constant__ CUtensorMap tmY, const __grid_constant__ TcArgs a, uint16_t *__restrict__ y) {
   using namespace sm100;
-  using L = TcSmem<BN, STAGES, CG, HS>;
+  using L = TcSmem<BN, STAGES, CG, HS, HR>;
   const int rank = CG == 2 ? (int)cluster_ctarank() : 0;
   const int unit0 = blockIdx.x / CG, unit_step = gridDim.x / CG;
   extern __shared__ __align__(1024) unsigned char smem_raw[];
@@ -517,14 +524,17 @@ __global__ void __launch_bounds__(kThreads, 1)
     // issues per stage: (group, channel slab) pairs; a K-major operand has
     // one group, an MN-major one ng groups of mnw rows (planner: <= 16);
     // halo mode: B issues one box per (tap s, slab), lane j -> s = j / spi
-    const int hsb = (HS && !isA) ? HS : 1;
+    // 2-D halo (HR): B issues one box per tap (r, s), lane j -> (j / S, j % S)
+    const int hsb = (HS && !isA) ? HS * (HR ? HR : 1) : 1;
     const bool active = j < om.ng * a.spi * hsb;
-    const int hs_s = (HS && !isA) ? j / a.spi : 0;
-    const int jj = (HS && !isA) ? j - hs_s * a.spi : j;
+    const int hs_t = (HS && !isA) ? j / a.spi : 0;  // the lane's tap slot
+    const int hs_s = HR ? hs_t % HS : hs_t, hr_r = HR ? hs_t / HS : 0;
+    const int jj = (HS && !isA) ? j - hs_t * a.spi : j;
     const int gi = om.mnw ? jj % om.ng : 0, si = om.mnw ? jj / om.ng : jj;
-    const int32_t hs_c[5] = {om.coef[0][V_S] * hs_s, om.coef[1][V_S] * hs_s, om.coef[2][V_S] * hs_s,
-                             om.coef[3][V_S] * hs_s, om.coef[4][V_S] * hs_s};
-    const uint32_t hs_off = (uint32_t)(hs_s * (BN / CG) * 128);
+    const int32_t hs_c[5] = {om.coef[0][V_S] * hs_s + om.coef[0][V_R] * hr_r, om.coef[1][V_S] * hs_s + om.coef[1][V_R] * hr_r,
+                             om.coef[2][V_S] * hs_s + om.coef[2][V_R] * hr_r, om.coef[3][V_S] * hs_s + om.coef[3][V_R] * hr_r,
+                             om.coef[4][V_S] * hs_s + om.coef[4][V_R] * hr_r};
+    const uint32_t hs_off = (uint32_t)(hs_t * (BN / CG) * 128);
     // this lane's group: rows [gi * mnw, (gi + 1) * mnw) of the tile
     int g_dn = 0, g_dh = 0, g_dw = 0;
     if (om.mnw && isA) {
@@ -565,7 +575,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         const bool bload = !(a.b_res && ti > 0);  // resident B: loaded with the first tile only
         for (int kit = k_begin; kit < k_end; kit++, it++) {
           if (it >= a.nst) mbar_wait(&empty[stage], ph ^ 1);
-          if (lane == 0 && rank == 0) mbar_expect_tx(&full[stage], CG * (kStageBytesA + (bload ? L::kB : 0)));
+          if (lane == 0 && rank == 0) mbar_expect_tx(&full[stage], CG * (a.a_bytes + (bload ? L::kB : 0)));
           __syncwarp();
           if (active && (isA || bload)) {
             const uint32_t ta = trow + (uint32_t)(kit * a.spi * 64);
@@ -591,7 +601,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         if (lane == 0 && ti == ALT_DBG_TILE && kit == k_begin) { DBG(25); }
         // the leader's full barrier counts the bytes of both CTAs of a pair
         const bool bload = !(a.b_res && ti > 0);
-        if (lane == 0 && rank == 0) mbar_expect_tx(&full[stage], CG * (kStageBytesA + (bload ? L::kB : 0)));
+        if (lane == 0 && rank == 0) mbar_expect_tx(&full[stage], CG * (a.a_bytes + (bload ? L::kB : 0)));
         __syncwarp();
         if (active && (isA || bload)) {
           const int slab = kit * a.spi + si;
@@ -603,6 +613,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           v[V_GT] = (int)om.fg.div((uint32_t)ga); v[V_GR] = ga - v[V_GT] * om.divg;
           int32_t c[5];
           v[V_S] += hs_s;  // halo mode: this lane's tap s (B); 0 otherwise
+          v[V_R] += hr_r;  // 2-D halo: this lane's tap r (B)
           coords<D3>(om, v, c);
           if (!valid) c[0] = om.oob0;
           if constexpr (CG == 2)
@@ -670,14 +681,18 @@ __global__ void __launch_bounds__(kThreads, 1)
                          oB = (uint64_t)(((a.b_res ? kit - k_begin : stage) * L::kB) >> 4);
           if (a.epi_dbg != 3) {  // developer knob 3: the TMA pipeline alone (no MMA, no drain)
 #pragma unroll
-            for (int hs = 0; hs < (HS ? HS : 1); hs++) {
+            for (int ht = 0; ht < (HS ? HS : 1) * (HR ? HR : 1); ht++) {
               // halo: tap s reads A rows shifted by s (128-byte rows: + s * 8
-              // in 16-byte units; base-offset field = s when requested)
-              const uint64_t sA_off = HS ? (uint64_t)(hs * 8) | (a.hboff ? ((uint64_t)hs << 49) : 0ull) : 0ull;
-              const uint64_t sB_off = HS ? (uint64_t)((hs * (BN / CG) * 128) >> 4) : 0ull;
+              // in 16-byte units; base-offset field = s when requested); 2-D
+              // halo: tap (r, s) reads rows shifted by r tile_w + s (r tile_w
+              // rows are whole 1024-byte swizzle atoms)
+              const int hs = HR ? ht % HS : ht, hr = HR ? ht / HS : 0;
+              const uint64_t sA_off = HS ? (uint64_t)((hr * a.tile_w + hs) * 8) | (a.hboff ? ((uint64_t)hs << 49) : 0ull)
+                                         : 0ull;
+              const uint64_t sB_off = HS ? (uint64_t)((ht * (BN / CG) * 128) >> 4) : 0ull;
 #pragma unroll
               for (int kk = 0; kk < 4; kk++) {
-                const uint32_t accum = (kit != k_begin || kk != 0 || hs != 0) ? 1u : 0u;
+                const uint32_t accum = (kit != k_begin || kk != 0 || ht != 0) ? 1u : 0u;
                 if constexpr (CG == 2) mma_bf16_2cta(d, dA[kk] + oA + sA_off, dB[kk] + oB + sB_off, idesc, accum);
                 else mma_bf16(d, dA[kk] + oA + sA_off, dB[kk] + oB + sB_off, idesc, accum);
               }
@@ -1697,13 +1712,13 @@ static int num_sms() {
   return n;
 }
 
-template <int BN, int STAGES, int CG_, bool RV, int SC = 1, int HS = 0, bool D3 = false>
+template <int BN, int STAGES, int CG_, bool RV, int SC = 1, int HS = 0, bool D3 = false, int HR = 0>
 static cudaError_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUtensorMap &ty, const TcArgs &a,
                              uint16_t *y, int grid, cudaStream_t s) {
   constexpr int CG = CG_;
-  auto kern = k_tc_conv<BN, STAGES, CG, RV, SC, HS, D3>;
-  const int smem = TcSmem<BN, STAGES, CG, HS>::kBytes;
-  static_assert(TcSmem<BN, STAGES, CG, HS>::kBytes <= 232448, "smem budget");
+  auto kern = k_tc_conv<BN, STAGES, CG, RV, SC, HS, D3, HR>;
+  const int smem = TcSmem<BN, STAGES, CG, HS, HR>::kBytes;
+  static_assert(TcSmem<BN, STAGES, CG, HS, HR>::kBytes <= 232448, "smem budget");
   static bool attr_set = false;  // once per instantiation (not capture-safe to repeat)
   if (!attr_set) {
     cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
@@ -1759,6 +1774,7 @@ struct TcPlan {
   int BN, stages, cg;
   int sc;  // cluster split-K factor (1 = off)
   int hs;  // halo mode: filter width S folded into row-shifted A reads (0 = off)
+  int hr;  // 2-D halo: filter height R folded too (0 = off)
   alt_kernel_cfg used;
 };
 static std::mutex g_tc_mu;
@@ -1772,8 +1788,11 @@ constexpr int stages_for(int BN, int CG) {
 }
 // halo-mode ring depth (A stage + 8 spare rows, three B tap slabs per stage)
 constexpr int stages_halo(int BN, int CG) { return BN / CG == 64 ? 4 : 2; }
+// 2-D halo ring: 33 KB A stages next to one resident 72 KB B slot (BN 64)
+constexpr int kStagesHalo2 = 3;
 template <bool RV>
 static cudaError_t launch_plan_rv(const TcPlan &pl, uint16_t *yy, cudaStream_t stream) {
+  if (pl.hr == 3) return launch_tc<64, kStagesHalo2, 1, RV, 1, 3, false, 3>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
   if (pl.hs == 3) {
     if (pl.cg == 2) {
       if (pl.BN == 128) return launch_tc<128, stages_halo(128, 2), 2, RV, 1, 3>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
@@ -1941,12 +1960,20 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
     const bool halo_ok = halo_want && P.is_conv && P.S == 3 && !P.pairs && P.ra[3].role == R_W && P.ra[3].V == 1 &&
                          P.ra[3].tap == 1 && (c.tw == 16 || c.tw == 32 || c.tw == 64) && P.Wo + P.S - 2 < c.tw &&
                          !(cfg && (cfg->split_k > 1 || cfg->split_cluster)) && BN / cg <= 128;
-    for (int hmode = halo_ok ? 1 : 0; hmode >= 0; hmode--)
+    // 2-D halo (hmode 2): R filter rows folded too — one 64-channel slab
+    // (C <= 64), one 64-channel N tile per CTA, one image per tile (tile_n 1,
+    // the tile's (tile_h + R - 1) x tile_w input rows in one box <= 256 rows)
+    static const int hrow_env = [] { const char *e = getenv("ALT_TC_HROW"); return e ? atoi(e) : 1; }();
+    const bool hrow_ok = halo_ok && hrow_env && P.R == 3 && P.C <= 64 && P.K <= 64 && BN == 64 && cg == 1 &&
+                         c.tn == 1 && (c.th + P.R - 1) * c.tw <= 256 && P.ra[2].role == R_H && P.ra[2].V == 1 &&
+                         P.ra[2].tap == 1 && P.T == 1 && !P.Do;
+    for (int hmode = hrow_ok ? 2 : (halo_ok ? 1 : 0); hmode >= 0; hmode--)
     for (int sw = 64; sw >= 8; sw /= 2) {
       if (hmode && sw != 64) continue;
       RoleInfo rah[kMaxL];
       memcpy(rah, ra, sizeof(rah));
       if (hmode) rah[3].tap = 0;  // the A box does not move with the tap s
+      if (hmode == 2) { rah[2].tap = 0; rah[2].tile = c.th + (int)P.R - 1; }  // nor with r: R - 1 extra rows
       View va, vb;
       // K-major first (the channel run innermost); otherwise an MN-major
       // view whose stride-1 dim is the M (A) / N (B) run: groups of mnw rows
@@ -1976,7 +2003,8 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       for (int i = 1; i < va.rank; i++) rowsA *= (va.d[i].box + va.d[i].estride - 1) / va.d[i].estride;
       for (int i = 1; i < vb.rank; i++) rowsB *= (vb.d[i].box + vb.d[i].estride - 1) / vb.d[i].estride;
       // K-major: a box holds the tile's rows; MN-major: sw K rows of one group
-      if (rowsA != (mnA ? sw : 128) || rowsB != (mnB ? sw : BN / cg)) {
+      const int64_t rowsA_want = mnA ? sw : (hmode == 2 ? (int64_t)(c.th + P.R - 1) * c.tw : 128);
+      if (rowsA != rowsA_want || rowsB != (mnB ? sw : BN / cg)) {
         snprintf(why, 160, "rows A %lld B %lld", (long long)rowsA, (long long)rowsB);
         continue;
       }
@@ -2065,21 +2093,24 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       a.num_n_tiles = (int32_t)ntiles;
       a.num_tiles = (int32_t)(((mtiles + cg - 1) / cg) * ntiles);  // work units
       a.S = (int32_t)(hmode ? 1 : P.S);  // halo: the slabs enumerate (r, g); the S taps ride in each stage
+      const int64_t Rsl = hmode == 2 ? 1 : P.R;  // 2-D halo: the slabs enumerate g; all R x S taps ride in each stage
+      a.a_bytes = (int32_t)((hmode == 2 ? rowsA_want : 128) * 64 * esize);  // one 64-channel stage
       a.Gc = (int32_t)((P.C + sw - 1) / sw);
       if (P.coff % sw) { snprintf(why, 160, "group channel offset %% slab"); continue; }
       a.a_goff = (int32_t)(P.coff / sw);
       a.b_koff = (int32_t)P.koff;
       a.y_koff = (int32_t)P.koff;
-      a.rsg = (int32_t)(P.R * a.S * a.Gc);
+      a.rsg = (int32_t)(Rsl * a.S * a.Gc);
       a.pairs = P.pairs;
       a.out_f32 = P.out_f32 ? 1 : 0;
       if (P.pairs && P.C % sw) { snprintf(why, 160, "split planes not slab-aligned"); continue; }
-      a.total_slabs = (int32_t)((P.pairs ? P.pairs : 1) * P.T * P.R * a.S * a.Gc);
+      a.total_slabs = (int32_t)((P.pairs ? P.pairs : 1) * P.T * Rsl * a.S * a.Gc);
       a.Do3 = (int32_t)P.Do;
-      a.RS3 = (int32_t)(P.R * a.S);
+      a.RS3 = (int32_t)(Rsl * a.S);
       a.f_Do3 = FastDiv((uint32_t)std::max<int64_t>(1, P.Do));
       a.f_RS3 = FastDiv((uint32_t)std::max(1, a.RS3));
       pl.hs = hmode ? (int)P.S : 0;
+      pl.hr = hmode == 2 ? (int)P.R : 0;
       {
         static const int hboff = [] { const char *e = getenv("ALT_HALO_BOFF"); return e ? atoi(e) : 0; }();
         a.hboff = hboff;
@@ -2181,7 +2212,7 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
                           : (int)std::min<int64_t>((int64_t)a.num_tiles * cg, num_sms() / cg * cg);
       pl.BN = BN;
       pl.cg = cg;
-      pl.stages = pl.hs ? stages_halo(BN, cg) : stages_for(BN, cg);
+      pl.stages = pl.hr ? kStagesHalo2 : (pl.hs ? stages_halo(BN, cg) : stages_for(BN, cg));
       // a shallower ring than the instantiation's (tuner knob; 2 .. STAGES)
       a.nst = (cfg && cfg->stages >= 2 && cfg->stages < pl.stages) ? cfg->stages : pl.stages;
       {
@@ -2191,6 +2222,15 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
         const int64_t ustep = pl.grid / cg;
         a.b_res = (!no_res && pl.sc == 1 && a.splits == 1 && a.full_units == 0 && a.num_iters <= a.nst &&
                    ustep % a.num_n_tiles == 0 && a.num_tiles > ustep) ? 1 : 0;
+        // 2-D halo: B lives in its one resident slot (the CTA keeps its N tile,
+        // the reduction is one stage), else this plan is not valid
+        if (pl.hr) {
+          if (!(pl.sc == 1 && a.splits == 1 && a.full_units == 0 && a.num_iters == 1 && ustep % a.num_n_tiles == 0)) {
+            snprintf(why, 160, "2-D halo needs one reduction stage and a fixed N tile per CTA");
+            continue;
+          }
+          a.b_res = 1;
+        }
       }
       alt_kernel_cfg u{};
       u.path = ALT_PATH_TC;
@@ -2202,7 +2242,7 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       u.tile_n = c.tn; u.tile_h = c.th; u.tile_w = c.tw;
       u.split_k = a.splits;
       u.split_cluster = pl.sc > 1 ? 1 : (a.full_units > 0 && a.splits > 1 ? 2 : 0);
-      u.block_k = pl.hs ? 1 : 64;  // 1 = halo mode (cfg->block_k: 1 request, 2 refuse)
+      u.block_k = pl.hr ? 3 : (pl.hs ? 1 : 64);  // 1 = halo, 3 = 2-D halo (cfg->block_k: 1 request, 2 refuse)
       pl.used = u;
       cudaError_t e = launch_plan(pl, P.y, stream);
       count_launch();
