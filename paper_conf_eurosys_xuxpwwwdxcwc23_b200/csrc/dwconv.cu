@@ -156,12 +156,17 @@ __global__ void __launch_bounds__(256, 2) k_dw_vec8(DwArgs a, const uint16_t *__
   }
 }
 
+#ifndef ALT_DW_MINB
+// resident CTAs per SM the fast form's register budget targets: measured on
+// the MV2 b16 chain 2 -> 0.666 ms, 3 -> 0.760 (spills), 4 -> 0.654 (64 registers)
+#define ALT_DW_MINB 4
+#endif
 // Fast 3x3 form (vector weights, vector output, aligned scale / bias,
 // vector or no residual): every tap's x and w vectors are requested before
 // any arithmetic (18 independent 16-byte loads in flight per thread; the
 // padded taps load a valid address and are zeroed), so the kernel is not
 // bound by one load latency per tap.  Same (r, s) accumulation order.
-__global__ void __launch_bounds__(256, 2) k_dw3x3_fast(DwArgs a, const uint16_t *__restrict__ x,
+__global__ void __launch_bounds__(256, ALT_DW_MINB) k_dw3x3_fast(DwArgs a, const uint16_t *__restrict__ x,
                                                        const uint16_t *__restrict__ w, uint16_t *__restrict__ y) {
   pdl_wait();
   for (uint32_t idx = blockIdx.x * blockDim.x + threadIdx.x; idx < a.total; idx += gridDim.x * blockDim.x) {
