@@ -993,7 +993,10 @@ static bool win_launch(Layout *S, const void *src, Layout *D, void *dst, int wb,
   P.blo = dt;
   // threads per CTA: each block's three phases are latency-bound, so more
   // threads per block shorten them (developer knob ALT_WIN_THREADS)
-  static const int win_threads = getenv("ALT_WIN_THREADS") ? atoi(getenv("ALT_WIN_THREADS")) : 512;
+  static const int win_threads = [] {
+    const int t = getenv("ALT_WIN_THREADS") ? atoi(getenv("ALT_WIN_THREADS")) : 512;
+    return t <= 128 ? 128 : (t <= 256 ? 256 : 512);  // the kernel's launch bound is 512
+  }();
   const int per_sm = std::max(1, (int)std::min<size_t>(2048 / win_threads, (size_t)(200 * 1024) / smem));
   const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(nouter, (int64_t)nsm * per_sm));
 #define WIN_LAUNCH(T, XX)                                                                                 \
