@@ -1783,7 +1783,7 @@ static std::unordered_map<TcKey, TcPlan, TcKeyHash> g_tc_cache;
 // smem-ring depth per (BLOCK_N, CTA group): the deepest ring that fits 227 KB
 // next to the kEpiWarps staging buffers and the slab table
 constexpr int stages_for(int BN, int CG) {
-  return kEpiWarps == 8 ? (CG == 2 ? (BN == 128 ? 7 : 5) : (BN == 64 ? 7 : (BN == 128 ? 5 : 3)))  // BN 192: pair, 5
+  return kEpiWarps == 8 ? (CG == 2 ? (BN == 128 ? 7 : 5) : (BN == 64 ? 7 : (BN == 128 ? 5 : (BN == 192 ? 4 : 3))))  // BN 192 pair: 5
                         : (CG == 2 ? (BN == 128 ? 5 : 4) : (BN == 64 ? 5 : (BN == 128 ? 4 : 3)));
 }
 // halo-mode ring depth (A stage + 8 spare rows, three B tap slabs per stage)
@@ -1808,6 +1808,7 @@ static cudaError_t launch_plan_rv(const TcPlan &pl, uint16_t *yy, cudaStream_t s
   }
   if (pl.BN == 64) return launch_tc<64, stages_for(64, 1), 1, RV>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
   if (pl.BN == 128) return launch_tc<128, stages_for(128, 1), 1, RV>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+  if (pl.BN == 192) return launch_tc<192, stages_for(192, 1), 1, RV>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
   return launch_tc<256, stages_for(256, 1), 1, RV>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
 }
 static cudaError_t launch_plan(const TcPlan &pl, void *y, cudaStream_t stream) {
@@ -1827,6 +1828,7 @@ static cudaError_t launch_plan(const TcPlan &pl, void *y, cudaStream_t stream) {
     }
     if (pl.BN == 64) return launch_tc<64, stages_for(64, 1), 1, false, 1, 0, true>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
     if (pl.BN == 128) return launch_tc<128, stages_for(128, 1), 1, false, 1, 0, true>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
+    if (pl.BN == 192) return launch_tc<192, stages_for(192, 1), 1, false, 1, 0, true>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
     return launch_tc<256, stages_for(256, 1), 1, false, 1, 0, true>(pl.ta, pl.tb, pl.ty, pl.a, yy, pl.grid, stream);
   }
   return pl.a.res_vec ? launch_plan_rv<true>(pl, yy, stream) : launch_plan_rv<false>(pl, yy, stream);
@@ -1931,7 +1933,6 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
   // 2 = single CTA, 0 = pair when BLOCK_N >= 128
   const int cg = (cfg && cfg->cta_pair == 2) ? 1 : ((cfg && cfg->cta_pair == 1) || BN >= 128 ? 2 : 1);
   if (cg == 2 && BN < 128) { set_error("tc: a CTA pair needs block_n >= 128"); return ALT_E_UNSUPPORTED; }
-  if (BN == 192 && cg != 2) { set_error("tc: block_n 192 runs as a CTA pair (96 B rows per CTA)"); return ALT_E_UNSUPPORTED; }
   for (const Cand &c : cands) {
     RoleInfo ra[kMaxL], rb[kMaxL], ry[kMaxL];
     memcpy(ra, P.ra, sizeof(ra));
@@ -2144,7 +2145,7 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
         // through DSMEM (single CTA, TMA-store output, no residual, sk 2 / 4)
         pl.sc = 1;
         if (cfg && cfg->split_cluster == 1 && sk > 1) {
-          if (cg != 1 || (sk != 2 && sk != 4) || BN < 128 || a.out_mode != 1 || P.epi.residual) {
+          if (cg != 1 || (sk != 2 && sk != 4) || BN < 128 || BN == 192 || a.out_mode != 1 || P.epi.residual) {
             set_error("tc: cluster split-K needs one CTA, block_n 128/256, split 2/4, a TMA-store output and no residual");
             return ALT_E_UNSUPPORTED;
           }

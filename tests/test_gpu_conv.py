@@ -354,6 +354,23 @@ def test_tc_gemm_block_n_192(M, N, K):
     assert plan["block_n"] == 192 and plan["cta_pair"] == 1
 
 
+@pytest.mark.parametrize("M,N,K", [(1024, 768, 256), (300, 384, 136), (8192, 768, 768)])
+def test_tc_gemm_block_n_192_single_cta(M, N, K):
+    """BLOCK_N 192 on one CTA (M = 128 tiles: 4 N tiles of a 768-wide GEMM
+    fill the persistent grid in 1.73 waves where 256-wide tiles need 1.3)"""
+    _, plan = run_gemm("g192s_%d" % N, M, N, K, [], LY.gemm_b_tiled_nk(K, N, 192, 8), [], torch.bfloat16, epi=True,
+                       cfg={"path": alt.PATH_TC, "block_n": 192, "cta_pair": 2}, expect_path=alt.PATH_TC)
+    assert plan["block_n"] == 192 and plan["cta_pair"] == 2
+
+
+def test_tc_conv_block_n_192_single_cta():
+    """BLOCK_N 192 on one CTA for a conv: a ragged last N tile (K = 320)"""
+    _, plan = run_conv("c192s", 2, 64, 14, 14, 320, 3, 3, 1, 1, LY.nchwxc(64, 64), LY.kcrs_yk_xc(320, 64, 64, 64),
+                       LY.nchwxc(320, 64), torch.bfloat16, epi=True, act=1,
+                       cfg={"path": alt.PATH_TC, "block_n": 192, "cta_pair": 2}, expect_path=alt.PATH_TC)
+    assert plan["block_n"] == 192 and plan["cta_pair"] == 2
+
+
 @pytest.mark.parametrize("sk", [2, 3])
 def test_tc_tail_split(sk):
     """tail split (split_cluster = 2): whole waves of tiles unsplit, the last
