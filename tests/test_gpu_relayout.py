@@ -138,3 +138,66 @@ def test_relayout_shape_mismatch_and_lossy():
         alt.relayout(gap, torch.zeros(gap.phys_shape, device="cuda"), ident,
                      torch.zeros(10, device="cuda"))
     assert e.value.code == alt._alt.ALT_E_LOSSY
+
+
+from tests.test_oracle_layout import random_prims  # noqa: E402
+
+
+@pytest.mark.parametrize("seed", range(240))
+def test_relayout_random_layout_pairs(seed):
+    """random primitive sequences on both sides (split / reorder / fuse / pad /
+    unfold), NCHW-like shapes with 8-multiple channel and width extents so the
+    vector kernels (permutation, K_ROW, K_WIN, K_PBLOCK, warp-staged stores)
+    are reached as well as the table and generic paths; bit-exact against the
+    oracle whenever the source holds every element"""
+    import random
+    rng = random.Random(1000 + seed)
+    shape = (rng.choice([1, 2, 3]), rng.choice([8, 16, 24, 32]), rng.randint(5, 20), rng.choice([8, 12, 16, 28]))
+    sp = random_prims(shape, rng, n=rng.randint(0, 3))
+    dp = random_prims(shape, rng, n=rng.randint(1, 4))
+    So = oracle.Layout(shape, sp)
+    try:  # the oracle decides losslessness: unmaterialize needs every element
+        So.unmaterialize(So.materialize(np.zeros(shape, np.uint16)))
+    except oracle.OracleError:
+        pytest.skip("lossy source")
+    dtype = torch.bfloat16 if seed % 2 == 0 else torch.float32
+    _gpu_relayout(shape, sp, dp, dtype, f"rand{seed}")
+
+
+@pytest.mark.parametrize("seed", range(60))
+def test_relayout_random_conv_templates(seed):
+    """random conv input templates (pad + unfold + NCHW[x]c with random
+    channel tile, spatial tile, stride, padding) from random sources (NCHW,
+    NHWC, NCHW[x]c) and back: the K_WIN / K_ROW / gather paths on ragged
+    shapes, bit-exact against the oracle"""
+    import random
+    rng = random.Random(5000 + seed)
+    it = rng.choice([4, 8, 16])
+    C = it * rng.randint(1, 4)
+    H, W = rng.randint(6, 30), rng.randint(6, 30)
+    R = rng.choice([1, 3, 5])
+    V = rng.choice([1, 2])
+    pad = rng.randint(0, R // 2)
+    # spatial tiles whose window fits the padded extent (reading A4: B <= D)
+    ht = rng.choice([t for t in (1, 2, 4, 7, 8) if V * (t - 1) + R <= H + 2 * pad])
+    wt = rng.choice([t for t in (1, 2, 4, 7, 8) if V * (t - 1) + R <= W + 2 * pad])
+    shape = (rng.randint(1, 3), C, H, W)
+    src = rng.choice([[], LY.nhwc(), LY.nchwxc(C, it)])
+    dst = LY.conv_input_tiled(C, it, H, W, R, R, ht, wt, V, pad)
+    dtype = torch.bfloat16 if seed % 2 == 0 else torch.float32
+    S, D, srcd, dstd = _gpu_relayout(shape, src, dst, dtype, f"rct{seed}")
+    # and back to the source layout when the template holds every element
+    # (a stride-V window narrower than V skips pixels: then the library must
+    # refuse with ALT_E_LOSSY, as the oracle's unmaterialize does)
+    Do = oracle.Layout(shape, dst)
+    try:
+        Do.unmaterialize(Do.materialize(np.zeros(shape, np.uint16)))
+    except oracle.OracleError:
+        with pytest.raises(alt.AltError) as e:
+            alt.relayout(D, dstd, S, torch.empty_like(srcd))
+        assert e.value.code == alt._alt.ALT_E_LOSSY
+        return
+    back = torch.empty_like(srcd)
+    alt.relayout(D, dstd, S, back)
+    torch.cuda.synchronize()
+    assert torch.equal(words_t(back), words_t(srcd))
