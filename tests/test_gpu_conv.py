@@ -523,3 +523,89 @@ def test_tc_conv_halo2d(case, pad_x):
                        LY.nchwxc(K, 64), torch.bfloat16, epi=True,
                        res_p=res, act=1, cfg={"path": alt.PATH_TC, "block_k": 1, **cfg}, expect_path=alt.PATH_TC)
     assert plan["block_k"] == 3, plan   # the 2-D halo plan ran
+
+
+def _divs(n, cands):
+    return [c for c in cands if n % c == 0]
+
+
+@pytest.mark.parametrize("seed", range(300))
+def test_tc_conv_random(seed):
+    """random tensor-core convs: shape (ragged channels, small / odd images,
+    stride 1 / 2, 1x1 / 3x3, padding), layouts (NCHW[x]c, padded, NHWC for x
+    and y; KCRS[y]k[x]c / KRSC for w), kernel configuration (BLOCK_N, CTA
+    pair, output-pixel tile, split-K, halo, residual, activation) drawn at
+    random; vs the oracle (normwise + per-element bound).  Configurations the
+    planner cannot serve on the tensor cores are skipped (ALT_E_UNSUPPORTED)."""
+    import random
+    rng = random.Random(7000 + seed)
+    C = 8 * rng.randint(1, 12)
+    K = 8 * rng.randint(1, 40)
+    N = rng.randint(1, 4)
+    H, W = rng.randint(4, 30), rng.randint(4, 30)
+    R = rng.choice([1, 3])
+    V = rng.choice([1, 1, 2])
+    pad = rng.randint(0, R // 2)
+    xc = rng.choice(_divs(C, (8, 16, 32, 64)))
+    xp = rng.choice([LY.nchwxc(C, xc), LY.nchwxc(C, xc, pad_hw=pad) if pad else LY.nchwxc(C, xc), LY.nhwc()])
+    wy, wx = rng.choice(_divs(K, (8, 16, 32, 64, 128, 256))), rng.choice(_divs(C, (8, 16, 32, 64)))
+    wp = rng.choice([LY.kcrs_yk_xc(K, C, wy, wx), [("reorder", [0, 2, 3, 1])]])
+    yc = rng.choice(_divs(K, (8, 16, 32, 64)))
+    yp = rng.choice([LY.nchwxc(K, yc), LY.nhwc()])
+    res = rng.choice([None, None, LY.nchwxc(K, yc)])
+    cfg = {"path": alt.PATH_TC, "block_n": rng.choice([64, 128, 256]), "cta_pair": rng.choice([0, 2])}
+    if rng.random() < 0.5:
+        tw = rng.choice([4, 8, 16, 32, 64])
+        th = rng.choice([t for t in (1, 2, 4, 8) if t * tw <= 128])
+        cfg.update(tile_n=128 // (th * tw), tile_h=th, tile_w=tw)
+    if rng.random() < 0.2:
+        cfg["split_k"] = 2
+    if R == 3 and V == 1 and rng.random() < 0.3:
+        cfg["block_k"] = 1
+    dtype = torch.float32 if rng.random() < 0.1 else torch.bfloat16  # fp32: three bf16 planes
+    if dtype == torch.float32:
+        cfg.pop("split_k", None)
+    if N == 1 and cfg.get("tile_n", 1) > 1:
+        cfg.update(tile_n=1, tile_h=min(128 // cfg["tile_w"], 8), tile_w=128 // min(128 // cfg["tile_w"], 8))
+    try:
+        run_conv(f"rnd{seed}", N, C, H, W, K, R, R, V, pad, xp, wp, yp, dtype, epi=True,
+                 res_p=res, act=rng.choice([0, 1, 2]), cfg=cfg, expect_path=alt.PATH_TC)
+    except alt.AltError as e:
+        if e.code != alt._alt.ALT_E_UNSUPPORTED:
+            raise
+        pytest.skip(f"no tensor-core plan: {e}")
+
+
+@pytest.mark.parametrize("seed", range(150))
+def test_tc_gemm_random(seed):
+    """random tensor-core GEMMs: ragged M / N / K, A in MK / KM / tiled
+    M/mt K/kt mt kt, B in KN / NK / tiled N/nt K/kt nt kt / the paper's
+    K/kt N/nt kt nt / NKn, C in MN / tiled, random BLOCK_N, CTA pair, split-K
+    (bf16 and the fp32 three-plane path); vs the oracle"""
+    import random
+    rng = random.Random(9000 + seed)
+    M = 8 * rng.randint(1, 80)
+    N = 8 * rng.randint(1, 60)
+    K = 8 * rng.randint(1, 60)
+    ap = rng.choice([[], LY.transpose2()] + ([LY.gemm_a_tiled(M, K, mt, kt) for mt in _divs(M, (64, 128))
+                                               for kt in _divs(K, (32, 64))][:1]))
+    bps = [[], LY.transpose2()]
+    bps += [LY.gemm_b_tiled_nk(K, N, nt, kt) for nt in _divs(N, (64, 128, 256)) for kt in _divs(K, (32, 64))][:1]
+    bps += [LY.gemm_b_tiled_kn(K, N, kt, nt) for nt in _divs(N, (64, 128)) for kt in _divs(K, (32, 64))][:1]
+    bps += [LY.gemm_nkn_b(K, N)] if N % 16 == 0 else []
+    bp = rng.choice(bps)
+    cp = rng.choice([[]] + [LY.gemm_c_tiled(M, N, mt, nt) for mt in _divs(M, (64, 128)) for nt in _divs(N, (64,))][:1])
+    cfg = {"path": alt.PATH_TC, "block_n": rng.choice([64, 128, 192, 256]), "cta_pair": rng.choice([0, 2])}
+    if cfg["block_n"] == 192 and N % 8:
+        cfg["block_n"] = 128
+    dtype = torch.float32 if rng.random() < 0.1 else torch.bfloat16
+    if dtype == torch.bfloat16 and rng.random() < 0.2:
+        cfg["split_k"] = rng.choice([2, 3])
+    try:
+        run_gemm(f"rg{seed}", M, N, K, ap, bp, cp, dtype, epi=True, cfg=cfg, expect_path=alt.PATH_TC)
+    except alt.AltError as e:
+        if e.code != alt._alt.ALT_E_UNSUPPORTED:
+            raise
+        # no tensor-core plan for these layouts: the automatic path (CUDA
+        # cores) must still be exact
+        run_gemm(f"rg{seed}", M, N, K, ap, bp, cp, dtype, epi=True, cfg={"path": alt.PATH_AUTO})
