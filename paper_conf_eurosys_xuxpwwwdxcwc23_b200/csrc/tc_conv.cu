@@ -790,6 +790,11 @@ __global__ void __launch_bounds__(kThreads, 1)
       // rows alias image n0 >= N, which a GEMM view (no image dim) maps back
       // onto rows 0..127 — such a tile stores nothing
       const bool tile_ok = tc.n0 < a.N;
+      // per-warp stores: this warp's 32-row sub-box lies inside the output.
+      // When y has a size-1 spatial dim the store view drops it, so a sub-box
+      // of rows past Ho (or N) would otherwise land on row 0 (TMA clips only
+      // the dims the view keeps)
+      const bool sub_ok = tc.n0 + sn0 < a.N && tc.p0 + sp0 < a.Ho && tc.q0 + sq0 < a.Wo;
       // TMA-store coordinates of this warp's 32-row sub-box (tile part),
       // computed while the MMA may still be running
       int32_t cbase[5] = {0, 0, 0, 0, 0};
@@ -1111,7 +1116,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             fence_async_smem();
             __syncwarp();
             if (lane == 0) {
-              for (int j = 0; j < nslab && tile_ok; j++) {
+              for (int j = 0; j < nslab && tile_ok && sub_ok; j++) {
                 if (kb + (j << lg_sw) >= a.K) break;  // channels past K: nothing to store
                 const int g = ((kb + a.y_koff) >> lg_sw) + j;
                 const int gt = (int)a.O.fg.div((uint32_t)g), gr = g - gt * a.O.divg;
@@ -1237,7 +1242,8 @@ __global__ void __launch_bounds__(kThreads, 1)
           vo[V_QT] = (int)a.O.fq.div((uint32_t)sq); vo[V_QR] = sq - vo[V_QT] * a.O.divq;
           vo[V_GT] = 0; vo[V_GR] = 0; vo[V_R] = 0; vo[V_S] = 0; vo[V_ONE] = 1; vo[V_DO] = tc.d0; vo[V_T] = 0;
           coords<D3>(a.O, vo, cbq);
-          for (int j = 0; j < nslab; j++) {
+          const bool q_ok = sn < a.N && spp < a.Ho && sq < a.Wo;  // as sub_ok above
+          for (int j = 0; j < nslab && q_ok; j++) {
             if (kb + (j << lg_sw) >= a.K) break;
             const int g = ((kb + a.y_koff) >> lg_sw) + j;
             const int gt = (int)a.O.fg.div((uint32_t)g), gr = g - gt * a.O.divg;

@@ -1,0 +1,27 @@
+"""Stress the randomized parity tests over many more seeds than the suite
+runs (developer tool): usage: stress_random.py CONV_SEEDS GEMM_SEEDS RELAYOUT_SEEDS"""
+import os
+import sys
+import traceback
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import pytest  # noqa: E402
+from tests import test_gpu_conv as TC, test_gpu_relayout as TR  # noqa: E402
+
+nc, ng, nr = (int(v) for v in sys.argv[1:4])
+fails = []
+for name, fn, n, base in (("conv", TC.test_tc_conv_random, nc, 300), ("gemm", TC.test_tc_gemm_random, ng, 150),
+                          ("relayout", TR.test_relayout_random_layout_pairs, nr, 240),
+                          ("template", TR.test_relayout_random_conv_templates, nr // 4, 60)):
+    ok = skip = 0
+    for seed in range(base, base + n):
+        try:
+            fn(seed)
+            ok += 1
+        except pytest.skip.Exception:
+            skip += 1
+        except Exception as e:  # noqa: BLE001
+            fails.append((name, seed, repr(e)[:300]))
+            traceback.print_exc(limit=2)
+    print(f"{name}: {ok} ok, {skip} skipped, {len([f for f in fails if f[0] == name])} failed", flush=True)
+for f in fails:
+    print("FAIL", f)

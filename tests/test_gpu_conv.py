@@ -525,6 +525,20 @@ def test_tc_conv_halo2d(case, pad_x):
     assert plan["block_k"] == 3, plan   # the 2-D halo plan ran
 
 
+@pytest.mark.parametrize("tile", [(4, 32), (2, 64), (8, 16)])
+@pytest.mark.parametrize("W", [8, 26])
+def test_tc_conv_single_output_row(tile, W):
+    """Ho = 1 (stride 2, H = 4) with output tiles of several rows: y's size-1
+    H dim drops out of the store view, so the warps whose 32-row sub-box lies
+    past Ho must not store (they used to land on row 0; found by the
+    randomized stress, seeds 842 / 844)"""
+    th, tw = tile
+    run_conv(f"ho1{th}{W}", 2, 32, 4, W, 64, 3, 3, 2, 0, LY.nchwxc(32, 32), LY.kcrs_yk_xc(64, 32, 64, 32),
+             LY.nchwxc(64, 64), torch.bfloat16, epi=True, act=1,
+             cfg={"path": alt.PATH_TC, "block_n": 64, "cta_pair": 2, "tile_n": 1, "tile_h": th, "tile_w": tw},
+             expect_path=alt.PATH_TC)
+
+
 def _divs(n, cands):
     return [c for c in cands if n % c == 0]
 
