@@ -623,3 +623,69 @@ def test_tc_gemm_random(seed):
         # no tensor-core plan for these layouts: the automatic path (CUDA
         # cores) must still be exact
         run_gemm(f"rg{seed}", M, N, K, ap, bp, cp, dtype, epi=True, cfg={"path": alt.PATH_AUTO})
+
+
+@pytest.mark.parametrize("seed", range(200))
+def test_conv_random_any_path(seed):
+    """random convs through the whole operator surface on the automatic path
+    and, when it applies, each forced path (tensor cores, CUDA cores,
+    depthwise): groups (1, 2, depthwise), dilation, stride, padding, the
+    paper's tiled input / output templates and weight order, padded and
+    plain layouts, fp32 / bf16; vs the oracle"""
+    import random
+    rng = random.Random(11000 + seed)
+    dtype = torch.float32 if rng.random() < 0.3 else torch.bfloat16
+    g = rng.choice([1, 1, 1, 2, "dw"])
+    C = 8 * rng.randint(1, 8)
+    K = C if g == "dw" else 8 * rng.randint(1, 8)
+    groups = C if g == "dw" else g
+    N, H, W = rng.randint(1, 3), rng.randint(5, 24), rng.randint(5, 24)
+    R = rng.choice([1, 3]) if g != "dw" else 3
+    V = rng.choice([1, 1, 2])
+    d = rng.choice([1, 1, 2]) if g != "dw" else 1
+    pad = rng.randint(0, d * (R // 2))
+    Ho, Wo = (H + 2 * pad - d * (R - 1) - 1) // V + 1, (W + 2 * pad - d * (R - 1) - 1) // V + 1
+    if Ho < 1 or Wo < 1:
+        pytest.skip("empty output")
+    it = rng.choice(_divs(C, (8, 16)))
+    xps = [[], LY.nhwc(), LY.nchwxc(C, it)]
+    if d == 1 and groups == 1 and R >= V:  # (R < V: the template skips pixels the oracle reads back)
+        ht, wt = rng.choice([1, 2, 4]), rng.choice([1, 2, 4])
+        if V * (ht - 1) + R <= H + 2 * pad and V * (wt - 1) + R <= W + 2 * pad:
+            xps.append(LY.conv_input_tiled(C, it, H, W, R, R, ht, wt, V, pad))
+    xp = rng.choice(xps)
+    wps = [[], [("reorder", [0, 2, 3, 1])]]
+    if groups == 1:
+        wps += [LY.kcrs_yk_xc(K, C, rng.choice(_divs(K, (8, 16))), it), LY.kcrs_paper(K, C, rng.choice(_divs(K, (8, 16))), it)]
+    if g == "dw":
+        wps = [[("reorder", [1, 2, 3, 0])], []]
+    wp = rng.choice(wps)
+    ot = rng.choice(_divs(K, (8, 16)))
+    yps = [[], LY.nhwc(), LY.nchwxc(K, ot)]
+    for ht2 in (2, 4):
+        if Ho % ht2 == 0 and Wo % ht2 == 0:
+            yps.append(LY.conv_output_tiled(K, ot, Ho, Wo, ht2, ht2))
+    yp = rng.choice(yps)
+    x = synth.activations(f"ra{seed}x", (N, C, H, W))
+    w = synth.weights(f"ra{seed}w", (K, C // groups, R, R))
+    Ox, xph, xd = make_operand(f"ra{seed}", xp, x, dtype)
+    Ow, wph, wd = make_operand(f"ra{seed}w", wp, w, dtype)
+    Lx, Lw, Ly = alt.Layout(x.shape, xp), alt.Layout(w.shape, wp), alt.Layout((N, K, Ho, Wo), yp)
+    p = alt.conv_params(N, C, H, W, K, R, R, V, pad, groups, dilation=d)
+    act = rng.choice([0, 1, 2])
+    sc, bi = synth.bn_scale(f"ra{seed}s", K), synth.bn_bias(f"ra{seed}b", K)
+    pd = dict(N=N, C=C, H=H, W=W, K=K, R=R, S=R, stride_h=V, stride_w=V, pad_h=pad, pad_w=pad, groups=groups,
+              dil_h=d, dil_w=d)
+    ref = oracle.conv2d(pd, Ox, xph, Ow, wph, act=act, scale=sc.double().numpy(), bias=bi.double().numpy())
+    ran = 0
+    for path in (alt.PATH_AUTO, alt.PATH_TC, alt.PATH_SIMT, alt.PATH_DW):
+        y = torch.full(Ly.phys_shape, 3.0, dtype=dtype, device="cuda")
+        try:
+            alt.conv2d(p, Lx, xd, Lw, wd, Ly, y, scale=sc.cuda(), bias=bi.cuda(), act=act, cfg={"path": path})
+        except alt.AltError as e:
+            assert path != alt.PATH_AUTO and e.code == alt._alt.ALT_E_UNSUPPORTED, e
+            continue
+        torch.cuda.synchronize()
+        assert_parity(read_output(oracle.Layout((N, K, Ho, Wo), yp), y, dtype), ref, dtype)
+        ran += 1
+    assert ran >= 2   # the automatic path plus at least the path it picked
