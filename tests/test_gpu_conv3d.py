@@ -127,3 +127,46 @@ def test_c3d_rejects_bad_shapes():
     with pytest.raises(alt.AltError) as e:
         alt.conv3d(p, Lx, x, Lw, w, Ly_bad, y)
     assert e.value.code == alt._alt.ALT_E_SHAPE
+
+
+def _divs(n, cands):
+    return [c for c in cands if n % c == 0]
+
+
+@pytest.mark.parametrize("seed", range(120))
+def test_c3d_random(seed):
+    """random 3-D convs (ragged channels, odd volumes, per-axis stride /
+    padding, 1x1x1 .. 3x3x3 windows, NCDHW[x]c / NDHWC layouts, BLOCK_N, CTA
+    pair, output-pixel tile) on the tensor cores (bf16), falling back to the
+    automatic path where no tensor-core plan exists (and fp32); vs O3b"""
+    import random
+    rng = random.Random(13000 + seed)
+    C, K = 8 * rng.randint(1, 8), 8 * rng.randint(1, 16)
+    N, D, H, W = rng.randint(1, 2), rng.randint(2, 7), rng.randint(3, 14), rng.randint(3, 14)
+    T, R = rng.choice([1, 3]), rng.choice([1, 3])
+    V = tuple(rng.choice([1, 1, 2]) for _ in range(3))
+    pad = (rng.randint(0, T // 2), rng.randint(0, R // 2), rng.randint(0, R // 2))
+    if (D + 2 * pad[0] - T) < 0 or (H + 2 * pad[1] - R) < 0 or (W + 2 * pad[2] - R) < 0:
+        pytest.skip("empty output")
+    xc, yc = rng.choice(_divs(C, (8, 16, 32, 64))), rng.choice(_divs(K, (8, 16, 32, 64)))
+    xp = rng.choice([ncdhwxc(C, xc), NDHWC])
+    wp = rng.choice([kctrs_yk_xc(K, C, rng.choice(_divs(K, (8, 16, 64))), rng.choice(_divs(C, (8, 16, 32)))),
+                     [("reorder", [0, 2, 3, 4, 1])]])
+    yp = rng.choice([ncdhwxc(K, yc), NDHWC])
+    dtype = torch.float32 if rng.random() < 0.15 else torch.bfloat16
+    cfg = {"path": alt.PATH_TC, "block_n": rng.choice([64, 128, 256]), "cta_pair": rng.choice([0, 2])}
+    if rng.random() < 0.5:
+        tw = rng.choice([4, 8, 16, 32])
+        th = 128 // tw if 128 // tw <= 32 else 32
+        cfg.update(tile_n=1, tile_h=th, tile_w=128 // th)
+    act = rng.choice([0, 1])
+    if dtype == torch.bfloat16:
+        try:
+            run_conv3d(f"r3d{seed}", N, C, D, H, W, K, T, R, R, V, pad, xp, wp, yp, dtype, epi=True,
+                       act=act, cfg=cfg, expect_path=alt.PATH_TC)
+            return
+        except alt.AltError as e:
+            if e.code != alt._alt.ALT_E_UNSUPPORTED:
+                raise
+    run_conv3d(f"r3d{seed}", N, C, D, H, W, K, T, R, R, V, pad, xp, wp, yp, dtype, epi=True,
+               act=act, cfg={"path": alt.PATH_AUTO})
