@@ -661,10 +661,15 @@ def test_conv_random_any_path(seed):
         wps = [[("reorder", [1, 2, 3, 0])], []]
     wp = rng.choice(wps)
     ot = rng.choice(_divs(K, (8, 16)))
-    yps = [[], LY.nhwc(), LY.nchwxc(K, ot)]
+    yps = [[], LY.nhwc(), LY.nchwxc(K, ot), LY.nchwxc(K, ot, pad_hw=rng.randint(1, 2))]
     for ht2 in (2, 4):
         if Ho % ht2 == 0 and Wo % ht2 == 0:
             yps.append(LY.conv_output_tiled(K, ot, Ho, Wo, ht2, ht2))
+    # the next 3x3 layer's input template (pad + unfold: the epilogue writes
+    # every overlapped copy and the pad zeros; checked by read_output)
+    ht3 = rng.choice([t for t in (1, 2, 4) if t <= Ho])
+    wt3 = rng.choice([t for t in (1, 2, 4) if t <= Wo])
+    yps.append(LY.conv_input_tiled(K, ot, Ho, Wo, 3, 3, ht3, wt3, 1, 1))
     yp = rng.choice(yps)
     x = synth.activations(f"ra{seed}x", (N, C, H, W))
     w = synth.weights(f"ra{seed}w", (K, C // groups, R, R))
