@@ -681,12 +681,21 @@ def test_conv_random_any_path(seed):
     sc, bi = synth.bn_scale(f"ra{seed}s", K), synth.bn_bias(f"ra{seed}b", K)
     pd = dict(N=N, C=C, H=H, W=W, K=K, R=R, S=R, stride_h=V, stride_w=V, pad_h=pad, pad_w=pad, groups=groups,
               dil_h=d, dil_w=d)
-    ref = oracle.conv2d(pd, Ox, xph, Ow, wph, act=act, scale=sc.double().numpy(), bias=bi.double().numpy())
+    rp = rng.choice([None, None, [], LY.nchwxc(K, ot), LY.nhwc()])
+    kw, ref_kw = {}, {}
+    if rp is not None:  # residual add in the epilogue, read through its own layout
+        r = synth.activations(f"ra{seed}r", (N, K, Ho, Wo))
+        Ro, rph, rd = make_operand(f"ra{seed}r", rp, r, dtype)
+        kw.update(residual=rd, residual_l=alt.Layout((N, K, Ho, Wo), rp))
+        ref_kw.update(res_l=Ro, residual=rph)
+    ref = oracle.conv2d(pd, Ox, xph, Ow, wph, act=act, scale=sc.double().numpy(), bias=bi.double().numpy(),
+                        **ref_kw)
     ran = 0
     for path in (alt.PATH_AUTO, alt.PATH_TC, alt.PATH_SIMT, alt.PATH_DW):
         y = torch.full(Ly.phys_shape, 3.0, dtype=dtype, device="cuda")
         try:
-            alt.conv2d(p, Lx, xd, Lw, wd, Ly, y, scale=sc.cuda(), bias=bi.cuda(), act=act, cfg={"path": path})
+            alt.conv2d(p, Lx, xd, Lw, wd, Ly, y, scale=sc.cuda(), bias=bi.cuda(), act=act, cfg={"path": path},
+                       **kw)
         except alt.AltError as e:
             assert path != alt.PATH_AUTO and e.code == alt._alt.ALT_E_UNSUPPORTED, e
             continue
