@@ -572,13 +572,15 @@ def test_tc_conv_random(seed):
         tw = rng.choice([4, 8, 16, 32, 64])
         th = rng.choice([t for t in (1, 2, 4, 8) if t * tw <= 128])
         cfg.update(tile_n=128 // (th * tw), tile_h=th, tile_w=tw)
-    if rng.random() < 0.2:
-        cfg["split_k"] = 2
+    if rng.random() < 0.25:
+        cfg["split_k"] = rng.choice([2, 3, 4])
+        cfg["split_cluster"] = rng.choice([0, 1, 2])  # workspace / cluster DSMEM / tail split
     if R == 3 and V == 1 and rng.random() < 0.3:
         cfg["block_k"] = 1
     dtype = torch.float32 if rng.random() < 0.1 else torch.bfloat16  # fp32: three bf16 planes
     if dtype == torch.float32:
         cfg.pop("split_k", None)
+        cfg.pop("split_cluster", None)
     if N == 1 and cfg.get("tile_n", 1) > 1:
         cfg.update(tile_n=1, tile_h=min(128 // cfg["tile_w"], 8), tile_w=128 // min(128 // cfg["tile_w"], 8))
     try:
@@ -587,7 +589,10 @@ def test_tc_conv_random(seed):
     except alt.AltError as e:
         if e.code != alt._alt.ALT_E_UNSUPPORTED:
             raise
-        pytest.skip(f"no tensor-core plan: {e}")
+        # this configuration has no tensor-core plan (e.g. cluster split-K with
+        # a residual): the automatic path must still be exact
+        run_conv(f"rnd{seed}", N, C, H, W, K, R, R, V, pad, xp, wp, yp, dtype, epi=True,
+                 res_p=res, act=1, cfg={"path": alt.PATH_AUTO})
 
 
 @pytest.mark.parametrize("seed", range(150))
