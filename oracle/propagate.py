@@ -83,44 +83,59 @@ def layout_propagation(ops, edges, e_T: int, p_T, logical_shape):
 
 
 def joint_stage(ops, edges, tuned_layouts: dict, logical_shapes: dict):
-    """§6: complex ops in topological order (edge order here),
-    each tuned output layout propagated with Algorithm 1; multi-producer
-    rule: when an elementwise op has several tuned inputs, the one in the
-    lowest input slot (X0) wins.
+    """§6: every complex op's tuned output layout is propagated
+    with Algorithm 1 (``layout_propagation``, verbatim); where several tuned
+    layouts reach the same tensor, the multi-producer rule decides: the
+    layout that enters the elementwise producer through its lowest input slot
+    (X0) wins.  Reading A31: the slot is judged by the layout each input
+    tensor finally carries — inputs are settled before outputs, in
+    topological order — so a layout that lost at an upstream elementwise op
+    does not enter downstream ops through that op's output.
 
     tuned_layouts: edge -> primitive sequence of each complex op's output.
     Returns (assign: edge -> (source edge, prims), conversions: set of edges).
     """
-    assign: dict[int, tuple[int, list]] = {}
+    reach: dict[int, dict] = {}   # tuned edge -> {edge: prims} (Alg. 1's P)
     conversions = set()
     for e_T in sorted(tuned_layouts):
         P, conv = layout_propagation(ops, edges, e_T, tuned_layouts[e_T], logical_shapes[e_T])
         if conv is not None:
             conversions.add(conv)
-        for e, prims in P.items():
-            if e in assign and e != e_T:
-                prev_src = assign[e][0]
-                # X0 heuristic: keep the source reaching e through the lowest
-                # input slot of e's producer
-                if _entry_slot(edges, prev_src, e) <= _entry_slot(edges, e_T, e):
-                    continue
-            assign[e] = (e_T, prims)
+        reach[e_T] = P
+    assign: dict[int, tuple[int, list]] = {}
+    for e in _topological_edges(ops, edges):
+        if e in tuned_layouts:                   # a tuned tensor keeps its own layout
+            assign[e] = (e, list(tuned_layouts[e]))
+            continue
+        cands = [T for T in reach if e in reach[T]]
+        if not cands:
+            continue
+        producer = edges[e][0]
+        inputs = sorted((edges[i][3], i) for i in range(len(edges)) if edges[i][1] == producer)
+        for _, i in inputs:                      # X0: the lowest slot carrying a candidate
+            if i in assign and assign[i][0] in cands:
+                T = assign[i][0]
+                assign[e] = (T, reach[T][e])
+                break
     return assign, conversions
 
 
-def _entry_slot(edges, src_edge: int, e: int) -> int:
-    """Input slot through which src_edge's chain enters the producer of e."""
-    producer = edges[e][0]
-    # walk the chain from src_edge forward: the edge consumed by `producer`
-    # that is reachable from src_edge
-    seen = {src_edge}
-    frontier = [src_edge]
-    while frontier:
-        f = frontier.pop()
-        if edges[f][1] == producer:
-            return edges[f][3]
-        for t, (a, b, _, _) in enumerate(edges):
-            if a is not None and a == edges[f][1] and t not in seen:
-                seen.add(t)
-                frontier.append(t)
-    return 1 << 30
+def _topological_edges(ops, edges):
+    """Edges ordered so that every input edge of an op precedes its output
+    edges (Kahn's algorithm over the ops; graph inputs first)."""
+    n = len(ops)
+    indeg = [0] * n
+    for a, b, _, _ in edges:
+        if a is not None and b is not None:
+            indeg[b] += 1
+    order, ready = [], [o for o in range(n) if indeg[o] == 0]
+    while ready:
+        o = ready.pop(0)
+        order.append(o)
+        for a, b, _, _ in edges:
+            if a == o and b is not None:
+                indeg[b] -= 1
+                if indeg[b] == 0:
+                    ready.append(b)
+    rank = {o: k for k, o in enumerate(order)}
+    return sorted(range(len(edges)), key=lambda e: (-1 if edges[e][0] is None else rank[edges[e][0]], e))

@@ -180,3 +180,47 @@ def test_store_at_argument_errors_without_gpu():
     assert codes["decouple shape"] == E_SHAPE
     assert codes["gemm z shape"] == E_SHAPE
     assert codes["host pointers"] == E_INVALID
+
+
+@pytest.mark.parametrize("seed", range(150))
+def test_plan_chain_random_dags_match_oracle(seed):
+    """random op DAGs (complex / elementwise ops, chains with skip edges and
+    two-input elementwise adds, several outputs) with random tuned output
+    layouts on the complex ops (tiled channels, a non-trivial pad + unfold):
+    alt_plan_chain (Alg. 1 + the multi-producer rule, plan.cpp) against the
+    oracle's joint stage (O7) edge by edge"""
+    rng = random.Random(17000 + seed)
+    S = (1, 64, 28, 28)
+    lays = [[("split", 1, [8, 8]), ("reorder", [0, 1, 3, 4, 2])],
+            [("split", 1, [4, 16]), ("reorder", [0, 1, 3, 4, 2])],
+            [("pad", 2, 1, 1), ("unfold", 2, 10, 8)],
+            [("reorder", [0, 2, 3, 1])]]
+    n = rng.randint(2, 7)
+    kinds = [rng.choice(["complex", "elementwise"]) for _ in range(n)]
+    edges = [(None, 0, S, 0)]
+    used = set()  # a complex op's output tensor has one tuned layout: one consumer edge
+    def pick(i, exclude=()):
+        cand = [j for j in range(i) if j not in exclude and not (kinds[j] == "complex" and j in used)]
+        if not cand:
+            return None
+        j = i - 1 if (i - 1 in cand and rng.random() < 0.7) else rng.choice(cand)
+        used.add(j)
+        return j
+    for i in range(1, n):
+        src = pick(i)
+        edges.append((src, i, S, 0))
+        if kinds[i] == "elementwise" and i >= 2 and rng.random() < 0.4:
+            src2 = pick(i, exclude=(src,))
+            if src2 is not None:
+                edges.append((src2, i, S, 1))
+    consumed = {s for (s, d, _, _) in edges if s is not None}
+    for i in range(n):
+        if i not in consumed or (kinds[i] != "complex" and rng.random() < 0.15):
+            edges.append((i, None, S, 0))
+    tuned = {}
+    for e, (s, d, _, _) in enumerate(edges):
+        if s is not None and kinds[s] == "complex" and rng.random() < 0.8:
+            tuned[e] = rng.choice(lays)
+    if not tuned:
+        pytest.skip("no tuned layout")
+    _plan_case(kinds, edges, tuned)
