@@ -176,3 +176,43 @@ def test_tune_gemm_small():
     res = alt.tune("matmul", g, alt.ALT_BF16, {0: [128], 1: [64], 2: [128, 256], 6: [256]}, max_points=4,
                    warmup=1, reps=3)
     assert res["measured"] >= 1 and res["best_us"] > 0
+
+
+@pytest.mark.parametrize("seed", range(80))
+def test_pool_random(seed):
+    """random max / average pooling (window 1-5, stride 1-3, padding up to
+    half the window, odd images, fp32 / bf16) through random layouts (NCHW,
+    NHWC, NCHW[x]c, padded, the next conv's pad + unfold template); max is
+    bit-exact, average within its single rounding"""
+    import random
+    rng = random.Random(19000 + seed)
+    C = 8 * rng.randint(1, 6)
+    N, H, W = rng.randint(1, 3), rng.randint(3, 20), rng.randint(3, 20)
+    k = rng.randint(1, 5)
+    s = rng.randint(1, 3)
+    p = rng.randint(0, k // 2)
+    Ho, Wo = (H + 2 * p - k) // s + 1, (W + 2 * p - k) // s + 1
+    if Ho < 1 or Wo < 1:
+        pytest.skip("empty output")
+    kind = rng.choice(["max", "avg"])
+    dtype = torch.float32 if rng.random() < 0.3 else torch.bfloat16
+    xc, yc = rng.choice([8, 16] if C % 16 == 0 else [8]), rng.choice([8, 16] if C % 16 == 0 else [8])
+    xp = rng.choice([[], LY.nhwc(), LY.nchwxc(C, xc), LY.nchwxc(C, xc, pad_hw=1)])
+    yps = [[], LY.nhwc(), LY.nchwxc(C, yc), LY.nchwxc(C, yc, pad_hw=rng.randint(1, 2))]
+    ht, wt = rng.choice([t for t in (1, 2, 4) if t <= Ho]), rng.choice([t for t in (1, 2, 4) if t <= Wo])
+    yps.append(LY.conv_input_tiled(C, yc, Ho, Wo, 3, 3, ht, wt, 1, 1))
+    yp = rng.choice(yps)
+    x = synth.activations(f"rpool{seed}", (N, C, H, W))
+    Ox, xph, xd = make_operand(f"rpool{seed}", xp, x, dtype)
+    Ly = alt.Layout((N, C, Ho, Wo), yp)
+    y = torch.full(Ly.phys_shape, 7.0, dtype=dtype, device="cuda")
+    alt.pool2d(alt.conv_params(N, C, H, W, C, k, k, s, p), alt.Layout(x.shape, xp), xd, Ly, y, kind)
+    torch.cuda.synchronize()
+    ref = oracle.pool2d_f64(Ox.read_f64(xph), k, k, s, p, kind)
+    got = read_output(oracle.Layout((N, C, Ho, Wo), yp), y, dtype)
+    if kind == "max":
+        assert np.array_equal(got, ref)
+    elif dtype == torch.bfloat16:
+        assert norm_rel(got, ref) <= 4e-3
+    else:
+        assert np.max(np.abs(got - ref)) <= 1e-6 * max(1.0, np.max(np.abs(ref)))
