@@ -1,5 +1,5 @@
 """Stress the randomized parity tests over many more seeds than the suite
-runs (developer tool): usage: stress_random.py CONV_SEEDS GEMM_SEEDS RELAYOUT_SEEDS [ANY_PATH_SEEDS [C3D_SEEDS [STORE_AT_SEEDS [POOL_SEEDS]]]]"""
+runs (developer tool): usage: stress_random.py CONV_SEEDS GEMM_SEEDS RELAYOUT_SEEDS [ANY_PATH_SEEDS [C3D_SEEDS [STORE_AT_SEEDS [POOL_SEEDS [CHAIN_SEEDS]]]]]"""
 import os
 import sys
 import traceback
@@ -14,6 +14,7 @@ na = int(sys.argv[4]) if len(sys.argv) > 4 else 0
 n3 = int(sys.argv[5]) if len(sys.argv) > 5 else 0
 ns = int(sys.argv[6]) if len(sys.argv) > 6 else 0
 npool = int(sys.argv[7]) if len(sys.argv) > 7 else 0
+nch = int(sys.argv[8]) if len(sys.argv) > 8 else 0
 fails = []
 for name, fn, n, base in (("conv", TC.test_tc_conv_random, nc, 300), ("gemm", TC.test_tc_gemm_random, ng, 150),
                           ("relayout", TR.test_relayout_random_layout_pairs, nr, 240),
@@ -21,7 +22,8 @@ for name, fn, n, base in (("conv", TC.test_tc_conv_random, nc, 300), ("gemm", TC
                           ("any_path", TC.test_conv_random_any_path, na, 200),
                           ("c3d", T3.test_c3d_random, n3, 120),
                           ("store_at", TS.test_store_at_random, ns, 100),
-                          ("pool", TCH.test_pool_random, npool, 80)):
+                          ("pool", TCH.test_pool_random, npool, 80),
+                          ("chain", TCH.test_chain_random, nch, 40)):
     ok = skip = 0
     for seed in range(base, base + n):
         try:
