@@ -80,6 +80,7 @@ def lib():
         L.orc_relayout.restype = c_i
         L.orc_read_logical.argtypes = [c_p, c_p, c_i, c_p]
         L.orc_read_logical.restype = c_i
+        L.orc_present_mask.argtypes = [c_p, c_p]
         L.orc_conv2d_f64.argtypes = [c_p, c_p, c_p, c_p, c_p, c_p, c_i, c_ll, c_ll, c_p]
         L.orc_conv3d_f64.argtypes = [c_p, c_p, c_p, c_p, c_p, c_p, c_i, c_p]
         L.orc_conv2d_points.argtypes = [c_p, c_p, c_p, c_p, c_p, c_i, c_p, c_p, c_p, c_p,
@@ -197,17 +198,24 @@ class Layout:
         phys = np.ascontiguousarray(phys).reshape(self.phys_shape)
         return int(lib().orc_check_consistent(self._buf, _ptr(phys), _wb(phys)))
 
-    def read_f64(self, phys: np.ndarray) -> np.ndarray:
+    def read_f64(self, phys: np.ndarray, allow_lossy: bool = False) -> np.ndarray:
         """Logical fp64 values of a physical buffer of fp32 (uint32 / float32)
-        or bf16 (uint16) words."""
+        or bf16 (uint16) words.  A lossy layout raises unless allow_lossy, in
+        which case elements without a copy read as 0 (see present())."""
         phys = np.ascontiguousarray(phys).reshape(self.phys_shape)
         if phys.dtype == np.float32:
             phys = phys.view(np.uint32)
         out = np.empty(self.logical_shape, np.float64)
         rc = lib().orc_read_logical(self._buf, _ptr(phys), _wb(phys), _ptr(out))
-        if rc != E_OK:
+        if rc != E_OK and not allow_lossy:
             raise OracleError(rc, "lossy")
         return out
+
+    def present(self) -> np.ndarray:
+        """bool mask over the logical tensor: elements that have a copy."""
+        m = np.empty(self.logical_shape, np.uint8)
+        lib().orc_present_mask(self._buf, _ptr(m))
+        return m.astype(bool)
 
 
 def relayout(src_l: Layout, src: np.ndarray, dst_l: Layout) -> np.ndarray:
@@ -249,8 +257,25 @@ def conv2d(p: dict, x_l: Layout, x: np.ndarray, w_l: Layout, w: np.ndarray,
            scale=None, bias=None, res_l: Layout | None = None, residual=None,
            act: int = 0, images: tuple | None = None) -> np.ndarray:
     """O3 + O6 with operands given as physical word buffers in declared
-    layouts (read exactly through each layout's F map)."""
-    xl = x_l.read_f64(x)
+    layouts (read exactly through each layout's F map).  The input may be a
+    lossy template (reading A32: e.g. a stride-2 window narrower than its
+    stride skips pixels): the conv's sum reads only pixels h = p V - pad +
+    r d, w = q V - pad + s d (Eq. (1)), so x may omit others — if a pixel the
+    sum reads has no copy, this refuses (OracleError)."""
+    xl = x_l.read_f64(x, allow_lossy=True)
+    present = x_l.present()
+    if not present.all():
+        g = lambda k, d=0: p.get(k, d)  # noqa: E731
+        V = (g("stride_h", 1), g("stride_w", 1)); pad = (g("pad_h"), g("pad_w")); dl = (g("dil_h", 1), g("dil_w", 1))
+        ext = (p["H"], p["W"])
+        win = (p["R"], p["S"])
+        need = []
+        for a in range(2):
+            out = (ext[a] + 2 * pad[a] - dl[a] * (win[a] - 1) - 1) // V[a] + 1
+            idx = {o * V[a] - pad[a] + t * dl[a] for o in range(out) for t in range(win[a])}
+            need.append(sorted(i for i in idx if 0 <= i < ext[a]))
+        if not present[:, :, need[0]][:, :, :, need[1]].all():
+            raise OracleError(E_LOSSY, "the conv reads a pixel the input layout does not hold")
     wl = w_l.read_f64(w)
     rl = res_l.read_f64(residual) if residual is not None else None
     return conv2d_f64(p, xl, wl, scale, bias, rl, act, images)

@@ -416,6 +416,17 @@ int orc_read_logical(const orc_layout *L, const void *phys, int wb, double *out)
   return lossy ? E_LOSSY : E_OK;
 }
 
+/* present[i] = 1 when logical element i has a copy in the layout (F defined) */
+void orc_present_mask(const orc_layout *L, unsigned char *present) {
+  long long n = orc_logical_numel(L);
+#pragma omp parallel for schedule(static)
+  for (long long i = 0; i < n; i++) {
+    long long l[OR_MAXR], c[OR_MAXR];
+    unlinear(i, L->shp[0], L->lrank, l);
+    present[i] = (unsigned char)(orc_F(L, l, c) ? 1 : 0);
+  }
+}
+
 /* ------------------------------------------------------------------ O6 --- */
 /* y = act(scale*acc + bias + residual); act 0 none, 1 ReLU, 2 ReLU6. */
 static double epilogue(double acc, const double *scale, const double *bias,

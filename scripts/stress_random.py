@@ -1,5 +1,5 @@
 """Stress the randomized parity tests over many more seeds than the suite
-runs (developer tool): usage: stress_random.py CONV_SEEDS GEMM_SEEDS RELAYOUT_SEEDS [ANY_PATH_SEEDS [C3D_SEEDS [STORE_AT_SEEDS [POOL_SEEDS [CHAIN_SEEDS]]]]]"""
+runs (developer tool): usage: stress_random.py CONV_SEEDS GEMM_SEEDS RELAYOUT_SEEDS [ANY_PATH_SEEDS [C3D_SEEDS [STORE_AT_SEEDS [POOL_SEEDS [CHAIN_SEEDS [TUNE_SEEDS]]]]]]"""
 import os
 import sys
 import traceback
@@ -15,6 +15,7 @@ n3 = int(sys.argv[5]) if len(sys.argv) > 5 else 0
 ns = int(sys.argv[6]) if len(sys.argv) > 6 else 0
 npool = int(sys.argv[7]) if len(sys.argv) > 7 else 0
 nch = int(sys.argv[8]) if len(sys.argv) > 8 else 0
+ntu = int(sys.argv[9]) if len(sys.argv) > 9 else 0
 fails = []
 for name, fn, n, base in (("conv", TC.test_tc_conv_random, nc, 300), ("gemm", TC.test_tc_gemm_random, ng, 150),
                           ("relayout", TR.test_relayout_random_layout_pairs, nr, 240),
@@ -23,7 +24,8 @@ for name, fn, n, base in (("conv", TC.test_tc_conv_random, nc, 300), ("gemm", TC
                           ("c3d", T3.test_c3d_random, n3, 120),
                           ("store_at", TS.test_store_at_random, ns, 100),
                           ("pool", TCH.test_pool_random, npool, 80),
-                          ("chain", TCH.test_chain_random, nch, 40)):
+                          ("chain", TCH.test_chain_random, nch, 40),
+                          ("tune", TCH.test_tune_random, ntu, 30)):
     ok = skip = 0
     for seed in range(base, base + n):
         try:

@@ -254,3 +254,41 @@ def test_chain_random(seed):
         shapes[f"t{i}"] = (L.K, Ho)
     ch = CH.Chain(ops, rng.randint(1, 3), torch.device("cuda"), name=f"rch{seed}", img_hw=img)
     _check_chain(ch, relu6=False, min_recorded=0)
+
+
+@pytest.mark.parametrize("seed", range(30))
+def test_tune_random(seed):
+    """alt_tune on random convs over random sub-grids (channel tiles, BLOCK_N,
+    spatial template ht / wt, weight order, stages, halo): whatever point
+    wins, its layouts and configuration give an oracle-exact conv"""
+    import random
+    rng = random.Random(23000 + seed)
+    C = rng.choice([16, 32, 64, 128])
+    K = rng.choice([32, 64, 128, 192])
+    N, H = rng.randint(1, 4), rng.choice([7, 12, 14, 20, 28])
+    R = rng.choice([1, 3])
+    stride = rng.choice([1, 1, 2])
+    pad = R // 2
+    sp = {0: rng.sample([v for v in (8, 16, 32, 64) if C % v == 0], k=1),
+          1: rng.sample([v for v in (8, 16, 32, 64) if K % v == 0], k=1),
+          6: rng.sample([v for v in (64, 128, 256) if v <= max(64, K)], k=1)}   # BLOCK_N <= K
+    Ho = (H + 2 * pad - R) // stride + 1
+    if rng.random() < 0.4:
+        t = rng.choice([v for v in (2, 4, 7) if Ho % v == 0] or [0])
+        if t:
+            sp[8], sp[9] = [t], [t]
+    if rng.random() < 0.3:
+        sp[11] = [0, 1]
+    if rng.random() < 0.3:
+        sp[10] = [0, rng.choice([2, 3, 4])]
+    if R == 3 and stride == 1 and rng.random() < 0.3:
+        sp[7] = [0, 1]
+    p = alt.conv_params(N, C, H, H, K, R, R, stride, pad)
+    try:
+        res = alt.tune("conv2d", p, alt.ALT_BF16, sp, max_points=8, warmup=1, reps=2)
+    except alt.AltError as e:   # a sub-grid with no tensor-core point (e.g. a ragged
+        if e.code != alt._alt.ALT_E_UNSUPPORTED:  # N tile under an MN-major weight order)
+            raise
+        pytest.skip(str(e))
+    assert res["measured"] >= 1 and res["best_us"] > 0
+    _check_tuned_conv(p, N, C, H, K, R, pad, res, stride=stride)

@@ -285,3 +285,46 @@ def test_dilated_conv_brute_force_and_special_cases():
     wz[:, :, ::2, ::2] = w
     pz = _params(1, 3, 9, 8, 2, 5, 5, 1, 2)
     np.testing.assert_allclose(y, oracle.conv2d_f64(pz, x, wz), rtol=1e-13, atol=1e-13)
+
+
+def _template(C, H, W, R, V, ht, wt, pad=0):
+    """the paper's C2D input template (reading A6) written out
+    here (the oracle tests do not import the product's layout helpers)"""
+    Bh, Sh, Bw, Sw = V * (ht - 1) + R, V * ht, V * (wt - 1) + R, V * wt
+    return [("pad", 2, pad, pad), ("pad", 3, pad, pad), ("unfold", 2, Bh, Sh), ("unfold", 4, Bw, Sw),
+            ("split", 1, [C // 8, 8]), ("reorder", [0, 3, 5, 1, 4, 6, 2])]
+
+
+@pytest.mark.parametrize("H,W,ht,wt", [(12, 12, 2, 2), (13, 9, 2, 4), (16, 10, 4, 1)])
+def test_conv_through_lossy_template_reads_only_needed_pixels(H, W, ht, wt):
+    """reading A32: a stride-2 1x1 template (windows B = 2(ht - 1) + 1 < S = 2 ht)
+    holds only the pixels the conv reads; the oracle's conv through it equals
+    torch's conv of the full tensor (the oracle reads the skipped pixels as 0,
+    torch sees their real values: equality proves they are never used)"""
+    rng = np.random.default_rng(H * 100 + W)
+    N, C, K = 2, 16, 8
+    x = rng.standard_normal((N, C, H, W))
+    w = rng.standard_normal((K, C, 1, 1))
+    Lx = oracle.Layout((N, C, H, W), _template(C, H, W, 1, 2, ht, wt))
+    assert not Lx.present().all()                 # the template is lossy
+    xw = x.astype(np.float32).view(np.uint32)
+    phys = Lx.materialize(xw)
+    Lw = oracle.Layout((K, C, 1, 1), [])
+    ww = w.astype(np.float32).view(np.uint32)
+    p = dict(N=N, C=C, H=H, W=W, K=K, R=1, S=1, stride_h=2, stride_w=2, pad_h=0, pad_w=0)
+    got = oracle.conv2d(p, Lx, phys, Lw, Lw.materialize(ww))
+    ref = torch.nn.functional.conv2d(torch.from_numpy(x.astype(np.float32).astype(np.float64)),
+                                     torch.from_numpy(w.astype(np.float32).astype(np.float64)), stride=2).numpy()
+    assert np.allclose(got, ref, rtol=1e-12, atol=1e-12)
+
+
+def test_conv_through_lossy_template_refuses_missing_pixels():
+    """the same lossy template under a conv that needs the skipped pixels
+    (3x3 stride 1) is refused, never silently read as zeros"""
+    N, C, H, W, K = 1, 8, 12, 12, 8
+    Lx = oracle.Layout((N, C, H, W), _template(C, H, W, 1, 2, 2, 2))
+    phys = Lx.materialize(np.zeros((N, C, H, W), np.uint32))
+    Lw = oracle.Layout((K, C, 3, 3), [])
+    p = dict(N=N, C=C, H=H, W=W, K=K, R=3, S=3, pad_h=1, pad_w=1)
+    with pytest.raises(oracle.OracleError):
+        oracle.conv2d(p, Lx, phys, Lw, Lw.materialize(np.zeros((K, C, 3, 3), np.uint32)))
