@@ -298,3 +298,51 @@ def test_store_at_random(seed):
     torch.cuda.synchronize()
     assert np.array_equal(OA.unmaterialize(words(a2).reshape(OA.phys_shape)), words(A.to(dtype)))
     assert np.array_equal(words(b2), bw)
+
+
+@pytest.mark.parametrize("seed", range(80))
+def test_matmul_store_at_random(seed):
+    """random GEMMs reading their bias from the attached row: ragged M / N /
+    K, Z stored column-attached with random row padding (or the fused
+    non-separable form), a tiled or plain A, random path / BLOCK_N, scale,
+    residual, activation, both dtypes; vs the O8 oracle"""
+    import random
+    rng = random.Random(25000 + seed)
+    M, N, K = 8 * rng.randint(1, 64), 8 * rng.randint(1, 40), 8 * rng.randint(1, 40)
+    dtype = torch.float32 if rng.random() < 0.3 else torch.bfloat16
+    pad = rng.choice([0, 7, 63 - (K % 64) if (K + 1) % 64 else 0, -1])
+    A = synth.activations(f"rmsa{seed}A", (M, K))
+    B = synth.weights(f"rmsa{seed}B", (K, N))
+    bias = synth.bn_bias(f"rmsa{seed}b", N)
+    scale = synth.bn_scale(f"rmsa{seed}s", N)
+    ap = rng.choice([[], [("split", 0, [M // 8, 8]), ("split", 2, [K // 8, 8]), ("reorder", [0, 2, 1, 3])]])
+    _, _, ad = make_operand(f"rmsa{seed}A", ap, A, dtype)
+    Lz = alt.Layout((K + 1, N), z_col(K, pad))
+    z = torch.empty(Lz.phys_shape, dtype=dtype, device="cuda")
+    alt.store_at(alt.Layout((K, N), []), B.to(dtype).cuda(), bias.to(dtype).cuda(), 0, Lz, z)
+    La, Lc = alt.Layout((M, K), ap), alt.Layout((M, N), [])
+    kw = {}
+    res = None
+    if rng.random() < 0.4:
+        res = synth.activations(f"rmsa{seed}r", (M, N))
+        _, _, rd = make_operand(f"rmsa{seed}r", [], res, dtype)
+        kw = dict(residual=rd, residual_l=Lc)
+    act = rng.choice(["none", "relu"])
+    path = rng.choice([alt.PATH_AUTO, alt.PATH_TC, alt.PATH_SIMT])
+    cfg = {"path": path}
+    if path == alt.PATH_TC:
+        cfg.update(block_n=rng.choice([64, 128, 256]), cta_pair=rng.choice([0, 2]))
+    c = torch.full((M, N), float("nan"), dtype=dtype, device="cuda")
+    try:
+        alt.matmul_store_at(M, N, K, La, ad, Lz, z, Lc, c, scale=scale.cuda(), act=0 if act == "none" else act,
+                            cfg=cfg, **kw)
+    except alt.AltError as e:
+        if e.code != alt._alt.ALT_E_UNSUPPORTED or path == alt.PATH_AUTO:
+            raise
+        pytest.skip(str(e))
+    torch.cuda.synchronize()
+    f64 = lambda t: t.to(dtype).double().numpy()  # noqa: E731
+    Z = o_store_at(f64(B), f64(bias), 0)
+    want = gemm_store_at_f64(f64(A), Z, scale=scale.double().numpy(),
+                             residual=f64(res) if res is not None else None, act=act)
+    assert_parity(read_output(oracle.Layout((M, N), []), c, dtype), want, dtype)
