@@ -2006,6 +2006,11 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       if (!view_of(P.va, rah, 128, c.tw, &va, &mnA)) continue;
       if (hmode && mnA) continue;
       if (!view_of(P.vb, rb, BN / cg, BN / cg, &vb, &mnB)) continue;
+      // halo modes issue one B box per (tap, slab) from lanes 16..31: an
+      // MN-major B (ng groups per slab) would need ng x taps boxes and its
+      // tap index would run past the stage (found by the randomized stress:
+      // an out-of-bounds shared-memory write with the paper's weight order)
+      if (hmode && mnB) continue;
       int64_t rowsA = 1, rowsB = 1;
       for (int i = 1; i < va.rank; i++) rowsA *= (va.d[i].box + va.d[i].estride - 1) / va.d[i].estride;
       for (int i = 1; i < vb.rank; i++) rowsB *= (vb.d[i].box + vb.d[i].estride - 1) / vb.d[i].estride;

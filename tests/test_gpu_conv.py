@@ -539,6 +539,18 @@ def test_tc_conv_single_output_row(tile, W):
              expect_path=alt.PATH_TC)
 
 
+def test_tc_conv_halo_request_with_paper_weight_order():
+    """halo requested (block_k 1) with the paper's weight order i't o't (an
+    MN-major B): the halo modes cannot issue MN-major B groups, so the plan
+    falls back to the plain tap loop instead of writing past the B stage (an
+    illegal address found by the randomized stress, seed 499)"""
+    _, plan = run_conv("halopaperw", 3, 64, 28, 18, 280, 3, 3, 1, 1, LY.nhwc(), LY.kcrs_paper(280, 64, 8, 64),
+                       LY.nchwxc(280, 8), torch.bfloat16, epi=True, act=1,
+                       cfg={"path": alt.PATH_TC, "block_n": 64, "cta_pair": 2, "tile_n": 4, "tile_h": 1,
+                            "tile_w": 32, "block_k": 1}, expect_path=alt.PATH_TC)
+    assert plan["block_k"] == 64, plan
+
+
 def _divs(n, cands):
     return [c for c in cands if n % c == 0]
 
@@ -561,9 +573,12 @@ def test_tc_conv_random(seed):
     V = rng.choice([1, 1, 2])
     pad = rng.randint(0, R // 2)
     xc = rng.choice(_divs(C, (8, 16, 32, 64)))
-    xp = rng.choice([LY.nchwxc(C, xc), LY.nchwxc(C, xc, pad_hw=pad) if pad else LY.nchwxc(C, xc), LY.nhwc()])
+    # plain NCHW (MN-major A: 1x1 unpadded convs with 8-multiple H W) and the
+    # paper's weight order i't o't (MN-major B) join the K-major layouts
+    xp = rng.choice([LY.nchwxc(C, xc), LY.nchwxc(C, xc, pad_hw=pad) if pad else LY.nchwxc(C, xc), LY.nhwc(), []])
     wy, wx = rng.choice(_divs(K, (8, 16, 32, 64, 128, 256))), rng.choice(_divs(C, (8, 16, 32, 64)))
-    wp = rng.choice([LY.kcrs_yk_xc(K, C, wy, wx), [("reorder", [0, 2, 3, 1])]])
+    wp = rng.choice([LY.kcrs_yk_xc(K, C, wy, wx), [("reorder", [0, 2, 3, 1])],
+                     LY.kcrs_paper(K, C, rng.choice(_divs(K, (8, 16, 32, 64))), wx)])
     yc = rng.choice(_divs(K, (8, 16, 32, 64)))
     yp = rng.choice([LY.nchwxc(K, yc), LY.nhwc()])
     res = rng.choice([None, None, LY.nchwxc(K, yc)])
