@@ -2011,6 +2011,14 @@ static alt_status tc_run(TcProblem &P, const alt_kernel_cfg *cfg, cudaStream_t s
       // tap index would run past the stage (found by the randomized stress:
       // an out-of-bounds shared-memory write with the paper's weight order)
       if (hmode && mnB) continue;
+      // a group's weight rows start at b_koff: when the weight layout splits
+      // K into tiles of divq rows the box origin must sit on a tile boundary
+      // (a box covers whole tiles; found by the randomized stress: K / groups
+      // = 144 on a K/32 weight layout read the wrong rows)
+      if (vb.divq > 1 && vb.divq < (1 << 30) && P.koff % vb.divq) {
+        snprintf(why, 160, "group weight offset %lld not a multiple of the weight k tile %d", (long long)P.koff, vb.divq);
+        continue;
+      }
       int64_t rowsA = 1, rowsB = 1;
       for (int i = 1; i < va.rank; i++) rowsA *= (va.d[i].box + va.d[i].estride - 1) / va.d[i].estride;
       for (int i = 1; i < vb.rank; i++) rowsB *= (vb.d[i].box + vb.d[i].estride - 1) / vb.d[i].estride;

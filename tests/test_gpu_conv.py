@@ -16,13 +16,13 @@ pytestmark = pytest.mark.gpu
 
 
 def run_conv(name, N, C, H, W, K, R, S, V, pad, xp, wp, yp, dtype, groups=1, epi=False,
-             res_p=None, act=0, cfg=None, expect_path=None):
+             res_p=None, act=0, cfg=None, expect_path=None, dil=1):
     x = synth.activations(name + "x", (N, C, H, W))
     w = synth.weights(name + "w", (K, C // groups, R, S))
-    Ho, Wo = (H + 2 * pad - R) // V + 1, (W + 2 * pad - S) // V + 1
+    Ho, Wo = (H + 2 * pad - dil * (R - 1) - 1) // V + 1, (W + 2 * pad - dil * (S - 1) - 1) // V + 1
     Xo, xph, xd = make_operand(name, xp, x, dtype)
     Wo_, wph, wd = make_operand(name, wp, w, dtype)
-    p = alt.conv_params(N, C, H, W, K, R, S, V, pad, groups)
+    p = alt.conv_params(N, C, H, W, K, R, S, V, pad, groups, dilation=dil)
     Lx, Lw, Ly = alt.Layout(x.shape, xp), alt.Layout(w.shape, wp), alt.Layout((N, K, Ho, Wo), yp)
     y = torch.full(Ly.phys_shape, 3.0, dtype=dtype, device="cuda")  # poison
     kw = {}
@@ -42,7 +42,7 @@ def run_conv(name, N, C, H, W, K, R, S, V, pad, xp, wp, yp, dtype, groups=1, epi
     if expect_path is not None:
         assert plan["path"] == expect_path, plan
     pd = dict(N=N, C=C, H=H, W=W, K=K, R=R, S=S, stride_h=V, stride_w=V, pad_h=pad, pad_w=pad,
-              groups=groups)
+              groups=groups, dil_h=dil, dil_w=dil)
     ref = oracle.conv2d(pd, Xo, xph, Wo_, wph, act=act, **ref_kw)
     got = read_output(oracle.Layout((N, K, Ho, Wo), yp), y, dtype)
     return assert_parity(got, ref, dtype), plan
@@ -551,6 +551,23 @@ def test_tc_conv_halo_request_with_paper_weight_order():
     assert plan["block_k"] == 64, plan
 
 
+def test_tc_grouped_conv_misaligned_group_weight_offset():
+    """grouped conv whose per-group weight offset (K / groups = 144) is not a
+    multiple of the weight layout's k tile (32): the tensor-core plan is
+    refused (its B box would start mid-tile and read the wrong rows — found by
+    the randomized stress) and the automatic path stays exact"""
+    args = ("grpmis", 2, 64, 12, 12, 288, 1, 1, 1, 0, LY.nchwxc(64, 8), LY.kcrs_yk_xc(288, 32, 32, 8),
+            LY.nchwxc(288, 8), torch.bfloat16)
+    with pytest.raises(alt.AltError) as e:
+        run_conv(*args, groups=2, cfg={"path": alt.PATH_TC, "block_n": 64, "cta_pair": 2})
+    assert e.value.code == alt._alt.ALT_E_UNSUPPORTED
+    run_conv(*args, groups=2, cfg={"path": alt.PATH_AUTO})
+    # aligned offsets (K / groups = 160 = 5 x 32) keep the tensor cores
+    run_conv("grpal", 2, 64, 12, 12, 320, 1, 1, 1, 0, LY.nchwxc(64, 8), LY.kcrs_yk_xc(320, 32, 32, 8),
+             LY.nchwxc(320, 8), torch.bfloat16, groups=2, cfg={"path": alt.PATH_TC, "block_n": 64, "cta_pair": 2},
+             expect_path=alt.PATH_TC)
+
+
 def _divs(n, cands):
     return [c for c in cands if n % c == 0]
 
@@ -572,13 +589,16 @@ def test_tc_conv_random(seed):
     R = rng.choice([1, 3])
     V = rng.choice([1, 1, 2])
     pad = rng.randint(0, R // 2)
+    g = rng.choice([1, 1, 1, 2]) if C % 16 == 0 and K % 16 == 0 else 1     # grouped (GRP)
+    dil = rng.choice([1, 1, 2]) if R == 3 and H >= 7 and W >= 7 else 1    # dilated (DIL)
     xc = rng.choice(_divs(C, (8, 16, 32, 64)))
     # plain NCHW (MN-major A: 1x1 unpadded convs with 8-multiple H W) and the
     # paper's weight order i't o't (MN-major B) join the K-major layouts
     xp = rng.choice([LY.nchwxc(C, xc), LY.nchwxc(C, xc, pad_hw=pad) if pad else LY.nchwxc(C, xc), LY.nhwc(), []])
-    wy, wx = rng.choice(_divs(K, (8, 16, 32, 64, 128, 256))), rng.choice(_divs(C, (8, 16, 32, 64)))
-    wp = rng.choice([LY.kcrs_yk_xc(K, C, wy, wx), [("reorder", [0, 2, 3, 1])],
-                     LY.kcrs_paper(K, C, rng.choice(_divs(K, (8, 16, 32, 64))), wx)])
+    Cg = C // g
+    wy, wx = rng.choice(_divs(K, (8, 16, 32, 64, 128, 256))), rng.choice(_divs(Cg, (8, 16, 32, 64)))
+    wp = rng.choice([LY.kcrs_yk_xc(K, Cg, wy, wx), [("reorder", [0, 2, 3, 1])],
+                     LY.kcrs_paper(K, Cg, rng.choice(_divs(K, (8, 16, 32, 64))), wx)])
     yc = rng.choice(_divs(K, (8, 16, 32, 64)))
     yp = rng.choice([LY.nchwxc(K, yc), LY.nhwc()])
     res = rng.choice([None, None, LY.nchwxc(K, yc)])
@@ -599,14 +619,14 @@ def test_tc_conv_random(seed):
     if N == 1 and cfg.get("tile_n", 1) > 1:
         cfg.update(tile_n=1, tile_h=min(128 // cfg["tile_w"], 8), tile_w=128 // min(128 // cfg["tile_w"], 8))
     try:
-        run_conv(f"rnd{seed}", N, C, H, W, K, R, R, V, pad, xp, wp, yp, dtype, epi=True,
+        run_conv(f"rnd{seed}", N, C, H, W, K, R, R, V, pad, xp, wp, yp, dtype, epi=True, groups=g, dil=dil,
                  res_p=res, act=rng.choice([0, 1, 2]), cfg=cfg, expect_path=alt.PATH_TC)
     except alt.AltError as e:
         if e.code != alt._alt.ALT_E_UNSUPPORTED:
             raise
         # this configuration has no tensor-core plan (e.g. cluster split-K with
         # a residual): the automatic path must still be exact
-        run_conv(f"rnd{seed}", N, C, H, W, K, R, R, V, pad, xp, wp, yp, dtype, epi=True,
+        run_conv(f"rnd{seed}", N, C, H, W, K, R, R, V, pad, xp, wp, yp, dtype, epi=True, groups=g, dil=dil,
                  res_p=res, act=1, cfg={"path": alt.PATH_AUTO})
 
 
