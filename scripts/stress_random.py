@@ -16,6 +16,7 @@ ns = int(sys.argv[6]) if len(sys.argv) > 6 else 0
 npool = int(sys.argv[7]) if len(sys.argv) > 7 else 0
 nch = int(sys.argv[8]) if len(sys.argv) > 8 else 0
 ntu = int(sys.argv[9]) if len(sys.argv) > 9 else 0
+off = int(os.environ.get("STRESS_SEED_OFFSET", "0"))  # explore seeds past the ones already run
 fails = []
 for name, fn, n, base in (("conv", TC.test_tc_conv_random, nc, 300), ("gemm", TC.test_tc_gemm_random, ng, 150),
                           ("relayout", TR.test_relayout_random_layout_pairs, nr, 240),
@@ -27,7 +28,7 @@ for name, fn, n, base in (("conv", TC.test_tc_conv_random, nc, 300), ("gemm", TC
                           ("chain", TCH.test_chain_random, nch, 40),
                           ("tune", TCH.test_tune_random, ntu, 30)):
     ok = skip = 0
-    for seed in range(base, base + n):
+    for seed in range(base + off, base + off + n):
         try:
             fn(seed)
             ok += 1
