@@ -371,7 +371,8 @@ def main():
                           f"batch {args.batch} per GPU, bf16, tuned ALT layouts, fused BN+ReLU",
               "global_batch": args.batch * ws, "per_gpu_batch": args.batch,
               "parallelism": f"dp{ws} (batch shards, no collective)",
-              "l2": "inputs larger than L2 (~726 MB touched per step at batch 32)"}
+              "l2": "inputs larger than L2 (~726 MB touched per step at batch 32)",
+              "warmup_note": "W eager warm-up steps, then one untimed replay of the K-step graph"}
 
     if args.impl == "reference":
         if rank != 0:
@@ -430,6 +431,11 @@ def main():
         except Exception as e:  # fall back to eager launches
             print(f"graph capture failed ({e}); timing eager launches", file=sys.stderr)
             graph = graph_ev = None
+    if graph is not None and os.environ.get("ALT_BENCH_PREREPLAY", "1") == "1":
+        # one untimed replay (more warm-up steps): uploads the graph's nodes to
+        # the device and brings the SM clock up before the timed replay
+        graph.replay()
+        torch.cuda.synchronize()
     with Clocks(local) as clk:
         barrier(ws)
         torch.cuda.synchronize()
@@ -451,6 +457,9 @@ def main():
     ms = max_over_ranks(ms, ws)
     # per-layer pass
     if graph_ev is not None:
+        if os.environ.get("ALT_BENCH_PREREPLAY", "1") == "1":
+            graph_ev.replay()  # untimed: upload
+            torch.cuda.synchronize()
         graph_ev.replay()
     else:
         for k in range(args.steps):
