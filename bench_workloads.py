@@ -212,24 +212,28 @@ def run(args):
         r = r18_strong(args.steps, args.warmup, ws, rank, dev)
         out = _line(args, ws, r["tflops"], "TFLOP/s", r["ms_per_step"],
                     {"workload": r["workload"], "global_batch": 256, "per_gpu_batch": r["per_gpu_batch"],
-                     "parallelism": f"dp{ws}"},
+                     "parallelism": f"dp{ws}",
+                     "l2": "inputs larger than L2 (R18 chain at batch 256 touches > 1 GB per step)"},
                     {"scaling": "strong", "gpu_launches": r["gpu_launches_per_step"] * args.steps,
                      "propagation": r["propagation"], "gathered_bytes": r["gathered_bytes"]})
     elif args.workload == "mv2":
         r = mv2_chain(args.steps, args.warmup, ws, dev)
         out = _line(args, ws, r["tflops"] * ws, "TFLOP/s", r["ms_per_step"],
                     {"workload": r["workload"], "global_batch": 16 * ws, "per_gpu_batch": 16,
-                     "parallelism": f"dp{ws}"},
+                     "parallelism": f"dp{ws}", "l2": f"inputs larger than L2 ({r['hbm_bytes_min'] / 1e6:.0f} MB "
+                                                      "of algorithmic HBM traffic per step)"},
                     {"scaling": "weak", "gpu_launches": r["gpu_launches_per_step"] * args.steps,
                      "propagation": r["propagation"], "hbm_gbs_min": r["hbm_gbs_min"]})
     elif args.workload == "bert":
         r = bert_set(args.steps, args.warmup, ws, dev, args.bert_bias)
         out = _line(args, ws, r["tflops"] * ws, "TFLOP/s", r["ms_per_step"],
-                    {"workload": r["workload"], "global_batch": 16 * ws, "seq_len": 512, "parallelism": f"dp{ws}"},
+                    {"workload": r["workload"], "global_batch": 16 * ws, "seq_len": 512, "parallelism": f"dp{ws}",
+                     "l2": "inputs larger than L2 (the three GEMMs touch ~161 MB of A, B and C per step; per_gemm repeats one GEMM, whose operands fit in L2)"},
                     {"scaling": "weak", "per_gemm": r["per_gemm"], "gpu_launches": 3 * args.steps})
     elif args.workload == "relayout":
         r = relayout_run(args.steps, ws, dev)
-        out = _line(args, ws, r["gbs"], "GB/s", r["ms"], {"workload": r["workload"], "parallelism": f"dp{ws}"},
+        out = _line(args, ws, r["gbs"], "GB/s", r["ms"], {"workload": r["workload"], "parallelism": f"dp{ws}",
+                                                      "l2": "no flush; each case moves src + dst >= 200 MB except R6 bf16 (101 MB, partly L2-resident across repetitions) and R7 (9.4 MB of weights, the offline a3 transform, L2-resident)"},
                     {"scaling": "weak", "hbm_peak_gbs": r["hbm_peak_gbs"], "cases": r["cases"]})
     elif args.workload == "fig12":
         out = fig12(args, ws)
