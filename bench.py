@@ -248,6 +248,9 @@ class LayerSet:
             for _ in range(steps):
                 self.step()
         torch.cuda.current_stream().wait_stream(s)
+        if os.environ.get("ALT_BENCH_PREREPLAY", "1") == "1":
+            g.replay()  # untimed (more warm-up steps): graph upload, allocator pools
+            torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record()
         g.replay()

@@ -80,3 +80,30 @@ def test_fp32_tc_r50_layer_full_size():
     err, _ = run_conv("f32l3", 32, 256, 14, 14, 256, 3, 3, 1, 1, LY.nchwxc(256, 64), LY.kcrs_yk_xc(256, 256, 256, 64),
                       LY.nchwxc(256, 64), F32, epi=True, act=1, cfg=TC, expect_path=alt.PATH_TC)
     assert err <= FP32_TOL
+
+
+def test_fp32_r50_layer_set_b32_bench_config():
+    """the R50 set at batch 32 in fp32 exactly as bench.py's aux.r50_fp32 runs
+    it (layouts and kernel configurations from the tune cache, split-K forms
+    dropped): every image of every layer against the oracle at the fp32 bar"""
+    import oracle
+    import bench
+    from tests.helpers import norm_rel, words
+    S = bench.LayerSet(32, torch.device("cuda", 0), F32)
+    S.step()
+    torch.cuda.synchronize()
+    for l in S.layers:
+        L = l["L"]
+        Ho, Wo = L.out_hw()
+        Ox = oracle.Layout((32, L.C, L.H, L.W), l["lx"].prims)
+        Ow = oracle.Layout((L.K, L.C, L.R, L.S), l["lw"].prims)
+        Oy = oracle.Layout((32, L.K, Ho, Wo), l["ly"].prims)
+        pd = dict(N=32, C=L.C, H=L.H, W=L.W, K=L.K, R=L.R, S=L.S, stride_h=L.stride, stride_w=L.stride,
+                  pad_h=L.pad, pad_w=L.pad)
+        ref = oracle.conv2d_f64(pd, Ox.read_f64(words(l["x"])), Ow.read_f64(words(l["w"])),
+                                l["sc"].double().cpu().numpy(), l["bi"].double().cpu().numpy(), None, 1)
+        yw = words(l["y"])
+        assert Oy.check_consistent(yw) == 0, L.name
+        got = Oy.read_f64(yw)
+        for n in range(32):
+            assert norm_rel(got[n], ref[n]) <= FP32_TOL, (L.name, n, l["cfg"])
