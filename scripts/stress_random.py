@@ -34,7 +34,7 @@ for name, fn, n, base in (("conv", TC.test_tc_conv_random, nc, 300), ("gemm", TC
             ok += 1
         except pytest.skip.Exception:
             skip += 1
-        except Exception as e:  # noqa: BLE001
+        except (Exception, pytest.fail.Exception) as e:  # noqa: BLE001
             fails.append((name, seed, repr(e)[:300]))
             traceback.print_exc(limit=2)
     print(f"{name}: {ok} ok, {skip} skipped, {len([f for f in fails if f[0] == name])} failed", flush=True)

@@ -287,17 +287,17 @@ def test_store_at_random(seed):
     bw = words(b.to(dtype))
     want = OZ.materialize(o_store_at(words(A.to(dtype)), bw, dim))
     La, Lz = alt.Layout(ashape, ap), alt.Layout(zshape, zp)
-    for Ll, prims in ((La, ap), (Lz, zp)):
-        if not Ll.flags & 1:
-            # reading A4: any unfold with B < S marks the layout lossy, even
-            # where another unfold re-covers the gap (the oracle's round trip
-            # then succeeds); the library refuses it — conservative, never wrong
-            assert any(p[0] == "unfold" and p[2] < p[3] for p in prims), prims
-            with pytest.raises(alt.AltError) as e:
-                alt.store_at(La, ad, from_words(bw, dtype), dim, Lz,
-                             torch.empty(Lz.phys_shape, dtype=dtype, device="cuda"))
-            assert e.value.code == alt._alt.ALT_E_LOSSY
-            pytest.skip("unfold B < S re-covered by another unfold: refused by the library (A4)")
+    if not La.flags & 1:
+        # reading A4: any unfold with B < S marks the layout lossy, even where
+        # another unfold re-covers the gap (the oracle's round trip then
+        # succeeds); store_at refuses such an A (it reads every element of A),
+        # and decouple_at such a Z below — conservative, never wrong
+        assert any(p[0] == "unfold" and p[2] < p[3] for p in ap), ap
+        with pytest.raises(alt.AltError) as e:
+            alt.store_at(La, ad, from_words(bw, dtype), dim, Lz,
+                         torch.empty(Lz.phys_shape, dtype=dtype, device="cuda"))
+        assert e.value.code == alt._alt.ALT_E_LOSSY
+        pytest.skip("unfold B < S re-covered by another unfold: refused by the library (A4)")
     z = torch.full(Lz.phys_shape, 7, dtype=dtype, device="cuda")
     alt.store_at(La, ad, from_words(bw, dtype), dim, Lz, z)
     torch.cuda.synchronize()
@@ -305,6 +305,12 @@ def test_store_at_random(seed):
     # decouple_at inverts it (A and the attached slice back, bit for bit)
     a2 = torch.empty(La.phys_shape, dtype=dtype, device="cuda")
     b2 = torch.empty(b.shape, dtype=dtype, device="cuda")
+    if not Lz.flags & 1:  # reading A4's static rule on Z (see above): refused
+        assert any(p[0] == "unfold" and p[2] < p[3] for p in zp), zp
+        with pytest.raises(alt.AltError) as e:
+            alt.decouple_at(Lz, z, dim, La, a2, b2)
+        assert e.value.code == alt._alt.ALT_E_LOSSY
+        return
     alt.decouple_at(Lz, z, dim, La, a2, b2)
     torch.cuda.synchronize()
     assert np.array_equal(OA.unmaterialize(words(a2).reshape(OA.phys_shape)), words(A.to(dtype)))
